@@ -1,0 +1,126 @@
+"""CPU oracle for the CUDAAdvisor trace analyses — TEST INFRASTRUCTURE ONLY.
+
+Only tests/, __graft_entry__.smoke() and bench.py (its cpu_baseline leg and
+--impl reference) may import this package.  The product path
+(paper_conf_cgo_shensll18_b200) never imports it and shares no code with it.
+
+Functions follow PAPER.md (see oracle.cpp header for the passages):
+  reuse(trace, ...)        LRU-stack reuse-distance histogram
+  reuse_rd(trace, ...)     per-record reuse distances
+  reuse_brute(trace, ...)  O(n^2) literal definition
+  mem_div(trace, ...)      unique lines per warp instruction
+  branch_div(trace, ...)   divergent warp-level block executions
+Every function is pinned in tests/test_oracle_pins.py.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "liboracle.so")
+_lib = None
+
+SCOPE_CTA, SCOPE_KERNEL = 0, 1
+BINS_LINEAR, BINS_LOG2 = 0, 1
+
+
+class OracleError(RuntimeError):
+    def __init__(self, code):
+        super().__init__({1: "invalid argument", 2: "bad trace"}.get(code, f"error {code}"))
+        self.code = code
+
+
+def _load():
+    global _lib
+    if _lib is not None:
+        return _lib
+    src = os.path.join(_HERE, "oracle.cpp")
+    if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
+        subprocess.check_call(["g++", "-O2", "-std=c++17", "-fopenmp", "-shared", "-fPIC", "-o", _SO, src])
+    lib = ctypes.CDLL(_SO)
+    P, u64, u32, i32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
+    lib.oracle_reuse.argtypes = [P, P, P, P, u64, u32, i32, i32, u32, P, P]
+    lib.oracle_reuse_rd.argtypes = [P, P, P, P, u64, u32, i32, P]
+    lib.oracle_reuse_brute.argtypes = [P, P, P, P, u64, u32, i32, i32, u32, P, P, P]
+    lib.oracle_mem_div.argtypes = [P, P, P, P, P, P, u64, u32, u32, u32, P, P]
+    lib.oracle_branch_div.argtypes = [P, P, P, P, P, u64, u32, u32, P, P]
+    for f in ("oracle_reuse", "oracle_reuse_rd", "oracle_reuse_brute", "oracle_mem_div",
+              "oracle_branch_div", "oracle_num_threads"):
+        getattr(lib, f).restype = ctypes.c_int
+    _lib = lib
+    return lib
+
+
+def _p(a):
+    return a.ctypes.data if a is not None else None
+
+
+def _check(rc):
+    if rc != 0:
+        raise OracleError(rc)
+
+
+def num_threads() -> int:
+    return int(_load().oracle_num_threads())
+
+
+def reuse(t, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66):
+    """Returns (hist[nbins] u64, stats dict)."""
+    lib = _load()
+    hist = np.zeros(nbins, np.uint64)
+    st = np.zeros(4, np.uint64)
+    _check(lib.oracle_reuse(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.meta), t.n, line_bytes, scope, binning,
+                            nbins, _p(hist), _p(st)))
+    return hist, dict(zip(("accesses", "inf", "streaming", "overflow"), map(int, st)))
+
+
+def reuse_rd(t, line_bytes=128, scope=SCOPE_CTA):
+    """Per-record reuse distance: >=0 finite, -1 = ∞, -2 = not a memory record."""
+    lib = _load()
+    rd = np.zeros(t.n, np.int64)
+    _check(lib.oracle_reuse_rd(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.meta), t.n, line_bytes, scope, _p(rd)))
+    return rd
+
+
+def reuse_brute(t, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66):
+    """O(n^2) literal definition; returns (hist, stats, rd per record)."""
+    lib = _load()
+    hist = np.zeros(nbins, np.uint64)
+    st = np.zeros(4, np.uint64)
+    rd = np.zeros(t.n, np.int64)
+    _check(lib.oracle_reuse_brute(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.meta), t.n, line_bytes, scope, binning,
+                                  nbins, _p(hist), _p(st), _p(rd)))
+    return hist, dict(zip(("accesses", "inf", "streaming", "overflow"), map(int, st))), rd
+
+
+def mem_div(t, line_bytes=128, warp_size=32, nsites=None, per_site=True):
+    """Returns (hist[2][W+1] u64, per_site[nsites][2] u64 or None)."""
+    lib = _load()
+    nsites = t.nsites if nsites is None else nsites
+    hist = np.zeros((2, warp_size + 1), np.uint64)
+    ps = np.zeros((nsites, 2), np.uint64) if per_site else None
+    _check(lib.oracle_mem_div(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.winst), _p(t.site), _p(t.meta), t.n,
+                              line_bytes, warp_size, nsites, _p(hist), _p(ps)))
+    return hist, ps
+
+
+def branch_div(t, warp_size=32, nsites=None, per_site=True):
+    """Returns (per_site[nsites][3] u64 or None, totals[3] u64 = exec, divergent, threads)."""
+    lib = _load()
+    nsites = t.nsites if nsites is None else nsites
+    ps = np.zeros((nsites, 3), np.uint64) if per_site else None
+    tot = np.zeros(3, np.uint64)
+    _check(lib.oracle_branch_div(_p(t.cta), _p(t.tid), _p(t.winst), _p(t.site), _p(t.meta), t.n, warp_size,
+                                 nsites, _p(ps), _p(tot)))
+    return ps, tot
+
+
+def md_degree(hist):
+    """Memory divergence degree: sum_k k*h_k / sum_k h_k over pooled loads+stores."""
+    h = np.asarray(hist, dtype=np.float64).sum(axis=0)
+    k = np.arange(len(h))
+    return float((k * h).sum() / h.sum()) if h.sum() else 0.0

@@ -1,0 +1,408 @@
+// oracle — plain, slow, obviously-correct CPU reference for the CUDAAdvisor
+// trace analyses.  TEST INFRASTRUCTURE ONLY: only tests/, __graft_entry__.smoke()
+// and bench.py's cpu_baseline / --impl reference legs may load this library.
+// It shares no code, header, table or helper with the CUDA path
+// (paper_conf_cgo_shensll18_b200/); the only common input is the record
+// layout produced by tracegen/.
+//
+// Each function follows the paper's definition step by step (PAPER.md =
+// /root/reference/PAPER.md; "P:Lnnn" = its line):
+//   * reuse distance: "the number of distinctive data elements accessed
+//     between two consecutive uses of the same element", with the write tweak
+//     "once an address A is written, we will restart its reuse distance
+//     counting as another address A'" and ∞ = "never reused ... or
+//     before the next write"; per CTA after regrouping by CTA id
+//     (P:L237); memory-element or cache-line model; streaming
+//     accesses "never reused by the same CTA".
+//       - oracle_reuse: explicit LRU stack of renamed (line, write-epoch) keys.
+//       - oracle_reuse_brute: literal O(n^2) definition (tiny traces only).
+//   * memory divergence: "the number of unique cache lines touched by each
+//     instruction", per dynamic warp-level instruction, a std::set
+//     of lines per group (group identity = (cta, tid / W, winst), DESIGN.md
+//     reading R9); degree = weighted average left to the caller.
+//   * branch divergence: how many times a block executes, how many threads,
+//     how often it makes the warp diverge; divergent = fewer active
+//     lanes than launched lanes of that warp (reading R12).
+//
+// Parity status: every function here is pinned by tests/test_oracle_pins.py
+// (paper-printed values, closed forms, brute force, invariants); see DESIGN.md
+// "Oracle pins".
+#include <algorithm>
+#include <cstdint>
+#include <cstring>
+#include <map>
+#include <set>
+#include <tuple>
+#include <unordered_map>
+#include <utility>
+#include <vector>
+#ifdef _OPENMP
+#include <omp.h>
+#endif
+
+namespace {
+
+enum { OK = 0, INVALID_ARG = 1, BAD_TRACE = 2 };
+enum { KIND_LOAD = 0, KIND_STORE = 1, KIND_BB = 2 };
+enum { SCOPE_CTA = 0, SCOPE_KERNEL = 1 };
+enum { BINS_LINEAR = 0, BINS_LOG2 = 1 };
+
+bool pow2(uint32_t x) { return x && !(x & (x - 1)); }
+
+// Per-record validity: kind <= 2, reserved meta
+// bits 5..7 zero, memory records naturally aligned and below 2^62, tid < 1024.
+bool record_ok(uint64_t addr, uint16_t tid, uint8_t meta) {
+  uint32_t kind = meta & 3u;
+  if (kind == 3 || (meta >> 5) != 0) return false;
+  if (tid >= 1024) return false;
+  if (kind != KIND_BB) {
+    uint32_t lg = (meta >> 2) & 7u;
+    if (lg > 4) return false;
+    uint64_t bytes = 1ull << lg;
+    if (addr % bytes != 0) return false;
+    if (addr >> 62) return false;
+  }
+  return true;
+}
+
+bool check_all(const uint64_t* addr, const uint16_t* tid, const uint8_t* meta, uint64_t n) {
+  for (uint64_t i = 0; i < n; ++i)
+    if (!record_ok(addr ? addr[i] : 0, tid ? tid[i] : 0, meta[i])) return false;
+  return true;
+}
+
+// Histogram index for a finite reuse distance d.
+uint32_t bin_of(uint64_t d, int binning, uint32_t nbins) {
+  if (binning == BINS_LINEAR) return d <= nbins - 3 ? (uint32_t)d : nbins - 2;
+  if (d == 0) return 0;
+  uint32_t k = 0;                      // k = floor(log2 d) + 1
+  while ((d >> k) != 0) ++k;
+  return k <= nbins - 3 ? k : nbins - 2;
+}
+
+struct KeyHash {
+  size_t operator()(const std::pair<uint64_t, uint64_t>& k) const {
+    return std::hash<uint64_t>()(k.first * 0x9e3779b97f4a7c15ull ^ k.second);
+  }
+};
+using RKey = std::pair<uint64_t, uint64_t>;  // renamed key: (line, write epoch)
+
+// Record indices of memory records, grouped by scope, trace order kept.
+std::vector<std::vector<uint64_t>> scopes_of(const uint32_t* cta, const uint8_t* meta, uint64_t n, int scope) {
+  std::map<uint32_t, std::vector<uint64_t>> m;
+  for (uint64_t i = 0; i < n; ++i) {
+    if ((meta[i] & 3u) == KIND_BB) continue;
+    m[scope == SCOPE_CTA ? cta[i] : 0u].push_back(i);
+  }
+  std::vector<std::vector<uint64_t>> out;
+  out.reserve(m.size());
+  for (auto& kv : m) out.push_back(std::move(kv.second));
+  return out;
+}
+
+int check_reuse_args(uint32_t line_bytes, int scope, int binning, uint32_t nbins) {
+  if (!pow2(line_bytes) || line_bytes > 4096) return INVALID_ARG;
+  if (scope != SCOPE_CTA && scope != SCOPE_KERNEL) return INVALID_ARG;
+  if (binning != BINS_LINEAR && binning != BINS_LOG2) return INVALID_ARG;
+  if (nbins < 3) return INVALID_ARG;
+  return OK;
+}
+
+// One scope's records walked with an explicit LRU stack (top = back()).
+// rd[k] = reuse distance of the k-th record of the scope, or -1 for ∞.
+void lru_scope(const std::vector<uint64_t>& idx, const uint64_t* addr, const uint8_t* meta, uint32_t line_bytes,
+               std::vector<int64_t>& rd, uint64_t& streaming) {
+  std::vector<RKey> stack;
+  std::unordered_map<uint64_t, uint64_t> epoch;            // e(s, line): stores seen so far
+  std::unordered_map<RKey, uint64_t, KeyHash> occurrences;  // per renamed key
+  std::vector<RKey> keys(idx.size());
+  rd.assign(idx.size(), -1);
+  for (size_t k = 0; k < idx.size(); ++k) {
+    uint64_t i = idx[k];
+    uint64_t line = addr[i] / line_bytes;
+    bool store = (meta[i] & 3u) == KIND_STORE;
+    if (store) {
+      uint64_t e = ++epoch[line];
+      RKey key{line, e};
+      stack.push_back(key);      // fresh key "A'": first access, RD = ∞
+      keys[k] = key;
+      rd[k] = -1;
+    } else {
+      RKey key{line, epoch[line]};
+      keys[k] = key;
+      int64_t found = -1;
+      for (size_t d = 0; d < stack.size(); ++d) {
+        if (stack[stack.size() - 1 - d] == key) { found = (int64_t)d; break; }
+      }
+      if (found >= 0) {
+        stack.erase(stack.end() - 1 - found);
+        rd[k] = found;
+      } else {
+        rd[k] = -1;
+      }
+      stack.push_back(key);
+    }
+    occurrences[keys[k]]++;
+  }
+  streaming = 0;
+  for (size_t k = 0; k < idx.size(); ++k)
+    if (occurrences[keys[k]] == 1) streaming++;
+}
+
+}  // namespace
+
+extern "C" {
+
+// Reuse-distance histogram (LRU-stack oracle).  hist[nbins]; stats[4] =
+// {accesses, inf, streaming, overflow}.  Returns 0 / 1 (invalid arg) / 2 (bad trace).
+int oracle_reuse(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid, const uint8_t* meta, uint64_t n,
+                 uint32_t line_bytes, int scope, int binning, uint32_t nbins, uint64_t* hist, uint64_t* stats) {
+  int rc = check_reuse_args(line_bytes, scope, binning, nbins);
+  if (rc) return rc;
+  if (!check_all(addr, tid, meta, n)) return BAD_TRACE;
+  auto sc = scopes_of(cta, meta, n, scope);
+  std::vector<uint64_t> h(nbins, 0);
+  uint64_t streaming = 0;
+#pragma omp parallel
+  {
+    std::vector<uint64_t> hl(nbins, 0);
+    uint64_t sl = 0;
+    std::vector<int64_t> rd;
+#pragma omp for schedule(dynamic, 1)
+    for (int64_t s = 0; s < (int64_t)sc.size(); ++s) {
+      uint64_t st = 0;
+      lru_scope(sc[s], addr, meta, line_bytes, rd, st);
+      sl += st;
+      for (int64_t d : rd) hl[d < 0 ? nbins - 1 : bin_of((uint64_t)d, binning, nbins)]++;
+    }
+#pragma omp critical
+    {
+      for (uint32_t b = 0; b < nbins; ++b) h[b] += hl[b];
+      streaming += sl;
+    }
+  }
+  uint64_t acc = 0;
+  for (uint32_t b = 0; b < nbins; ++b) { hist[b] = h[b]; acc += h[b]; }
+  stats[0] = acc;
+  stats[1] = h[nbins - 1];
+  stats[2] = streaming;
+  stats[3] = h[nbins - 2];
+  return OK;
+}
+
+// Per-record reuse distance (LRU-stack oracle): rd[i] = distance, -1 = ∞,
+// -2 = not a memory record.
+int oracle_reuse_rd(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid, const uint8_t* meta, uint64_t n,
+                    uint32_t line_bytes, int scope, int64_t* rd_out) {
+  int rc = check_reuse_args(line_bytes, scope, BINS_LINEAR, 3);
+  if (rc) return rc;
+  if (!check_all(addr, tid, meta, n)) return BAD_TRACE;
+  for (uint64_t i = 0; i < n; ++i) rd_out[i] = -2;
+  auto sc = scopes_of(cta, meta, n, scope);
+#pragma omp parallel for schedule(dynamic, 1)
+  for (int64_t s = 0; s < (int64_t)sc.size(); ++s) {
+    std::vector<int64_t> rd;
+    uint64_t st;
+    lru_scope(sc[s], addr, meta, line_bytes, rd, st);
+    for (size_t k = 0; k < rd.size(); ++k) rd_out[sc[s][k]] = rd[k];
+  }
+  return OK;
+}
+
+// Literal O(n^2) definition: for each access, find the previous use
+// of the same renamed element in the same scope and count the distinct
+// renamed elements of that scope accessed strictly in between.
+int oracle_reuse_brute(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid, const uint8_t* meta,
+                       uint64_t n, uint32_t line_bytes, int scope, int binning, uint32_t nbins, uint64_t* hist,
+                       uint64_t* stats, int64_t* rd_out) {
+  int rc = check_reuse_args(line_bytes, scope, binning, nbins);
+  if (rc) return rc;
+  if (!check_all(addr, tid, meta, n)) return BAD_TRACE;
+  // renamed element of every access: (scope, line, number of stores to that
+  // (scope, line) at positions <= i)
+  std::vector<std::tuple<uint32_t, uint64_t, uint64_t>> key(n);
+  std::vector<bool> mem(n);
+  for (uint64_t i = 0; i < n; ++i) {
+    mem[i] = (meta[i] & 3u) != KIND_BB;
+    if (!mem[i]) continue;
+    uint32_t s = scope == SCOPE_CTA ? cta[i] : 0u;
+    uint64_t line = addr[i] / line_bytes;
+    uint64_t stores = 0;
+    for (uint64_t j = 0; j <= i; ++j)
+      if (mem[j] && (meta[j] & 3u) == KIND_STORE && (scope == SCOPE_CTA ? cta[j] : 0u) == s &&
+          addr[j] / line_bytes == line)
+        stores++;
+    key[i] = std::make_tuple(s, line, stores);
+  }
+  std::vector<uint64_t> h(nbins, 0);
+  for (uint64_t i = 0; i < n; ++i) {
+    if (!mem[i]) { if (rd_out) rd_out[i] = -2; continue; }
+    int64_t rd = -1;
+    if ((meta[i] & 3u) == KIND_LOAD) {
+      for (int64_t j = (int64_t)i - 1; j >= 0; --j) {
+        if (mem[j] && key[j] == key[i]) {
+          std::set<std::tuple<uint32_t, uint64_t, uint64_t>> between;
+          for (uint64_t m = (uint64_t)j + 1; m < i; ++m)
+            if (mem[m] && std::get<0>(key[m]) == std::get<0>(key[i])) between.insert(key[m]);
+          rd = (int64_t)between.size();
+          break;
+        }
+      }
+    }
+    if (rd_out) rd_out[i] = rd;
+    h[rd < 0 ? nbins - 1 : bin_of((uint64_t)rd, binning, nbins)]++;
+  }
+  uint64_t streaming = 0;
+  for (uint64_t i = 0; i < n; ++i) {
+    if (!mem[i]) continue;
+    uint64_t c = 0;
+    for (uint64_t j = 0; j < n; ++j) if (mem[j] && key[j] == key[i]) c++;
+    if (c == 1) streaming++;
+  }
+  uint64_t acc = 0;
+  for (uint32_t b = 0; b < nbins; ++b) { hist[b] = h[b]; acc += h[b]; }
+  stats[0] = acc; stats[1] = h[nbins - 1]; stats[2] = streaming; stats[3] = h[nbins - 2];
+  return OK;
+}
+
+// Memory divergence: per dynamic warp-level load/store, the number
+// of unique cache lines touched.  Group = (cta, tid / W, winst) over memory
+// records.  hist[2][W+1] (row 0 loads, row 1 stores; column = degree);
+// per_site[nsites][2] = {groups, sum of degrees} (nullable).
+int oracle_mem_div(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid, const uint32_t* winst,
+                   const uint32_t* site, const uint8_t* meta, uint64_t n, uint32_t line_bytes, uint32_t warp_size,
+                   uint32_t nsites, uint64_t* hist, uint64_t* per_site) {
+  if (!pow2(line_bytes) || line_bytes > 4096) return INVALID_ARG;
+  if (!pow2(warp_size) || warp_size > 32) return INVALID_ARG;
+  if (!check_all(addr, tid, meta, n)) return BAD_TRACE;
+  for (uint64_t i = 0; i < n; ++i)
+    if ((meta[i] & 3u) != KIND_BB && per_site && site[i] >= nsites) return INVALID_ARG;
+  const uint32_t W = warp_size;
+  // bucket memory records by CTA (trace order kept inside each bucket)
+  std::map<uint32_t, std::vector<uint64_t>> by_cta;
+  for (uint64_t i = 0; i < n; ++i)
+    if ((meta[i] & 3u) != KIND_BB) by_cta[cta[i]].push_back(i);
+  std::vector<const std::vector<uint64_t>*> lists;
+  for (auto& kv : by_cta) lists.push_back(&kv.second);
+  std::vector<uint64_t> H(2 * (W + 1), 0), S(per_site ? 2ull * nsites : 0, 0);
+  int bad = 0;
+#pragma omp parallel
+  {
+    std::vector<uint64_t> Hl(2 * (W + 1), 0), Sl(per_site ? 2ull * nsites : 0, 0);
+#pragma omp for schedule(dynamic, 4)
+    for (int64_t c = 0; c < (int64_t)lists.size(); ++c) {
+      struct Group { uint64_t first; std::set<uint64_t> lines; std::set<uint32_t> lanes; uint64_t count = 0; };
+      std::map<std::pair<uint32_t, uint32_t>, Group> groups;  // (tid / W, winst)
+      for (uint64_t i : *lists[c]) {
+        auto key = std::make_pair((uint32_t)(tid[i] / W), winst[i]);
+        auto it = groups.find(key);
+        if (it == groups.end()) { it = groups.emplace(key, Group()).first; it->second.first = i; }
+        it->second.lines.insert(addr[i] / line_bytes);
+        it->second.lanes.insert(tid[i] % W);
+        it->second.count++;
+      }
+      for (auto& kv : groups) {
+        const Group& g = kv.second;
+        if (g.lanes.size() != g.count) {
+#pragma omp atomic write
+          bad = 1;
+          continue;
+        }
+        uint64_t deg = g.lines.size();
+        uint32_t kind = meta[g.first] & 3u;
+        Hl[kind * (W + 1) + deg]++;
+        if (per_site) { Sl[2ull * site[g.first]] += 1; Sl[2ull * site[g.first] + 1] += deg; }
+      }
+    }
+#pragma omp critical
+    {
+      for (size_t k = 0; k < H.size(); ++k) H[k] += Hl[k];
+      for (size_t k = 0; k < S.size(); ++k) S[k] += Sl[k];
+    }
+  }
+  if (bad) return BAD_TRACE;
+  std::memcpy(hist, H.data(), H.size() * 8);
+  if (per_site) std::memcpy(per_site, S.data(), S.size() * 8);
+  return OK;
+}
+
+// Branch divergence (Table 3): per dynamic warp-level basic-block
+// execution g = (cta, tid / W, winst) over BB records:
+//   active(g) = number of distinct lanes (tid % W) in g
+//   live(g)   = clamp(T_c - w*W, 0, W), T_c = 1 + max tid over CTA c's BB records
+//   divergent = active < live
+// per_site[nsites][3] = {exec, divergent, threads}; totals[3] = their sums.
+int oracle_branch_div(const uint32_t* cta, const uint16_t* tid, const uint32_t* winst, const uint32_t* site,
+                      const uint8_t* meta, uint64_t n, uint32_t warp_size, uint32_t nsites, uint64_t* per_site,
+                      uint64_t* totals) {
+  if (!pow2(warp_size) || warp_size > 32) return INVALID_ARG;
+  if (!check_all(nullptr, tid, meta, n)) return BAD_TRACE;
+  for (uint64_t i = 0; i < n; ++i)
+    if ((meta[i] & 3u) == KIND_BB && per_site && site[i] >= nsites) return INVALID_ARG;
+  const uint32_t W = warp_size;
+  std::map<uint32_t, std::vector<uint64_t>> by_cta;
+  for (uint64_t i = 0; i < n; ++i)
+    if ((meta[i] & 3u) == KIND_BB) by_cta[cta[i]].push_back(i);
+  std::vector<const std::vector<uint64_t>*> lists;
+  for (auto& kv : by_cta) lists.push_back(&kv.second);
+  std::vector<uint64_t> S(per_site ? 3ull * nsites : 0, 0);
+  uint64_t T[3] = {0, 0, 0};
+  int bad = 0;
+#pragma omp parallel
+  {
+    std::vector<uint64_t> Sl(S.size(), 0);
+    uint64_t Tl[3] = {0, 0, 0};
+#pragma omp for schedule(dynamic, 4)
+    for (int64_t c = 0; c < (int64_t)lists.size(); ++c) {
+      uint32_t Tc = 0;
+      for (uint64_t i : *lists[c]) Tc = std::max<uint32_t>(Tc, (uint32_t)tid[i] + 1);
+      struct Group { uint64_t first; std::set<uint32_t> lanes; uint64_t count = 0; };
+      std::map<std::pair<uint32_t, uint32_t>, Group> groups;
+      for (uint64_t i : *lists[c]) {
+        auto key = std::make_pair((uint32_t)(tid[i] / W), winst[i]);
+        auto it = groups.find(key);
+        if (it == groups.end()) { it = groups.emplace(key, Group()).first; it->second.first = i; }
+        it->second.lanes.insert(tid[i] % W);
+        it->second.count++;
+      }
+      for (auto& kv : groups) {
+        const Group& g = kv.second;
+        if (g.lanes.size() != g.count) {
+#pragma omp atomic write
+          bad = 1;
+          continue;
+        }
+        uint64_t w = kv.first.first;
+        int64_t live = (int64_t)Tc - (int64_t)(w * W);
+        if (live < 0) live = 0;
+        if (live > (int64_t)W) live = W;
+        uint64_t active = g.lanes.size();
+        uint64_t div = (int64_t)active < live ? 1 : 0;
+        Tl[0] += 1; Tl[1] += div; Tl[2] += active;
+        if (per_site) {
+          uint32_t s = site[g.first];
+          Sl[3ull * s] += 1; Sl[3ull * s + 1] += div; Sl[3ull * s + 2] += active;
+        }
+      }
+    }
+#pragma omp critical
+    {
+      for (size_t k = 0; k < S.size(); ++k) S[k] += Sl[k];
+      for (int k = 0; k < 3; ++k) T[k] += Tl[k];
+    }
+  }
+  if (bad) return BAD_TRACE;
+  if (per_site) std::memcpy(per_site, S.data(), S.size() * 8);
+  for (int k = 0; k < 3; ++k) totals[k] = T[k];
+  return OK;
+}
+
+int oracle_num_threads(void) {
+#ifdef _OPENMP
+  return omp_get_max_threads();
+#else
+  return 1;
+#endif
+}
+
+}  // extern "C"

@@ -1,0 +1,142 @@
+"""Seeded synthetic trace generator (shared input module).
+
+Holds no analysis arithmetic: it only emits the records an instrumented
+kernel would produce (PAPER.md L235-237 Record(), L322/L345 passBasicBlock()).
+Both the oracle side and the CUDA side of the tests and of bench.py read the
+arrays it produces.  See tracegen.cpp for the record layout and the virtual
+scheduler, DESIGN.md "Input recipe" for the workloads.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+import subprocess
+from dataclasses import dataclass, field
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+_SO = os.path.join(_HERE, "libtracegen.so")
+_lib = None
+
+COLUMNS = (("addr", np.uint64), ("cta", np.uint32), ("tid", np.uint16),
+           ("site", np.uint32), ("winst", np.uint32), ("meta", np.uint8))
+
+KIND_LOAD, KIND_STORE, KIND_BB = 0, 1, 2
+
+
+def _load():
+    global _lib
+    if _lib is not None:
+        return _lib
+    src = os.path.join(_HERE, "tracegen.cpp")
+    if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
+        subprocess.check_call(["g++", "-O2", "-std=c++17", "-fopenmp", "-shared", "-fPIC",
+                               "-o", _SO, src])
+    lib = ctypes.CDLL(_SO)
+    P, u64, u32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32
+    lib.tg_plan.restype = P
+    lib.tg_plan.argtypes = [ctypes.c_char_p, ctypes.c_char_p, ctypes.c_char_p, ctypes.c_int]
+    for fn, rt in (("tg_num_records", u64), ("tg_num_sites", u32), ("tg_num_ctas", u32),
+                   ("tg_num_launches", u32), ("tg_info", ctypes.c_char_p)):
+        getattr(lib, fn).restype = rt
+        getattr(lib, fn).argtypes = [P]
+    lib.tg_fill_range.restype = ctypes.c_int
+    lib.tg_fill_range.argtypes = [P, u64, u64] + [P] * 6
+    lib.tg_free.restype = None
+    lib.tg_free.argtypes = [P]
+    _lib = lib
+    return lib
+
+
+@dataclass
+class Trace:
+    """One synthetic trace (or one position-range shard of it), SoA columns."""
+    workload: str
+    params: dict
+    n: int                      # records in this object
+    n_total: int                # records in the whole trace
+    nsites: int
+    nctas: int
+    nlaunches: int
+    info: str
+    lo: int = 0                 # first global position held here
+    cols: dict = field(default_factory=dict)
+
+    def __getattr__(self, k):
+        cols = self.__dict__.get("cols", {})
+        if k in cols:
+            return cols[k]
+        raise AttributeError(k)
+
+    def nbytes(self) -> int:
+        return sum(a.nbytes for a in self.cols.values())
+
+
+def _param_str(params: dict) -> str:
+    return ",".join(f"{k}={v}" for k, v in params.items())
+
+
+def plan(workload: str, **params):
+    """Returns (handle, n_total, nsites, nctas, nlaunches, info) without generating."""
+    lib = _load()
+    err = ctypes.create_string_buffer(256)
+    h = lib.tg_plan(workload.encode(), _param_str(params).encode(), err, 256)
+    if not h:
+        raise ValueError(err.value.decode())
+    return (h, int(lib.tg_num_records(h)), int(lib.tg_num_sites(h)), int(lib.tg_num_ctas(h)),
+            int(lib.tg_num_launches(h)), lib.tg_info(h).decode())
+
+
+def generate(workload: str, lo: int | None = None, hi: int | None = None, alloc=None, **params) -> Trace:
+    """Generates records [lo, hi) (default: all) of a workload.
+
+    alloc(n, dtype) -> numpy array may be given to place the columns in
+    caller-owned memory (e.g. pinned host memory for bench.py's e2e leg).
+    """
+    lib = _load()
+    h, n_total, nsites, nctas, nl, info = plan(workload, **params)
+    try:
+        lo = 0 if lo is None else int(lo)
+        hi = n_total if hi is None else int(hi)
+        n = hi - lo
+        alloc = alloc or (lambda m, dt: np.empty(m, dtype=dt))
+        cols = {name: alloc(n, dt) for name, dt in COLUMNS}
+        for name, dt in COLUMNS:
+            a = cols[name]
+            assert a.dtype == dt and a.flags.c_contiguous and a.shape == (n,)
+        if n > 0:
+            rc = lib.tg_fill_range(h, lo, hi, *[cols[name].ctypes.data for name, _ in COLUMNS])
+            if rc != 0:
+                raise ValueError(f"tg_fill_range failed ({rc})")
+        return Trace(workload, dict(params), n, n_total, nsites, nctas, nl, info, lo, cols)
+    finally:
+        lib.tg_free(h)
+
+
+def from_arrays(addr, cta, tid, site, winst, meta, nsites=None, workload="custom") -> Trace:
+    """Wraps hand-built columns (tests, golden fixtures) as a Trace."""
+    cols = {}
+    for (name, dt), a in zip(COLUMNS, (addr, cta, tid, site, winst, meta)):
+        cols[name] = np.ascontiguousarray(np.asarray(a, dtype=dt))
+    n = len(cols["addr"])
+    assert all(len(a) == n for a in cols.values())
+    ns = int(nsites) if nsites is not None else (int(cols["site"].max()) + 1 if n else 1)
+    nc = int(cols["cta"].max()) + 1 if n else 0
+    return Trace(workload, {}, n, n, ns, nc, 1, "", 0, cols)
+
+
+def concat(traces) -> Trace:
+    cols = {name: np.concatenate([t.cols[name] for t in traces]) for name, _ in COLUMNS}
+    return from_arrays(*[cols[name] for name, _ in COLUMNS],
+                       nsites=max(t.nsites for t in traces), workload="+".join(t.workload for t in traces))
+
+
+# Named configurations of BASELINE.json; params per workload.
+CONFIGS = {
+    "c1_vecadd": ("vecadd", {}),
+    "c2_sgemm": ("sgemm", {"n": 256}),
+    "c3_bfs": ("bfs", {"nodes": 1000000, "seed": 42}),
+    "c4_srad": ("srad", {"rows": 2048, "cols": 2048, "iters": 6}),
+    "c4_backprop": ("backprop", {"in": 4194304}),
+}
