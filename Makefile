@@ -3,21 +3,21 @@
 #   oracle/liboracle.so       CPU oracle (test infrastructure only)
 #   paper_conf_cgo_shensll18_b200/libcadv.so   the product: sm_100a CUDA + C-ABI
 NVCC      ?= /usr/local/cuda/bin/nvcc
-CXX       ?= g++
+HOSTCXX   := /usr/bin/g++
 ARCH      := -gencode arch=compute_100a,code=sm_100a
 PKG       := paper_conf_cgo_shensll18_b200
 CADV_SRC  := $(wildcard $(PKG)/csrc/*.cu) $(wildcard $(PKG)/csrc/*.cpp)
 CADV_HDR  := $(wildcard $(PKG)/csrc/*.cuh) $(wildcard $(PKG)/csrc/*.h) include/cadv.h
-NVFLAGS   := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
+NVFLAGS   := -ccbin $(HOSTCXX) $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
              -Iinclude --expt-relaxed-constexpr -Xptxas -v
 
 all: tracegen/libtracegen.so oracle/liboracle.so $(PKG)/libcadv.so
 
 tracegen/libtracegen.so: tracegen/tracegen.cpp
-	$(CXX) -O2 -std=c++17 -fopenmp -shared -fPIC -o $@ $<
+	$(HOSTCXX) -O2 -std=c++17 -fopenmp -shared -fPIC -o $@ $<
 
 oracle/liboracle.so: oracle/oracle.cpp
-	$(CXX) -O2 -std=c++17 -fopenmp -shared -fPIC -o $@ $<
+	$(HOSTCXX) -O2 -std=c++17 -fopenmp -shared -fPIC -o $@ $<
 
 $(PKG)/libcadv.so: $(CADV_SRC) $(CADV_HDR)
 	$(NVCC) $(NVFLAGS) -shared -o $@ $(CADV_SRC) -ldl 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)

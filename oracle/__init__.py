@@ -40,7 +40,7 @@ def _load():
         return _lib
     src = os.path.join(_HERE, "oracle.cpp")
     if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
-        subprocess.check_call(["g++", "-O2", "-std=c++17", "-fopenmp", "-shared", "-fPIC", "-o", _SO, src])
+        subprocess.check_call(["/usr/bin/g++" if os.path.exists("/usr/bin/g++") else "g++", "-O2", "-std=c++17", "-fopenmp", "-shared", "-fPIC", "-o", _SO, src])
     lib = ctypes.CDLL(_SO)
     P, u64, u32, i32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32, ctypes.c_int
     lib.oracle_reuse.argtypes = [P, P, P, P, u64, u32, i32, i32, u32, P, P]

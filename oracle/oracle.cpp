@@ -49,25 +49,29 @@ enum { BINS_LINEAR = 0, BINS_LOG2 = 1 };
 
 bool pow2(uint32_t x) { return x && !(x & (x - 1)); }
 
-// Per-record validity: kind <= 2, reserved meta
-// bits 5..7 zero, memory records naturally aligned and below 2^62, tid < 1024.
-bool record_ok(uint64_t addr, uint16_t tid, uint8_t meta) {
-  uint32_t kind = meta & 3u;
-  if (kind == 3 || (meta >> 5) != 0) return false;
-  if (tid >= 1024) return false;
+// Per-record validity (include/cadv.h "Per-record validity"), checked over
+// the columns an analysis reads: kind <= 2, reserved meta bits 5..7 zero;
+// memory records: log2 bytes <= 4, naturally aligned, addr < 2^58 (when the
+// address column is read); tid < 1024 (when the tid column is read).
+bool record_ok(const uint64_t* addr, const uint16_t* tid, const uint8_t* meta, uint64_t i) {
+  uint32_t kind = meta[i] & 3u;
+  if (kind == 3 || (meta[i] >> 5) != 0) return false;
+  if (tid && tid[i] >= 1024) return false;
   if (kind != KIND_BB) {
-    uint32_t lg = (meta >> 2) & 7u;
+    uint32_t lg = (meta[i] >> 2) & 7u;
     if (lg > 4) return false;
-    uint64_t bytes = 1ull << lg;
-    if (addr % bytes != 0) return false;
-    if (addr >> 62) return false;
+    if (addr) {
+      uint64_t bytes = 1ull << lg;
+      if (addr[i] % bytes != 0) return false;
+      if (addr[i] >> 58) return false;
+    }
   }
   return true;
 }
 
 bool check_all(const uint64_t* addr, const uint16_t* tid, const uint8_t* meta, uint64_t n) {
   for (uint64_t i = 0; i < n; ++i)
-    if (!record_ok(addr ? addr[i] : 0, tid ? tid[i] : 0, meta[i])) return false;
+    if (!record_ok(addr, tid, meta, i)) return false;
   return true;
 }
 
@@ -159,7 +163,7 @@ int oracle_reuse(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid,
                  uint32_t line_bytes, int scope, int binning, uint32_t nbins, uint64_t* hist, uint64_t* stats) {
   int rc = check_reuse_args(line_bytes, scope, binning, nbins);
   if (rc) return rc;
-  if (!check_all(addr, tid, meta, n)) return BAD_TRACE;
+  if (!check_all(addr, nullptr, meta, n)) return BAD_TRACE;
   auto sc = scopes_of(cta, meta, n, scope);
   std::vector<uint64_t> h(nbins, 0);
   uint64_t streaming = 0;
@@ -196,7 +200,7 @@ int oracle_reuse_rd(const uint64_t* addr, const uint32_t* cta, const uint16_t* t
                     uint32_t line_bytes, int scope, int64_t* rd_out) {
   int rc = check_reuse_args(line_bytes, scope, BINS_LINEAR, 3);
   if (rc) return rc;
-  if (!check_all(addr, tid, meta, n)) return BAD_TRACE;
+  if (!check_all(addr, nullptr, meta, n)) return BAD_TRACE;
   for (uint64_t i = 0; i < n; ++i) rd_out[i] = -2;
   auto sc = scopes_of(cta, meta, n, scope);
 #pragma omp parallel for schedule(dynamic, 1)
@@ -217,7 +221,7 @@ int oracle_reuse_brute(const uint64_t* addr, const uint32_t* cta, const uint16_t
                        uint64_t* stats, int64_t* rd_out) {
   int rc = check_reuse_args(line_bytes, scope, binning, nbins);
   if (rc) return rc;
-  if (!check_all(addr, tid, meta, n)) return BAD_TRACE;
+  if (!check_all(addr, nullptr, meta, n)) return BAD_TRACE;
   // renamed element of every access: (scope, line, number of stores to that
   // (scope, line) at positions <= i)
   std::vector<std::tuple<uint32_t, uint64_t, uint64_t>> key(n);

@@ -1,0 +1,207 @@
+"""paper_conf_cgo_shensll18_b200 — B200-native CUDAAdvisor trace analysis.
+
+Thin ctypes binding over libcadv.so (include/cadv.h).  Argument marshalling
+only: every step of every analysis runs in the library's sm_100a kernels.
+There is no CPU fallback — without the built library or without an sm_100
+device every call raises CadvError.
+
+Names mirror the C ABI:
+    ctx = create(device=0, stream=None)          # cadv_create
+    ctx.load_trace(cols, warp_contiguous=True)   # cadv_load_trace
+    ctx.reuse_histogram(line_bytes, scope, binning, nbins)   # cadv_reuse_histogram
+    ctx.mem_divergence(line_bytes, warp_size, nsites)        # cadv_mem_divergence
+    ctx.branch_divergence(warp_size, nsites)                 # cadv_branch_divergence
+    ctx.destroy()                                            # cadv_destroy
+Trace columns may be torch CUDA tensors (borrowed, zero copy) or host numpy
+arrays / CPU tensors (copied by cadv_load_trace).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_HERE = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_HERE, "libcadv.so")
+
+CADV_OK, CADV_ERR_INVALID_ARG, CADV_ERR_BAD_TRACE, CADV_ERR_NO_TRACE = 0, 1, 2, 3
+CADV_ERR_OOM, CADV_ERR_CUDA, CADV_ERR_NCCL, CADV_ERR_UNSUPPORTED = 4, 5, 6, 7
+SCOPE_CTA, SCOPE_KERNEL = 0, 1
+BINS_LINEAR, BINS_LOG2 = 0, 1
+STATUS_NAMES = {0: "OK", 1: "INVALID_ARG", 2: "BAD_TRACE", 3: "NO_TRACE", 4: "OOM", 5: "CUDA", 6: "NCCL",
+                7: "UNSUPPORTED"}
+COLUMNS = ("addr", "cta", "tid", "site", "winst", "meta")
+_DTYPES = {"addr": np.uint64, "cta": np.uint32, "tid": np.uint16, "site": np.uint32, "winst": np.uint32,
+           "meta": np.uint8}
+
+
+class CadvError(RuntimeError):
+    def __init__(self, status, msg=""):
+        super().__init__(f"cadv error {STATUS_NAMES.get(status, status)}: {msg}")
+        self.status = status
+
+
+class TraceDesc(ctypes.Structure):
+    _fields_ = [("addr", ctypes.c_void_p), ("cta", ctypes.c_void_p), ("tid", ctypes.c_void_p),
+                ("site", ctypes.c_void_p), ("winst", ctypes.c_void_p), ("meta", ctypes.c_void_p),
+                ("n", ctypes.c_uint64), ("on_device", ctypes.c_int), ("warp_contiguous", ctypes.c_int)]
+
+
+class ReuseStats(ctypes.Structure):
+    _fields_ = [("accesses", ctypes.c_uint64), ("inf", ctypes.c_uint64), ("streaming", ctypes.c_uint64),
+                ("overflow", ctypes.c_uint64)]
+
+
+_lib = None
+
+
+def lib():
+    """Loads libcadv.so (built by `make` / __graft_entry__.build()); raises if absent."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(LIB_PATH):
+        raise CadvError(CADV_ERR_CUDA, f"{LIB_PATH} is not built (run `make` or __graft_entry__.build())")
+    L = ctypes.CDLL(LIB_PATH)
+    P, u32, u64, i32 = ctypes.c_void_p, ctypes.c_uint32, ctypes.c_uint64, ctypes.c_int
+    L.cadv_create.argtypes = [ctypes.POINTER(P), i32, P, P, i32, i32]
+    L.cadv_load_trace.argtypes = [P, ctypes.POINTER(TraceDesc), u64]
+    L.cadv_reuse_histogram.argtypes = [P, u32, i32, i32, P, u32, ctypes.POINTER(ReuseStats)]
+    L.cadv_mem_divergence.argtypes = [P, u32, u32, P, P, u32]
+    L.cadv_branch_divergence.argtypes = [P, u32, P, u32, P]
+    L.cadv_destroy.argtypes = [P]
+    for f in ("cadv_create", "cadv_load_trace", "cadv_reuse_histogram", "cadv_mem_divergence",
+              "cadv_branch_divergence", "cadv_destroy"):
+        getattr(L, f).restype = i32
+    L.cadv_last_error.argtypes = [P]
+    L.cadv_last_error.restype = ctypes.c_char_p
+    L.cadv_last_elapsed_ms.argtypes = [P]
+    L.cadv_last_elapsed_ms.restype = ctypes.c_float
+    L.cadv_last_launches.argtypes = [P]
+    L.cadv_last_launches.restype = u32
+    L.cadv_version.restype = ctypes.c_char_p
+    _lib = L
+    return L
+
+
+def _ptr_and_kind(a, name):
+    """(pointer, on_device, keepalive) for a torch tensor or numpy array column."""
+    dt = _DTYPES[name]
+    try:
+        import torch
+        if isinstance(a, torch.Tensor):
+            tmap = {np.uint64: torch.uint64, np.uint32: torch.uint32, np.uint16: torch.uint16, np.uint8: torch.uint8}
+            if a.dtype != tmap[dt] or not a.is_contiguous() or a.dim() != 1:
+                raise CadvError(CADV_ERR_INVALID_ARG, f"column {name}: need contiguous 1-D {tmap[dt]}")
+            return a.data_ptr(), bool(a.is_cuda), a
+    except ImportError:
+        pass
+    arr = np.ascontiguousarray(a)
+    if arr.dtype != dt or arr.ndim != 1:
+        raise CadvError(CADV_ERR_INVALID_ARG, f"column {name}: need 1-D {np.dtype(dt)}")
+    return arr.ctypes.data, False, arr
+
+
+class Context:
+    """One analysis context (one per GPU / rank): cadv_create ... cadv_destroy."""
+
+    def __init__(self, device: int = 0, stream=None):
+        L = lib()
+        h = ctypes.c_void_p()
+        s = L.cadv_create(ctypes.byref(h), int(device), ctypes.c_void_p(stream or 0), None, 0, 1)
+        if s != CADV_OK:
+            raise CadvError(s, "cadv_create failed (needs an sm_100 GPU and the CUDA driver)")
+        self._h = h
+        self._keep = None
+        self.device = device
+
+    # -- helpers
+    def _check(self, s):
+        if s != CADV_OK:
+            raise CadvError(s, lib().cadv_last_error(self._h).decode())
+
+    @property
+    def handle(self):
+        return self._h
+
+    def last_elapsed_ms(self) -> float:
+        return float(lib().cadv_last_elapsed_ms(self._h))
+
+    def last_launches(self) -> int:
+        return int(lib().cadv_last_launches(self._h))
+
+    # -- cadv_load_trace
+    def load_trace(self, cols, n=None, warp_contiguous=True, global_offset=0):
+        """cols: mapping (or object with attributes) addr/cta/tid/site/winst/meta."""
+        get = (lambda k: cols[k]) if isinstance(cols, dict) else (lambda k: getattr(cols, k))
+        ptrs, devs, keep = {}, set(), []
+        for k in COLUMNS:
+            p, d, ka = _ptr_and_kind(get(k), k)
+            ptrs[k] = p
+            devs.add(d)
+            keep.append(ka)
+        if len(devs) != 1:
+            raise CadvError(CADV_ERR_INVALID_ARG, "all columns must be on the device or all on the host")
+        n = len(keep[0]) if n is None else int(n)
+        d = TraceDesc(ptrs["addr"], ptrs["cta"], ptrs["tid"], ptrs["site"], ptrs["winst"], ptrs["meta"], n,
+                      1 if devs.pop() else 0, 1 if warp_contiguous else 0)
+        self._check(lib().cadv_load_trace(self._h, ctypes.byref(d), int(global_offset)))
+        self._keep = keep  # borrowed device columns stay alive while loaded
+
+    # -- cadv_reuse_histogram
+    def reuse_histogram(self, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66):
+        hist = np.zeros(nbins, np.uint64)
+        st = ReuseStats()
+        self._check(lib().cadv_reuse_histogram(self._h, line_bytes, scope, binning, hist.ctypes.data, nbins,
+                                               ctypes.byref(st)))
+        return hist, {"accesses": st.accesses, "inf": st.inf, "streaming": st.streaming, "overflow": st.overflow}
+
+    # -- cadv_mem_divergence
+    def mem_divergence(self, line_bytes=128, warp_size=32, nsites=0):
+        hist = np.zeros((2, warp_size + 1), np.uint64)
+        ps = np.zeros((nsites, 2), np.uint64) if nsites else None
+        self._check(lib().cadv_mem_divergence(self._h, line_bytes, warp_size, hist.ctypes.data,
+                                              ps.ctypes.data if ps is not None else None, nsites))
+        return hist, ps
+
+    # -- cadv_branch_divergence
+    def branch_divergence(self, warp_size=32, nsites=0):
+        ps = np.zeros((nsites, 3), np.uint64) if nsites else None
+        tot = np.zeros(3, np.uint64)
+        self._check(lib().cadv_branch_divergence(self._h, warp_size, ps.ctypes.data if ps is not None else None,
+                                                 nsites, tot.ctypes.data))
+        return ps, tot
+
+    # -- cadv_destroy
+    def destroy(self):
+        if getattr(self, "_h", None):
+            lib().cadv_destroy(self._h)
+            self._h = None
+            self._keep = None
+
+    def __del__(self):
+        try:
+            self.destroy()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.destroy()
+
+
+def create(device: int = 0, stream=None) -> Context:
+    return Context(device, stream)
+
+
+def version() -> str:
+    return lib().cadv_version().decode()
+
+
+def to_device(trace, device="cuda"):
+    """Copies a tracegen.Trace's columns to torch CUDA tensors (plumbing only)."""
+    import torch
+    return {k: torch.from_numpy(np.ascontiguousarray(trace.cols[k])).to(device) for k in COLUMNS}

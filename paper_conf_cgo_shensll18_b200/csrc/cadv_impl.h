@@ -1,0 +1,105 @@
+// cadv_impl.h — internal context and launcher declarations of libcadv.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+#include <vector>
+
+#include "../../include/cadv.h"
+
+namespace cadv {
+
+// Device workspace buffer that only grows (allocation happens on the first
+// call that needs it; later calls of the same size allocate nothing).
+struct DevBuf {
+  void* p = nullptr;
+  size_t bytes = 0;
+};
+
+// Small per-call device scalars (zeroed at the start of every analysis).
+struct Scalars {
+  unsigned long long err_index;  // first offending record (ULLONG_MAX = none)
+  unsigned int err_code;         // 1 = bad record, 2 = run longer than 32 / duplicate lane
+  unsigned int tile_counter;     // dynamic tile assignment
+  unsigned long long count[8];   // generic counters (kept records, entries, ...)
+  unsigned long long max_cta;    // ingest: max CTA id
+  unsigned long long n_kind[4];  // ingest: records per kind
+};
+
+enum BufId {
+  B_SCALARS, B_HOST_COPY0, B_HOST_COPY1, B_HOST_COPY2, B_HOST_COPY3, B_HOST_COPY4, B_HOST_COPY5,
+  B_HIST, B_SITES, B_TC,
+  B_SORT_K0, B_SORT_K1, B_SORT_V0, B_SORT_V1, B_SORT_HIST, B_SCAN_TMP,
+  B_GATHER,
+  B_RD_KEY, B_RD_VAL, B_RD_TILESTAT, B_RD_TILEW, B_RD_TILEQ, B_RD_ENT, B_RD_ENT_KEY0, B_RD_ENT_KEY1,
+  B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP,
+  B_COUNT
+};
+
+}  // namespace cadv
+
+struct cadv_ctx {
+  int device = 0;
+  cudaStream_t stream = nullptr;
+  int rank = 0, nranks = 1;
+  void* comm = nullptr;  // ncclComm_t when nranks > 1
+  int num_sms = 148;
+  // registered trace (device pointers)
+  bool loaded = false;
+  cadv_trace_desc t{};
+  uint64_t global_offset = 0;
+  // ingest results (R0)
+  uint32_t max_cta = 0;
+  uint64_t n_kind[4] = {0, 0, 0, 0};
+  // bookkeeping
+  std::string err;
+  float elapsed_ms = 0.f;
+  uint32_t launches = 0;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  cadv::DevBuf buf[cadv::B_COUNT];
+  void* host_pinned = nullptr;
+  size_t host_pinned_bytes = 0;
+};
+
+namespace cadv {
+
+// Returns a device buffer of at least `bytes` (grown if needed).
+cudaError_t ensure(cadv_ctx* c, BufId id, size_t bytes, void** out);
+// Pinned host staging area for results.
+cudaError_t ensure_host(cadv_ctx* c, size_t bytes, void** out);
+Scalars* scalars(cadv_ctx* c);
+
+// ---- launchers (each returns cudaSuccess or the launch error; they add the
+// number of kernels they launched to c->launches)
+cudaError_t launch_ingest(cadv_ctx* c);
+cudaError_t launch_mem_div(cadv_ctx* c, const cadv_trace_desc& t, uint32_t lb_shift, uint32_t w_shift,
+                           uint64_t* d_hist, uint64_t* d_sites, uint32_t nsites);
+cudaError_t launch_cta_maxtid(cadv_ctx* c, const cadv_trace_desc& t, uint32_t* d_tc, uint32_t ncta);
+cudaError_t launch_branch_div(cadv_ctx* c, const cadv_trace_desc& t, uint32_t w_shift, const uint32_t* d_tc,
+                              uint64_t* d_sites, uint32_t nsites, uint64_t* d_totals);
+// Stable (cta, tid/32) ordering of a non-warp-contiguous trace: fills `out`
+// with device copies of every column in that order.
+cudaError_t regroup_by_warp(cadv_ctx* c, cadv_trace_desc* out);
+// Reuse distance (reuse.cu): fills d_hist[nbins] and d_stats[4] on the device.
+cudaError_t run_reuse(cadv_ctx* c, uint32_t lb_shift, int scope, int log2bins, uint32_t nbins, uint64_t* d_hist,
+                      uint64_t* d_stats);
+
+// ---- device-wide primitives (sort.cu)
+// Stable LSD radix sort of (key, value) pairs on bits [bit_lo, bit_hi) of the
+// key.  Ping-pongs between (k0,v0) and (k1,v1); returns 0 if the result is in
+// (k0,v0), 1 if in (k1,v1).
+template <typename K, typename V>
+cudaError_t radix_sort_pairs(cadv_ctx* c, K* k0, V* v0, K* k1, V* v1, uint64_t n, int bit_lo, int bit_hi,
+                             int* result_in);
+// Exclusive scan of n u32 values in place (out may alias in); *d_total (nullable) = sum.
+cudaError_t exclusive_scan_u32(cadv_ctx* c, const uint32_t* in, uint32_t* out, uint64_t n, uint32_t* d_total);
+cudaError_t exclusive_scan_u64(cadv_ctx* c, const uint64_t* in, uint64_t* out, uint64_t n);
+
+}  // namespace cadv
+
+#define CADV_LAUNCH(c, ...)   \
+  do {                        \
+    __VA_ARGS__;              \
+    (c)->launches++;          \
+  } while (0)

@@ -1,0 +1,943 @@
+// reuse.cu — reuse-distance histograms on B200.
+//
+// Definition (PAPER.md L248 + DESIGN.md readings R1-R8): per scope (CTA, or
+// the whole kernel), walk the memory records in trace order; the element of
+// an access is its line (addr / line_bytes) renamed by write epoch (a store
+// starts a new element A'); RD(i) = number of distinct elements accessed
+// strictly between the previous use P(i) of i's element and i; ∞ if none.
+//
+// Identity used on the device:
+//   RD(i) = |window (P(i), i)| - #{ j < i : P(j) > P(i) }
+// (the second term counts the window's records whose element is used again
+// inside the window).  The pipeline:
+//   R1 k_rd_compact  one streaming pass over (addr, cta, meta): validation,
+//                    line keys, and run compression of raw-adjacent records
+//                    of the same (scope, line): a load repeating the previous
+//                    record's element has RD 0 and is dropped (counted in
+//                    bin 0); consecutive stores are merged into one record of
+//                    weight w (they are w distinct one-shot elements).  Kept
+//                    records are written in trace order (decoupled look-back).
+//   R1b              stable radix sort of kept records by CTA id (CTA scope).
+//   R2/R3 k_rd_tile  fixed-capacity tiles of the CTA-major kept sequence
+//                    (boundaries snapped to segment starts): in shared memory,
+//                    a stable merge sort by line gives the local previous
+//                    occurrence P, a counting merge sort of the local queries
+//                    by P gives #{j < i : P(j) > P(i)} (merge-path,
+//                    inversion counting), and R4 bins every local RD.
+//   R3 (cross-tile)  only for segments cut by a tile boundary: one entry per
+//                    (tile piece, line) carries first/last occurrence data;
+//                    entries are sorted by (segment, line, tile) and linked;
+//                    cross-tile queries get RD from prefix sums plus a global
+//                    inversion count on the compacted cross-tile set.
+#include <cuda_runtime.h>
+#include <stdio.h>
+
+#include "cadv_impl.h"
+#include "common.cuh"
+
+namespace cadv {
+namespace {
+
+// kept-record value layout
+constexpr uint64_t LINE_MASK = (1ull << 58) - 1;
+constexpr int VB_STORE = 58, VB_DUP = 59, VB_W = 60;  // weight - 1 in bits 60..63
+
+// ------------------------------------------------------------------ R1 compaction
+constexpr int CP_NT = 256, CP_IPT = 16, CP_TILE = CP_NT * CP_IPT;  // 4096 raw records per tile
+constexpr uint32_t CP_ROWS = CP_TILE + 2;
+constexpr uint32_t CP_OFF_ADDR = 0;
+constexpr uint32_t CP_OFF_CTA = CP_OFF_ADDR + stage_bytes<uint64_t>(CP_ROWS);
+constexpr uint32_t CP_OFF_META = CP_OFF_CTA + stage_bytes<uint32_t>(CP_ROWS);
+constexpr uint32_t CP_SMEM = CP_OFF_META + stage_bytes<uint8_t>(CP_ROWS);
+
+constexpr uint64_t LB_AGG = 1ull << 62, LB_PRE = 2ull << 62, LB_VAL = (1ull << 62) - 1;
+
+__device__ __forceinline__ uint64_t ld_volatile(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
+  return v;
+}
+
+__global__ void __launch_bounds__(CP_NT) k_rd_compact(const uint64_t* __restrict__ addr, const uint32_t* __restrict__ cta,
+                                                      const uint8_t* __restrict__ meta, uint64_t n, uint32_t lbs,
+                                                      int cta_scope, uint32_t* __restrict__ kout,
+                                                      uint64_t* __restrict__ vout, uint64_t* status, uint64_t* hist0,
+                                                      Scalars* sc) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ uint64_t bar;
+  __shared__ uint32_t s_tile;
+  __shared__ uint32_t ws[CP_NT / 32 + 1];
+  __shared__ uint64_t s_base;
+  const uint32_t tx = threadIdx.x;
+  if (tx == 0) {
+    s_tile = atomicAdd(&sc->tile_counter, 1u);
+    mbar_init(&bar, 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  const uint64_t tile = s_tile;
+  const uint64_t t0 = tile * CP_TILE;
+  const uint64_t lo = t0 ? t0 - 1 : 0;
+  const uint64_t hi = (t0 + CP_TILE + 1) < n ? (t0 + CP_TILE + 1) : n;
+  if (tx == 0) {
+    auto hull = [](uintptr_t b, uintptr_t e) {
+      return (uint32_t)(((e + 15) & ~(uintptr_t)15) - (b & ~(uintptr_t)15));
+    };
+    uint32_t bytes = hull((uintptr_t)(addr + lo), (uintptr_t)(addr + hi)) +
+                     hull((uintptr_t)(cta + lo), (uintptr_t)(cta + hi)) +
+                     hull((uintptr_t)(meta + lo), (uintptr_t)(meta + hi));
+    mbar_arrive_expect_tx(&bar, bytes);
+    uint32_t d;
+    stage_column(addr, lo, hi, smem + CP_OFF_ADDR, &bar, &d);
+    stage_column(cta, lo, hi, smem + CP_OFF_CTA, &bar, &d);
+    stage_column(meta, lo, hi, smem + CP_OFF_META, &bar, &d);
+  }
+  const uint32_t da = (uint32_t)((uintptr_t)(addr + lo) & 15), dc = (uint32_t)((uintptr_t)(cta + lo) & 15),
+                 dm = (uint32_t)((uintptr_t)(meta + lo) & 15);
+  auto A = [&](uint64_t i) { return *(const uint64_t*)(smem + CP_OFF_ADDR + da + (i - lo) * 8); };
+  auto C = [&](uint64_t i) { return *(const uint32_t*)(smem + CP_OFF_CTA + dc + (i - lo) * 4); };
+  auto M = [&](uint64_t i) { return smem[CP_OFF_META + dm + (i - lo)]; };
+  mbar_wait(&bar, 0);
+
+  const uint64_t i0 = t0 + (uint64_t)tx * CP_IPT;
+  // state of the previous record (record i - 1)
+  bool pmem = false, pst = false;
+  uint64_t pline = 0;
+  uint32_t pscope = 0;
+  if (i0 > 0 && i0 - 1 < n) {
+    uint8_t m = M(i0 - 1);
+    pmem = is_mem(m) && meta_ok(m);
+    if (pmem) {
+      pline = A(i0 - 1) >> lbs;
+      pscope = cta_scope ? C(i0 - 1) : 0u;
+      pst = is_store(m);
+    }
+  }
+  uint64_t kline[CP_IPT];
+  uint32_t kcta[CP_IPT];
+  uint32_t kflag[CP_IPT];  // store | has_dup << 1 | (w - 1) << 2
+  int nk = 0;
+  uint32_t ndup = 0;
+#pragma unroll
+  for (int k = 0; k <= CP_IPT; ++k) {
+    uint64_t i = i0 + k;
+    if (i >= n) break;
+    uint8_t m = M(i);
+    bool mem = is_mem(m);
+    bool ok = meta_ok(m);
+    uint64_t a = 0;
+    if (mem && ok) {
+      a = A(i);
+      ok = addr_ok(a, m);
+    }
+    if (k == CP_IPT) {
+      // first record of the next chunk: only "is it a repeat of our last run?"
+      if (mem && ok && !is_store(m) && pmem && nk > 0) {
+        uint32_t s = cta_scope ? C(i) : 0u;
+        if (s == pscope && (a >> lbs) == pline) kflag[nk - 1] |= 2u;
+      }
+      break;
+    }
+    if (!ok) {
+      atomicMin(&sc->err_index, (unsigned long long)i);
+      atomicMax(&sc->err_code, 1u);
+      mem = false;
+    }
+    if (!mem) {
+      pmem = false;
+      continue;
+    }
+    uint64_t line = a >> lbs;
+    uint32_t s = cta_scope ? C(i) : 0u;
+    bool st = is_store(m);
+    bool same = pmem && s == pscope && line == pline;
+    if (same && !st) {
+      // a load of the element the previous record used: RD 0, dropped
+      ndup++;
+      if (k > 0 && nk > 0) kflag[nk - 1] |= 2u;
+    } else if (same && st && pst && k > 0 && nk > 0 && (kflag[nk - 1] >> 2) < 15u) {
+      // store right after a store to the same line: one more one-shot element
+      kflag[nk - 1] += 4u;
+    } else {
+      kline[nk] = line;
+      kcta[nk] = s;
+      kflag[nk] = st ? 1u : 0u;
+      nk++;
+    }
+    pmem = true;
+    pst = st;
+    pline = line;
+    pscope = s;
+  }
+  uint32_t tot;
+  uint32_t off = block_exclusive_scan<CP_NT>((uint32_t)nk, ws, &tot);
+  {
+    uint32_t d = __reduce_add_sync(FULL, ndup);
+    if (lane_id() == 0 && d) atomicAdd((unsigned long long*)hist0, (unsigned long long)d);
+  }
+  // decoupled look-back: global offset of this tile's kept records
+  if (tx == 0) {
+    uint64_t excl = 0;
+    if (tile == 0) {
+      atomicExch((unsigned long long*)&status[0], (unsigned long long)(LB_PRE | tot));
+    } else {
+      atomicExch((unsigned long long*)&status[tile], (unsigned long long)(LB_AGG | tot));
+      int64_t k = (int64_t)tile - 1;
+      while (k >= 0) {
+        uint64_t s = ld_volatile(status + k);
+        if (s & LB_PRE) { excl += s & LB_VAL; break; }
+        if (s & LB_AGG) { excl += s & LB_VAL; --k; continue; }
+      }
+      __threadfence();
+      atomicExch((unsigned long long*)&status[tile], (unsigned long long)(LB_PRE | (excl + tot)));
+    }
+    s_base = excl;
+  }
+  __syncthreads();
+  uint64_t g = s_base + off;
+  for (int k = 0; k < nk; ++k) {
+    uint64_t v = kline[k] | ((uint64_t)(kflag[k] & 1u) << VB_STORE) | ((uint64_t)((kflag[k] >> 1) & 1u) << VB_DUP) |
+                 ((uint64_t)(kflag[k] >> 2) << VB_W);
+    vout[g + k] = v;
+    if (kout) kout[g + k] = kcta[k];
+  }
+}
+
+// ------------------------------------------------------------------ tile bounds
+constexpr int TL_CAP = 4096;   // tile capacity (kept records)
+constexpr int TL_NOM = 3072;   // nominal tile length
+constexpr int TL_SNAP = 1024;  // boundary snapped to a segment start within this window
+
+__global__ void k_tile_bounds(const uint32_t* __restrict__ key, uint64_t K, uint32_t* __restrict__ bounds,
+                              uint64_t ntiles) {
+  const uint32_t lane = lane_id();
+  uint64_t w = (blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5;
+  uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t k = w; k <= ntiles; k += nw) {
+    uint64_t b;
+    if (k == 0) b = 0;
+    else if (k == ntiles) b = K;
+    else {
+      uint64_t x0 = k * TL_NOM;
+      b = x0;
+      if (key) {
+        uint64_t end = x0 + TL_SNAP < K ? x0 + TL_SNAP : K;
+        for (uint64_t base = x0; base < end; base += 32) {
+          uint64_t x = base + lane;
+          bool ss = x < end && __ldg(key + x) != __ldg(key + x - 1);
+          uint32_t bm = __ballot_sync(FULL, ss);
+          if (bm) { b = base + __ffs(bm) - 1; break; }
+        }
+      }
+    }
+    if (lane == 0) bounds[k] = (uint32_t)b;
+  }
+}
+
+// ------------------------------------------------------------------ block merge sort (shared memory)
+// Stable merge sort of N = NT*IPT items held in (ka, pa); result ends in the
+// buffer returned (0 = a, 1 = b).  COUNT: for every item from the right run
+// of a merge, cnt[idx(key)] += number of left-run items still unmerged =
+// number of earlier items with a larger key (inversion count per item;
+// keys are distinct when COUNT is used).
+template <int NT, int IPT, typename K, typename P, bool COUNT>
+__device__ int block_merge_sort(K* ka, P* pa, K* kb, P* pb, uint16_t* cnt, K pad_key) {
+  constexpr int N = NT * IPT;
+  const uint32_t t = threadIdx.x;
+  // thread-local sort of IPT consecutive items (insertion sort, stable)
+  {
+    K k[IPT];
+    P p[IPT];
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) { k[j] = ka[t * IPT + j]; p[j] = pa[t * IPT + j]; }
+    if (COUNT) {
+#pragma unroll
+      for (int j = 0; j < IPT; ++j) {
+        uint32_t c = 0;
+#pragma unroll
+        for (int q = 0; q < j; ++q) c += k[q] > k[j] ? 1u : 0u;
+        if (c && k[j] != pad_key) cnt[(uint32_t)(k[j] & 0xfffu)] += (uint16_t)c;
+      }
+    }
+#pragma unroll
+    for (int j = 1; j < IPT; ++j) {
+      K kk = k[j];
+      P pp = p[j];
+      int q = j - 1;
+      while (q >= 0 && k[q] > kk) { k[q + 1] = k[q]; p[q + 1] = p[q]; --q; }
+      k[q + 1] = kk;
+      p[q + 1] = pp;
+    }
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) { ka[t * IPT + j] = k[j]; pa[t * IPT + j] = p[j]; }
+  }
+  __syncthreads();
+  K* ks = ka; P* ps = pa; K* kd = kb; P* pd = pb;
+  int res = 0;
+  for (int w = IPT; w < N; w <<= 1) {
+    const uint32_t o = t * IPT;
+    const uint32_t s0 = (o / (2 * w)) * (2 * w);
+    const K* Ak = ks + s0;
+    const K* Bk = ks + s0 + w;
+    const P* Ap = ps + s0;
+    const P* Bp = ps + s0 + w;
+    const uint32_t d = o - s0;
+    uint32_t lo = d > (uint32_t)w ? d - w : 0, hi = d < (uint32_t)w ? d : (uint32_t)w;
+    while (lo < hi) {
+      uint32_t mid = (lo + hi) >> 1;
+      if (!(Bk[d - 1 - mid] < Ak[mid])) lo = mid + 1;
+      else hi = mid;
+    }
+    uint32_t a = lo, b = d - lo;
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) {
+      bool takeA = a < (uint32_t)w && (b >= (uint32_t)w || !(Bk[b] < Ak[a]));
+      if (takeA) {
+        kd[o + j] = Ak[a];
+        pd[o + j] = Ap[a];
+        ++a;
+      } else {
+        K kk = Bk[b];
+        kd[o + j] = kk;
+        pd[o + j] = Bp[b];
+        if (COUNT && kk != pad_key && a < (uint32_t)w) cnt[(uint32_t)(kk & 0xfffu)] += (uint16_t)(w - a);
+        ++b;
+      }
+    }
+    __syncthreads();
+    K* tk = ks; ks = kd; kd = tk;
+    P* tp = ps; ps = pd; pd = tp;
+    res ^= 1;
+  }
+  return res;
+}
+
+// ------------------------------------------------------------------ R2-R4 tile kernel
+constexpr int TL_NT = 1024, TL_IPT = 4;  // 4096 = TL_CAP
+constexpr int TL_SMEM_BINS = 2048;
+constexpr uint16_t NONE16 = 0xffff;
+
+struct TileSmem {
+  uint64_t ln[2][TL_CAP];     // lines (merge sort ping-pong); later: weighted prefix / query keys
+  uint16_t ps[2][TL_CAP];     // positions (payload); later: counts
+  uint8_t sdw[TL_CAP];        // store | has_dup << 1 | weight << 2
+  uint8_t ffl[TL_CAP];        // first_in_piece | last_in_piece << 1
+  uint8_t fnx[TL_CAP];        // the record's element is used again later in the tile
+  uint16_t sgs[TL_CAP];       // local start of the record's segment
+  uint16_t pl[TL_CAP];        // local previous use + 1 (0 = none)
+  uint16_t qx[TL_CAP];        // number of local queries before the record
+  uint16_t es[TL_CAP];        // entry slot + 1 (0 = none)
+  uint32_t tmax[TL_NT];       // per-thread inclusive max (segment-start scan)
+  uint32_t hist[TL_SMEM_BINS];
+  uint32_t ws[TL_NT / 32 + 1];
+  uint32_t misc[8];
+};
+
+struct EntryCols {
+  uint32_t* seg;
+  uint64_t* line;
+  uint32_t* tile;
+  uint32_t* f;      // global kept position of the piece's first use of the line
+  uint32_t* fa;     // local queries of the piece before f
+  uint32_t* fw;     // tile-local weighted position of f
+  uint8_t* ff;      // bit0 load, bit1 no dup, bit2 local next, bit3 head piece, bit4 f == l
+  uint32_t* l;      // global kept position of the piece's last use of the line
+  uint32_t* lw;     // tile-local weighted position of l
+  uint32_t* ld;     // local queries of the piece whose previous use lies after l
+  uint8_t* lf;      // bit0 store, bit1 no dup, bits 2.. weight of l
+};
+
+// One CTA per tile [bounds[t], bounds[t+1]) of the CTA-major kept sequence.
+// A "piece" is the part of one segment (CTA, or the whole trace for kernel
+// scope) inside the tile; pieces cut by the tile's start (head) or end
+// (tail) are "partial" and emit one entry per distinct line for the
+// cross-tile phase.
+__global__ void __launch_bounds__(TL_NT, 1)
+    k_rd_tile(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val, uint64_t K,
+              const uint32_t* __restrict__ bounds, uint32_t ntiles, int log2bins, uint32_t nbins,
+              uint64_t* __restrict__ g_hist, uint64_t* __restrict__ g_stream, uint32_t* __restrict__ tile_w,
+              uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
+  const uint32_t tx = threadIdx.x;
+  const uint32_t tile = blockIdx.x;
+  const uint64_t b = bounds[tile], e = bounds[tile + 1];
+  const uint32_t m = (uint32_t)(e - b);
+  const bool smem_hist = nbins <= TL_SMEM_BINS;
+  if (smem_hist)
+    for (uint32_t k = tx; k < nbins; k += TL_NT) S.hist[k] = 0;
+  if (tx == 0) S.misc[2] = m;
+  // ---- load (striped)
+  for (uint32_t x = tx; x < TL_CAP; x += TL_NT) {
+    if (x < m) {
+      uint64_t v = __ldg(val + b + x);
+      S.ln[0][x] = v & LINE_MASK;
+      uint32_t w = (uint32_t)(v >> VB_W) + 1u;
+      S.sdw[x] = (uint8_t)(((v >> VB_STORE) & 1u) | (((v >> VB_DUP) & 1u) << 1) | (w << 2));
+    } else {
+      S.ln[0][x] = ~0ull;
+      S.sdw[x] = 0;
+    }
+    S.ps[0][x] = (uint16_t)x;
+    S.fnx[x] = 0;
+    S.es[x] = 0;
+  }
+  // ---- segment starts (blocked: thread owns 4 consecutive positions)
+  bool ssf[TL_IPT];
+  uint32_t ss_local = 0;
+#pragma unroll
+  for (int j = 0; j < TL_IPT; ++j) {
+    uint32_t x = tx * TL_IPT + j;
+    uint64_t gx = b + x;
+    bool s = x < m && (gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1)));
+    ssf[j] = s;
+    if (s) ss_local = x;
+  }
+  S.tmax[tx] = block_inclusive_max<TL_NT>(ss_local, S.ws);
+  __syncthreads();
+  {
+    uint32_t cur = tx ? S.tmax[tx - 1] : 0u;
+#pragma unroll
+    for (int j = 0; j < TL_IPT; ++j) {
+      uint32_t x = tx * TL_IPT + j;
+      if (ssf[j]) cur = x;
+      S.sgs[x] = (uint16_t)cur;
+      if (ssf[j] && x > 0) atomicMin(&S.misc[2], x);  // start of the tile's second segment
+    }
+  }
+  const bool head_cont = m > 0 && b > 0 && (!key || __ldg(key + b) == __ldg(key + b - 1));
+  const bool tail_cont = m > 0 && e < K && (!key || __ldg(key + e) == __ldg(key + e - 1));
+  __syncthreads();
+  const uint32_t lastseg = m ? S.sgs[m - 1] : 0u;
+  const uint32_t second = S.misc[2];
+  auto partial = [&](uint32_t x) {
+    uint32_t sg = S.sgs[x];
+    return (sg == 0 && head_cont) || (sg == lastseg && tail_cont);
+  };
+  // ---- stable merge sort of (line, position): runs of equal lines in position order
+  int r = block_merge_sort<TL_NT, TL_IPT, uint64_t, uint16_t, false>(S.ln[0], S.ps[0], S.ln[1], S.ps[1], nullptr,
+                                                                     ~0ull);
+  const uint64_t* L = S.ln[r];
+  const uint16_t* PS = S.ps[r];
+  // ---- previous local use; first / last use of the line in its piece
+  uint32_t isent[TL_IPT];
+  uint32_t nent = 0;
+#pragma unroll
+  for (int j = 0; j < TL_IPT; ++j) {
+    uint32_t s = tx * TL_IPT + j;
+    isent[j] = 0;
+    if (s >= m) continue;
+    uint32_t x = PS[s];
+    uint64_t l = L[s];
+    uint32_t sg = S.sgs[x];
+    bool prev_same = s > 0 && L[s - 1] == l && S.sgs[PS[s - 1]] == sg;
+    bool next_same = s + 1 < m && L[s + 1] == l && S.sgs[PS[s + 1]] == sg;
+    bool st = S.sdw[x] & 1u;
+    uint32_t p = 0;
+    if (prev_same && !st) {
+      p = PS[s - 1] + 1u;
+      S.fnx[p - 1] = 1;
+    }
+    S.pl[x] = (uint16_t)p;
+    S.ffl[x] = (uint8_t)((prev_same ? 0u : 1u) | (next_same ? 0u : 2u));
+    if (!prev_same && partial(x)) {
+      isent[j] = 1;
+      nent++;
+    }
+  }
+  // ---- entry slots, one per (partial piece, line), allocated in sorted order
+  uint32_t etot;
+  uint32_t eoff = block_exclusive_scan<TL_NT>(nent, S.ws, &etot);
+  if (tx == 0)
+    S.misc[1] = etot ? (uint32_t)atomicAdd((unsigned long long*)&sc->count[1], (unsigned long long)etot) : 0u;
+  __syncthreads();
+  const uint32_t ebase = S.misc[1];
+  {
+    uint32_t run = eoff;
+#pragma unroll
+    for (int j = 0; j < TL_IPT; ++j) {
+      uint32_t s = tx * TL_IPT + j;
+      if (!isent[j]) continue;
+      uint32_t x = PS[s];
+      uint32_t slot = ebase + run;
+      E.seg[slot] = key ? __ldg(key + b + x) : 0u;
+      E.line[slot] = L[s];
+      E.tile[slot] = tile;
+      S.es[x] = (uint16_t)(run + 1);
+      run++;
+    }
+  }
+  __syncthreads();
+  // the last use of a run (if different from the first) shares the run's slot
+#pragma unroll
+  for (int j = 0; j < TL_IPT; ++j) {
+    uint32_t s = tx * TL_IPT + j;
+    if (s >= m) continue;
+    uint32_t x = PS[s];
+    uint32_t f = S.ffl[x];
+    if ((f & 2u) && !(f & 1u) && partial(x)) {
+      uint32_t q = s;
+      while (!(S.ffl[PS[q]] & 1u)) --q;
+      S.es[x] = S.es[PS[q]];
+    }
+  }
+  __syncthreads();
+  // ---- position-order prefix counts: local queries and weights
+  uint32_t* WP = reinterpret_cast<uint32_t*>(S.ln[r ^ 1]);  // weighted exclusive prefix
+  uint32_t* QK = reinterpret_cast<uint32_t*>(S.ln[r]);      // query keys (2 x TL_CAP u32)
+  uint32_t* QK2 = QK + TL_CAP;
+  uint16_t* CNT = S.ps[r ^ 1];
+  uint32_t nq = 0, wsum = 0;
+#pragma unroll
+  for (int j = 0; j < TL_IPT; ++j) {
+    uint32_t x = tx * TL_IPT + j;
+    if (x < m) {
+      nq += S.pl[x] ? 1u : 0u;
+      wsum += S.sdw[x] >> 2;
+    }
+  }
+  uint32_t Q, WT;
+  uint32_t qoff = block_exclusive_scan<TL_NT>(nq, S.ws, &Q);
+  uint32_t woff = block_exclusive_scan<TL_NT>(wsum, S.ws, &WT);
+#pragma unroll
+  for (int j = 0; j < TL_IPT; ++j) {
+    uint32_t x = tx * TL_IPT + j;
+    S.qx[x] = (uint16_t)qoff;
+    WP[x] = woff;
+    if (x < m) {
+      if (S.pl[x]) {
+        QK[qoff] = ((uint32_t)(S.pl[x] - 1u) << 12) | x;
+        qoff++;
+      }
+      woff += S.sdw[x] >> 2;
+    }
+  }
+  for (uint32_t k = Q + tx; k < TL_CAP; k += TL_NT) QK[k] = 0xffffffffu;
+  for (uint32_t x = tx; x < TL_CAP; x += TL_NT) CNT[x] = 0;
+  __syncthreads();
+  // ---- counting merge sort of the queries by previous use:
+  //      CNT[x] = #{ local queries y < x : P(y) > P(x) }
+  int r2 = block_merge_sort<TL_NT, TL_IPT, uint32_t, uint32_t, true>(QK, QK, QK2, QK2, CNT, 0xffffffffu);
+  const uint32_t* QS = r2 ? QK2 : QK;
+  // ---- R4: bin the local accesses
+  uint32_t stream = 0;
+#pragma unroll
+  for (int j = 0; j < TL_IPT; ++j) {
+    uint32_t x = tx * TL_IPT + j;
+    if (x >= m) continue;
+    uint32_t sdw = S.sdw[x];
+    bool st = sdw & 1u, hd = (sdw >> 1) & 1u;
+    uint32_t w = sdw >> 2;
+    uint32_t bin = 0xffffffffu, cntb = 1;
+    bool head_first = S.sgs[x] == 0 && head_cont && (S.ffl[x] & 1u);
+    if (S.pl[x]) {
+      uint32_t p = S.pl[x] - 1u;
+      uint32_t rd = (WP[x] - WP[p] - (uint32_t)(S.sdw[p] >> 2)) - CNT[x];
+      bin = rd_bin(rd, log2bins, nbins);
+    } else if (st) {
+      bin = nbins - 1;
+      cntb = w;
+    } else if (!head_first) {
+      bin = nbins - 1;
+    }
+    if (bin != 0xffffffffu) {
+      if (smem_hist) atomicAdd(&S.hist[bin], cntb);
+      else atomicAdd((unsigned long long*)&g_hist[bin], (unsigned long long)cntb);
+    }
+    if (st) stream += w - 1;  // all but the last of merged stores are one-shot elements
+    bool deferred = partial(x) && S.ffl[x] != 0;
+    if (!deferred && !S.pl[x] && !hd && !S.fnx[x]) stream += 1;
+  }
+  // ---- entry payloads of partial pieces
+  for (uint32_t x = tx; x < m; x += TL_NT) {
+    if (!S.es[x]) continue;
+    uint32_t slot = ebase + S.es[x] - 1;
+    uint32_t f = S.ffl[x];
+    uint32_t sdw = S.sdw[x];
+    if (f & 1u) {
+      bool head_piece = S.sgs[x] == 0 && head_cont;
+      E.f[slot] = (uint32_t)(b + x);
+      E.fa[slot] = (uint32_t)S.qx[x] - (uint32_t)S.qx[S.sgs[x]];
+      E.fw[slot] = WP[x];
+      E.ff[slot] = (uint8_t)(((sdw & 1u) ? 0u : 1u) | (((sdw >> 1) & 1u) ? 0u : 2u) | (S.fnx[x] ? 4u : 0u) |
+                             (head_piece ? 8u : 0u) | ((f & 2u) ? 16u : 0u));
+    }
+    if (f & 2u) {
+      uint32_t pend = (S.sgs[x] == lastseg && tail_cont) ? m : second;
+      // queries of the piece whose previous use lies in (x, pend)
+      uint32_t lo_key = (x + 1) << 12, hi_key = pend << 12;
+      uint32_t a0 = 0, a1 = Q;
+      while (a0 < a1) { uint32_t md = (a0 + a1) >> 1; if (QS[md] < lo_key) a0 = md + 1; else a1 = md; }
+      uint32_t c0 = a0, c1 = Q;
+      while (c0 < c1) { uint32_t md = (c0 + c1) >> 1; if (QS[md] < hi_key) c0 = md + 1; else c1 = md; }
+      E.l[slot] = (uint32_t)(b + x);
+      E.lw[slot] = WP[x];
+      E.ld[slot] = c0 - a0;
+      E.lf[slot] = (uint8_t)((sdw & 1u) | (((sdw >> 1) & 1u) ? 0u : 2u) | ((sdw >> 2) << 2));
+    }
+  }
+  // ---- flush
+  stream = __reduce_add_sync(FULL, stream);
+  if (lane_id() == 0 && stream) atomicAdd((unsigned long long*)g_stream, (unsigned long long)stream);
+  if (tx == 0) {
+    tile_w[tile] = WT;
+    tile_q[tile] = Q;
+  }
+  __syncthreads();
+  if (smem_hist)
+    for (uint32_t k = tx; k < nbins; k += TL_NT)
+      if (S.hist[k]) atomicAdd((unsigned long long*)&g_hist[k], (unsigned long long)S.hist[k]);
+}
+
+// ------------------------------------------------------------------ cross-tile phase
+__global__ void k_ent_line_range(const uint64_t* __restrict__ line, uint64_t E, unsigned long long* mn,
+                                 unsigned long long* mx) {
+  uint64_t a = ~0ull, z = 0;
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < E; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint64_t v = line[i];
+    a = v < a ? v : a;
+    z = v > z ? v : z;
+  }
+  for (int o = 16; o; o >>= 1) {
+    uint64_t a2 = __shfl_xor_sync(FULL, a, o), z2 = __shfl_xor_sync(FULL, z, o);
+    a = a2 < a ? a2 : a;
+    z = z2 > z ? z2 : z;
+  }
+  if (lane_id() == 0) { atomicMin(mn, (unsigned long long)a); atomicMax(mx, (unsigned long long)z); }
+}
+
+// composite sort key (seg, line - minl, tile) when it fits in 64 bits; else
+// one field at a time (field 0 = tile, 1 = line, 2 = seg) through idx.
+__global__ void k_ent_key(const uint32_t* __restrict__ seg, const uint64_t* __restrict__ line,
+                          const uint32_t* __restrict__ tile, uint64_t E, uint64_t minl, int lb, int tb, int field,
+                          const uint32_t* __restrict__ idx_in, uint64_t* __restrict__ key, uint32_t* __restrict__ idx) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < E; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t j = idx_in ? idx_in[i] : (uint32_t)i;
+    uint64_t k;
+    if (field < 0) k = ((uint64_t)seg[j] << (lb + tb)) | ((line[j] - minl) << tb) | tile[j];
+    else if (field == 0) k = tile[j];
+    else if (field == 1) k = line[j] - minl;
+    else k = seg[j];
+    key[i] = k;
+    idx[i] = j;
+  }
+}
+
+struct CrossOut {
+  uint32_t* xpos;   // query global kept position
+  uint32_t* xq;     // its previous use (global kept position)
+  int64_t* part;    // RD before subtracting the cross-tile dominance count
+};
+
+__global__ void k_link(const uint32_t* __restrict__ order, uint64_t E, EntryCols En,
+                       const unsigned long long* __restrict__ tile_wb, const unsigned long long* __restrict__ tile_qb,
+                       uint32_t nbins, uint64_t* g_hist, uint64_t* g_stream, CrossOut X, Scalars* sc) {
+  uint32_t stream = 0;
+  for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < E; k += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t e = order[k];
+    int64_t pv = -1, nx = -1;
+    if (k > 0) {
+      uint32_t p = order[k - 1];
+      if (En.seg[p] == En.seg[e] && En.line[p] == En.line[e]) pv = p;
+    }
+    if (k + 1 < E) {
+      uint32_t q = order[k + 1];
+      if (En.seg[q] == En.seg[e] && En.line[q] == En.line[e]) nx = q;
+    }
+    uint8_t ff = En.ff[e], lf = En.lf[e];
+    bool f_load = ff & 1u, f_nodup = ff & 2u, f_next = ff & 4u, head = ff & 8u, f_is_l = ff & 16u;
+    bool next_load = nx >= 0 && (En.ff[nx] & 1u);
+    // RD of the piece's first use (deferred by the tile kernel when the piece is a head piece)
+    bool linked = false;
+    if (head && f_load) {
+      if (pv >= 0) {
+        linked = true;
+        uint32_t p = (uint32_t)pv;
+        uint64_t gwf = tile_wb[En.tile[e]] + En.fw[e];
+        uint64_t gwl = tile_wb[En.tile[p]] + En.lw[p];
+        uint32_t wl = En.lf[p] >> 2;
+        uint64_t B = tile_qb[En.tile[e]] - tile_qb[En.tile[p] + 1];
+        int64_t part = (int64_t)(gwf - gwl - wl) - (int64_t)En.fa[e] - (int64_t)B - (int64_t)En.ld[p];
+        unsigned long long slot = atomicAdd((unsigned long long*)&sc->count[2], 1ull);
+        X.xpos[slot] = En.f[e];
+        X.xq[slot] = En.l[p];
+        X.part[slot] = part;
+      } else {
+        atomicAdd((unsigned long long*)&g_hist[nbins - 1], 1ull);
+      }
+    }
+    // streaming of the deferred first / last uses
+    bool f_pnone = !f_load || !linked;
+    bool f_next_any = f_is_l ? next_load : f_next;
+    if (f_pnone && f_nodup && !f_next_any) stream++;
+    if (!f_is_l) {
+      bool l_store = lf & 1u, l_nodup = lf & 2u;
+      if (l_store && l_nodup && !next_load) stream++;
+    }
+  }
+  stream = __reduce_add_sync(FULL, stream);
+  if (lane_id() == 0 && stream) atomicAdd((unsigned long long*)g_stream, (unsigned long long)stream);
+}
+
+// one level of a device-wide merge sort with inversion counting: runs of
+// width w are merged pairwise; items of the right run add the number of
+// larger items in the left run to cnt[id].
+__global__ void k_merge_count(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ iin,
+                              uint32_t* __restrict__ kout, uint32_t* __restrict__ iout, uint64_t M, uint64_t w,
+                              uint32_t* __restrict__ cnt) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint64_t s = (i / (2 * w)) * (2 * w);
+    uint32_t k = kin[i];
+    uint64_t dst;
+    if (i < s + w) {
+      uint64_t b0 = s + w, b1 = s + 2 * w < M ? s + 2 * w : M;
+      uint64_t lo = b0, hi = b1 > b0 ? b1 : b0;
+      while (lo < hi) { uint64_t md = (lo + hi) >> 1; if (kin[md] < k) lo = md + 1; else hi = md; }
+      dst = s + (i - s) + (lo - b0);
+    } else {
+      uint64_t a0 = s, a1 = s + w;
+      uint64_t lo = a0, hi = a1;
+      while (lo < hi) { uint64_t md = (lo + hi) >> 1; if (kin[md] < k) lo = md + 1; else hi = md; }
+      uint64_t less = lo - a0;
+      cnt[iin[i]] += (uint32_t)(w - less);
+      dst = s + (i - s - w) + less;
+    }
+    kout[dst] = k;
+    iout[dst] = iin[i];
+  }
+}
+
+__global__ void k_iota_gather(const uint32_t* __restrict__ order, const uint32_t* __restrict__ xq, uint64_t M,
+                              uint32_t* __restrict__ k, uint32_t* __restrict__ id, uint32_t* __restrict__ cnt) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
+    uint32_t j = order[i];
+    k[i] = xq[j];
+    id[i] = j;
+    cnt[j] = 0;
+  }
+}
+
+__global__ void k_cross_final(const int64_t* __restrict__ part, const uint32_t* __restrict__ cnt, uint64_t M,
+                              int log2bins, uint32_t nbins, uint64_t* g_hist, Scalars* sc) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
+    int64_t rd = part[i] - (int64_t)cnt[i];
+    if (rd < 0) {
+      atomicMax(&sc->err_code, 3u);
+      rd = 0;
+    }
+    atomicAdd((unsigned long long*)&g_hist[rd_bin((uint64_t)rd, log2bins, nbins)], 1ull);
+  }
+}
+
+__global__ void k_widen(const uint32_t* a, unsigned long long* o, uint64_t nvalid, uint64_t n) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    o[i] = i < nvalid ? a[i] : 0ull;
+}
+
+__global__ void k_iota(uint32_t* p, uint64_t n) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x)
+    p[i] = (uint32_t)i;
+}
+
+int bits_for(uint64_t maxv) {
+  int b = 0;
+  while (b < 64 && (maxv >> b)) ++b;
+  return b;
+}
+
+int g_tile_smem_set = 0, g_compact_smem_set = 0;
+
+}  // namespace
+
+cudaError_t run_reuse(cadv_ctx* c, uint32_t lbs, int scope, int log2bins, uint32_t nbins, uint64_t* d_hist,
+                      uint64_t* d_stats) {
+  cudaError_t e;
+  const uint64_t n = c->t.n;
+  const uint64_t nmem = c->n_kind[0] + c->n_kind[1];
+  const int cta_scope = scope == CADV_SCOPE_CTA;
+  const int grid_ls = c->num_sms * 4;
+  Scalars* sc = scalars(c);
+  void *k0 = nullptr, *k1 = nullptr, *v0, *v1, *st;
+  uint64_t cap = nmem + 16;
+  if ((e = ensure(c, B_RD_VAL, cap * 8, &v0)) || (e = ensure(c, B_SORT_V1, cap * 8, &v1))) return e;
+  if (cta_scope && ((e = ensure(c, B_RD_KEY, cap * 4, &k0)) || (e = ensure(c, B_SORT_K1, cap * 4, &k1)))) return e;
+  // ---- R1 compaction
+  uint64_t ctiles = (n + CP_TILE - 1) / CP_TILE;
+  if ((e = ensure(c, B_RD_TILESTAT, ctiles * 8 + 64, &st))) return e;
+  if ((e = cudaMemsetAsync(st, 0, ctiles * 8, c->stream))) return e;
+  if (!g_compact_smem_set) {
+    if ((e = cudaFuncSetAttribute(k_rd_compact, cudaFuncAttributeMaxDynamicSharedMemorySize, CP_SMEM))) return e;
+    g_compact_smem_set = 1;
+  }
+  CADV_LAUNCH(c, k_rd_compact<<<(unsigned)ctiles, CP_NT, CP_SMEM, c->stream>>>(
+                     c->t.addr, c->t.cta, c->t.meta, n, lbs, cta_scope, (uint32_t*)k0, (uint64_t*)v0,
+                     (uint64_t*)st, d_hist, sc));
+  if ((e = cudaGetLastError())) return e;
+  // kept count = inclusive prefix of the last compaction tile
+  uint64_t last;
+  if ((e = cudaMemcpyAsync(&last, (uint64_t*)st + (ctiles - 1), 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  const uint64_t K = last & LB_VAL;
+  if (K == 0) return cudaSuccess;
+  // ---- R1b regroup by CTA (stable)
+  const uint32_t* key = nullptr;
+  const uint64_t* val = (const uint64_t*)v0;
+  if (cta_scope) {
+    int res;
+    int bits = bits_for(c->max_cta);
+    if (bits == 0) bits = 1;
+    if ((e = radix_sort_pairs<uint32_t, uint64_t>(c, (uint32_t*)k0, (uint64_t*)v0, (uint32_t*)k1, (uint64_t*)v1, K, 0,
+                                                  bits, &res)))
+      return e;
+    key = res ? (const uint32_t*)k1 : (const uint32_t*)k0;
+    val = res ? (const uint64_t*)v1 : (const uint64_t*)v0;
+  }
+  // ---- tiles
+  uint64_t ntiles = (K + TL_NOM - 1) / TL_NOM;
+  void *bnd, *tw, *tq;
+  if ((e = ensure(c, B_RD_XTMP, (ntiles + 2) * 4 + 64, &bnd))) return e;
+  if ((e = ensure(c, B_RD_TILEW, (ntiles + 2) * 8 * 2, &tw))) return e;
+  if ((e = ensure(c, B_RD_TILEQ, (ntiles + 2) * 8 * 2, &tq))) return e;
+  CADV_LAUNCH(c, k_tile_bounds<<<(unsigned)((ntiles + 1 + 7) / 8), 256, 0, c->stream>>>(key, K, (uint32_t*)bnd,
+                                                                                       ntiles));
+  // entries: at most one per kept record
+  void* ent;
+  size_t ent_bytes = K * (4 + 8 + 4 + 4 + 4 + 4 + 1 + 4 + 4 + 4 + 1) + 16 * 16;
+  if ((e = ensure(c, B_RD_ENT, ent_bytes, &ent))) return e;
+  EntryCols En;
+  {
+    uint8_t* p = (uint8_t*)ent;
+    auto take = [&](size_t bytes) { uint8_t* q = p; p += (bytes + 15) & ~size_t(15); return q; };
+    En.line = (uint64_t*)take(K * 8);
+    En.seg = (uint32_t*)take(K * 4);
+    En.tile = (uint32_t*)take(K * 4);
+    En.f = (uint32_t*)take(K * 4);
+    En.fa = (uint32_t*)take(K * 4);
+    En.fw = (uint32_t*)take(K * 4);
+    En.l = (uint32_t*)take(K * 4);
+    En.lw = (uint32_t*)take(K * 4);
+    En.ld = (uint32_t*)take(K * 4);
+    En.ff = (uint8_t*)take(K);
+    En.lf = (uint8_t*)take(K);
+  }
+  if (!g_tile_smem_set) {
+    if ((e = cudaFuncSetAttribute(k_rd_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))))
+      return e;
+    g_tile_smem_set = 1;
+  }
+  uint32_t* tile_w = (uint32_t*)tw;
+  uint32_t* tile_q = (uint32_t*)tq;
+  CADV_LAUNCH(c, k_rd_tile<<<(unsigned)ntiles, TL_NT, sizeof(TileSmem), c->stream>>>(
+                     key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
+                     tile_q, En, sc));
+  if ((e = cudaGetLastError())) return e;
+  unsigned long long nent;
+  if ((e = cudaMemcpyAsync(&nent, &sc->count[1], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  if (nent == 0) return cudaSuccess;
+  // ---- cross-tile phase
+  // tile prefix sums of weights and local query counts (u64)
+  unsigned long long* twb = (unsigned long long*)((uint8_t*)tw + (ntiles + 2) * 8);
+  unsigned long long* tqb = (unsigned long long*)((uint8_t*)tq + (ntiles + 2) * 8);
+  void* wide;
+  if ((e = ensure(c, B_RD_XQ2, (ntiles + 2) * 16 + 64, &wide))) return e;
+  {
+    unsigned long long* w64 = (unsigned long long*)wide;
+    unsigned long long* q64 = w64 + (ntiles + 2);
+    CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_w, w64, ntiles, ntiles + 1));
+    CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_q, q64, ntiles, ntiles + 1));
+    if ((e = exclusive_scan_u64(c, (const uint64_t*)w64, (uint64_t*)twb, ntiles + 1))) return e;
+    if ((e = exclusive_scan_u64(c, (const uint64_t*)q64, (uint64_t*)tqb, ntiles + 1))) return e;
+  }
+  // sort entries by (seg, line, tile)
+  void *ek0, *ek1, *ei0, *ei1;
+  if ((e = ensure(c, B_RD_ENT_KEY0, nent * 8, &ek0)) || (e = ensure(c, B_RD_ENT_KEY1, nent * 8, &ek1)) ||
+      (e = ensure(c, B_RD_ENT_IDX0, nent * 4, &ei0)) || (e = ensure(c, B_RD_ENT_IDX1, nent * 4, &ei1)))
+    return e;
+  unsigned long long* mm = (unsigned long long*)&sc->count[4];
+  if ((e = cudaMemsetAsync(mm, 0xff, 8, c->stream)) || (e = cudaMemsetAsync(mm + 1, 0, 8, c->stream))) return e;
+  CADV_LAUNCH(c, k_ent_line_range<<<grid_ls, 256, 0, c->stream>>>(En.line, nent, mm, mm + 1));
+  unsigned long long hmm[2];
+  if ((e = cudaMemcpyAsync(hmm, mm, 16, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  uint64_t minl = hmm[0];
+  int lb = bits_for(hmm[1] - hmm[0]);
+  int tb = bits_for(ntiles);
+  int sb = cta_scope ? bits_for(c->max_cta) : 0;
+  const uint32_t* order;
+  if (sb + lb + tb <= 64) {
+    CADV_LAUNCH(c, k_ent_key<<<grid_ls, 256, 0, c->stream>>>(En.seg, En.line, En.tile, nent, minl, lb, tb, -1, nullptr,
+                                                             (uint64_t*)ek0, (uint32_t*)ei0));
+    int res;
+    if ((e = radix_sort_pairs<uint64_t, uint32_t>(c, (uint64_t*)ek0, (uint32_t*)ei0, (uint64_t*)ek1, (uint32_t*)ei1,
+                                                  nent, 0, sb + lb + tb, &res)))
+      return e;
+    order = res ? (const uint32_t*)ei1 : (const uint32_t*)ei0;
+  } else {
+    // one field at a time, least significant first (stable passes)
+    const uint32_t* idx = nullptr;
+    uint32_t* ib[2] = {(uint32_t*)ei0, (uint32_t*)ei1};
+    int cur = 0;
+    int fb[3] = {tb, lb, sb};
+    for (int field = 0; field < 3; ++field) {
+      if (fb[field] == 0) continue;
+      uint32_t* dst = ib[cur];
+      uint32_t* alt = ib[cur ^ 1];
+      CADV_LAUNCH(c, k_ent_key<<<grid_ls, 256, 0, c->stream>>>(En.seg, En.line, En.tile, nent, minl, lb, tb, field,
+                                                               idx, (uint64_t*)ek1, alt));
+      // keys in ek1, idx in alt -> sort into (ek0, dst) or back
+      int res;
+      if ((e = radix_sort_pairs<uint64_t, uint32_t>(c, (uint64_t*)ek1, alt, (uint64_t*)ek0, dst, nent, 0, fb[field],
+                                                    &res)))
+        return e;
+      idx = res ? dst : alt;
+      cur = (idx == ib[0]) ? 1 : 0;
+    }
+    order = idx ? idx : (const uint32_t*)ei0;
+  }
+  // link
+  void *xq, *xq2;
+  if ((e = ensure(c, B_RD_XQ, nent * (4 + 4 + 8) + 64, &xq))) return e;
+  CrossOut X;
+  X.xpos = (uint32_t*)xq;
+  X.xq = X.xpos + nent;
+  X.part = (int64_t*)(((uintptr_t)(X.xq + nent) + 15) & ~(uintptr_t)15);
+  CADV_LAUNCH(c, k_link<<<grid_ls, 256, 0, c->stream>>>(order, nent, En, twb, tqb, nbins, d_hist, d_stats, X, sc));
+  unsigned long long M;
+  if ((e = cudaMemcpyAsync(&M, &sc->count[2], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  if (M == 0) return cudaSuccess;
+  // sort cross queries by position, then count inversions of their previous uses
+  if ((e = ensure(c, B_RD_ENT_KEY1, M * 8 + nent * 8, &ek1))) return e;
+  if ((e = ensure(c, B_SORT_K0, M * 4 * 2 + 64, &xq2))) return e;
+  uint32_t* pk0 = (uint32_t*)xq2;
+  uint32_t* pk1 = pk0 + M;
+  uint32_t* pi0 = (uint32_t*)ei0;  // nent >= M
+  uint32_t* pi1 = (uint32_t*)ei1;
+  if ((e = cudaMemcpyAsync(pk0, X.xpos, M * 4, cudaMemcpyDeviceToDevice, c->stream))) return e;
+  CADV_LAUNCH(c, k_iota<<<grid_ls, 256, 0, c->stream>>>(pi0, M));
+  int res;
+  if ((e = radix_sort_pairs<uint32_t, uint32_t>(c, pk0, pi0, pk1, pi1, M, 0, 32, &res))) return e;
+  const uint32_t* ord = res ? pi1 : pi0;
+  // keys = previous use in position order; ids = cross-query index
+  uint32_t* ka = (uint32_t*)ek0;
+  uint32_t* kb = ka + M;
+  uint32_t* ia = (uint32_t*)ek1;
+  uint32_t* ib = ia + M;
+  void* cntb;
+  if ((e = ensure(c, B_GATHER, M * 4 + 64, &cntb))) return e;
+  uint32_t* cnt = (uint32_t*)cntb;
+  if ((e = ensure(c, B_RD_ENT_KEY0, M * 8 + 64, &ek0))) return e;
+  ka = (uint32_t*)ek0;
+  kb = ka + M;
+  CADV_LAUNCH(c, k_iota_gather<<<grid_ls, 256, 0, c->stream>>>(ord, X.xq, M, ka, ia, cnt));
+  for (uint64_t w = 1; w < M; w <<= 1) {
+    CADV_LAUNCH(c, k_merge_count<<<grid_ls, 256, 0, c->stream>>>(ka, ia, kb, ib, M, w, cnt));
+    std::swap(ka, kb);
+    std::swap(ia, ib);
+  }
+  CADV_LAUNCH(c, k_cross_final<<<grid_ls, 256, 0, c->stream>>>(X.part, cnt, M, log2bins, nbins, d_hist, sc));
+  return cudaGetLastError();
+}
+
+}  // namespace cadv

@@ -1,0 +1,309 @@
+"""GPU parity: the CUDA path (through the C ABI) == the CPU oracle, bit-exact.
+
+Every output is an integer, so comparisons are exact (`==`), element by
+element: histograms, stats, per-site counters.  Inputs are seeded synthetic
+traces from tracegen/ (DESIGN.md "Input recipe").
+"""
+import numpy as np
+import pytest
+
+import oracle as orc
+import tracegen as tg
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def cadv():
+    import paper_conf_cgo_shensll18_b200 as m
+    return m
+
+
+@pytest.fixture(scope="module")
+def ctx(cadv):
+    c = cadv.create(0)
+    yield c
+    c.destroy()
+
+
+def load(ctx, cadv, t, contiguous=True, host=False):
+    if host:
+        ctx.load_trace(t.cols, warp_contiguous=contiguous)
+    else:
+        ctx.load_trace(cadv.to_device(t), warp_contiguous=contiguous)
+
+
+def check_reuse(ctx, t, lb, scope, binning=0, nbins=66):
+    h_gpu, s_gpu = ctx.reuse_histogram(lb, scope, binning, nbins)
+    h_ref, s_ref = orc.reuse(t, lb, scope, binning, nbins)
+    assert (h_gpu == h_ref).all(), (lb, scope, binning, np.nonzero(h_gpu != h_ref), h_gpu, h_ref)
+    assert s_gpu == s_ref, (lb, scope, s_gpu, s_ref)
+
+
+def check_md(ctx, t, lb, W=32):
+    h_gpu, ps_gpu = ctx.mem_divergence(lb, W, t.nsites)
+    h_ref, ps_ref = orc.mem_div(t, lb, W)
+    assert (h_gpu == h_ref).all(), (lb, W, h_gpu, h_ref)
+    assert (ps_gpu == ps_ref).all()
+
+
+def check_bd(ctx, t, W=32):
+    ps_gpu, tot_gpu = ctx.branch_divergence(W, t.nsites)
+    ps_ref, tot_ref = orc.branch_div(t, W)
+    assert (tot_gpu == tot_ref).all(), (W, tot_gpu, tot_ref)
+    assert (ps_gpu == ps_ref).all()
+
+
+def full_check(ctx, cadv, t, lbs=(128, 32), scopes=(0, 1), contiguous=True, W=(32,)):
+    load(ctx, cadv, t, contiguous)
+    for lb in lbs:
+        for sc in scopes:
+            check_reuse(ctx, t, lb, sc)
+        check_md(ctx, t, lb)
+    for w in W:
+        check_bd(ctx, t, w)
+
+
+# ----------------------------------------------------------------- config 1 + closed forms
+
+def test_c1_vecadd_all(ctx, cadv):
+    t = tg.generate("vecadd")
+    load(ctx, cadv, t)
+    for lb in (1, 4, 32, 128):
+        for sc in (0, 1):
+            for binning, nb in ((0, 66), (1, 12), (0, 3)):
+                check_reuse(ctx, t, lb, sc, binning, nb)
+        for W in (32, 16, 8, 4, 2, 1):
+            check_md(ctx, t, lb, W)
+    for W in (32, 16, 8, 1):
+        check_bd(ctx, t, W)
+    # closed forms through the GPU path too
+    h, st = ctx.reuse_histogram(128, 0, 0, 66)
+    assert h[0] == 1322 and h[-1] == 727
+    ps, tot = ctx.branch_divergence(32, t.nsites)
+    assert list(tot) == [50, 2, 1558]
+
+
+def test_host_pointer_load(ctx, cadv):
+    t = tg.generate("vecadd")
+    load(ctx, cadv, t, host=True)
+    check_reuse(ctx, t, 128, 0)
+    check_md(ctx, t, 32)
+    check_bd(ctx, t)
+
+
+def test_paper_example_gpu(ctx, cadv):
+    """ABCCDEFAAAB, RD(B) = 5; full histogram {0:3, 5:2, ∞:6}."""
+    addr = [0x7F0000000000 + 4 * "ABCDEF".index(ch) for ch in "ABCCDEFAAAB"]
+    n = len(addr)
+    t = tg.from_arrays(addr, np.zeros(n), np.zeros(n), np.zeros(n), np.arange(n), [2 << 2] * n, nsites=1)
+    load(ctx, cadv, t)
+    h, st = ctx.reuse_histogram(4, 0, 0, 8)
+    assert list(h) == [3, 0, 0, 0, 0, 2, 0, 6]
+
+
+@pytest.mark.parametrize("K,R", [(3, 4), (100, 3), (5000, 2), (9000, 3)])
+def test_cyclic_closed_form_gpu(ctx, cadv, K, R):
+    """K lines read cyclically R times: K ∞ + K(R-1) at distance K-1 (spans tiles for K > 4096)."""
+    n = K * R
+    addr = 0x7F0000000000 + 128 * (np.arange(n) % K)
+    t = tg.from_arrays(addr, np.zeros(n), np.zeros(n), np.zeros(n), np.arange(n), np.full(n, 2 << 2), nsites=1)
+    load(ctx, cadv, t)
+    h, st = ctx.reuse_histogram(128, 0, 0, K + 3)
+    assert h[-1] == K and h[K - 1] == K * (R - 1) and h.sum() == n
+
+
+# ----------------------------------------------------------------- random traces
+
+RAND_CASES = [
+    dict(ctas=1, threads=32, instrs=4, lines=4),
+    dict(ctas=3, threads=64, instrs=10, lines=16, pstore=0.3),
+    dict(ctas=8, threads=96, instrs=20, lines=40, pbb=0.5),
+    dict(ctas=2, threads=1024, instrs=30, lines=200),        # large CTA segments -> several tiles
+    dict(ctas=40, threads=128, instrs=12, lines=8, pfull=0.9),
+    dict(ctas=5, threads=33, instrs=50, lines=3, pstore=0.5),
+    dict(ctas=1, threads=1024, instrs=80, lines=2000, pstore=0.1),  # one giant CTA, many lines
+    dict(ctas=200, threads=64, instrs=6, lines=64, launches=3),
+]
+
+
+@pytest.mark.parametrize("case", range(len(RAND_CASES)))
+@pytest.mark.parametrize("seed", [1, 2, 3])
+def test_random_traces(ctx, cadv, case, seed):
+    t = tg.generate("rand", seed=seed, **RAND_CASES[case])
+    full_check(ctx, cadv, t, lbs=(1, 32, 128), W=(32, 8))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_non_contiguous_traces(ctx, cadv, seed):
+    """warp_contiguous = 0: records of the per-(cta, warp) streams randomly merged."""
+    t = tg.generate("rand", seed=seed, ctas=6, threads=128, instrs=15, lines=30, scramble=1, scramble_seed=seed)
+    full_check(ctx, cadv, t, lbs=(32, 128), contiguous=False, W=(32, 16))
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_lane_order_independence(ctx, cadv, seed):
+    """Divergence depends on lane sets, not on the order lanes appear in a warp instruction."""
+    t = tg.generate("rand", seed=seed, ctas=4, threads=64, instrs=20, lines=20)
+    rng = np.random.default_rng(seed)
+    # permute records inside each run of equal (cta, warp, winst, family)
+    key = (t.cta.astype(np.int64) << 32) | ((t.tid.astype(np.int64) >> 5) << 24) | (t.winst.astype(np.int64) << 1) \
+        | ((t.meta & 3) == 2)
+    starts = np.r_[0, np.nonzero(np.diff(key))[0] + 1, t.n]
+    order = np.arange(t.n)
+    for a, b in zip(starts[:-1], starts[1:]):
+        order[a:b] = a + rng.permutation(b - a)
+    t2 = tg.from_arrays(*(t.cols[k][order] for k, _ in tg.COLUMNS), nsites=t.nsites)
+    load(ctx, cadv, t2)
+    check_md(ctx, t2, 32)
+    check_bd(ctx, t2)
+    h1, _ = orc.mem_div(t, 32)
+    h2, _ = ctx.mem_divergence(32, 32, t.nsites)
+    assert (h1 == h2).all()
+
+
+# ----------------------------------------------------------------- adversarial / edge cases
+
+def _mk(addr, cta, tid=None, meta=None, winst=None):
+    n = len(addr)
+    tid = np.zeros(n) if tid is None else tid
+    meta = np.full(n, 2 << 2) if meta is None else meta
+    winst = np.arange(n) if winst is None else winst
+    return tg.from_arrays(addr, cta, tid, np.zeros(n), winst, meta, nsites=1)
+
+
+def test_all_same_line(ctx, cadv):
+    n = 20000
+    t = _mk(np.full(n, 0x7F0000000000), np.zeros(n))
+    full_check(ctx, cadv, t, lbs=(128,), W=(32,))
+
+
+def test_all_distinct_lines(ctx, cadv):
+    n = 20000
+    t = _mk(0x7F0000000000 + 128 * np.arange(n), np.zeros(n))
+    full_check(ctx, cadv, t, lbs=(128, 4096), W=(32,))
+
+
+@pytest.mark.parametrize("k", [1, 2, 7])
+def test_stores_every_k(ctx, cadv, k):
+    rng = np.random.default_rng(k)
+    n = 30000
+    addr = 0x7F0000000000 + 4 * rng.integers(0, 300, n)
+    meta = np.where(np.arange(n) % k == 0, (2 << 2) | 1, 2 << 2)
+    t = _mk(addr, rng.integers(0, 3, n), meta=meta)
+    full_check(ctx, cadv, t, lbs=(4, 32, 128), W=(32,))
+
+
+def test_many_tiny_ctas(ctx, cadv):
+    rng = np.random.default_rng(5)
+    n = 100000
+    cta = np.sort(rng.integers(0, 60000, n))
+    addr = 0x7F0000000000 + 8 * rng.integers(0, 50, n)
+    t = _mk(addr, cta)
+    full_check(ctx, cadv, t, lbs=(8, 128), W=(32,))
+
+
+def test_empty_and_bb_only(ctx, cadv):
+    t = _mk(np.zeros(0, np.uint64), np.zeros(0))
+    load(ctx, cadv, t)
+    h, st = ctx.reuse_histogram(128, 0, 0, 10)
+    assert h.sum() == 0 and st["accesses"] == 0
+    hm, _ = ctx.mem_divergence(128, 32, 1)
+    assert hm.sum() == 0
+    _, tot = ctx.branch_divergence(32, 1)
+    assert tot.sum() == 0
+    t = tg.generate("nw", ctas=3)
+    full_check(ctx, cadv, t, lbs=(128,), W=(32, 16))
+
+
+def test_large_nbins_global_atomics(ctx, cadv):
+    t = tg.generate("rand", seed=9, ctas=2, threads=512, instrs=40, lines=900)
+    load(ctx, cadv, t)
+    check_reuse(ctx, t, 32, 0, 0, 5000)
+    check_reuse(ctx, t, 32, 1, 0, 5000)
+
+
+def test_bad_trace_detected(ctx, cadv):
+    t = tg.generate("vecadd")
+    cols = {k: v.copy() for k, v in t.cols.items()}
+    cols["meta"][100] = 3
+    ctx.load_trace(cadv.to_device(tg.from_arrays(*(cols[k] for k, _ in tg.COLUMNS), nsites=t.nsites)))
+    for call in (lambda: ctx.reuse_histogram(128, 0, 0, 10), lambda: ctx.mem_divergence(128, 32, 7),
+                 lambda: ctx.branch_divergence(32, 7)):
+        with pytest.raises(cadv.CadvError) as e:
+            call()
+        assert e.value.status == cadv.CADV_ERR_BAD_TRACE
+    cols = {k: v.copy() for k, v in t.cols.items()}
+    mem = np.nonzero((cols["meta"] & 3) < 2)[0]
+    cols["addr"][mem[5]] += 1
+    ctx.load_trace(cadv.to_device(tg.from_arrays(*(cols[k] for k, _ in tg.COLUMNS), nsites=t.nsites)))
+    with pytest.raises(cadv.CadvError) as e:
+        ctx.reuse_histogram(128, 0, 0, 10)
+    assert e.value.status == cadv.CADV_ERR_BAD_TRACE
+
+
+def test_long_run_detected(ctx, cadv):
+    """A warp-level group of 40 records (same cta, warp, winst) violates the format."""
+    n = 40
+    t = _mk(0x7F0000000000 + 4 * np.arange(n), np.zeros(n), tid=np.arange(n) % 32, winst=np.zeros(n))
+    ctx.load_trace(cadv.to_device(t))
+    with pytest.raises(cadv.CadvError) as e:
+        ctx.mem_divergence(128, 32, 1)
+    assert e.value.status == cadv.CADV_ERR_BAD_TRACE
+
+
+def test_invalid_args(ctx, cadv):
+    t = tg.generate("vecadd")
+    load(ctx, cadv, t)
+    for args in ((48, 0, 0, 10), (128, 2, 0, 10), (128, 0, 5, 10), (128, 0, 0, 2), (8192, 0, 0, 10)):
+        with pytest.raises(cadv.CadvError) as e:
+            ctx.reuse_histogram(*args)
+        assert e.value.status == cadv.CADV_ERR_INVALID_ARG
+    with pytest.raises(cadv.CadvError):
+        ctx.mem_divergence(128, 64, 7)
+    with pytest.raises(cadv.CadvError) as e:
+        ctx.mem_divergence(128, 32, 3)  # sites up to 6 exist
+    assert e.value.status == cadv.CADV_ERR_INVALID_ARG
+
+
+# ----------------------------------------------------------------- shaped workloads (reduced sizes)
+
+def test_sgemm_small(ctx, cadv):
+    full_check(ctx, cadv, tg.generate("sgemm", n=64, bb=1), lbs=(32, 128))
+
+
+def test_srad_small(ctx, cadv):
+    full_check(ctx, cadv, tg.generate("srad", rows=128, cols=128, iters=2), lbs=(32, 128))
+
+
+def test_bfs_small(ctx, cadv):
+    full_check(ctx, cadv, tg.generate("bfs", nodes=20000, seed=3), lbs=(32, 128))
+
+
+def test_backprop_small(ctx, cadv):
+    full_check(ctx, cadv, tg.generate("backprop", **{"in": 4096}), lbs=(32, 128))
+
+
+def test_polybench_md_printed_gpu(ctx, cadv):
+    """The paper's printed BICG/Syrk memory-divergence shares, via the GPU path."""
+    t = tg.generate("bicg", nx=1024, ny=1024)
+    load(ctx, cadv, t)
+    h, _ = ctx.mem_divergence(128, 32, t.nsites)
+    pooled = h.sum(axis=0).astype(float)
+    assert round(100 * pooled[1] / pooled.sum()) == 75 and round(100 * pooled[32] / pooled.sum()) == 25
+    check_md(ctx, t, 32)
+    t = tg.generate("syrk", ni=8, nj=32, m=1024)
+    load(ctx, cadv, t)
+    h, _ = ctx.mem_divergence(128, 32, t.nsites)
+    pooled = h.sum(axis=0).astype(float)
+    assert round(100 * pooled[1] / pooled.sum(), 2) == 50.02
+
+
+# ----------------------------------------------------------------- full-size configs
+
+@pytest.mark.slow
+def test_c2_sgemm_full(ctx, cadv):
+    """Config 2 at full size (35,782,656 records), both line sizes, bit-exact."""
+    t = tg.generate("sgemm", n=256)
+    assert t.n == 35782656
+    full_check(ctx, cadv, t, lbs=(32, 128), scopes=(0,))

@@ -31,7 +31,7 @@ def _load():
         return _lib
     src = os.path.join(_HERE, "tracegen.cpp")
     if not os.path.exists(_SO) or os.path.getmtime(_SO) < os.path.getmtime(src):
-        subprocess.check_call(["g++", "-O2", "-std=c++17", "-fopenmp", "-shared", "-fPIC",
+        subprocess.check_call(["/usr/bin/g++" if os.path.exists("/usr/bin/g++") else "g++", "-O2", "-std=c++17", "-fopenmp", "-shared", "-fPIC",
                                "-o", _SO, src])
     lib = ctypes.CDLL(_SO)
     P, u64, u32 = ctypes.c_void_p, ctypes.c_uint64, ctypes.c_uint32
