@@ -1,0 +1,368 @@
+#!/usr/bin/env python
+"""bench.py — throughput of the CUDAAdvisor trace-analysis hot path on B200.
+
+One step = the whole hot path over
+one synthetic trace resident in HBM:
+    cadv_load_trace (R0 ingest) + cadv_reuse_histogram (128 B lines, CTA
+    scope) + cadv_mem_divergence (128 B, warp 32) + cadv_branch_divergence.
+Metric (BASELINE.json): trace records analysed per second (reuse +
+divergence), whole job, plus the dominant kernel's HBM roofline fraction.
+
+Workload (N=1): config 4, Rodinia-shaped SRAD 2048x2048, 6 iterations, with
+its basic-block trace (tracegen "srad"); 478,150,656 memory records.
+N>1 (torchrun, one rank per GPU): weak scaling, every rank analyses its own
+SRAD trace of the same size (seed = 42 + rank); histograms are summed over
+ranks with one NCCL all-reduce per step (ranks share no other data: CTA
+scope and divergence never cross kernel instances).
+
+--impl reference: the CPU oracle (oracle/) as it stands, on this host's
+cores, on a bounded sample of the same workload.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+WORKLOADS = {
+    "c4_srad": ("srad", dict(rows=2048, cols=2048, iters=6, bb=1)),
+    "c2_sgemm": ("sgemm", dict(n=256, bb=1)),
+    "c3_bfs": ("bfs", dict(nodes=1000000, seed=42)),
+    "c4_backprop": ("backprop", {"in": 4194304}),
+}
+METRIC = "trace records analysed/sec (reuse+divergence)"
+UNIT = "records/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="cadv", choices=["cadv", "reference"])
+    ap.add_argument("--workload", default="c4_srad", choices=sorted(WORKLOADS))
+    ap.add_argument("--line-bytes", type=int, default=128)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--profile-run", action="store_true", help="short run for ncu (no clocks / baselines)")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------- helpers
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device):
+        self.device = device
+        self.p = None
+
+    def start(self):
+        try:
+            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                       "-lms", "200", "-i", str(self.device)], stdout=subprocess.PIPE,
+                                      stderr=subprocess.DEVNULL, text=True)
+        except Exception:
+            self.p = None
+
+    def stop(self):
+        if not self.p:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.p.terminate()
+        out, _ = self.p.communicate(timeout=10)
+        sm, mx, reasons = [], [], set()
+        names = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
+        for line in out.strip().splitlines():
+            f = [x.strip() for x in line.split(",")]
+            if len(f) < 9:
+                continue
+            try:
+                sm.append(float(f[1]))
+                mx.append(float(f[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[5:9]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        under = [s for s in sm if s > 300] or sm
+        return {"sm_mhz": statistics.median(under) if under else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def make_trace(workload, rank, pinned):
+    import tracegen as tg
+    name, params = WORKLOADS[workload]
+    params = dict(params)
+    if rank and "seed" in params:
+        params["seed"] = params["seed"] + rank
+    elif rank:
+        params["seed"] = 42 + rank
+    alloc = None
+    if pinned:
+        import torch
+        tmap = {np.uint64: torch.uint64, np.uint32: torch.uint32, np.uint16: torch.uint16, np.uint8: torch.uint8}
+
+        def alloc(n, dt):
+            return torch.empty(n, dtype=tmap[dt], pin_memory=True).numpy()
+    t0 = time.time()
+    t = tg.generate(name, alloc=alloc, **params)
+    log(f"[bench] rank {rank}: generated {workload} ({name} {params}): {t.n:,} records in {time.time() - t0:.1f}s")
+    return t
+
+
+# Algorithmic bytes per launch of each kernel.
+def algorithmic_bytes(kname, st):
+    n, kept, mgroups, bgroups = st["n"], st["kept"], st["md_groups"], st["bd_groups"]
+    table = {
+        "k_ingest": 5 * n,                          # cta 4 + meta 1
+        "k_rd_compact": 13 * n + 12 * kept,         # read addr 8 + cta 4 + meta 1; write key 4 + value 8 per kept
+        "k_divergence<0>": 19 * n + 4 * mgroups,    # addr 8 + cta 4 + tid 2 + winst 4 + meta 1; site per group
+        "k_cta_maxtid": 7 * n,                      # cta 4 + tid 2 + meta 1
+        "k_divergence<1>": 11 * n + 4 * bgroups,    # cta 4 + tid 2 + winst 4 + meta 1; site per group
+        "k_rd_tile": 12 * kept,                     # key 4 + value 8 per kept record
+    }
+    return table.get(kname)
+
+
+# ----------------------------------------------------------------- CPU oracle (baseline / reference arm)
+
+def oracle_sample(t, target_s, line_bytes):
+    """Times the oracle (reuse + MD + BD, as it stands) on a growing prefix of
+    the trace until one sample takes >= target_s/3; returns the last sample's
+    (records, seconds, cores, description)."""
+    import oracle as orc
+    import tracegen as tg
+    n = min(t.n, 200_000)
+    while True:
+        sub = tg.from_arrays(*(t.cols[k][:n] for k, _ in tg.COLUMNS), nsites=t.nsites)
+        t0 = time.time()
+        orc.reuse(sub, line_bytes, 0, 0, 66)
+        orc.mem_div(sub, line_bytes, 32)
+        orc.branch_div(sub, 32)
+        dt = time.time() - t0
+        if dt >= target_s / 3 or n >= t.n:
+            return n, dt, orc.num_threads(), f"first {n:,} records of the trace (reuse + MD + BD)"
+        n = min(t.n, int(n * max(2.0, min(8.0, (target_s / 3) / max(dt, 1e-3)))))
+
+
+# ----------------------------------------------------------------- main
+
+def main():
+    args = parse()
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        return run_reference(args, rank, world)
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_cgo_shensll18_b200 as cadv
+    torch.cuda.set_device(local)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    t = make_trace(args.workload, rank, pinned=True)
+    n = t.n
+    nsites = t.nsites
+    dev = {k: torch.from_numpy(t.cols[k]).to(f"cuda:{local}", non_blocking=True) for k in cadv.COLUMNS}
+    torch.cuda.synchronize()
+    stream = torch.cuda.current_stream()
+    ctx = cadv.create(local, stream.cuda_stream)
+    lb = args.line_bytes
+    NB = 66
+
+    def step(cols, allreduce=True):
+        launches = 0
+        ktimes = []
+        ctx.load_trace(cols)
+        launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+        h, st = ctx.reuse_histogram(lb, cadv.SCOPE_CTA, cadv.BINS_LINEAR, NB)
+        launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+        kept = ctx.last_count(0)
+        hm, _ = ctx.mem_divergence(lb, 32, nsites)
+        launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+        _, tot = ctx.branch_divergence(32, nsites)
+        launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+        if world > 1 and allreduce:
+            r = torch.from_numpy(np.concatenate([h, hm.ravel(), tot]).astype(np.int64)).cuda()
+            dist.all_reduce(r)
+            launches += 1
+        return launches, ktimes, dict(n=n, kept=kept, md_groups=int(hm.sum()), bd_groups=int(tot[0]))
+
+    # ---- warm-up (allocates the library workspace)
+    for _ in range(max(args.warmup, 0)):
+        step(dev)
+    # ---- timed region
+    ctx.set_profiling(True)
+    clocks = Clocks(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    if not args.profile_run:
+        clocks.start()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    launches, kt, stats = 0, [], None
+    for _ in range(args.steps):
+        L, k, stats = step(dev)
+        launches += L
+        kt += k
+    e1.record(stream)
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    ck = clocks.stop() if not args.profile_run else {}
+    ctx.set_profiling(False)
+    ms = e0.elapsed_time(e1)
+    ms_max = ms
+    total_records = n
+    if world > 1:
+        v = torch.tensor([ms, float(n)], dtype=torch.float64, device="cuda")
+        mx = v.clone()
+        dist.all_reduce(mx, op=dist.ReduceOp.MAX)
+        sm = v.clone()
+        dist.all_reduce(sm, op=dist.ReduceOp.SUM)
+        ms_max = float(mx[0])
+        total_records = int(sm[1])
+    ms_step = ms_max / max(args.steps, 1)
+    value = total_records * args.steps / (ms_max / 1e3)
+
+    # ---- dominant kernel roofline (live CUDA-event durations of the timed region)
+    agg = {}
+    for name, t_ms in kt:
+        a = agg.setdefault(name, [0.0, 0])
+        a[0] += t_ms
+        a[1] += 1
+    dom = max(agg.items(), key=lambda kv: kv[1][0])[0] if agg else None
+    peak, peak_src = peaks()
+    roof = None
+    if dom:
+        tot_ms, cnt = agg[dom]
+        per = algorithmic_bytes(dom, stats)
+        avg_ms = tot_ms / cnt
+        if per is not None:
+            gbs = per / (avg_ms / 1e3) / 1e9
+            roof = {"bound": "hbm", "kernel": dom, "achieved": round(gbs, 1), "peak": peak, "unit": "GB/s",
+                    "frac": round(gbs / peak, 4), "traffic": None, "peak_source": peak_src,
+                    "avg_launch_ms": round(avg_ms, 4), "algorithmic_bytes_per_launch": per,
+                    "share_of_step": round(tot_ms / (ms * 1.0), 4)}
+    kernels = {k: {"launches": v[1], "total_ms": round(v[0], 3)} for k, v in sorted(agg.items(), key=lambda kv: -kv[1][0])}
+
+    # ---- e2e: the same step through the C ABI with HOST buffers (H2D inside the timed region)
+    e2e = None
+    if args.e2e_steps > 0 and not args.profile_run:
+        host = {k: t.cols[k] for k in cadv.COLUMNS}
+        step(host, allreduce=False)  # warm the host-copy workspace
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+        f0, f1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        f0.record(stream)
+        for _ in range(args.e2e_steps):
+            step(host)
+        f1.record(stream)
+        torch.cuda.synchronize()
+        ems = f0.elapsed_time(f1)
+        if world > 1:
+            v = torch.tensor([ems], dtype=torch.float64, device="cuda")
+            dist.all_reduce(v, op=dist.ReduceOp.MAX)
+            ems = float(v[0])
+        h2d = int(sum(t.cols[k].nbytes for k in cadv.COLUMNS))
+        d2h = 8 * (NB + 4) + 8 * 2 * 33 + 8 * 2 * nsites + 8 * 3 + 8 * 3 * nsites
+        e2e = {"value": round(total_records * args.e2e_steps / (ems / 1e3), 1), "unit": UNIT,
+               "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h}
+
+    # ---- CPU oracle baseline (rank 0, N = 1 only)
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile_run:
+        rec, dt, cores, desc = oracle_sample(t, args.cpu_seconds, lb)
+        cpu = {"value": round(rec / dt, 1), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc,
+               "seconds": round(dt, 2)}
+
+    if rank == 0:
+        name, params = WORKLOADS[args.workload]
+        line = {
+            "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": round(ms_step, 3), "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "config": {"workload": args.workload, "generator": name, "params": params,
+                       "records_per_gpu": n, "mem_records_per_gpu": int(((t.meta & 3) < 2).sum()),
+                       "line_bytes": lb, "warp_size": 32, "rd_scope": "cta", "rd_bins": "linear 66",
+                       "analyses": "load_trace+reuse+mem_div+branch_div",
+                       "l2": "inputs larger than L2 (trace >> 126 MB), no flush needed",
+                       "parallelism": f"dp{world} (independent trace per GPU, histograms all-reduced)"},
+            "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
+            "clocks": ck, "kernels": kernels,
+        }
+        print(json.dumps(line), flush=True)
+    ctx.destroy()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def run_reference(args, rank, world):
+    """The oracle as it stands, on this host's cores, one bounded sample per step."""
+    if rank != 0:
+        return
+    import oracle as orc
+    import tracegen as tg
+    name, params = WORKLOADS[args.workload]
+    lb = args.line_bytes
+    # a bounded sample: the first launch's worth of records, capped
+    t = make_trace(args.workload, 0, pinned=False)
+    nsamp, dt_probe, cores, desc = oracle_sample(t, max(args.cpu_seconds / 2, 2.0), lb)
+    sub = tg.from_arrays(*(t.cols[k][:nsamp] for k, _ in tg.COLUMNS), nsites=t.nsites)
+
+    def step():
+        orc.reuse(sub, lb, 0, 0, 66)
+        orc.mem_div(sub, lb, 32)
+        orc.branch_div(sub, 32)
+
+    for _ in range(args.warmup):
+        step()
+    t0 = time.time()
+    for _ in range(args.steps):
+        step()
+    dt = time.time() - t0
+    value = nsamp * args.steps / dt
+    line = {
+        "impl": "reference", "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(1e3 * dt / max(args.steps, 1), 3),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+        "config": {"workload": args.workload, "generator": name, "params": params, "line_bytes": lb,
+                   "sample_records": nsamp},
+        "cpu_baseline": {"value": round(value, 1), "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": desc},
+        "e2e": {"value": round(value, 1), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+if __name__ == "__main__":
+    main()

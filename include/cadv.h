@@ -169,6 +169,21 @@ CADV_API float cadv_last_elapsed_ms(const cadv_ctx *ctx);
 /* Number of kernels the last call launched (for bench.py's gpu_launches). */
 CADV_API uint32_t cadv_last_launches(const cadv_ctx *ctx);
 
+/* Per-kernel timing of the calls that follow (enable != 0): CUDA events are
+ * recorded on the context's stream around every kernel launch.  Off by
+ * default (it adds two event records per launch). */
+CADV_API cadv_status cadv_set_profiling(cadv_ctx *ctx, int enable);
+
+/* Kernel names and device times (ms) of the last call's launches, in launch
+ * order, when profiling was enabled.  Returns the number of launches and
+ * fills at most `max` entries; names stay valid until the next call. */
+CADV_API uint32_t cadv_last_kernel_times(const cadv_ctx *ctx, const char **names, float *ms, uint32_t max);
+
+/* Work counters of the last cadv_reuse_histogram call (for roofline
+ * accounting): which = 0 kept records after run compression, 1 cross-tile
+ * entries, 2 cross-tile queries, 3 tiles.  0 for unknown `which`. */
+CADV_API uint64_t cadv_last_count(const cadv_ctx *ctx, int which);
+
 /* Library version string. */
 CADV_API const char *cadv_version(void);
 

@@ -80,6 +80,12 @@ def lib():
     L.cadv_last_elapsed_ms.restype = ctypes.c_float
     L.cadv_last_launches.argtypes = [P]
     L.cadv_last_launches.restype = u32
+    L.cadv_set_profiling.argtypes = [P, i32]
+    L.cadv_set_profiling.restype = i32
+    L.cadv_last_kernel_times.argtypes = [P, P, P, u32]
+    L.cadv_last_kernel_times.restype = u32
+    L.cadv_last_count.argtypes = [P, i32]
+    L.cadv_last_count.restype = u64
     L.cadv_version.restype = ctypes.c_char_p
     _lib = L
     return L
@@ -130,6 +136,23 @@ class Context:
 
     def last_launches(self) -> int:
         return int(lib().cadv_last_launches(self._h))
+
+    def set_profiling(self, enable: bool):
+        """cadv_set_profiling: CUDA events around every kernel launch."""
+        self._check(lib().cadv_set_profiling(self._h, 1 if enable else 0))
+
+    def last_kernel_times(self):
+        """cadv_last_kernel_times: [(kernel name, device ms)] of the last call."""
+        L = lib()
+        k = L.cadv_last_kernel_times(self._h, None, None, 0)
+        names = (ctypes.c_char_p * max(k, 1))()
+        ms = (ctypes.c_float * max(k, 1))()
+        k = L.cadv_last_kernel_times(self._h, ctypes.cast(names, ctypes.c_void_p), ctypes.cast(ms, ctypes.c_void_p), k)
+        return [(names[i].decode(), float(ms[i])) for i in range(k)]
+
+    def last_count(self, which: int) -> int:
+        """cadv_last_count: 0 kept records, 1 cross-tile entries, 2 cross-tile queries, 3 tiles."""
+        return int(lib().cadv_last_count(self._h, which))
 
     # -- cadv_load_trace
     def load_trace(self, cols, n=None, warp_contiguous=True, global_offset=0):

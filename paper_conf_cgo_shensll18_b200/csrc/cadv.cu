@@ -51,6 +51,40 @@ cudaError_t ensure_host(cadv_ctx* c, size_t bytes, void** out) {
 
 Scalars* scalars(cadv_ctx* c) { return (Scalars*)c->buf[B_SCALARS].p; }
 
+void prof_begin(cadv_ctx* c, const char* src) {
+  if (!c->profiling) return;
+  uint32_t k = c->nprof;
+  while (c->prof_ev.size() < 2ull * (k + 1)) {
+    cudaEvent_t e;
+    if (cudaEventCreate(&e) != cudaSuccess) { c->profiling = false; return; }
+    c->prof_ev.push_back(e);
+  }
+  if (c->prof_src.size() <= k) c->prof_src.resize(k + 1);
+  c->prof_src[k] = src;
+  cudaEventRecord(c->prof_ev[2 * k], c->stream);
+}
+
+void prof_end(cadv_ctx* c) {
+  if (!c->profiling || c->prof_ev.size() < 2ull * (c->nprof + 1)) return;
+  cudaEventRecord(c->prof_ev[2 * c->nprof + 1], c->stream);
+  c->nprof++;
+}
+
+// after the stream is synchronised: per-launch times and kernel names
+static void prof_collect(cadv_ctx* c) {
+  c->prof_ms.assign(c->nprof, 0.f);
+  c->prof_name.assign(c->nprof, std::string());
+  for (uint32_t k = 0; k < c->nprof; ++k) {
+    cudaEventElapsedTime(&c->prof_ms[k], c->prof_ev[2 * k], c->prof_ev[2 * k + 1]);
+    std::string src = c->prof_src[k] ? c->prof_src[k] : "";
+    size_t a = src.find("<<<");
+    std::string nm = src.substr(0, a);
+    size_t sp = nm.find_last_of(" (,");
+    if (sp != std::string::npos) nm = nm.substr(sp + 1);
+    c->prof_name[k] = nm;
+  }
+}
+
 // ------------------------------------------------------------------ R0 ingest
 // One streaming pass over (cta, meta): max CTA id and record count per kind.
 __global__ void __launch_bounds__(256) k_ingest(const uint32_t* __restrict__ cta, const uint8_t* __restrict__ meta,
@@ -118,6 +152,8 @@ cadv_status begin_call(cadv_ctx* c) {
   CK(cudaMemsetAsync(p, 0, sizeof(Scalars), c->stream), "memset");
   CK(cudaMemsetAsync(&((Scalars*)p)->err_index, 0xff, sizeof(unsigned long long), c->stream), "memset");
   c->launches = 0;
+  c->nprof = 0;
+  for (auto& v : c->counts) v = 0;
   CK(cudaEventRecord(c->ev0, c->stream), "event");
   return CADV_OK;
 }
@@ -136,6 +172,7 @@ cadv_status end_call(cadv_ctx* c, const void* d_out, size_t nout, void** h_out) 
   float ms = 0.f;
   CK(cudaEventElapsedTime(&ms, c->ev0, c->ev1), "event");
   c->elapsed_ms = ms;
+  prof_collect(c);
   if (hs->err_code) {
     char b[200];
     snprintf(b, sizeof b, "%s at trace position %llu",
@@ -198,6 +235,7 @@ CADV_API cadv_status cadv_destroy(cadv_ctx* c) {
   if (c->host_pinned) cudaFreeHost(c->host_pinned);
   if (c->ev0) cudaEventDestroy(c->ev0);
   if (c->ev1) cudaEventDestroy(c->ev1);
+  for (auto e : c->prof_ev) cudaEventDestroy(e);
   delete c;
   return CADV_OK;
 }
@@ -205,6 +243,26 @@ CADV_API cadv_status cadv_destroy(cadv_ctx* c) {
 CADV_API const char* cadv_last_error(const cadv_ctx* c) { return c ? c->err.c_str() : "null context"; }
 CADV_API float cadv_last_elapsed_ms(const cadv_ctx* c) { return c ? c->elapsed_ms : 0.f; }
 CADV_API uint32_t cadv_last_launches(const cadv_ctx* c) { return c ? c->launches : 0; }
+
+CADV_API uint64_t cadv_last_count(const cadv_ctx* c, int which) {
+  return (c && which >= 0 && which < 4) ? c->counts[which] : 0;
+}
+
+CADV_API cadv_status cadv_set_profiling(cadv_ctx* c, int enable) {
+  if (!c) return CADV_ERR_INVALID_ARG;
+  c->profiling = enable != 0;
+  return CADV_OK;
+}
+
+CADV_API uint32_t cadv_last_kernel_times(const cadv_ctx* c, const char** names, float* ms, uint32_t max) {
+  if (!c) return 0;
+  uint32_t k = (uint32_t)c->prof_ms.size();
+  for (uint32_t i = 0; i < k && i < max; ++i) {
+    if (names) names[i] = c->prof_name[i].c_str();
+    if (ms) ms[i] = c->prof_ms[i];
+  }
+  return k;
+}
 
 CADV_API cadv_status cadv_load_trace(cadv_ctx* c, const cadv_trace_desc* d, uint64_t global_offset) {
   if (!c || !d) return CADV_ERR_INVALID_ARG;
@@ -262,8 +320,8 @@ CADV_API cadv_status cadv_mem_divergence(cadv_ctx* c, uint32_t line_bytes, uint3
   if (s != CADV_OK) return s;
   size_t hbytes = 2ull * (warp_size + 1) * 8, sbytes = per_site ? 2ull * nsites * 8 : 0;
   void* d_out;
-  CK(ensure(c, B_HIST, hbytes + sbytes, &d_out), "workspace");
-  CK(cudaMemsetAsync(d_out, 0, hbytes + sbytes, c->stream), "memset");
+  CK(ensure(c, B_HIST, hbytes + sbytes + 8, &d_out), "workspace");
+  CK(cudaMemsetAsync(d_out, 0, hbytes + sbytes + 8, c->stream), "memset");
   cadv_trace_desc t = c->t;
   if (!t.warp_contiguous && t.n) CK(regroup_by_warp(c, &t), "regroup by warp");
   CK(launch_mem_div(c, t, ilog2(line_bytes), ilog2(warp_size), (uint64_t*)d_out,

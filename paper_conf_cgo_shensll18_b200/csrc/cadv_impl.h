@@ -60,6 +60,14 @@ struct cadv_ctx {
   cadv::DevBuf buf[cadv::B_COUNT];
   void* host_pinned = nullptr;
   size_t host_pinned_bytes = 0;
+  // per-kernel profiling (cadv_set_profiling)
+  bool profiling = false;
+  std::vector<cudaEvent_t> prof_ev;   // 2 per launch
+  std::vector<const char*> prof_src;  // stringified launch expression
+  std::vector<std::string> prof_name;
+  std::vector<float> prof_ms;
+  uint32_t nprof = 0;
+  uint64_t counts[4] = {0, 0, 0, 0};  // cadv_last_count
 };
 
 namespace cadv {
@@ -98,8 +106,15 @@ cudaError_t exclusive_scan_u64(cadv_ctx* c, const uint64_t* in, uint64_t* out, u
 
 }  // namespace cadv
 
-#define CADV_LAUNCH(c, ...)   \
-  do {                        \
-    __VA_ARGS__;              \
-    (c)->launches++;          \
+namespace cadv {
+void prof_begin(cadv_ctx* c, const char* src);
+void prof_end(cadv_ctx* c);
+}  // namespace cadv
+
+#define CADV_LAUNCH(c, ...)                 \
+  do {                                      \
+    cadv::prof_begin((c), #__VA_ARGS__);    \
+    __VA_ARGS__;                            \
+    cadv::prof_end((c));                    \
+    (c)->launches++;                        \
   } while (0)

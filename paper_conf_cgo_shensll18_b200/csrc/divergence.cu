@@ -397,7 +397,12 @@ cudaError_t launch_div(cadv_ctx* c, const cadv_trace_desc& d, uint32_t lbs, uint
   uint64_t cap = (uint64_t)g_dv_blocks[MODE] * c->num_sms;
   int grid = (int)(ntiles < cap ? ntiles : cap);
   TraceCols t{d.addr, d.cta, d.tid, d.site, d.winst, d.meta, d.n};
-  CADV_LAUNCH(c, kern<<<grid, DV_NT, smem, c->stream>>>(t, lbs, ws, hist, sites, nsites, flag, tc, scalars(c), ntiles));
+  if (MODE == 0)
+    CADV_LAUNCH(c, k_divergence<0><<<grid, DV_NT, smem, c->stream>>>(t, lbs, ws, hist, sites, nsites, flag, tc,
+                                                                      scalars(c), ntiles));
+  else
+    CADV_LAUNCH(c, k_divergence<1><<<grid, DV_NT, smem, c->stream>>>(t, lbs, ws, hist, sites, nsites, flag, tc,
+                                                                      scalars(c), ntiles));
   return cudaGetLastError();
 }
 

@@ -778,6 +778,7 @@ cudaError_t run_reuse(cadv_ctx* c, uint32_t lbs, int scope, int log2bins, uint32
   if ((e = cudaMemcpyAsync(&last, (uint64_t*)st + (ctiles - 1), 8, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
   const uint64_t K = last & LB_VAL;
+  c->counts[0] = K;
   if (K == 0) return cudaSuccess;
   // ---- R1b regroup by CTA (stable)
   const uint32_t* key = nullptr;
@@ -794,6 +795,7 @@ cudaError_t run_reuse(cadv_ctx* c, uint32_t lbs, int scope, int log2bins, uint32
   }
   // ---- tiles
   uint64_t ntiles = (K + TL_NOM - 1) / TL_NOM;
+  c->counts[3] = ntiles;
   void *bnd, *tw, *tq;
   if ((e = ensure(c, B_RD_XTMP, (ntiles + 2) * 4 + 64, &bnd))) return e;
   if ((e = ensure(c, B_RD_TILEW, (ntiles + 2) * 8 * 2, &tw))) return e;
@@ -834,6 +836,7 @@ cudaError_t run_reuse(cadv_ctx* c, uint32_t lbs, int scope, int log2bins, uint32
   unsigned long long nent;
   if ((e = cudaMemcpyAsync(&nent, &sc->count[1], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
+  c->counts[1] = nent;
   if (nent == 0) return cudaSuccess;
   // ---- cross-tile phase
   // tile prefix sums of weights and local query counts (u64)
@@ -906,6 +909,7 @@ cudaError_t run_reuse(cadv_ctx* c, uint32_t lbs, int scope, int log2bins, uint32
   unsigned long long M;
   if ((e = cudaMemcpyAsync(&M, &sc->count[2], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
+  c->counts[2] = M;
   if (M == 0) return cudaSuccess;
   // sort cross queries by position, then count inversions of their previous uses
   if ((e = ensure(c, B_RD_ENT_KEY1, M * 8 + nent * 8, &ek1))) return e;

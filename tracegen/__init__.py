@@ -43,6 +43,8 @@ def _load():
         getattr(lib, fn).argtypes = [P]
     lib.tg_fill_range.restype = ctypes.c_int
     lib.tg_fill_range.argtypes = [P, u64, u64] + [P] * 6
+    lib.tg_launch_offsets.restype = None
+    lib.tg_launch_offsets.argtypes = [P, P]
     lib.tg_free.restype = None
     lib.tg_free.argtypes = [P]
     _lib = lib
@@ -86,6 +88,32 @@ def plan(workload: str, **params):
         raise ValueError(err.value.decode())
     return (h, int(lib.tg_num_records(h)), int(lib.tg_num_sites(h)), int(lib.tg_num_ctas(h)),
             int(lib.tg_num_launches(h)), lib.tg_info(h).decode())
+
+
+def launch_offsets(workload: str, **params) -> np.ndarray:
+    """Start position of every kernel launch in the trace, plus the total."""
+    lib = _load()
+    h, n_total, nsites, nctas, nl, info = plan(workload, **params)
+    try:
+        out = np.zeros(nl + 1, np.uint64)
+        lib.tg_launch_offsets(h, out.ctypes.data)
+        return out
+    finally:
+        lib.tg_free(h)
+
+
+def shard_bounds(workload: str, rank: int, world: int, **params):
+    """[lo, hi) of this rank's shard: launch-aligned position ranges of about
+    equal size (no CTA spans two shards: CTAs never span launches)."""
+    off = launch_offsets(workload, **params).astype(np.int64)
+    n = int(off[-1])
+    cut = [0]
+    for r in range(1, world):
+        target = r * n // world
+        k = int(np.argmin(np.abs(off - target)))
+        cut.append(max(cut[-1], int(off[k])))
+    cut.append(n)
+    return cut[rank], cut[rank + 1]
 
 
 def generate(workload: str, lo: int | None = None, hi: int | None = None, alloc=None, **params) -> Trace:

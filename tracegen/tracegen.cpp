@@ -867,6 +867,13 @@ uint32_t tg_num_ctas(const tg_trace* t) { return reinterpret_cast<const Trace*>(
 uint32_t tg_num_launches(const tg_trace* t) { return (uint32_t)reinterpret_cast<const Trace*>(t)->launches.size(); }
 const char* tg_info(const tg_trace* t) { return reinterpret_cast<const Trace*>(t)->info.c_str(); }
 
+// First record position of every launch, plus the total (nlaunches + 1 values).
+void tg_launch_offsets(const tg_trace* t, uint64_t* out) {
+  const Trace* T = reinterpret_cast<const Trace*>(t);
+  for (size_t k = 0; k < T->launches.size(); ++k) out[k] = T->launches[k].offset;
+  out[T->launches.size()] = T->n;
+}
+
 // Writes records [lo, hi) of the trace into the caller's arrays (indexed from 0).
 int tg_fill_range(tg_trace* t, uint64_t lo, uint64_t hi, uint64_t* addr, uint32_t* cta, uint16_t* tid,
                   uint32_t* site, uint32_t* winst, uint8_t* meta) {
