@@ -55,6 +55,8 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-run", action="store_true", help="short run for ncu (no clocks / baselines)")
+    ap.add_argument("--separate", action="store_true",
+                    help="one library call per analysis (three passes) instead of the fused cadv_analyze")
     return ap.parse_args()
 
 
@@ -140,6 +142,10 @@ def make_trace(workload, rank, pinned):
 def algorithmic_bytes(kname, st):
     n, kept, mgroups, bgroups = st["n"], st["kept"], st["md_groups"], st["bd_groups"]
     table = {
+        "k_scan<7>": 23 * n + 12 * kept,            # every column once + kept records written (fused pass)
+        "k_scan<1>": 13 * n + 12 * kept,            # addr, cta, meta + kept records
+        "k_scan<2>": 23 * n,                        # addr, cta, tid, winst, site, meta
+        "k_scan<4>": 15 * n,                        # cta, tid, winst, site, meta
         "k_ingest": 5 * n,                          # cta 4 + meta 1
         "k_rd_compact": 13 * n + 12 * kept,         # read addr 8 + cta 4 + meta 1; write key 4 + value 8 per kept
         "k_divergence<0>": 19 * n + 4 * mgroups,    # addr 8 + cta 4 + tid 2 + winst 4 + meta 1; site per group
@@ -202,13 +208,21 @@ def main():
         ktimes = []
         ctx.load_trace(cols)
         launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
-        h, st = ctx.reuse_histogram(lb, cadv.SCOPE_CTA, cadv.BINS_LINEAR, NB)
-        launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
-        kept = ctx.last_count(0)
-        hm, _ = ctx.mem_divergence(lb, 32, nsites)
-        launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
-        _, tot = ctx.branch_divergence(32, nsites)
-        launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+        if args.separate:
+            h, st = ctx.reuse_histogram(lb, cadv.SCOPE_CTA, cadv.BINS_LINEAR, NB)
+            launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+            kept = ctx.last_count(0)
+            hm, _ = ctx.mem_divergence(lb, 32, nsites)
+            launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+            _, tot = ctx.branch_divergence(32, nsites)
+            launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+        else:
+            out = ctx.analyze(rd=(lb, cadv.SCOPE_CTA, cadv.BINS_LINEAR, NB), md=(lb, 32), bd=32, nsites=nsites)
+            launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
+            kept = ctx.last_count(0)
+            h, st = out["reuse"]
+            hm, _ = out["mem_div"]
+            _, tot = out["branch_div"]
         if world > 1 and allreduce:
             r = torch.from_numpy(np.concatenate([h, hm.ravel(), tot]).astype(np.int64)).cuda()
             dist.all_reduce(r)
@@ -314,7 +328,8 @@ def main():
             "config": {"workload": args.workload, "generator": name, "params": params,
                        "records_per_gpu": n, "mem_records_per_gpu": int(((t.meta & 3) < 2).sum()),
                        "line_bytes": lb, "warp_size": 32, "rd_scope": "cta", "rd_bins": "linear 66",
-                       "analyses": "load_trace+reuse+mem_div+branch_div",
+                       "analyses": ("load_trace + reuse + mem_div + branch_div (three calls)" if args.separate else
+                                    "load_trace + cadv_analyze(reuse, mem_div, branch_div: one fused pass)"),
                        "l2": "inputs larger than L2 (trace >> 126 MB), no flush needed",
                        "parallelism": f"dp{world} (independent trace per GPU, histograms all-reduced)"},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,

@@ -156,6 +156,23 @@ CADV_API cadv_status cadv_mem_divergence(cadv_ctx *ctx, uint32_t line_bytes, uin
 CADV_API cadv_status cadv_branch_divergence(cadv_ctx *ctx, uint32_t warp_size, cadv_site_branch *per_site,
                                             uint32_t nsites, uint64_t totals[3]);
 
+/* Parameters of cadv_analyze (one fused pass for several analyses). */
+typedef struct {
+  uint32_t rd_line_bytes; int rd_scope; int rd_binning; uint32_t rd_nbins;  /* as cadv_reuse_histogram */
+  uint32_t md_line_bytes; uint32_t md_warp_size;                            /* as cadv_mem_divergence */
+  uint32_t bd_warp_size;                                                    /* as cadv_branch_divergence */
+  uint32_t nsites;                                                          /* for md_sites / bd_sites */
+} cadv_analysis;
+
+/* Runs every analysis whose output pointer is non-NULL (rd_hist: reuse;
+ * md_hist: memory divergence; bd_totals: branch divergence) with ONE
+ * streaming pass over the trace (the passes above share it), and writes the
+ * same outputs as the individual calls with the same parameters would.
+ * rd_stats, md_sites, bd_sites are optional as in the individual calls. */
+CADV_API cadv_status cadv_analyze(cadv_ctx *ctx, const cadv_analysis *a, uint64_t *rd_hist,
+                                  cadv_reuse_stats *rd_stats, uint64_t *md_hist, cadv_site_mem *md_sites,
+                                  uint64_t *bd_totals, cadv_site_branch *bd_sites);
+
 /* Releases the context and all its device workspace. */
 CADV_API cadv_status cadv_destroy(cadv_ctx *ctx);
 

@@ -48,6 +48,12 @@ class TraceDesc(ctypes.Structure):
                 ("n", ctypes.c_uint64), ("on_device", ctypes.c_int), ("warp_contiguous", ctypes.c_int)]
 
 
+class Analysis(ctypes.Structure):
+    _fields_ = [("rd_line_bytes", ctypes.c_uint32), ("rd_scope", ctypes.c_int), ("rd_binning", ctypes.c_int),
+                ("rd_nbins", ctypes.c_uint32), ("md_line_bytes", ctypes.c_uint32), ("md_warp_size", ctypes.c_uint32),
+                ("bd_warp_size", ctypes.c_uint32), ("nsites", ctypes.c_uint32)]
+
+
 class ReuseStats(ctypes.Structure):
     _fields_ = [("accesses", ctypes.c_uint64), ("inf", ctypes.c_uint64), ("streaming", ctypes.c_uint64),
                 ("overflow", ctypes.c_uint64)]
@@ -70,9 +76,10 @@ def lib():
     L.cadv_reuse_histogram.argtypes = [P, u32, i32, i32, P, u32, ctypes.POINTER(ReuseStats)]
     L.cadv_mem_divergence.argtypes = [P, u32, u32, P, P, u32]
     L.cadv_branch_divergence.argtypes = [P, u32, P, u32, P]
+    L.cadv_analyze.argtypes = [P, ctypes.POINTER(Analysis), P, ctypes.POINTER(ReuseStats), P, P, P, P]
     L.cadv_destroy.argtypes = [P]
     for f in ("cadv_create", "cadv_load_trace", "cadv_reuse_histogram", "cadv_mem_divergence",
-              "cadv_branch_divergence", "cadv_destroy"):
+              "cadv_branch_divergence", "cadv_analyze", "cadv_destroy"):
         getattr(L, f).restype = i32
     L.cadv_last_error.argtypes = [P]
     L.cadv_last_error.restype = ctypes.c_char_p
@@ -195,6 +202,31 @@ class Context:
         self._check(lib().cadv_branch_divergence(self._h, warp_size, ps.ctypes.data if ps is not None else None,
                                                  nsites, tot.ctypes.data))
         return ps, tot
+
+    # -- cadv_analyze (one fused pass)
+    def analyze(self, rd=(128, SCOPE_CTA, BINS_LINEAR, 66), md=(128, 32), bd=32, nsites=0, per_site=True):
+        """Any of rd / md / bd may be None.  Returns dict with the outputs of
+        reuse_histogram / mem_divergence / branch_divergence."""
+        a = Analysis(rd[0] if rd else 1, rd[1] if rd else 0, rd[2] if rd else 0, rd[3] if rd else 3,
+                     md[0] if md else 1, md[1] if md else 32, bd if bd else 32, nsites)
+        out = {}
+        rh = np.zeros(rd[3], np.uint64) if rd else None
+        st = ReuseStats()
+        mh = np.zeros((2, md[1] + 1), np.uint64) if md else None
+        ms = np.zeros((nsites, 2), np.uint64) if (md and per_site and nsites) else None
+        bt = np.zeros(3, np.uint64) if bd else None
+        bs = np.zeros((nsites, 3), np.uint64) if (bd and per_site and nsites) else None
+        p = lambda x: x.ctypes.data if x is not None else None
+        self._check(lib().cadv_analyze(self._h, ctypes.byref(a), p(rh), ctypes.byref(st) if rd else None, p(mh),
+                                       p(ms), p(bt), p(bs)))
+        if rd:
+            out["reuse"] = (rh, {"accesses": st.accesses, "inf": st.inf, "streaming": st.streaming,
+                                 "overflow": st.overflow})
+        if md:
+            out["mem_div"] = (mh, ms)
+        if bd:
+            out["branch_div"] = (bs, bt)
+        return out
 
     # -- cadv_destroy
     def destroy(self):

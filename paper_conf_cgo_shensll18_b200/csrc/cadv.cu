@@ -306,109 +306,220 @@ CADV_API cadv_status cadv_load_trace(cadv_ctx* c, const cadv_trace_desc* d, uint
   return CADV_OK;
 }
 
+}  // extern "C"
+
+namespace {
+
+struct Req {
+  bool rd = false, md = false, bd = false;
+  uint32_t rd_lbs = 7, md_lbs = 7, md_ws = 5, bd_ws = 5;
+  int scope = CADV_SCOPE_CTA, log2bins = 0;
+  uint32_t nbins = 66, nsites = 0;
+  bool md_sites = false, bd_sites = false;
+};
+
+cadv_status check_args(cadv_ctx* c, uint32_t line_bytes, uint32_t warp_size, bool check_line, bool check_warp) {
+  if (check_line && (!pow2(line_bytes) || line_bytes > 4096))
+    return fail(c, CADV_ERR_INVALID_ARG, "line_bytes must be 2^k <= 4096");
+  if (check_warp && (!pow2(warp_size) || warp_size > 32))
+    return fail(c, CADV_ERR_INVALID_ARG, "warp_size must be 2^k <= 32");
+  return CADV_OK;
+}
+
+// Runs the requested analyses with ONE streaming pass over the trace (k_scan)
+// followed by the reuse tail (regroup, tiles, cross-tile) and the deferred
+// branch-divergence resolution.  Device output layout in B_OUT2:
+//   [rd hist nbins][rd stats 4][md hist 2(W+1)][md sites 2 nsites][md flag]
+//   [bd totals 3][bd flag][bd sites 3 nsites]
+cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_stats* rd_stats, uint64_t* md_hist,
+                         cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites) {
+  if (!c->loaded) return fail(c, CADV_ERR_NO_TRACE, "no trace loaded");
+  if (q.bd && c->t.n && c->max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
+  CK(cudaSetDevice(c->device), "cudaSetDevice");
+  cadv_status s = begin_call(c);
+  if (s != CADV_OK) return s;
+  const uint32_t mdW = 1u << q.md_ws;
+  const size_t o_rdh = 0, o_rds = o_rdh + (q.rd ? q.nbins : 0), o_mdh = o_rds + (q.rd ? 4 : 0);
+  const size_t o_mds = o_mdh + (q.md ? 2 * (mdW + 1) : 0);
+  const size_t o_mdf = o_mds + (q.md && q.md_sites ? 2ull * q.nsites : 0);
+  const size_t o_bdt = o_mdf + (q.md ? 1 : 0);
+  const size_t o_bdf = o_bdt + 3;
+  const size_t o_bds = o_bdf + 1;
+  const size_t total = o_bds + (q.bd && q.bd_sites ? 3ull * q.nsites : 0);
+  void* dv;
+  CK(ensure(c, B_OUT2, total * 8 + 64, &dv), "workspace");
+  CK(cudaMemsetAsync(dv, 0, total * 8 + 64, c->stream), "memset");
+  uint64_t* d = (uint64_t*)dv;
+  cadv_trace_desc t = c->t;
+  if ((q.md || q.bd) && !t.warp_contiguous && t.n) CK(regroup_by_warp(c, &t), "regroup by warp");
+  ScanParams P;
+  P.t = t;
+  int flags = 0;
+  RdState rs;
+  if (q.rd && t.n) {
+    CK(rd_begin(c, q.scope, &rs), "reuse workspace");
+    flags |= F_RD;
+    P.lbs_rd = q.rd_lbs;
+    P.cta_scope = q.scope == CADV_SCOPE_CTA;
+    P.kout = rs.cta_scope ? rs.k0 : nullptr;
+    P.vout = rs.v0;
+    P.status = rs.status;
+    P.hist0 = d + o_rdh;
+  }
+  if (q.md) {
+    flags |= F_MD;
+    P.lbs_md = q.md_lbs;
+    P.ws_md = q.md_ws;
+    P.md_hist = d + o_mdh;
+    P.md_sites = q.md_sites ? d + o_mds : nullptr;
+  }
+  void* tc = nullptr;
+  void* defer = nullptr;
+  if (q.bd && t.n) {
+    flags |= F_BD;
+    uint32_t ncta = c->max_cta + 1;
+    CK(ensure(c, B_TC, 4ull * ncta, &tc), "workspace");
+    CK(cudaMemsetAsync(tc, 0, 4ull * ncta, c->stream), "memset");
+    CK(ensure(c, B_DEFER, 16ull * (c->n_kind[2] + 1), &defer), "workspace");
+    P.ws_bd = q.bd_ws;
+    P.tc = (uint32_t*)tc;
+    P.bd_tot = d + o_bdt;
+    P.bd_sites = q.bd_sites ? d + o_bds : nullptr;
+    P.defer = defer;
+    P.ndefer = (unsigned long long*)&scalars(c)->count[5];
+  }
+  P.nsites = (q.md_sites || q.bd_sites) ? q.nsites : 0;
+  // one flag word for both site checks
+  P.site_flag = d + (q.md ? o_mdf : o_bdf);
+  if (flags) CK(launch_scan(c, flags, P), "scan launch");
+  if (q.rd && t.n) CK(rd_finish(c, rs, q.log2bins, q.nbins, d + o_rdh, d + o_rds), "reuse");
+  if (q.bd && t.n) {
+    unsigned long long m = 0;
+    CK(cudaMemcpyAsync(&m, P.ndefer, 8, cudaMemcpyDeviceToHost, c->stream), "D2H");
+    CK(cudaStreamSynchronize(c->stream), "scan");
+    CK(launch_bd_resolve(c, defer, m, (const uint32_t*)tc, q.bd_ws, d + o_bdt, q.bd_sites ? d + o_bds : nullptr,
+                         q.bd_sites ? q.nsites : 0),
+       "bd resolve");
+  }
+  void* h;
+  s = end_call(c, d, total * 8, &h);
+  if (s != CADV_OK) return s;
+  const uint64_t* hr = (const uint64_t*)h;
+  if ((q.md && hr[o_mdf]) || (q.bd && hr[o_bdf]))
+    return fail(c, CADV_ERR_INVALID_ARG, "a record's site id is >= nsites");
+  if (q.rd) {
+    memcpy(rd_hist, hr + o_rdh, q.nbins * 8);
+    if (rd_stats) {
+      uint64_t acc = 0;
+      for (uint32_t b = 0; b < q.nbins; ++b) acc += hr[o_rdh + b];
+      rd_stats->accesses = acc;
+      rd_stats->inf = hr[o_rdh + q.nbins - 1];
+      rd_stats->overflow = hr[o_rdh + q.nbins - 2];
+      rd_stats->streaming = hr[o_rds];
+    }
+  }
+  if (q.md) {
+    memcpy(md_hist, hr + o_mdh, 2ull * (mdW + 1) * 8);
+    if (q.md_sites) memcpy(md_sites, hr + o_mds, 2ull * q.nsites * 8);
+  }
+  if (q.bd) {
+    memcpy(bd_tot, hr + o_bdt, 3 * 8);
+    if (q.bd_sites) memcpy(bd_sites, hr + o_bds, 3ull * q.nsites * 8);
+  }
+  return CADV_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
 CADV_API cadv_status cadv_mem_divergence(cadv_ctx* c, uint32_t line_bytes, uint32_t warp_size, uint64_t* hist,
                                          cadv_site_mem* per_site, uint32_t nsites) {
   if (!c) return CADV_ERR_INVALID_ARG;
   c->err.clear();
-  if (!c->loaded) return fail(c, CADV_ERR_NO_TRACE, "no trace loaded");
-  if (!pow2(line_bytes) || line_bytes > 4096) return fail(c, CADV_ERR_INVALID_ARG, "line_bytes must be 2^k <= 4096");
-  if (!pow2(warp_size) || warp_size > 32) return fail(c, CADV_ERR_INVALID_ARG, "warp_size must be 2^k <= 32");
+  cadv_status s = check_args(c, line_bytes, warp_size, true, true);
+  if (s != CADV_OK) return s;
   if (!hist) return fail(c, CADV_ERR_INVALID_ARG, "hist is NULL");
   if (per_site && nsites == 0) return fail(c, CADV_ERR_INVALID_ARG, "nsites must be > 0 with per_site");
-  CK(cudaSetDevice(c->device), "cudaSetDevice");
-  cadv_status s = begin_call(c);
-  if (s != CADV_OK) return s;
-  size_t hbytes = 2ull * (warp_size + 1) * 8, sbytes = per_site ? 2ull * nsites * 8 : 0;
-  void* d_out;
-  CK(ensure(c, B_HIST, hbytes + sbytes + 8, &d_out), "workspace");
-  CK(cudaMemsetAsync(d_out, 0, hbytes + sbytes + 8, c->stream), "memset");
-  cadv_trace_desc t = c->t;
-  if (!t.warp_contiguous && t.n) CK(regroup_by_warp(c, &t), "regroup by warp");
-  CK(launch_mem_div(c, t, ilog2(line_bytes), ilog2(warp_size), (uint64_t*)d_out,
-                    per_site ? (uint64_t*)d_out + 2 * (warp_size + 1) : nullptr, per_site ? nsites : 0),
-     "mem_div launch");
-  void* h;
-  s = end_call(c, d_out, hbytes + sbytes + 8, &h);
-  if (s != CADV_OK) return s;
-  const uint64_t* hr = (const uint64_t*)h;
-  if (per_site && hr[2 * (warp_size + 1) + 2 * nsites])
-    return fail(c, CADV_ERR_INVALID_ARG, "a memory record's site id is >= nsites");
-  memcpy(hist, hr, hbytes);
-  if (per_site) memcpy(per_site, hr + 2 * (warp_size + 1), sbytes);
-  return CADV_OK;
+  Req q;
+  q.md = true;
+  q.md_lbs = ilog2(line_bytes);
+  q.md_ws = ilog2(warp_size);
+  q.md_sites = per_site != nullptr;
+  q.nsites = per_site ? nsites : 0;
+  return run_analyses(c, q, nullptr, nullptr, hist, per_site, nullptr, nullptr);
 }
 
 CADV_API cadv_status cadv_branch_divergence(cadv_ctx* c, uint32_t warp_size, cadv_site_branch* per_site,
                                             uint32_t nsites, uint64_t totals[3]) {
   if (!c) return CADV_ERR_INVALID_ARG;
   c->err.clear();
-  if (!c->loaded) return fail(c, CADV_ERR_NO_TRACE, "no trace loaded");
-  if (!pow2(warp_size) || warp_size > 32) return fail(c, CADV_ERR_INVALID_ARG, "warp_size must be 2^k <= 32");
+  cadv_status s = check_args(c, 1, warp_size, false, true);
+  if (s != CADV_OK) return s;
   if (!totals) return fail(c, CADV_ERR_INVALID_ARG, "totals is NULL");
   if (per_site && nsites == 0) return fail(c, CADV_ERR_INVALID_ARG, "nsites must be > 0 with per_site");
-  if (c->t.n && c->max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
-  CK(cudaSetDevice(c->device), "cudaSetDevice");
-  cadv_status s = begin_call(c);
-  if (s != CADV_OK) return s;
-  size_t tbytes = 4 * 8, sbytes = per_site ? 3ull * nsites * 8 : 0;
-  void* d_out;
-  CK(ensure(c, B_HIST, tbytes + sbytes, &d_out), "workspace");
-  CK(cudaMemsetAsync(d_out, 0, tbytes + sbytes, c->stream), "memset");
-  uint32_t ncta = c->t.n ? c->max_cta + 1 : 1;
-  void* d_tc;
-  CK(ensure(c, B_TC, 4ull * ncta, &d_tc), "workspace");
-  CK(cudaMemsetAsync(d_tc, 0, 4ull * ncta, c->stream), "memset");
-  cadv_trace_desc t = c->t;
-  if (t.n) {
-    CK(launch_cta_maxtid(c, t, (uint32_t*)d_tc, ncta), "maxtid launch");
-    if (!t.warp_contiguous) CK(regroup_by_warp(c, &t), "regroup by warp");
-    CK(launch_branch_div(c, t, ilog2(warp_size), (const uint32_t*)d_tc,
-                         per_site ? (uint64_t*)d_out + 4 : nullptr, per_site ? nsites : 0, (uint64_t*)d_out),
-       "branch_div launch");
-  }
-  void* h;
-  s = end_call(c, d_out, tbytes + sbytes, &h);
-  if (s != CADV_OK) return s;
-  const uint64_t* hr = (const uint64_t*)h;
-  if (per_site && hr[3]) return fail(c, CADV_ERR_INVALID_ARG, "a basic-block record's site id is >= nsites");
-  memcpy(totals, hr, 3 * 8);
-  if (per_site) memcpy(per_site, hr + 4, sbytes);
-  return CADV_OK;
+  Req q;
+  q.bd = true;
+  q.bd_ws = ilog2(warp_size);
+  q.bd_sites = per_site != nullptr;
+  q.nsites = per_site ? nsites : 0;
+  return run_analyses(c, q, nullptr, nullptr, nullptr, nullptr, totals, per_site);
 }
 
 CADV_API cadv_status cadv_reuse_histogram(cadv_ctx* c, uint32_t line_bytes, int scope, int binning, uint64_t* hist,
                                           uint32_t nbins, cadv_reuse_stats* stats) {
   if (!c) return CADV_ERR_INVALID_ARG;
   c->err.clear();
-  if (!c->loaded) return fail(c, CADV_ERR_NO_TRACE, "no trace loaded");
-  if (!pow2(line_bytes) || line_bytes > 4096) return fail(c, CADV_ERR_INVALID_ARG, "line_bytes must be 2^k <= 4096");
+  cadv_status s = check_args(c, line_bytes, 32, true, false);
+  if (s != CADV_OK) return s;
   if (scope != CADV_SCOPE_CTA && scope != CADV_SCOPE_KERNEL) return fail(c, CADV_ERR_INVALID_ARG, "bad scope");
   if (binning != CADV_BINS_LINEAR && binning != CADV_BINS_LOG2) return fail(c, CADV_ERR_INVALID_ARG, "bad binning");
   if (nbins < 3 || !hist) return fail(c, CADV_ERR_INVALID_ARG, "nbins must be >= 3 and hist non-NULL");
-  CK(cudaSetDevice(c->device), "cudaSetDevice");
-  cadv_status s = begin_call(c);
+  Req q;
+  q.rd = true;
+  q.rd_lbs = ilog2(line_bytes);
+  q.scope = scope;
+  q.log2bins = binning == CADV_BINS_LOG2;
+  q.nbins = nbins;
+  return run_analyses(c, q, hist, stats, nullptr, nullptr, nullptr, nullptr);
+}
+
+CADV_API cadv_status cadv_analyze(cadv_ctx* c, const cadv_analysis* a, uint64_t* rd_hist, cadv_reuse_stats* rd_stats,
+                                  uint64_t* md_hist, cadv_site_mem* md_sites, uint64_t* bd_totals,
+                                  cadv_site_branch* bd_sites) {
+  if (!c || !a) return CADV_ERR_INVALID_ARG;
+  c->err.clear();
+  Req q;
+  q.rd = rd_hist != nullptr;
+  q.md = md_hist != nullptr;
+  q.bd = bd_totals != nullptr;
+  if (!q.rd && !q.md && !q.bd) return fail(c, CADV_ERR_INVALID_ARG, "no analysis requested");
+  cadv_status s = check_args(c, q.rd ? a->rd_line_bytes : 1, 32, q.rd, false);
+  if (s == CADV_OK) s = check_args(c, q.md ? a->md_line_bytes : 1, q.md ? a->md_warp_size : 32, q.md, q.md);
+  if (s == CADV_OK) s = check_args(c, 1, q.bd ? a->bd_warp_size : 32, false, q.bd);
   if (s != CADV_OK) return s;
-  size_t hbytes = (size_t)nbins * 8;
-  void* d_out;
-  CK(ensure(c, B_HIST, hbytes + 64, &d_out), "workspace");
-  CK(cudaMemsetAsync(d_out, 0, hbytes + 64, c->stream), "memset");
-  uint64_t* d_stats = (uint64_t*)((uint8_t*)d_out + hbytes);
-  if (c->t.n) CK(run_reuse(c, ilog2(line_bytes), scope, binning == CADV_BINS_LOG2, nbins, (uint64_t*)d_out, d_stats),
-                 "reuse");
-  void* h;
-  s = end_call(c, d_out, hbytes + 32, &h);
-  if (s != CADV_OK) return s;
-  const uint64_t* hr = (const uint64_t*)h;
-  memcpy(hist, hr, hbytes);
-  if (stats) {
-    uint64_t acc = 0;
-    for (uint32_t b = 0; b < nbins; ++b) acc += hr[b];
-    stats->accesses = acc;
-    stats->inf = hr[nbins - 1];
-    stats->overflow = hr[nbins - 2];
-    stats->streaming = hr[nbins + 0];
+  if (q.rd) {
+    if (a->rd_scope != CADV_SCOPE_CTA && a->rd_scope != CADV_SCOPE_KERNEL) return fail(c, CADV_ERR_INVALID_ARG, "bad scope");
+    if (a->rd_binning != CADV_BINS_LINEAR && a->rd_binning != CADV_BINS_LOG2)
+      return fail(c, CADV_ERR_INVALID_ARG, "bad binning");
+    if (a->rd_nbins < 3) return fail(c, CADV_ERR_INVALID_ARG, "nbins must be >= 3");
+    q.rd_lbs = ilog2(a->rd_line_bytes);
+    q.scope = a->rd_scope;
+    q.log2bins = a->rd_binning == CADV_BINS_LOG2;
+    q.nbins = a->rd_nbins;
   }
-  return CADV_OK;
+  if ((md_sites || bd_sites) && a->nsites == 0) return fail(c, CADV_ERR_INVALID_ARG, "nsites must be > 0 with per_site");
+  if (q.md) {
+    q.md_lbs = ilog2(a->md_line_bytes);
+    q.md_ws = ilog2(a->md_warp_size);
+    q.md_sites = md_sites != nullptr;
+  }
+  if (q.bd) {
+    q.bd_ws = ilog2(a->bd_warp_size);
+    q.bd_sites = bd_sites != nullptr;
+  }
+  q.nsites = a->nsites;
+  return run_analyses(c, q, rd_hist, rd_stats, md_hist, md_sites, bd_totals, bd_sites);
 }
 
 }  // extern "C"

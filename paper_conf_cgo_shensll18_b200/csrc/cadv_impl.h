@@ -33,7 +33,7 @@ enum BufId {
   B_SORT_K0, B_SORT_K1, B_SORT_V0, B_SORT_V1, B_SORT_HIST, B_SCAN_TMP,
   B_GATHER,
   B_RD_KEY, B_RD_VAL, B_RD_TILESTAT, B_RD_TILEW, B_RD_TILEQ, B_RD_ENT, B_RD_ENT_KEY0, B_RD_ENT_KEY1,
-  B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP,
+  B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP, B_DEFER, B_OUT2,
   B_COUNT
 };
 
@@ -81,16 +81,54 @@ Scalars* scalars(cadv_ctx* c);
 // ---- launchers (each returns cudaSuccess or the launch error; they add the
 // number of kernels they launched to c->launches)
 cudaError_t launch_ingest(cadv_ctx* c);
-cudaError_t launch_mem_div(cadv_ctx* c, const cadv_trace_desc& t, uint32_t lb_shift, uint32_t w_shift,
-                           uint64_t* d_hist, uint64_t* d_sites, uint32_t nsites);
-cudaError_t launch_cta_maxtid(cadv_ctx* c, const cadv_trace_desc& t, uint32_t* d_tc, uint32_t ncta);
-cudaError_t launch_branch_div(cadv_ctx* c, const cadv_trace_desc& t, uint32_t w_shift, const uint32_t* d_tc,
-                              uint64_t* d_sites, uint32_t nsites, uint64_t* d_totals);
 // Stable (cta, tid/32) ordering of a non-warp-contiguous trace: fills `out`
 // with device copies of every column in that order.
 cudaError_t regroup_by_warp(cadv_ctx* c, cadv_trace_desc* out);
-// Reuse distance (reuse.cu): fills d_hist[nbins] and d_stats[4] on the device.
-cudaError_t run_reuse(cadv_ctx* c, uint32_t lb_shift, int scope, int log2bins, uint32_t nbins, uint64_t* d_hist,
+
+// ---- the fused streaming pass (scan.cu)
+enum { F_RD = 1, F_MD = 2, F_BD = 4 };
+struct ScanParams {
+  cadv_trace_desc t;
+  // reuse distance: run compression output
+  uint32_t lbs_rd = 0;
+  int cta_scope = 1;
+  uint32_t* kout = nullptr;
+  uint64_t* vout = nullptr;
+  uint64_t* status = nullptr;
+  uint64_t* hist0 = nullptr;
+  // memory divergence
+  uint32_t lbs_md = 0, ws_md = 5;
+  uint64_t* md_hist = nullptr;
+  uint64_t* md_sites = nullptr;
+  // branch divergence
+  uint32_t ws_bd = 5;
+  uint32_t* tc = nullptr;
+  uint64_t* bd_tot = nullptr;
+  uint64_t* bd_sites = nullptr;
+  void* defer = nullptr;
+  unsigned long long* ndefer = nullptr;
+  uint32_t nsites = 0;
+  uint64_t* site_flag = nullptr;
+};
+uint64_t scan_tiles(uint64_t n);
+cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P);
+cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const uint32_t* tc, uint32_t ws,
+                              uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites);
+
+// ---- reuse distance around the scan (reuse.cu)
+struct RdState {
+  int cta_scope = 1;
+  uint32_t* k0 = nullptr;
+  uint32_t* k1 = nullptr;
+  uint64_t* v0 = nullptr;
+  uint64_t* v1 = nullptr;
+  uint64_t* status = nullptr;
+  uint64_t stiles = 0;
+};
+// workspace for the run-compression output of the scan
+cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st);
+// CTA regroup, tiles, cross-tile phase after the scan wrote the kept records
+cudaError_t rd_finish(cadv_ctx* c, const RdState& st, int log2bins, uint32_t nbins, uint64_t* d_hist,
                       uint64_t* d_stats);
 
 // ---- device-wide primitives (sort.cu)

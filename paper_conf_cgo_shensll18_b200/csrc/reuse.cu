@@ -10,13 +10,13 @@
 //   RD(i) = |window (P(i), i)| - #{ j < i : P(j) > P(i) }
 // (the second term counts the window's records whose element is used again
 // inside the window).  The pipeline:
-//   R1 k_rd_compact  one streaming pass over (addr, cta, meta): validation,
-//                    line keys, and run compression of raw-adjacent records
-//                    of the same (scope, line): a load repeating the previous
-//                    record's element has RD 0 and is dropped (counted in
-//                    bin 0); consecutive stores are merged into one record of
-//                    weight w (they are w distinct one-shot elements).  Kept
-//                    records are written in trace order (decoupled look-back).
+//   R1 k_scan<F_RD>  (scan.cu) one streaming pass over (addr, cta, meta):
+//                    validation, line keys, and run compression of
+//                    raw-adjacent records of the same (scope, line): a load
+//                    repeating the previous record's element has RD 0 and is
+//                    dropped (counted in bin 0); consecutive stores are merged
+//                    into one record of weight w (w distinct one-shot
+//                    elements).  Kept records are written in trace order.
 //   R1b              stable radix sort of kept records by CTA id (CTA scope).
 //   R2/R3 k_rd_tile  fixed-capacity tiles of the CTA-major kept sequence
 //                    (boundaries snapped to segment starts): in shared memory,
@@ -42,166 +42,7 @@ namespace {
 constexpr uint64_t LINE_MASK = (1ull << 58) - 1;
 constexpr int VB_STORE = 58, VB_DUP = 59, VB_W = 60;  // weight - 1 in bits 60..63
 
-// ------------------------------------------------------------------ R1 compaction
-constexpr int CP_NT = 256, CP_IPT = 16, CP_TILE = CP_NT * CP_IPT;  // 4096 raw records per tile
-constexpr uint32_t CP_ROWS = CP_TILE + 2;
-constexpr uint32_t CP_OFF_ADDR = 0;
-constexpr uint32_t CP_OFF_CTA = CP_OFF_ADDR + stage_bytes<uint64_t>(CP_ROWS);
-constexpr uint32_t CP_OFF_META = CP_OFF_CTA + stage_bytes<uint32_t>(CP_ROWS);
-constexpr uint32_t CP_SMEM = CP_OFF_META + stage_bytes<uint8_t>(CP_ROWS);
-
-constexpr uint64_t LB_AGG = 1ull << 62, LB_PRE = 2ull << 62, LB_VAL = (1ull << 62) - 1;
-
-__device__ __forceinline__ uint64_t ld_volatile(const uint64_t* p) {
-  uint64_t v;
-  asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(v) : "l"(p));
-  return v;
-}
-
-__global__ void __launch_bounds__(CP_NT) k_rd_compact(const uint64_t* __restrict__ addr, const uint32_t* __restrict__ cta,
-                                                      const uint8_t* __restrict__ meta, uint64_t n, uint32_t lbs,
-                                                      int cta_scope, uint32_t* __restrict__ kout,
-                                                      uint64_t* __restrict__ vout, uint64_t* status, uint64_t* hist0,
-                                                      Scalars* sc) {
-  extern __shared__ __align__(128) uint8_t smem[];
-  __shared__ uint64_t bar;
-  __shared__ uint32_t s_tile;
-  __shared__ uint32_t ws[CP_NT / 32 + 1];
-  __shared__ uint64_t s_base;
-  const uint32_t tx = threadIdx.x;
-  if (tx == 0) {
-    s_tile = atomicAdd(&sc->tile_counter, 1u);
-    mbar_init(&bar, 1);
-    fence_barrier_init();
-  }
-  __syncthreads();
-  const uint64_t tile = s_tile;
-  const uint64_t t0 = tile * CP_TILE;
-  const uint64_t lo = t0 ? t0 - 1 : 0;
-  const uint64_t hi = (t0 + CP_TILE + 1) < n ? (t0 + CP_TILE + 1) : n;
-  if (tx == 0) {
-    auto hull = [](uintptr_t b, uintptr_t e) {
-      return (uint32_t)(((e + 15) & ~(uintptr_t)15) - (b & ~(uintptr_t)15));
-    };
-    uint32_t bytes = hull((uintptr_t)(addr + lo), (uintptr_t)(addr + hi)) +
-                     hull((uintptr_t)(cta + lo), (uintptr_t)(cta + hi)) +
-                     hull((uintptr_t)(meta + lo), (uintptr_t)(meta + hi));
-    mbar_arrive_expect_tx(&bar, bytes);
-    uint32_t d;
-    stage_column(addr, lo, hi, smem + CP_OFF_ADDR, &bar, &d);
-    stage_column(cta, lo, hi, smem + CP_OFF_CTA, &bar, &d);
-    stage_column(meta, lo, hi, smem + CP_OFF_META, &bar, &d);
-  }
-  const uint32_t da = (uint32_t)((uintptr_t)(addr + lo) & 15), dc = (uint32_t)((uintptr_t)(cta + lo) & 15),
-                 dm = (uint32_t)((uintptr_t)(meta + lo) & 15);
-  auto A = [&](uint64_t i) { return *(const uint64_t*)(smem + CP_OFF_ADDR + da + (i - lo) * 8); };
-  auto C = [&](uint64_t i) { return *(const uint32_t*)(smem + CP_OFF_CTA + dc + (i - lo) * 4); };
-  auto M = [&](uint64_t i) { return smem[CP_OFF_META + dm + (i - lo)]; };
-  mbar_wait(&bar, 0);
-
-  const uint64_t i0 = t0 + (uint64_t)tx * CP_IPT;
-  // state of the previous record (record i - 1)
-  bool pmem = false, pst = false;
-  uint64_t pline = 0;
-  uint32_t pscope = 0;
-  if (i0 > 0 && i0 - 1 < n) {
-    uint8_t m = M(i0 - 1);
-    pmem = is_mem(m) && meta_ok(m);
-    if (pmem) {
-      pline = A(i0 - 1) >> lbs;
-      pscope = cta_scope ? C(i0 - 1) : 0u;
-      pst = is_store(m);
-    }
-  }
-  uint64_t kline[CP_IPT];
-  uint32_t kcta[CP_IPT];
-  uint32_t kflag[CP_IPT];  // store | has_dup << 1 | (w - 1) << 2
-  int nk = 0;
-  uint32_t ndup = 0;
-#pragma unroll
-  for (int k = 0; k <= CP_IPT; ++k) {
-    uint64_t i = i0 + k;
-    if (i >= n) break;
-    uint8_t m = M(i);
-    bool mem = is_mem(m);
-    bool ok = meta_ok(m);
-    uint64_t a = 0;
-    if (mem && ok) {
-      a = A(i);
-      ok = addr_ok(a, m);
-    }
-    if (k == CP_IPT) {
-      // first record of the next chunk: only "is it a repeat of our last run?"
-      if (mem && ok && !is_store(m) && pmem && nk > 0) {
-        uint32_t s = cta_scope ? C(i) : 0u;
-        if (s == pscope && (a >> lbs) == pline) kflag[nk - 1] |= 2u;
-      }
-      break;
-    }
-    if (!ok) {
-      atomicMin(&sc->err_index, (unsigned long long)i);
-      atomicMax(&sc->err_code, 1u);
-      mem = false;
-    }
-    if (!mem) {
-      pmem = false;
-      continue;
-    }
-    uint64_t line = a >> lbs;
-    uint32_t s = cta_scope ? C(i) : 0u;
-    bool st = is_store(m);
-    bool same = pmem && s == pscope && line == pline;
-    if (same && !st) {
-      // a load of the element the previous record used: RD 0, dropped
-      ndup++;
-      if (k > 0 && nk > 0) kflag[nk - 1] |= 2u;
-    } else if (same && st && pst && k > 0 && nk > 0 && (kflag[nk - 1] >> 2) < 15u) {
-      // store right after a store to the same line: one more one-shot element
-      kflag[nk - 1] += 4u;
-    } else {
-      kline[nk] = line;
-      kcta[nk] = s;
-      kflag[nk] = st ? 1u : 0u;
-      nk++;
-    }
-    pmem = true;
-    pst = st;
-    pline = line;
-    pscope = s;
-  }
-  uint32_t tot;
-  uint32_t off = block_exclusive_scan<CP_NT>((uint32_t)nk, ws, &tot);
-  {
-    uint32_t d = __reduce_add_sync(FULL, ndup);
-    if (lane_id() == 0 && d) atomicAdd((unsigned long long*)hist0, (unsigned long long)d);
-  }
-  // decoupled look-back: global offset of this tile's kept records
-  if (tx == 0) {
-    uint64_t excl = 0;
-    if (tile == 0) {
-      atomicExch((unsigned long long*)&status[0], (unsigned long long)(LB_PRE | tot));
-    } else {
-      atomicExch((unsigned long long*)&status[tile], (unsigned long long)(LB_AGG | tot));
-      int64_t k = (int64_t)tile - 1;
-      while (k >= 0) {
-        uint64_t s = ld_volatile(status + k);
-        if (s & LB_PRE) { excl += s & LB_VAL; break; }
-        if (s & LB_AGG) { excl += s & LB_VAL; --k; continue; }
-      }
-      __threadfence();
-      atomicExch((unsigned long long*)&status[tile], (unsigned long long)(LB_PRE | (excl + tot)));
-    }
-    s_base = excl;
-  }
-  __syncthreads();
-  uint64_t g = s_base + off;
-  for (int k = 0; k < nk; ++k) {
-    uint64_t v = kline[k] | ((uint64_t)(kflag[k] & 1u) << VB_STORE) | ((uint64_t)((kflag[k] >> 1) & 1u) << VB_DUP) |
-                 ((uint64_t)(kflag[k] >> 2) << VB_W);
-    vout[g + k] = v;
-    if (kout) kout[g + k] = kcta[k];
-  }
-}
+constexpr uint64_t LB_VAL = (1ull << 62) - 1;  // look-back status value bits (scan.cu)
 
 // ------------------------------------------------------------------ tile bounds
 constexpr int TL_CAP = 4096;   // tile capacity (kept records)
@@ -745,37 +586,41 @@ int bits_for(uint64_t maxv) {
   return b;
 }
 
-int g_tile_smem_set = 0, g_compact_smem_set = 0;
+int g_tile_smem_set = 0;
 
 }  // namespace
 
-cudaError_t run_reuse(cadv_ctx* c, uint32_t lbs, int scope, int log2bins, uint32_t nbins, uint64_t* d_hist,
-                      uint64_t* d_stats) {
+cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st) {
   cudaError_t e;
   const uint64_t n = c->t.n;
   const uint64_t nmem = c->n_kind[0] + c->n_kind[1];
-  const int cta_scope = scope == CADV_SCOPE_CTA;
-  const int grid_ls = c->num_sms * 4;
-  Scalars* sc = scalars(c);
-  void *k0 = nullptr, *k1 = nullptr, *v0, *v1, *st;
+  st->cta_scope = scope == CADV_SCOPE_CTA;
+  void *k0 = nullptr, *k1 = nullptr, *v0, *v1, *stt;
   uint64_t cap = nmem + 16;
   if ((e = ensure(c, B_RD_VAL, cap * 8, &v0)) || (e = ensure(c, B_SORT_V1, cap * 8, &v1))) return e;
-  if (cta_scope && ((e = ensure(c, B_RD_KEY, cap * 4, &k0)) || (e = ensure(c, B_SORT_K1, cap * 4, &k1)))) return e;
-  // ---- R1 compaction
-  uint64_t ctiles = (n + CP_TILE - 1) / CP_TILE;
-  if ((e = ensure(c, B_RD_TILESTAT, ctiles * 8 + 64, &st))) return e;
-  if ((e = cudaMemsetAsync(st, 0, ctiles * 8, c->stream))) return e;
-  if (!g_compact_smem_set) {
-    if ((e = cudaFuncSetAttribute(k_rd_compact, cudaFuncAttributeMaxDynamicSharedMemorySize, CP_SMEM))) return e;
-    g_compact_smem_set = 1;
-  }
-  CADV_LAUNCH(c, k_rd_compact<<<(unsigned)ctiles, CP_NT, CP_SMEM, c->stream>>>(
-                     c->t.addr, c->t.cta, c->t.meta, n, lbs, cta_scope, (uint32_t*)k0, (uint64_t*)v0,
-                     (uint64_t*)st, d_hist, sc));
-  if ((e = cudaGetLastError())) return e;
-  // kept count = inclusive prefix of the last compaction tile
+  if (st->cta_scope && ((e = ensure(c, B_RD_KEY, cap * 4, &k0)) || (e = ensure(c, B_SORT_K1, cap * 4, &k1)))) return e;
+  st->stiles = scan_tiles(n);
+  if ((e = ensure(c, B_RD_TILESTAT, st->stiles * 8 + 64, &stt))) return e;
+  if ((e = cudaMemsetAsync(stt, 0, st->stiles * 8, c->stream))) return e;
+  st->k0 = (uint32_t*)k0;
+  st->k1 = (uint32_t*)k1;
+  st->v0 = (uint64_t*)v0;
+  st->v1 = (uint64_t*)v1;
+  st->status = (uint64_t*)stt;
+  return cudaSuccess;
+}
+
+cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbins, uint64_t* d_hist,
+                      uint64_t* d_stats) {
+  cudaError_t e;
+  const int cta_scope = S.cta_scope;
+  const int grid_ls = c->num_sms * 4;
+  Scalars* sc = scalars(c);
+  if (S.stiles == 0) return cudaSuccess;
+  void *k0 = S.k0, *k1 = S.k1, *v0 = S.v0, *v1 = S.v1;
+  // kept count = inclusive prefix of the last scan tile
   uint64_t last;
-  if ((e = cudaMemcpyAsync(&last, (uint64_t*)st + (ctiles - 1), 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaMemcpyAsync(&last, S.status + (S.stiles - 1), 8, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
   const uint64_t K = last & LB_VAL;
   c->counts[0] = K;

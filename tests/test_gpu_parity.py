@@ -266,6 +266,33 @@ def test_invalid_args(ctx, cadv):
     assert e.value.status == cadv.CADV_ERR_INVALID_ARG
 
 
+# ----------------------------------------------------------------- fused pass (cadv_analyze)
+
+@pytest.mark.parametrize("seed", range(4))
+def test_fused_analyze_equals_oracle(ctx, cadv, seed):
+    t = tg.generate("rand", seed=seed, ctas=7, threads=160, instrs=40, lines=80, pstore=0.2, pbb=0.4)
+    load(ctx, cadv, t)
+    for (lb_rd, scope, lb_md, W, Wb) in ((128, 0, 32, 32, 32), (32, 1, 128, 16, 8), (4, 0, 4, 8, 32)):
+        out = ctx.analyze(rd=(lb_rd, scope, 0, 66), md=(lb_md, W), bd=Wb, nsites=t.nsites)
+        h_ref, s_ref = orc.reuse(t, lb_rd, scope, 0, 66)
+        assert (out["reuse"][0] == h_ref).all() and out["reuse"][1] == s_ref
+        mh, ms = orc.mem_div(t, lb_md, W)
+        assert (out["mem_div"][0] == mh).all() and (out["mem_div"][1] == ms).all()
+        bs, bt = orc.branch_div(t, Wb)
+        assert (out["branch_div"][1] == bt).all() and (out["branch_div"][0] == bs).all()
+
+
+def test_fused_subsets(ctx, cadv):
+    t = tg.generate("srad", rows=64, cols=64, iters=1)
+    load(ctx, cadv, t)
+    out = ctx.analyze(rd=None, md=(128, 32), bd=None, nsites=t.nsites)
+    assert set(out) == {"mem_div"}
+    assert (out["mem_div"][0] == orc.mem_div(t, 128, 32)[0]).all()
+    out = ctx.analyze(rd=(128, 0, 1, 20), md=None, bd=32, nsites=t.nsites, per_site=False)
+    assert (out["reuse"][0] == orc.reuse(t, 128, 0, 1, 20)[0]).all()
+    assert (out["branch_div"][1] == orc.branch_div(t, 32)[1]).all()
+
+
 # ----------------------------------------------------------------- shaped workloads (reduced sizes)
 
 def test_sgemm_small(ctx, cadv):
