@@ -87,14 +87,44 @@ static void prof_collect(cadv_ctx* c) {
 
 // ------------------------------------------------------------------ R0 ingest
 // One streaming pass over (cta, meta): max CTA id and record count per kind.
+// 16 records per thread and step: four 16-byte loads of cta, one of meta.
+__device__ __forceinline__ void ingest_one(uint32_t c, uint32_t m, uint32_t& mx, uint32_t (&cnt)[4]) {
+  mx = max(mx, c);
+  const uint32_t k = m & 3u;
+  cnt[0] += k == 0;
+  cnt[1] += k == 1;
+  cnt[2] += k == 2;
+  cnt[3] += k == 3;
+}
+
 __global__ void __launch_bounds__(256) k_ingest(const uint32_t* __restrict__ cta, const uint8_t* __restrict__ meta,
                                                 uint64_t n, Scalars* s) {
   uint32_t mx = 0;
   uint32_t cnt[4] = {0, 0, 0, 0};
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
-    mx = max(mx, __ldg(cta + i));
-    cnt[__ldg(meta + i) & 3u]++;
+  const bool vec = (((uintptr_t)cta | (uintptr_t)meta) & 15) == 0;
+  const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, nth = (uint64_t)gridDim.x * blockDim.x;
+  uint64_t done = 0;
+  if (vec) {
+    const uint64_t ng = n / 16;
+    const uint4* c4 = (const uint4*)cta;
+    const uint4* m4 = (const uint4*)meta;
+    for (uint64_t gi = tid; gi < ng; gi += nth) {
+      const uint4 mm = __ldg(m4 + gi);
+      uint4 cc[4];
+#pragma unroll
+      for (int k = 0; k < 4; ++k) cc[k] = __ldg(c4 + 4 * gi + k);
+      const uint32_t mw[4] = {mm.x, mm.y, mm.z, mm.w};
+#pragma unroll
+      for (int k = 0; k < 4; ++k) {
+        ingest_one(cc[k].x, mw[k] & 0xffu, mx, cnt);
+        ingest_one(cc[k].y, (mw[k] >> 8) & 0xffu, mx, cnt);
+        ingest_one(cc[k].z, (mw[k] >> 16) & 0xffu, mx, cnt);
+        ingest_one(cc[k].w, mw[k] >> 24, mx, cnt);
+      }
+    }
+    done = ng * 16;
   }
+  for (uint64_t i = done + tid; i < n; i += nth) ingest_one(__ldg(cta + i), __ldg(meta + i), mx, cnt);
   mx = __reduce_max_sync(FULL, mx);
 #pragma unroll
   for (int k = 0; k < 4; ++k) cnt[k] = __reduce_add_sync(FULL, cnt[k]);
@@ -109,7 +139,7 @@ __global__ void __launch_bounds__(256) k_ingest(const uint32_t* __restrict__ cta
 cudaError_t launch_ingest(cadv_ctx* c) {
   uint64_t n = c->t.n;
   if (n == 0) return cudaSuccess;
-  uint64_t want = (n + 255) / 256;
+  uint64_t want = (n / 16 + 255) / 256 + 1;
   int grid = (int)(want < (uint64_t)c->num_sms * 8 ? want : (uint64_t)c->num_sms * 8);
   CADV_LAUNCH(c, k_ingest<<<grid, 256, 0, c->stream>>>(c->t.cta, c->t.meta, n, scalars(c)));
   return cudaGetLastError();
@@ -352,6 +382,20 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
   uint64_t* d = (uint64_t*)dv;
   cadv_trace_desc t = c->t;
   if ((q.md || q.bd) && !t.warp_contiguous && t.n) CK(regroup_by_warp(c, &t), "regroup by warp");
+  // the scan's 1-D TMA copies need 16-byte aligned column bases
+  if (t.n && (((uintptr_t)t.addr | (uintptr_t)t.cta | (uintptr_t)t.tid | (uintptr_t)t.site | (uintptr_t)t.winst |
+               (uintptr_t)t.meta) & 15)) {
+    const void* src[6] = {t.addr, t.cta, t.tid, t.site, t.winst, t.meta};
+    const size_t es[6] = {8, 4, 2, 4, 4, 1};
+    void* dst[6];
+    for (int k = 0; k < 6; ++k) {
+      if (!((uintptr_t)src[k] & 15)) { dst[k] = (void*)src[k]; continue; }
+      CK(ensure(c, (BufId)(B_ALIGN0 + k), es[k] * t.n + 16, &dst[k]), "workspace");
+      CK(cudaMemcpyAsync(dst[k], src[k], es[k] * t.n, cudaMemcpyDeviceToDevice, c->stream), "align copy");
+    }
+    t.addr = (const uint64_t*)dst[0]; t.cta = (const uint32_t*)dst[1]; t.tid = (const uint16_t*)dst[2];
+    t.site = (const uint32_t*)dst[3]; t.winst = (const uint32_t*)dst[4]; t.meta = (const uint8_t*)dst[5];
+  }
   ScanParams P;
   P.t = t;
   int flags = 0;
@@ -361,9 +405,9 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
     flags |= F_RD;
     P.lbs_rd = q.rd_lbs;
     P.cta_scope = q.scope == CADV_SCOPE_CTA;
-    P.kout = rs.cta_scope ? rs.k0 : nullptr;
-    P.vout = rs.v0;
-    P.status = rs.status;
+    P.kout = rs.cta_scope ? rs.k1 : nullptr;
+    P.vout = rs.v1;
+    P.blkcnt = rs.blkcnt;
     P.hist0 = d + o_rdh;
   }
   if (q.md) {
@@ -386,7 +430,7 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
     P.bd_tot = d + o_bdt;
     P.bd_sites = q.bd_sites ? d + o_bds : nullptr;
     P.defer = defer;
-    P.ndefer = (unsigned long long*)&scalars(c)->count[5];
+    P.ndefer = &scalars(c)->ndefer;
   }
   P.nsites = (q.md_sites || q.bd_sites) ? q.nsites : 0;
   // one flag word for both site checks

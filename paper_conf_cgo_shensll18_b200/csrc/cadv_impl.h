@@ -25,6 +25,8 @@ struct Scalars {
   unsigned long long count[8];   // generic counters (kept records, entries, ...)
   unsigned long long max_cta;    // ingest: max CTA id
   unsigned long long n_kind[4];  // ingest: records per kind
+  unsigned long long ndefer;     // branch divergence: deferred partial groups
+  unsigned long long rd_line_min, rd_line_max;  // reuse cross-tile phase: entry line range
 };
 
 enum BufId {
@@ -34,6 +36,7 @@ enum BufId {
   B_GATHER,
   B_RD_KEY, B_RD_VAL, B_RD_TILESTAT, B_RD_TILEW, B_RD_TILEQ, B_RD_ENT, B_RD_ENT_KEY0, B_RD_ENT_KEY1,
   B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP, B_DEFER, B_OUT2,
+  B_ALIGN0, B_ALIGN1, B_ALIGN2, B_ALIGN3, B_ALIGN4, B_ALIGN5,
   B_COUNT
 };
 
@@ -92,9 +95,9 @@ struct ScanParams {
   // reuse distance: run compression output
   uint32_t lbs_rd = 0;
   int cta_scope = 1;
-  uint32_t* kout = nullptr;
+  uint32_t* kout = nullptr;    // gapped per-block regions (scan_geometry)
   uint64_t* vout = nullptr;
-  uint64_t* status = nullptr;
+  uint64_t* blkcnt = nullptr;  // kept records per scan warp chunk
   uint64_t* hist0 = nullptr;
   // memory divergence
   uint32_t lbs_md = 0, ws_md = 5;
@@ -111,6 +114,9 @@ struct ScanParams {
   uint64_t* site_flag = nullptr;
 };
 uint64_t scan_tiles(uint64_t n);
+void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nwarps, uint64_t* chunk);
+cudaError_t launch_squeeze(cadv_ctx* c, const uint32_t* kin, const uint64_t* vin, uint32_t* kout, uint64_t* vout,
+                           const uint64_t* cnt, const uint64_t* off, uint64_t nblocks, uint64_t chunk_cap);
 cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P);
 cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const uint32_t* tc, uint32_t ws,
                               uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites);
@@ -118,12 +124,12 @@ cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const 
 // ---- reuse distance around the scan (reuse.cu)
 struct RdState {
   int cta_scope = 1;
-  uint32_t* k0 = nullptr;
-  uint32_t* k1 = nullptr;
+  uint32_t* k0 = nullptr;   // final kept records (after the squeeze) / radix sort ping
+  uint32_t* k1 = nullptr;   // scan output (gapped) / radix sort pong
   uint64_t* v0 = nullptr;
   uint64_t* v1 = nullptr;
-  uint64_t* status = nullptr;
-  uint64_t stiles = 0;
+  uint64_t* blkcnt = nullptr;  // [grid] kept per scan block, then [grid] offsets
+  uint64_t grid = 0, chunk_cap = 0;
 };
 // workspace for the run-compression output of the scan
 cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st);
@@ -148,6 +154,14 @@ namespace cadv {
 void prof_begin(cadv_ctx* c, const char* src);
 void prof_end(cadv_ctx* c);
 }  // namespace cadv
+
+#define CADV_LAUNCH_N(c, name, ...)         \
+  do {                                      \
+    cadv::prof_begin((c), (name));          \
+    __VA_ARGS__;                            \
+    cadv::prof_end((c));                    \
+    (c)->launches++;                        \
+  } while (0)
 
 #define CADV_LAUNCH(c, ...)                 \
   do {                                      \

@@ -153,25 +153,112 @@ __device__ int block_merge_sort(K* ka, P* pa, K* kb, P* pb, uint16_t* cnt, K pad
   return res;
 }
 
-// ------------------------------------------------------------------ R2-R4 tile kernel
-constexpr int TL_NT = 1024, TL_IPT = 4;  // 4096 = TL_CAP
-constexpr int TL_SMEM_BINS = 2048;
-constexpr uint16_t NONE16 = 0xffff;
+// Compare-exchange for the base-case sorting network.
+template <typename K>
+__device__ __forceinline__ void cas(K& a, K& b) {
+  K lo = a < b ? a : b, hi = a < b ? b : a;
+  a = lo;
+  b = hi;
+}
 
+// Merge sort of N = NT*8 DISTINCT keys in shared memory (no payload): base
+// case = Batcher's 19-comparator network on 8 registers per thread, then
+// log2(NT) merge-path levels.  COUNT: cnt[key & 0xfff] += number of earlier
+// (left) keys greater than the key, i.e. the per-element inversion count.
+template <int NT, typename K, bool COUNT>
+__device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key) {
+  constexpr int IPT = 8, N = NT * IPT;
+  const uint32_t t = threadIdx.x;
+  {
+    K k[IPT];
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) k[j] = ka[t * IPT + j];
+    if (COUNT) {
+#pragma unroll
+      for (int j = 1; j < IPT; ++j) {
+        uint32_t c = 0;
+#pragma unroll
+        for (int q = 0; q < j; ++q) c += k[q] > k[j] ? 1u : 0u;
+        if (c && k[j] != pad_key) cnt[(uint32_t)(k[j] & 0xfffu)] += (uint16_t)c;
+      }
+    }
+    cas(k[0], k[1]); cas(k[2], k[3]); cas(k[4], k[5]); cas(k[6], k[7]);
+    cas(k[0], k[2]); cas(k[1], k[3]); cas(k[4], k[6]); cas(k[5], k[7]);
+    cas(k[1], k[2]); cas(k[5], k[6]);
+    cas(k[0], k[4]); cas(k[1], k[5]); cas(k[2], k[6]); cas(k[3], k[7]);
+    cas(k[2], k[4]); cas(k[3], k[5]);
+    cas(k[1], k[2]); cas(k[3], k[4]); cas(k[5], k[6]);
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) ka[t * IPT + j] = k[j];
+  }
+  __syncthreads();
+  K* ks = ka;
+  K* kd = kb;
+  int res = 0;
+  for (uint32_t w = IPT; w < (uint32_t)N; w <<= 1) {
+    const uint32_t o = t * IPT;
+    const uint32_t s0 = (o / (2 * w)) * (2 * w);
+    const K* Ak = ks + s0;
+    const K* Bk = ks + s0 + w;
+    const uint32_t d = o - s0;
+    uint32_t lo = d > w ? d - w : 0, hi = d < w ? d : w;
+    while (lo < hi) {
+      const uint32_t mid = (lo + hi) >> 1;
+      if (Ak[mid] < Bk[d - 1 - mid]) lo = mid + 1;
+      else hi = mid;
+    }
+    uint32_t a = lo, b = d - lo;
+    K va = a < w ? Ak[a] : pad_key, vb = b < w ? Bk[b] : pad_key;
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) {
+      const bool takeA = a < w && (b >= w || va < vb);
+      if (takeA) {
+        kd[o + j] = va;
+        ++a;
+        va = a < w ? Ak[a] : pad_key;
+      } else {
+        kd[o + j] = vb;
+        if (COUNT && vb != pad_key && a < w) cnt[(uint32_t)(vb & 0xfffu)] += (uint16_t)(w - a);
+        ++b;
+        vb = b < w ? Bk[b] : pad_key;
+      }
+    }
+    __syncthreads();
+    K* tk = ks;
+    ks = kd;
+    kd = tk;
+    res ^= 1;
+  }
+  return res;
+}
+
+// ------------------------------------------------------------------ R2-R4 tile kernel
+constexpr int TL_NT = 512;            // 8 keys per thread -> TL_CAP
+constexpr int TL_SMEM_BINS = 1024;
+
+// Shared memory of one tile (<= 113 KB so that two CTAs fit on an SM).
+// key[2] holds the packed (line - min line) << 12 | position sort keys;
+// after P is known, key[r] is reused for the query keys (2 x u32 arrays) and
+// key[r^1] for the weighted prefix (u32) and the inversion counts (u16).
 struct TileSmem {
-  uint64_t ln[2][TL_CAP];     // lines (merge sort ping-pong); later: weighted prefix / query keys
-  uint16_t ps[2][TL_CAP];     // positions (payload); later: counts
+  uint64_t key[2][TL_CAP];
   uint8_t sdw[TL_CAP];        // store | has_dup << 1 | weight << 2
   uint8_t ffl[TL_CAP];        // first_in_piece | last_in_piece << 1
   uint8_t fnx[TL_CAP];        // the record's element is used again later in the tile
   uint16_t sgs[TL_CAP];       // local start of the record's segment
   uint16_t pl[TL_CAP];        // local previous use + 1 (0 = none)
   uint16_t qx[TL_CAP];        // number of local queries before the record
-  uint16_t es[TL_CAP];        // entry slot + 1 (0 = none)
-  uint32_t tmax[TL_NT];       // per-thread inclusive max (segment-start scan)
+  uint16_t es[TL_CAP];        // entry slot + 1 (0 = none); earlier: per-thread scan temp
   uint32_t hist[TL_SMEM_BINS];
   uint32_t ws[TL_NT / 32 + 1];
   uint32_t misc[8];
+  unsigned long long lmin, lmax;
+};
+// WIDE tiles (line range >= 2^52, practically never) keep lines and positions
+// in separate arrays.
+struct TileSmemWide {
+  TileSmem base;
+  uint16_t ps[2][TL_CAP];
 };
 
 struct EntryCols {
@@ -193,145 +280,193 @@ struct EntryCols {
 // scope) inside the tile; pieces cut by the tile's start (head) or end
 // (tail) are "partial" and emit one entry per distinct line for the
 // cross-tile phase.
-__global__ void __launch_bounds__(TL_NT, 1)
+// WIDE = 0: tiles whose line range fits 52 bits (the others are counted in
+// sc->count[3] / listed in wide_list and handled by the WIDE = 1 instance).
+template <bool WIDE>
+__global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
     k_rd_tile(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val, uint64_t K,
               const uint32_t* __restrict__ bounds, uint32_t ntiles, int log2bins, uint32_t nbins,
               uint64_t* __restrict__ g_hist, uint64_t* __restrict__ g_stream, uint32_t* __restrict__ tile_w,
-              uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc) {
+              uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc, uint32_t* wide_list) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
   const uint32_t tx = threadIdx.x;
-  const uint32_t tile = blockIdx.x;
+  const uint32_t tile = WIDE ? wide_list[blockIdx.x] : blockIdx.x;
   const uint64_t b = bounds[tile], e = bounds[tile + 1];
   const uint32_t m = (uint32_t)(e - b);
   const bool smem_hist = nbins <= TL_SMEM_BINS;
+  // ---- line range of the tile (packed keys need < 2^52)
+  if (tx == 0) {
+    S.lmin = ~0ull;
+    S.lmax = 0;
+    S.misc[2] = m;
+  }
+  __syncthreads();
+  {
+    uint64_t mn = ~0ull, mx = 0;
+    for (uint32_t x = tx; x < m; x += TL_NT) {
+      uint64_t l = __ldg(val + b + x) & LINE_MASK;
+      mn = l < mn ? l : mn;
+      mx = l > mx ? l : mx;
+    }
+    for (int o = 16; o; o >>= 1) {
+      uint64_t a2 = __shfl_xor_sync(FULL, mn, o), z2 = __shfl_xor_sync(FULL, mx, o);
+      mn = a2 < mn ? a2 : mn;
+      mx = z2 > mx ? z2 : mx;
+    }
+    if (lane_id() == 0 && m) {
+      atomicMin(&S.lmin, (unsigned long long)mn);
+      atomicMax(&S.lmax, (unsigned long long)mx);
+    }
+  }
+  __syncthreads();
+  const uint64_t lmin = m ? S.lmin : 0;
+  if (!WIDE && m && ((S.lmax - lmin) >> 52)) {
+    // handled by the WIDE instance
+    if (tx == 0) {
+      unsigned long long k = atomicAdd((unsigned long long*)&sc->count[3], 1ull);
+      wide_list[k] = tile;
+    }
+    return;
+  }
   if (smem_hist)
     for (uint32_t k = tx; k < nbins; k += TL_NT) S.hist[k] = 0;
-  if (tx == 0) S.misc[2] = m;
   // ---- load (striped)
+  uint16_t* PSW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[0] : nullptr;
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) {
     if (x < m) {
       uint64_t v = __ldg(val + b + x);
-      S.ln[0][x] = v & LINE_MASK;
+      uint64_t l = v & LINE_MASK;
+      S.key[0][x] = WIDE ? l : (((l - lmin) << 12) | x);
       uint32_t w = (uint32_t)(v >> VB_W) + 1u;
       S.sdw[x] = (uint8_t)(((v >> VB_STORE) & 1u) | (((v >> VB_DUP) & 1u) << 1) | (w << 2));
     } else {
-      S.ln[0][x] = ~0ull;
+      S.key[0][x] = ~0ull;
       S.sdw[x] = 0;
     }
-    S.ps[0][x] = (uint16_t)x;
+    if (WIDE) PSW[x] = (uint16_t)x;
     S.fnx[x] = 0;
-    S.es[x] = 0;
   }
-  // ---- segment starts (blocked: thread owns 4 consecutive positions)
-  bool ssf[TL_IPT];
-  uint32_t ss_local = 0;
+  // ---- segment starts (blocked: thread owns 8 consecutive positions)
+  constexpr int IPT = TL_CAP / TL_NT;
+  uint32_t ssm = 0, ss_local = 0;
 #pragma unroll
-  for (int j = 0; j < TL_IPT; ++j) {
-    uint32_t x = tx * TL_IPT + j;
+  for (int j = 0; j < IPT; ++j) {
+    uint32_t x = tx * IPT + j;
     uint64_t gx = b + x;
-    bool s = x < m && (gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1)));
-    ssf[j] = s;
-    if (s) ss_local = x;
+    bool sflag = x < m && (gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1)));
+    if (sflag) { ssm |= 1u << j; ss_local = x; }
   }
-  S.tmax[tx] = block_inclusive_max<TL_NT>(ss_local, S.ws);
+  uint32_t* tmax = reinterpret_cast<uint32_t*>(S.es);
+  tmax[tx] = block_inclusive_max<TL_NT>(ss_local, S.ws);
   __syncthreads();
   {
-    uint32_t cur = tx ? S.tmax[tx - 1] : 0u;
+    uint32_t cur = tx ? tmax[tx - 1] : 0u;
 #pragma unroll
-    for (int j = 0; j < TL_IPT; ++j) {
-      uint32_t x = tx * TL_IPT + j;
-      if (ssf[j]) cur = x;
+    for (int j = 0; j < IPT; ++j) {
+      uint32_t x = tx * IPT + j;
+      if ((ssm >> j) & 1u) {
+        cur = x;
+        if (x > 0) atomicMin(&S.misc[2], x);  // start of the tile's second segment
+      }
       S.sgs[x] = (uint16_t)cur;
-      if (ssf[j] && x > 0) atomicMin(&S.misc[2], x);  // start of the tile's second segment
     }
   }
   const bool head_cont = m > 0 && b > 0 && (!key || __ldg(key + b) == __ldg(key + b - 1));
   const bool tail_cont = m > 0 && e < K && (!key || __ldg(key + e) == __ldg(key + e - 1));
   __syncthreads();
+  for (uint32_t x = tx; x < TL_CAP; x += TL_NT) S.es[x] = 0;
   const uint32_t lastseg = m ? S.sgs[m - 1] : 0u;
   const uint32_t second = S.misc[2];
   auto partial = [&](uint32_t x) {
     uint32_t sg = S.sgs[x];
     return (sg == 0 && head_cont) || (sg == lastseg && tail_cont);
   };
-  // ---- stable merge sort of (line, position): runs of equal lines in position order
-  int r = block_merge_sort<TL_NT, TL_IPT, uint64_t, uint16_t, false>(S.ln[0], S.ps[0], S.ln[1], S.ps[1], nullptr,
-                                                                     ~0ull);
-  const uint64_t* L = S.ln[r];
-  const uint16_t* PS = S.ps[r];
+  // ---- sort by (line, position): runs of equal lines in position order
+  int r;
+  if (WIDE) {
+    TileSmemWide& SW = *reinterpret_cast<TileSmemWide*>(smem_raw);
+    r = block_merge_sort<TL_NT, IPT, uint64_t, uint16_t, false>(S.key[0], SW.ps[0], S.key[1], SW.ps[1], nullptr,
+                                                                ~0ull);
+  } else {
+    r = block_sort_keys<TL_NT, uint64_t, false>(S.key[0], S.key[1], nullptr, ~0ull);
+  }
+  const uint64_t* KS = S.key[r];
+  const uint16_t* PW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[r] : nullptr;
+  auto POS = [&](uint32_t s_) -> uint32_t { return WIDE ? PW[s_] : (uint32_t)(KS[s_] & 0xfffu); };
+  auto LN = [&](uint32_t s_) -> uint64_t { return WIDE ? KS[s_] : (KS[s_] >> 12); };
   // ---- previous local use; first / last use of the line in its piece
-  uint32_t isent[TL_IPT];
-  uint32_t nent = 0;
+  uint32_t isent = 0, nent = 0;
 #pragma unroll
-  for (int j = 0; j < TL_IPT; ++j) {
-    uint32_t s = tx * TL_IPT + j;
-    isent[j] = 0;
-    if (s >= m) continue;
-    uint32_t x = PS[s];
-    uint64_t l = L[s];
-    uint32_t sg = S.sgs[x];
-    bool prev_same = s > 0 && L[s - 1] == l && S.sgs[PS[s - 1]] == sg;
-    bool next_same = s + 1 < m && L[s + 1] == l && S.sgs[PS[s + 1]] == sg;
-    bool st = S.sdw[x] & 1u;
+  for (int j = 0; j < IPT; ++j) {
+    const uint32_t s_ = tx * IPT + j;
+    if (s_ >= m) continue;
+    const uint32_t x = POS(s_);
+    const uint64_t l = LN(s_);
+    const uint32_t sg = S.sgs[x];
+    const bool prev_same = s_ > 0 && LN(s_ - 1) == l && S.sgs[POS(s_ - 1)] == sg;
+    const bool next_same = s_ + 1 < m && LN(s_ + 1) == l && S.sgs[POS(s_ + 1)] == sg;
+    const bool st = S.sdw[x] & 1u;
     uint32_t p = 0;
     if (prev_same && !st) {
-      p = PS[s - 1] + 1u;
+      p = POS(s_ - 1) + 1u;
       S.fnx[p - 1] = 1;
     }
     S.pl[x] = (uint16_t)p;
     S.ffl[x] = (uint8_t)((prev_same ? 0u : 1u) | (next_same ? 0u : 2u));
     if (!prev_same && partial(x)) {
-      isent[j] = 1;
+      isent |= 1u << j;
       nent++;
     }
   }
   // ---- entry slots, one per (partial piece, line), allocated in sorted order
   uint32_t etot;
-  uint32_t eoff = block_exclusive_scan<TL_NT>(nent, S.ws, &etot);
+  const uint32_t eoff = block_exclusive_scan<TL_NT>(nent, S.ws, &etot);
   if (tx == 0)
     S.misc[1] = etot ? (uint32_t)atomicAdd((unsigned long long*)&sc->count[1], (unsigned long long)etot) : 0u;
   __syncthreads();
   const uint32_t ebase = S.misc[1];
-  {
+  if (isent) {
     uint32_t run = eoff;
 #pragma unroll
-    for (int j = 0; j < TL_IPT; ++j) {
-      uint32_t s = tx * TL_IPT + j;
-      if (!isent[j]) continue;
-      uint32_t x = PS[s];
-      uint32_t slot = ebase + run;
+    for (int j = 0; j < IPT; ++j) {
+      if (!((isent >> j) & 1u)) continue;
+      const uint32_t s_ = tx * IPT + j;
+      const uint32_t x = POS(s_);
+      const uint32_t slot = ebase + run;
       E.seg[slot] = key ? __ldg(key + b + x) : 0u;
-      E.line[slot] = L[s];
+      E.line[slot] = WIDE ? LN(s_) : LN(s_) + lmin;
       E.tile[slot] = tile;
       S.es[x] = (uint16_t)(run + 1);
       run++;
     }
   }
   __syncthreads();
-  // the last use of a run (if different from the first) shares the run's slot
+  if (etot) {
+    // the last use of a run (if different from the first) shares the run's slot
 #pragma unroll
-  for (int j = 0; j < TL_IPT; ++j) {
-    uint32_t s = tx * TL_IPT + j;
-    if (s >= m) continue;
-    uint32_t x = PS[s];
-    uint32_t f = S.ffl[x];
-    if ((f & 2u) && !(f & 1u) && partial(x)) {
-      uint32_t q = s;
-      while (!(S.ffl[PS[q]] & 1u)) --q;
-      S.es[x] = S.es[PS[q]];
+    for (int j = 0; j < IPT; ++j) {
+      const uint32_t s_ = tx * IPT + j;
+      if (s_ >= m) continue;
+      const uint32_t x = POS(s_);
+      const uint32_t f = S.ffl[x];
+      if ((f & 2u) && !(f & 1u) && partial(x)) {
+        uint32_t q = s_;
+        while (!(S.ffl[POS(q)] & 1u)) --q;
+        S.es[x] = S.es[POS(q)];
+      }
     }
+    __syncthreads();
   }
-  __syncthreads();
   // ---- position-order prefix counts: local queries and weights
-  uint32_t* WP = reinterpret_cast<uint32_t*>(S.ln[r ^ 1]);  // weighted exclusive prefix
-  uint32_t* QK = reinterpret_cast<uint32_t*>(S.ln[r]);      // query keys (2 x TL_CAP u32)
+  uint32_t* QK = reinterpret_cast<uint32_t*>(S.key[r]);          // 2 x TL_CAP u32 (the sorted keys are dead now)
   uint32_t* QK2 = QK + TL_CAP;
-  uint16_t* CNT = S.ps[r ^ 1];
+  uint32_t* WP = reinterpret_cast<uint32_t*>(S.key[r ^ 1]);      // TL_CAP u32
+  uint16_t* CNT = reinterpret_cast<uint16_t*>(WP + TL_CAP);       // TL_CAP u16
   uint32_t nq = 0, wsum = 0;
 #pragma unroll
-  for (int j = 0; j < TL_IPT; ++j) {
-    uint32_t x = tx * TL_IPT + j;
+  for (int j = 0; j < IPT; ++j) {
+    const uint32_t x = tx * IPT + j;
     if (x < m) {
       nq += S.pl[x] ? 1u : 0u;
       wsum += S.sdw[x] >> 2;
@@ -341,8 +476,8 @@ __global__ void __launch_bounds__(TL_NT, 1)
   uint32_t qoff = block_exclusive_scan<TL_NT>(nq, S.ws, &Q);
   uint32_t woff = block_exclusive_scan<TL_NT>(wsum, S.ws, &WT);
 #pragma unroll
-  for (int j = 0; j < TL_IPT; ++j) {
-    uint32_t x = tx * TL_IPT + j;
+  for (int j = 0; j < IPT; ++j) {
+    const uint32_t x = tx * IPT + j;
     S.qx[x] = (uint16_t)qoff;
     WP[x] = woff;
     if (x < m) {
@@ -356,24 +491,24 @@ __global__ void __launch_bounds__(TL_NT, 1)
   for (uint32_t k = Q + tx; k < TL_CAP; k += TL_NT) QK[k] = 0xffffffffu;
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) CNT[x] = 0;
   __syncthreads();
-  // ---- counting merge sort of the queries by previous use:
+  // ---- counting sort of the queries by previous use:
   //      CNT[x] = #{ local queries y < x : P(y) > P(x) }
-  int r2 = block_merge_sort<TL_NT, TL_IPT, uint32_t, uint32_t, true>(QK, QK, QK2, QK2, CNT, 0xffffffffu);
+  const int r2 = block_sort_keys<TL_NT, uint32_t, true>(QK, QK2, CNT, 0xffffffffu);
   const uint32_t* QS = r2 ? QK2 : QK;
   // ---- R4: bin the local accesses
   uint32_t stream = 0;
 #pragma unroll
-  for (int j = 0; j < TL_IPT; ++j) {
-    uint32_t x = tx * TL_IPT + j;
+  for (int j = 0; j < IPT; ++j) {
+    const uint32_t x = tx * IPT + j;
     if (x >= m) continue;
-    uint32_t sdw = S.sdw[x];
-    bool st = sdw & 1u, hd = (sdw >> 1) & 1u;
-    uint32_t w = sdw >> 2;
+    const uint32_t sdw = S.sdw[x];
+    const bool st = sdw & 1u, hd = (sdw >> 1) & 1u;
+    const uint32_t w = sdw >> 2;
     uint32_t bin = 0xffffffffu, cntb = 1;
-    bool head_first = S.sgs[x] == 0 && head_cont && (S.ffl[x] & 1u);
+    const bool head_first = S.sgs[x] == 0 && head_cont && (S.ffl[x] & 1u);
     if (S.pl[x]) {
-      uint32_t p = S.pl[x] - 1u;
-      uint32_t rd = (WP[x] - WP[p] - (uint32_t)(S.sdw[p] >> 2)) - CNT[x];
+      const uint32_t p = S.pl[x] - 1u;
+      const uint32_t rd = (WP[x] - WP[p] - (uint32_t)(S.sdw[p] >> 2)) - CNT[x];
       bin = rd_bin(rd, log2bins, nbins);
     } else if (st) {
       bin = nbins - 1;
@@ -386,35 +521,37 @@ __global__ void __launch_bounds__(TL_NT, 1)
       else atomicAdd((unsigned long long*)&g_hist[bin], (unsigned long long)cntb);
     }
     if (st) stream += w - 1;  // all but the last of merged stores are one-shot elements
-    bool deferred = partial(x) && S.ffl[x] != 0;
+    const bool deferred = partial(x) && S.ffl[x] != 0;
     if (!deferred && !S.pl[x] && !hd && !S.fnx[x]) stream += 1;
   }
   // ---- entry payloads of partial pieces
-  for (uint32_t x = tx; x < m; x += TL_NT) {
-    if (!S.es[x]) continue;
-    uint32_t slot = ebase + S.es[x] - 1;
-    uint32_t f = S.ffl[x];
-    uint32_t sdw = S.sdw[x];
-    if (f & 1u) {
-      bool head_piece = S.sgs[x] == 0 && head_cont;
-      E.f[slot] = (uint32_t)(b + x);
-      E.fa[slot] = (uint32_t)S.qx[x] - (uint32_t)S.qx[S.sgs[x]];
-      E.fw[slot] = WP[x];
-      E.ff[slot] = (uint8_t)(((sdw & 1u) ? 0u : 1u) | (((sdw >> 1) & 1u) ? 0u : 2u) | (S.fnx[x] ? 4u : 0u) |
-                             (head_piece ? 8u : 0u) | ((f & 2u) ? 16u : 0u));
-    }
-    if (f & 2u) {
-      uint32_t pend = (S.sgs[x] == lastseg && tail_cont) ? m : second;
-      // queries of the piece whose previous use lies in (x, pend)
-      uint32_t lo_key = (x + 1) << 12, hi_key = pend << 12;
-      uint32_t a0 = 0, a1 = Q;
-      while (a0 < a1) { uint32_t md = (a0 + a1) >> 1; if (QS[md] < lo_key) a0 = md + 1; else a1 = md; }
-      uint32_t c0 = a0, c1 = Q;
-      while (c0 < c1) { uint32_t md = (c0 + c1) >> 1; if (QS[md] < hi_key) c0 = md + 1; else c1 = md; }
-      E.l[slot] = (uint32_t)(b + x);
-      E.lw[slot] = WP[x];
-      E.ld[slot] = c0 - a0;
-      E.lf[slot] = (uint8_t)((sdw & 1u) | (((sdw >> 1) & 1u) ? 0u : 2u) | ((sdw >> 2) << 2));
+  if (etot) {
+    for (uint32_t x = tx; x < m; x += TL_NT) {
+      if (!S.es[x]) continue;
+      const uint32_t slot = ebase + S.es[x] - 1;
+      const uint32_t f = S.ffl[x];
+      const uint32_t sdw = S.sdw[x];
+      if (f & 1u) {
+        const bool head_piece = S.sgs[x] == 0 && head_cont;
+        E.f[slot] = (uint32_t)(b + x);
+        E.fa[slot] = (uint32_t)S.qx[x] - (uint32_t)S.qx[S.sgs[x]];
+        E.fw[slot] = WP[x];
+        E.ff[slot] = (uint8_t)(((sdw & 1u) ? 0u : 1u) | (((sdw >> 1) & 1u) ? 0u : 2u) | (S.fnx[x] ? 4u : 0u) |
+                               (head_piece ? 8u : 0u) | ((f & 2u) ? 16u : 0u));
+      }
+      if (f & 2u) {
+        const uint32_t pend = (S.sgs[x] == lastseg && tail_cont) ? m : second;
+        // queries of the piece whose previous use lies in (x, pend)
+        const uint32_t lo_key = (x + 1) << 12, hi_key = pend << 12;
+        uint32_t a0 = 0, a1 = Q;
+        while (a0 < a1) { uint32_t md = (a0 + a1) >> 1; if (QS[md] < lo_key) a0 = md + 1; else a1 = md; }
+        uint32_t c0 = a0, c1 = Q;
+        while (c0 < c1) { uint32_t md = (c0 + c1) >> 1; if (QS[md] < hi_key) c0 = md + 1; else c1 = md; }
+        E.l[slot] = (uint32_t)(b + x);
+        E.lw[slot] = WP[x];
+        E.ld[slot] = c0 - a0;
+        E.lf[slot] = (uint8_t)((sdw & 1u) | (((sdw >> 1) & 1u) ? 0u : 2u) | ((sdw >> 2) << 2));
+      }
     }
   }
   // ---- flush
@@ -595,18 +732,26 @@ cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st) {
   const uint64_t n = c->t.n;
   const uint64_t nmem = c->n_kind[0] + c->n_kind[1];
   st->cta_scope = scope == CADV_SCOPE_CTA;
-  void *k0 = nullptr, *k1 = nullptr, *v0, *v1, *stt;
-  uint64_t cap = nmem + 16;
-  if ((e = ensure(c, B_RD_VAL, cap * 8, &v0)) || (e = ensure(c, B_SORT_V1, cap * 8, &v1))) return e;
-  if (st->cta_scope && ((e = ensure(c, B_RD_KEY, cap * 4, &k0)) || (e = ensure(c, B_SORT_K1, cap * 4, &k1)))) return e;
-  st->stiles = scan_tiles(n);
-  if ((e = ensure(c, B_RD_TILESTAT, st->stiles * 8 + 64, &stt))) return e;
-  if ((e = cudaMemsetAsync(stt, 0, st->stiles * 8, c->stream))) return e;
+  uint64_t grid, nw, chunk;
+  scan_geometry(c, n, &grid, &nw, &chunk);
+  st->grid = nw;  // one kept-record region per scan warp
+  st->chunk_cap = chunk;
+  // the scan writes kept records into per-block regions of (k1, v1) (capacity
+  // grid * chunk >= n); the squeeze packs them into (k0, v0); the CTA radix
+  // sort then ping-pongs between the two pairs.
+  const uint64_t gap = nw * chunk + 16, cap = (nmem > gap ? gap : nmem) + 16;
+  void *k0 = nullptr, *k1 = nullptr, *v0, *v1, *bc;
+  if ((e = ensure(c, B_RD_VAL, (gap > cap ? gap : cap) * 8, &v0)) || (e = ensure(c, B_SORT_V1, gap * 8, &v1))) return e;
+  if (st->cta_scope && ((e = ensure(c, B_RD_KEY, (gap > cap ? gap : cap) * 4, &k0)) ||
+                        (e = ensure(c, B_SORT_K1, gap * 4, &k1))))
+    return e;
+  if ((e = ensure(c, B_RD_TILESTAT, (2 * nw + 8) * 8, &bc))) return e;
+  if ((e = cudaMemsetAsync(bc, 0, (2 * nw + 8) * 8, c->stream))) return e;
   st->k0 = (uint32_t*)k0;
   st->k1 = (uint32_t*)k1;
   st->v0 = (uint64_t*)v0;
   st->v1 = (uint64_t*)v1;
-  st->status = (uint64_t*)stt;
+  st->blkcnt = (uint64_t*)bc;
   return cudaSuccess;
 }
 
@@ -616,13 +761,17 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   const int cta_scope = S.cta_scope;
   const int grid_ls = c->num_sms * 4;
   Scalars* sc = scalars(c);
-  if (S.stiles == 0) return cudaSuccess;
+  if (S.grid == 0) return cudaSuccess;
   void *k0 = S.k0, *k1 = S.k1, *v0 = S.v0, *v1 = S.v1;
-  // kept count = inclusive prefix of the last scan tile
-  uint64_t last;
-  if ((e = cudaMemcpyAsync(&last, S.status + (S.stiles - 1), 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  // pack the per-block regions: offsets = exclusive scan of the block counts
+  uint64_t* off = S.blkcnt + S.grid + 4;
+  if ((e = exclusive_scan_u64(c, S.blkcnt, off, S.grid + 1))) return e;
+  uint64_t K;
+  if ((e = cudaMemcpyAsync(&K, off + S.grid, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = launch_squeeze(c, (const uint32_t*)k1, (const uint64_t*)v1, (uint32_t*)k0, (uint64_t*)v0, S.blkcnt, off,
+                          S.grid, S.chunk_cap)))
+    return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
-  const uint64_t K = last & LB_VAL;
   c->counts[0] = K;
   if (K == 0) return cudaSuccess;
   // ---- R1b regroup by CTA (stable)
@@ -642,7 +791,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   uint64_t ntiles = (K + TL_NOM - 1) / TL_NOM;
   c->counts[3] = ntiles;
   void *bnd, *tw, *tq;
-  if ((e = ensure(c, B_RD_XTMP, (ntiles + 2) * 4 + 64, &bnd))) return e;
+  if ((e = ensure(c, B_RD_XTMP, (2 * ntiles + 4) * 4 + 64, &bnd))) return e;  // bounds + wide-tile list
   if ((e = ensure(c, B_RD_TILEW, (ntiles + 2) * 8 * 2, &tw))) return e;
   if ((e = ensure(c, B_RD_TILEQ, (ntiles + 2) * 8 * 2, &tq))) return e;
   CADV_LAUNCH(c, k_tile_bounds<<<(unsigned)((ntiles + 1 + 7) / 8), 256, 0, c->stream>>>(key, K, (uint32_t*)bnd,
@@ -668,16 +817,29 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     En.lf = (uint8_t*)take(K);
   }
   if (!g_tile_smem_set) {
-    if ((e = cudaFuncSetAttribute(k_rd_tile, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))))
+    if ((e = cudaFuncSetAttribute(k_rd_tile<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)sizeof(TileSmem))) ||
+        (e = cudaFuncSetAttribute(k_rd_tile<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)sizeof(TileSmemWide))))
       return e;
     g_tile_smem_set = 1;
   }
   uint32_t* tile_w = (uint32_t*)tw;
   uint32_t* tile_q = (uint32_t*)tq;
-  CADV_LAUNCH(c, k_rd_tile<<<(unsigned)ntiles, TL_NT, sizeof(TileSmem), c->stream>>>(
+  uint32_t* wide_list = (uint32_t*)bnd + (ntiles + 2);
+  CADV_LAUNCH(c, k_rd_tile<false><<<(unsigned)ntiles, TL_NT, sizeof(TileSmem), c->stream>>>(
                      key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
-                     tile_q, En, sc));
+                     tile_q, En, sc, wide_list));
   if ((e = cudaGetLastError())) return e;
+  unsigned long long cnt13[3];
+  if ((e = cudaMemcpyAsync(cnt13, &sc->count[1], 24, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  if (cnt13[2]) {
+    CADV_LAUNCH(c, k_rd_tile<true><<<(unsigned)cnt13[2], TL_NT, sizeof(TileSmemWide), c->stream>>>(
+                       key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
+                       tile_q, En, sc, wide_list));
+    if ((e = cudaGetLastError())) return e;
+  }
   unsigned long long nent;
   if ((e = cudaMemcpyAsync(&nent, &sc->count[1], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
@@ -702,7 +864,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   if ((e = ensure(c, B_RD_ENT_KEY0, nent * 8, &ek0)) || (e = ensure(c, B_RD_ENT_KEY1, nent * 8, &ek1)) ||
       (e = ensure(c, B_RD_ENT_IDX0, nent * 4, &ei0)) || (e = ensure(c, B_RD_ENT_IDX1, nent * 4, &ei1)))
     return e;
-  unsigned long long* mm = (unsigned long long*)&sc->count[4];
+  unsigned long long* mm = &sc->rd_line_min;  // rd_line_min, rd_line_max are adjacent
   if ((e = cudaMemsetAsync(mm, 0xff, 8, c->stream)) || (e = cudaMemsetAsync(mm + 1, 0, 8, c->stream))) return e;
   CADV_LAUNCH(c, k_ent_line_range<<<grid_ls, 256, 0, c->stream>>>(En.line, nent, mm, mm + 1));
   unsigned long long hmm[2];
