@@ -153,6 +153,15 @@ __device__ int block_merge_sort(K* ka, P* pa, K* kb, P* pb, uint16_t* cnt, K pad
   return res;
 }
 
+// Bank-conflict-free placement of sort keys: thread t owns logical items
+// 8t..8t+7; XOR-swizzling the low 3 index bits with bits of the 8-group index
+// spreads a warp's same-j accesses over all banks (u32: bits 5..7, u64: bits
+// 4..6, matching 32 resp. 16 lanes per shared-memory wavefront).
+template <typename K>
+__device__ __forceinline__ uint32_t swz(uint32_t i) {
+  return sizeof(K) == 8 ? (i ^ ((i >> 4) & 7u)) : (i ^ ((i >> 5) & 7u));
+}
+
 // Compare-exchange for the base-case sorting network.
 template <typename K>
 __device__ __forceinline__ void cas(K& a, K& b) {
@@ -172,7 +181,7 @@ __device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key) {
   {
     K k[IPT];
 #pragma unroll
-    for (int j = 0; j < IPT; ++j) k[j] = ka[t * IPT + j];
+    for (int j = 0; j < IPT; ++j) k[j] = ka[swz<K>(t * IPT + j)];
     if (COUNT) {
 #pragma unroll
       for (int j = 1; j < IPT; ++j) {
@@ -189,7 +198,7 @@ __device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key) {
     cas(k[2], k[4]); cas(k[3], k[5]);
     cas(k[1], k[2]); cas(k[3], k[4]); cas(k[5], k[6]);
 #pragma unroll
-    for (int j = 0; j < IPT; ++j) ka[t * IPT + j] = k[j];
+    for (int j = 0; j < IPT; ++j) ka[swz<K>(t * IPT + j)] = k[j];
   }
   __syncthreads();
   K* ks = ka;
@@ -198,29 +207,29 @@ __device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key) {
   for (uint32_t w = IPT; w < (uint32_t)N; w <<= 1) {
     const uint32_t o = t * IPT;
     const uint32_t s0 = (o / (2 * w)) * (2 * w);
-    const K* Ak = ks + s0;
-    const K* Bk = ks + s0 + w;
     const uint32_t d = o - s0;
+    auto A_ = [&](uint32_t i) { return ks[swz<K>(s0 + i)]; };
+    auto B_ = [&](uint32_t i) { return ks[swz<K>(s0 + w + i)]; };
     uint32_t lo = d > w ? d - w : 0, hi = d < w ? d : w;
     while (lo < hi) {
       const uint32_t mid = (lo + hi) >> 1;
-      if (Ak[mid] < Bk[d - 1 - mid]) lo = mid + 1;
+      if (A_(mid) < B_(d - 1 - mid)) lo = mid + 1;
       else hi = mid;
     }
     uint32_t a = lo, b = d - lo;
-    K va = a < w ? Ak[a] : pad_key, vb = b < w ? Bk[b] : pad_key;
+    K va = a < w ? A_(a) : pad_key, vb = b < w ? B_(b) : pad_key;
 #pragma unroll
     for (int j = 0; j < IPT; ++j) {
       const bool takeA = a < w && (b >= w || va < vb);
       if (takeA) {
-        kd[o + j] = va;
+        kd[swz<K>(o + j)] = va;
         ++a;
-        va = a < w ? Ak[a] : pad_key;
+        va = a < w ? A_(a) : pad_key;
       } else {
-        kd[o + j] = vb;
+        kd[swz<K>(o + j)] = vb;
         if (COUNT && vb != pad_key && a < w) cnt[(uint32_t)(vb & 0xfffu)] += (uint16_t)(w - a);
         ++b;
-        vb = b < w ? Bk[b] : pad_key;
+        vb = b < w ? B_(b) : pad_key;
       }
     }
     __syncthreads();
@@ -337,11 +346,11 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
     if (x < m) {
       uint64_t v = __ldg(val + b + x);
       uint64_t l = v & LINE_MASK;
-      S.key[0][x] = WIDE ? l : (((l - lmin) << 12) | x);
+      S.key[0][WIDE ? x : swz<uint64_t>(x)] = WIDE ? l : (((l - lmin) << 12) | x);
       uint32_t w = (uint32_t)(v >> VB_W) + 1u;
       S.sdw[x] = (uint8_t)(((v >> VB_STORE) & 1u) | (((v >> VB_DUP) & 1u) << 1) | (w << 2));
     } else {
-      S.key[0][x] = ~0ull;
+      S.key[0][WIDE ? x : swz<uint64_t>(x)] = ~0ull;
       S.sdw[x] = 0;
     }
     if (WIDE) PSW[x] = (uint16_t)x;
@@ -393,8 +402,8 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
   }
   const uint64_t* KS = S.key[r];
   const uint16_t* PW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[r] : nullptr;
-  auto POS = [&](uint32_t s_) -> uint32_t { return WIDE ? PW[s_] : (uint32_t)(KS[s_] & 0xfffu); };
-  auto LN = [&](uint32_t s_) -> uint64_t { return WIDE ? KS[s_] : (KS[s_] >> 12); };
+  auto POS = [&](uint32_t s_) -> uint32_t { return WIDE ? PW[s_] : (uint32_t)(KS[swz<uint64_t>(s_)] & 0xfffu); };
+  auto LN = [&](uint32_t s_) -> uint64_t { return WIDE ? KS[s_] : (KS[swz<uint64_t>(s_)] >> 12); };
   // ---- previous local use; first / last use of the line in its piece
   uint32_t isent = 0, nent = 0;
 #pragma unroll
@@ -482,13 +491,13 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
     WP[x] = woff;
     if (x < m) {
       if (S.pl[x]) {
-        QK[qoff] = ((uint32_t)(S.pl[x] - 1u) << 12) | x;
+        QK[swz<uint32_t>(qoff)] = ((uint32_t)(S.pl[x] - 1u) << 12) | x;
         qoff++;
       }
       woff += S.sdw[x] >> 2;
     }
   }
-  for (uint32_t k = Q + tx; k < TL_CAP; k += TL_NT) QK[k] = 0xffffffffu;
+  for (uint32_t k = Q + tx; k < TL_CAP; k += TL_NT) QK[swz<uint32_t>(k)] = 0xffffffffu;
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) CNT[x] = 0;
   __syncthreads();
   // ---- counting sort of the queries by previous use:
@@ -544,9 +553,9 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
         // queries of the piece whose previous use lies in (x, pend)
         const uint32_t lo_key = (x + 1) << 12, hi_key = pend << 12;
         uint32_t a0 = 0, a1 = Q;
-        while (a0 < a1) { uint32_t md = (a0 + a1) >> 1; if (QS[md] < lo_key) a0 = md + 1; else a1 = md; }
+        while (a0 < a1) { uint32_t md = (a0 + a1) >> 1; if (QS[swz<uint32_t>(md)] < lo_key) a0 = md + 1; else a1 = md; }
         uint32_t c0 = a0, c1 = Q;
-        while (c0 < c1) { uint32_t md = (c0 + c1) >> 1; if (QS[md] < hi_key) c0 = md + 1; else c1 = md; }
+        while (c0 < c1) { uint32_t md = (c0 + c1) >> 1; if (QS[swz<uint32_t>(md)] < hi_key) c0 = md + 1; else c1 = md; }
         E.l[slot] = (uint32_t)(b + x);
         E.lw[slot] = WP[x];
         E.ld[slot] = c0 - a0;
