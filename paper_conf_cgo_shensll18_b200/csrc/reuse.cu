@@ -46,8 +46,8 @@ constexpr uint64_t LB_VAL = (1ull << 62) - 1;  // look-back status value bits (s
 
 // ------------------------------------------------------------------ tile bounds
 constexpr int TL_CAP = 4096;   // tile capacity (kept records)
-constexpr int TL_NOM = 3072;   // nominal tile length
-constexpr int TL_SNAP = 1024;  // boundary snapped to a segment start within this window
+constexpr int TL_NOM = 3584;   // nominal tile length
+constexpr int TL_SNAP = 512;   // boundary snapped to a segment start within this window
 
 __global__ void k_tile_bounds(const uint32_t* __restrict__ key, uint64_t K, uint32_t* __restrict__ bounds,
                               uint64_t ntiles) {
@@ -175,10 +175,12 @@ __device__ __forceinline__ void cas(K& a, K& b) {
 // log2(NT) merge-path levels.  COUNT: cnt[key & 0xfff] += number of earlier
 // (left) keys greater than the key, i.e. the per-element inversion count.
 template <int NT, typename K, bool COUNT>
-__device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key) {
-  constexpr int IPT = 8, N = NT * IPT;
+__device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key, uint32_t N = NT * 8) {
+  // N: power of two <= NT * 8; keys [0, N) are sorted (callers pad with pad_key)
+  constexpr int IPT = 8;
   const uint32_t t = threadIdx.x;
-  {
+  const bool act = t * IPT < N;
+  if (act) {
     K k[IPT];
 #pragma unroll
     for (int j = 0; j < IPT; ++j) k[j] = ka[swz<K>(t * IPT + j)];
@@ -204,8 +206,9 @@ __device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key) {
   K* ks = ka;
   K* kd = kb;
   int res = 0;
-  for (uint32_t w = IPT; w < (uint32_t)N; w <<= 1) {
+  for (uint32_t w = IPT; w < N; w <<= 1) {
     const uint32_t o = t * IPT;
+    if (act) {
     const uint32_t s0 = (o / (2 * w)) * (2 * w);
     const uint32_t d = o - s0;
     auto A_ = [&](uint32_t i) { return ks[swz<K>(s0 + i)]; };
@@ -231,6 +234,7 @@ __device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key) {
         ++b;
         vb = b < w ? B_(b) : pad_key;
       }
+    }
     }
     __syncthreads();
     K* tk = ks;
@@ -497,12 +501,14 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
       woff += S.sdw[x] >> 2;
     }
   }
-  for (uint32_t k = Q + tx; k < TL_CAP; k += TL_NT) QK[swz<uint32_t>(k)] = 0xffffffffu;
+  uint32_t NQ = 64;
+  while (NQ < Q) NQ <<= 1;
+  for (uint32_t k = Q + tx; k < NQ; k += TL_NT) QK[swz<uint32_t>(k)] = 0xffffffffu;
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) CNT[x] = 0;
   __syncthreads();
   // ---- counting sort of the queries by previous use:
   //      CNT[x] = #{ local queries y < x : P(y) > P(x) }
-  const int r2 = block_sort_keys<TL_NT, uint32_t, true>(QK, QK2, CNT, 0xffffffffu);
+  const int r2 = block_sort_keys<TL_NT, uint32_t, true>(QK, QK2, CNT, 0xffffffffu, NQ);
   const uint32_t* QS = r2 ? QK2 : QK;
   // ---- R4: bin the local accesses
   uint32_t stream = 0;
