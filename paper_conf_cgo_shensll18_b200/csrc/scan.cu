@@ -124,26 +124,63 @@ __device__ __forceinline__ void site_add(const ScanArgs& A, uint32_t* smem_tab, 
   }
 }
 
+// Per-warp TMA issuer: global column pointers at the chunk start, ring
+// shared-memory addresses, and the byte count of a full piece, computed once.
 template <int F>
-__device__ __forceinline__ void issue_piece(const ScanArgs& A, uint8_t* ring, uint64_t* bar, uint64_t q0,
-                                            uint64_t q1, int stage) {
-  constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
-  const uint32_t cnt = (uint32_t)(q1 - q0);
-  auto r16 = [](uint32_t b) { return (b + 15u) & ~15u; };
-  uint32_t bytes = r16(cnt * 4) + r16(cnt);
-  if (NA) bytes += r16(cnt * 8);
-  if (NG) bytes += r16(cnt * 2) + r16(cnt * 4) + r16(cnt * 4);
-  mbar_arrive_expect_tx(bar, bytes);
-  const uint32_t so = (uint32_t)stage * KR;
-  if (NA) tma_load_1d(ring + R_ADDR + so * 8, A.addr + q0, r16(cnt * 8), bar);
-  tma_load_1d(ring + R_CTA + so * 4, A.cta + q0, r16(cnt * 4), bar);
-  if (NG) {
-    tma_load_1d(ring + R_TID + so * 2, A.tid + q0, r16(cnt * 2), bar);
-    tma_load_1d(ring + R_WINST + so * 4, A.winst + q0, r16(cnt * 4), bar);
-    tma_load_1d(ring + R_SITE + so * 4, A.site + q0, r16(cnt * 4), bar);
+struct Issuer {
+  static constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
+  static constexpr uint32_t FULL_BYTES = KR * (4 + 1 + (NA ? 8 : 0) + (NG ? 2 + 4 + 4 : 0));
+  const uint8_t *ga, *gc, *gt, *gw, *gs, *gm;  // column bytes at record c_lo
+  uint32_t sa, sc, st, sw, ss, sm, sbar;       // shared addresses of stage 0 / barrier 0
+  uint64_t c_lo, s_end;
+  __device__ __forceinline__ void init(const ScanArgs& A, uint8_t* ring, uint64_t* bar, uint64_t lo, uint64_t end) {
+    c_lo = lo;
+    s_end = end;
+    ga = (const uint8_t*)(A.addr + lo); gc = (const uint8_t*)(A.cta + lo); gt = (const uint8_t*)(A.tid + lo);
+    gw = (const uint8_t*)(A.winst + lo); gs = (const uint8_t*)(A.site + lo); gm = (const uint8_t*)(A.meta + lo);
+    const uint32_t r = smem_u32(ring);
+    sa = r + R_ADDR; sc = r + R_CTA; st = r + R_TID; sw = r + R_WINST; ss = r + R_SITE; sm = r + R_META;
+    sbar = smem_u32(bar);
   }
-  tma_load_1d(ring + R_META + so, A.meta + q0, r16(cnt), bar);
-}
+  __device__ __forceinline__ static void cp(uint32_t dst, const uint8_t* src, uint32_t bytes, uint32_t bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+                 "l"(src), "r"(bytes), "r"(bar)
+                 : "memory");
+  }
+  // piece p -> stage p % KS
+  __device__ __forceinline__ void issue(uint32_t p) const {
+    const uint32_t stg = p % KS, bar = sbar + stg * 8;
+    const uint64_t q0 = c_lo + (uint64_t)p * KR;
+    const uint32_t off = p * KR;
+    if (q0 + KR <= s_end) {
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(FULL_BYTES) : "memory");
+      if (NA) cp(sa + stg * KR * 8, ga + (size_t)off * 8, KR * 8, bar);
+      cp(sc + stg * KR * 4, gc + (size_t)off * 4, KR * 4, bar);
+      if (NG) {
+        cp(st + stg * KR * 2, gt + (size_t)off * 2, KR * 2, bar);
+        cp(sw + stg * KR * 4, gw + (size_t)off * 4, KR * 4, bar);
+        cp(ss + stg * KR * 4, gs + (size_t)off * 4, KR * 4, bar);
+      }
+      cp(sm + stg * KR, gm + off, KR, bar);
+    } else {
+      // the last (partial) piece: sizes rounded up to 16 bytes
+      const uint32_t cnt = (uint32_t)(s_end - q0);
+      auto r16 = [](uint32_t b) { return (b + 15u) & ~15u; };
+      uint32_t bytes = r16(cnt * 4) + r16(cnt);
+      if (NA) bytes += r16(cnt * 8);
+      if (NG) bytes += r16(cnt * 2) + 2 * r16(cnt * 4);
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+      if (NA) cp(sa + stg * KR * 8, ga + (size_t)off * 8, r16(cnt * 8), bar);
+      cp(sc + stg * KR * 4, gc + (size_t)off * 4, r16(cnt * 4), bar);
+      if (NG) {
+        cp(st + stg * KR * 2, gt + (size_t)off * 2, r16(cnt * 2), bar);
+        cp(sw + stg * KR * 4, gw + (size_t)off * 4, r16(cnt * 4), bar);
+        cp(ss + stg * KR * 4, gs + (size_t)off * 4, r16(cnt * 4), bar);
+      }
+      cp(sm + stg * KR, gm + off, r16(cnt), bar);
+    }
+  }
+};
 
 // run identity: (cta, warp32, winst, family)
 __device__ __forceinline__ uint32_t run_hi(uint32_t tid, uint32_t meta) {
@@ -192,12 +229,10 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
     }
     __syncwarp();
     uint32_t issued = 0, waited = 0;
+    Issuer<F> io;
+    io.init(A, ring, bar, c_lo, s_end);
     if (lane == 0)
-      for (; issued < (uint32_t)KS && issued < npieces; ++issued) {
-        const uint64_t q0 = c_lo + (uint64_t)issued * KR;
-        const uint64_t q1 = q0 + KR < s_end ? q0 + KR : s_end;
-        issue_piece<F>(A, ring, &bar[issued], q0, q1, (int)issued);
-      }
+      for (; issued < (uint32_t)KS && issued < npieces; ++issued) io.issue(issued);
     issued = __shfl_sync(FULL, issued, 0);
     const uint64_t* r_addr = (const uint64_t*)(ring + R_ADDR);
     const uint32_t* r_cta = (const uint32_t*)(ring + R_CTA);
@@ -250,6 +285,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       }
       // predecessor record
       uint32_t pc = __shfl_up_sync(FULL, c, 1), ptm = __shfl_up_sync(FULL, tm, 1), pwi = __shfl_up_sync(FULL, w, 1);
+      const uint32_t rk = run_hi(tm & 0xffffu, tm >> 16);
       uint64_t pa = __shfl_up_sync(FULL, a, 1);
       if (lane == 0) { pc = p_cta; ptm = p_tm; pwi = p_winst; pa = p_addr; }
       uint32_t m = tm >> 16;
@@ -259,17 +295,16 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       uint32_t S = 0, e32 = 1;
       bool rs = true;
       if (NG) {
-        rs = !inb || c != pc || w != pwi || run_hi(t, m) != run_hi(pt, pm);
+        rs = !inb || c != pc || w != pwi || rk != run_hi(pt, pm);
         S = __ballot_sync(FULL, rs);
         // does the record after the batch start a new run?
         const uint32_t j32 = g + 32;
-        const uint32_t c31 = __shfl_sync(FULL, c, 31), tm31 = __shfl_sync(FULL, tm, 31),
+        const uint32_t c31 = __shfl_sync(FULL, c, 31), rk31 = __shfl_sync(FULL, rk, 31),
                        w31 = __shfl_sync(FULL, w, 31);
         if (j32 < nrel) {
           const uint32_t s32 = j32 & (RING - 1);
           const uint32_t c32 = r_cta[s32], tm32 = ((uint32_t)r_meta[s32] << 16) | r_tid[s32], w32 = r_winst[s32];
-          e32 = (c32 != c31 || w32 != w31 || run_hi(tm32 & 0xffffu, tm32 >> 16) != run_hi(tm31 & 0xffffu, tm31 >> 16))
-                    ? 1u : 0u;
+          e32 = (c32 != c31 || w32 != w31 || run_hi(tm32 & 0xffffu, tm32 >> 16) != rk31) ? 1u : 0u;
         }
       }
       const uint32_t S1 = S | 1u;                                   // lane 0 always opens a (pseudo) run
@@ -328,13 +363,19 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
           LEAD = __ballot_sync(FULL, pmem && (uint32_t)(__ffs(mt) - 1) == lane);
         }
         const uint32_t s = inb ? r_site[slot] : 0u;
-        for (uint32_t L = LEAD; L; L &= L - 1) {  // one group at a time (warp-uniform)
+        // one group at a time (warp-uniform): the warp-private histogram takes plain updates
+        for (uint32_t L = LEAD; L; L &= L - 1) {
           const uint32_t l = __ffs(L) - 1;
-          const uint32_t kd = __shfl_sync(FULL, m & 3u, l), dg = __shfl_sync(FULL, deg, l), ss = __shfl_sync(FULL, s, l);
-          if (lane == 0) {
-            whist[kd * 33 + dg] += 1;
-            if (A.nsites) site_add(A, C.md_sites, A.md_sites, 2, ss, 1, dg);
+          if (lane == l) {
+            whist[(m & 3u) * 33 + deg] += 1;
+            if (sites_smem) {
+              if (s < A.nsites) { atomicAdd(&C.md_sites[2 * s], 1u); atomicAdd(&C.md_sites[2 * s + 1], deg); }
+              else *A.site_flag = 1;
+            } else if (A.nsites) {
+              site_add(A, nullptr, A.md_sites, 2, s, 1, deg);
+            }
           }
+          __syncwarp();
         }
       }
       // ---- B1-B3 branch divergence
@@ -365,17 +406,26 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
         bd_exec += __popc(LEAD);
         bd_threads += __popc(CN);
         const uint32_t s = inb ? r_site[slot] : 0u;
-        for (uint32_t L = LEAD; L; L &= L - 1) {  // one group at a time (warp-uniform)
-          const uint32_t l = __ffs(L) - 1;
-          const uint32_t cn = __shfl_sync(FULL, cnt, l), ss = __shfl_sync(FULL, s, l);
-          const uint32_t cc = __shfl_sync(FULL, c, l), wv = __shfl_sync(FULL, t >> ws_bd, l);
-          if (lane == 0) {
-            if (A.nsites) site_add(A, C.bd_sites, A.bd_sites, 3, ss, 1, cn);
-            if (cn < W) {  // fewer than W lanes: divergence decided once T_c is known
-              const unsigned long long k = atomicAdd(A.ndefer, 1ull);
-              A.defer[k] = make_uint4(cc, wv, cn, (A.nsites && ss < A.nsites) ? ss : 0xffffffffu);
-            }
+        // leaders update the per-site counters (shared-memory atomics, different sites in parallel)
+        const bool lead = (LEAD >> lane) & 1u;
+        if (lead) {
+          if (sites_smem) {
+            if (s < A.nsites) { atomicAdd(&C.bd_sites[3 * s], 1u); atomicAdd(&C.bd_sites[3 * s + 2], cnt); }
+            else *A.site_flag = 1;
+          } else if (A.nsites) {
+            site_add(A, nullptr, A.bd_sites, 3, s, 1, cnt);
           }
+        }
+        // groups with fewer than W lanes: divergence decided once T_c is known
+        const bool dfr = lead && cnt < W;
+        const uint32_t MDF = __ballot_sync(FULL, dfr);
+        if (MDF) {
+          unsigned long long base = 0;
+          if (lane == 0) base = atomicAdd(A.ndefer, (unsigned long long)__popc(MDF));
+          base = __shfl_sync(FULL, base, 0);
+          if (dfr)
+            A.defer[base + __popc(MDF & lanemask_lt())] =
+                make_uint4(c, t >> ws_bd, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
         }
       }
       // ---- R1 run compression over the consumed records of this chunk
@@ -465,9 +515,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
         __syncwarp();
         if (lane == 0) {
           fence_proxy_async();
-          const uint64_t q0 = c_lo + (uint64_t)issued * KR;
-          const uint64_t q1 = q0 + KR < s_end ? q0 + KR : s_end;
-          issue_piece<F>(A, ring, &bar[issued % KS], q0, q1, (int)(issued % KS));
+          io.issue(issued);
         }
         ++issued;
       }
