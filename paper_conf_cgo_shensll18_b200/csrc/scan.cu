@@ -13,9 +13,9 @@
 //         k_bd_resolve classifies once T_c (1 + max tid of the CTA's BB
 //         records, reduced with fire-and-forget RED.MAX) is complete.
 //
-// Data movement (B200): one persistent CTA per SM, 24 independent warps.
+// Data movement (B200): one persistent CTA per SM, 20 independent warps.
 // Every warp owns a contiguous chunk of the trace and streams it through a
-// private ring of 4 x 64-record pieces in shared memory, filled by 1-D TMA
+// private ring of 3 x 128-record pieces in shared memory, filled by 1-D TMA
 // bulk copies (cp.async.bulk + a per-warp mbarrier per piece).  There is no
 // block-level barrier in the loop.  A warp walks its chunk in batches of 32
 // records that start at a run start (run = records of one (cta, warp32,
@@ -37,12 +37,17 @@
 namespace cadv {
 namespace {
 
-constexpr int KR = 64;                 // records per piece
-constexpr int KS = 4;                  // pieces in flight per warp
-constexpr int RING = KR * KS;          // 256 records
-constexpr int NWARP = 24;              // warps per CTA (one CTA per SM)
+constexpr int KR = 128;                // records per piece
+constexpr int KS = 3;                  // pieces in flight per warp
+constexpr int RING = KR * KS;          // 384 ring slots: record j lives in stage (j / KR) % KS
+constexpr int NWARP = 20;              // warps per CTA (one CTA per SM)
 constexpr int NTHR = NWARP * 32;
 constexpr int NSITE_SMEM = 1024;       // per-site counters kept in shared memory up to this many sites
+
+__device__ __forceinline__ uint32_t ring_slot(uint32_t j) {  // chunk-relative record -> ring slot
+  const uint32_t p = j >> 7;                                    // KR = 128
+  return (p - (p / KS) * KS) * KR + (j & (KR - 1));
+}
 
 // per-warp ring (bytes); every column region is a multiple of 128 B
 constexpr uint32_t R_ADDR = 0;
@@ -253,6 +258,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       p_tm = (pm0 << 16) | (NG ? (uint32_t)__ldg(A.tid + c_lo - 1) : 0u);
       if (NG) p_winst = __ldg(A.winst + c_lo - 1);
     }
+    uint32_t p_rk = run_hi(p_tm & 0xffffu, p_tm >> 16);
     // RD carried state; r_* = the chunk's last record seen by the compression
     bool pv = false, pst = false, r_mem = false;
     uint64_t r_line = 0;
@@ -274,7 +280,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       // ---- this batch's records (tm = tid | meta << 16)
       const uint32_t j = g + lane;
       const bool inb = j < slen;
-      const uint32_t slot = j & (RING - 1);
+      const uint32_t slot = ring_slot(j);
       uint32_t c = 0xfffffffeu, tm = 3u << 16, w = 0;
       uint64_t a = 0;
       if (inb) {
@@ -286,6 +292,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       // predecessor record
       uint32_t pc = __shfl_up_sync(FULL, c, 1), ptm = __shfl_up_sync(FULL, tm, 1), pwi = __shfl_up_sync(FULL, w, 1);
       const uint32_t rk = run_hi(tm & 0xffffu, tm >> 16);
+      uint32_t prk = __shfl_up_sync(FULL, rk, 1);
+      if (lane == 0) prk = p_rk;
       uint64_t pa = __shfl_up_sync(FULL, a, 1);
       if (lane == 0) { pc = p_cta; ptm = p_tm; pwi = p_winst; pa = p_addr; }
       uint32_t m = tm >> 16;
@@ -295,14 +303,14 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       uint32_t S = 0, e32 = 1;
       bool rs = true;
       if (NG) {
-        rs = !inb || c != pc || w != pwi || rk != run_hi(pt, pm);
+        rs = !inb || c != pc || w != pwi || rk != prk;
         S = __ballot_sync(FULL, rs);
         // does the record after the batch start a new run?
         const uint32_t j32 = g + 32;
         const uint32_t c31 = __shfl_sync(FULL, c, 31), rk31 = __shfl_sync(FULL, rk, 31),
                        w31 = __shfl_sync(FULL, w, 31);
         if (j32 < nrel) {
-          const uint32_t s32 = j32 & (RING - 1);
+          const uint32_t s32 = ring_slot(j32);
           const uint32_t c32 = r_cta[s32], tm32 = ((uint32_t)r_meta[s32] << 16) | r_tid[s32], w32 = r_winst[s32];
           e32 = (c32 != c31 || w32 != w31 || run_hi(tm32 & 0xffffu, tm32 >> 16) != rk31) ? 1u : 0u;
         }
@@ -363,19 +371,15 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
           LEAD = __ballot_sync(FULL, pmem && (uint32_t)(__ffs(mt) - 1) == lane);
         }
         const uint32_t s = inb ? r_site[slot] : 0u;
-        // one group at a time (warp-uniform): the warp-private histogram takes plain updates
-        for (uint32_t L = LEAD; L; L &= L - 1) {
-          const uint32_t l = __ffs(L) - 1;
-          if (lane == l) {
-            whist[(m & 3u) * 33 + deg] += 1;
-            if (sites_smem) {
-              if (s < A.nsites) { atomicAdd(&C.md_sites[2 * s], 1u); atomicAdd(&C.md_sites[2 * s + 1], deg); }
-              else *A.site_flag = 1;
-            } else if (A.nsites) {
-              site_add(A, nullptr, A.md_sites, 2, s, 1, deg);
-            }
+        // leaders update the counters in parallel (shared-memory atomics)
+        if ((LEAD >> lane) & 1u) {
+          atomicAdd(&whist[(m & 3u) * 33 + deg], 1u);
+          if (sites_smem) {
+            if (s < A.nsites) { atomicAdd(&C.md_sites[2 * s], 1u); atomicAdd(&C.md_sites[2 * s + 1], deg); }
+            else *A.site_flag = 1;
+          } else if (A.nsites) {
+            site_add(A, nullptr, A.md_sites, 2, s, 1, deg);
           }
-          __syncwarp();
         }
       }
       // ---- B1-B3 branch divergence
@@ -508,6 +512,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       const uint32_t last = adv - 1;
       p_cta = __shfl_sync(FULL, c, last);
       p_tm = __shfl_sync(FULL, (m << 16) | t, last);
+      p_rk = __shfl_sync(FULL, rk, last);
       p_winst = __shfl_sync(FULL, w, last);
       p_addr = __shfl_sync(FULL, a, last);
       g += adv;
