@@ -37,15 +37,17 @@
 namespace cadv {
 namespace {
 
-constexpr int KR = 128;                // records per piece
-constexpr int KS = 3;                  // pieces in flight per warp
-constexpr int RING = KR * KS;          // 384 ring slots: record j lives in stage (j / KR) % KS
-constexpr int NWARP = 20;              // warps per CTA (one CTA per SM)
+constexpr int LPR = 8;                 // consecutive records per lane in one warp step
+constexpr int KR = 32 * LPR;           // records per piece = one warp step
+constexpr int KS = 3;                  // ring stages per warp (pieces p - 1, p, p + 1)
+constexpr int RING = KR * KS;          // ring slots: record j lives in stage (j / KR) % KS
+constexpr int NWARP = 11;              // warps per CTA (one CTA per SM)
 constexpr int NTHR = NWARP * 32;
-constexpr int NSITE_SMEM = 1024;       // per-site counters kept in shared memory up to this many sites
+constexpr int NSITE_SMEM = 512;        // per-site counters kept in shared memory up to this many sites
+constexpr int QCAP = 160;              // per-warp queue of complete runs awaiting finalization
 
 __device__ __forceinline__ uint32_t ring_slot(uint32_t j) {  // chunk-relative record -> ring slot
-  const uint32_t p = j >> 7;                                    // KR = 128
+  const uint32_t p = j / KR;
   return (p - (p / KS) * KS) * KR + (j & (KR - 1));
 }
 
@@ -192,6 +194,176 @@ __device__ __forceinline__ uint32_t run_hi(uint32_t tid, uint32_t meta) {
   return (tid >> 5) | (((meta & 3u) == 2u) ? 64u : 0u);
 }
 
+// ------------------------------------------------------------------ group finishing
+struct Acc {              // per-lane BD accumulators, reduced at the end
+  uint32_t bd_exec, bd_threads;
+};
+
+__device__ __forceinline__ void finish_md(const ScanArgs& A, const Counters& C, uint32_t* whist, bool sites_smem,
+                                          uint32_t kind, uint32_t deg, uint32_t s) {
+  atomicAdd(&whist[kind * 33 + deg], 1u);
+  if (sites_smem) {
+    if (s < A.nsites) { atomicAdd(&C.md_sites[2 * s], 1u); atomicAdd(&C.md_sites[2 * s + 1], deg); }
+    else *A.site_flag = 1;
+  } else if (A.nsites) {
+    site_add(A, nullptr, A.md_sites, 2, s, 1, deg);
+  }
+}
+
+// One BB group: exec / threads, T_c candidate, per-site counters; groups with
+// fewer than W active lanes are deferred until T_c is known (k_bd_resolve).
+__device__ __forceinline__ void finish_bd(const ScanArgs& A, const Counters& C, Acc& acc, bool sites_smem,
+                                          uint32_t cnt, uint32_t s, uint32_t cta, uint32_t wsub, uint32_t maxtid) {
+  acc.bd_exec += 1;
+  acc.bd_threads += cnt;
+  red_max(A.tc + cta, maxtid + 1u);
+  if (sites_smem) {
+    if (s < A.nsites) { atomicAdd(&C.bd_sites[3 * s], 1u); atomicAdd(&C.bd_sites[3 * s + 2], cnt); }
+    else *A.site_flag = 1;
+  } else if (A.nsites) {
+    site_add(A, nullptr, A.bd_sites, 3, s, 1, cnt);
+  }
+  if (cnt < (1u << A.ws_bd)) {
+    const unsigned long long k = atomicAdd(A.ndefer, 1ull);
+    A.defer[k] = make_uint4(cta, wsub, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
+  }
+}
+
+struct RingView {
+  const uint64_t* addr;
+  const uint32_t* cta;
+  const uint16_t* tid;
+  const uint32_t* winst;
+  const uint32_t* site;
+  const uint8_t* meta;
+};
+
+// Exact resolution of one run [j0, j0 + nrec) read back from the ring: every
+// sub-warp group's distinct lines (MD) / lanes (BD) by pairwise comparison.
+// Used for runs whose lines are not non-decreasing (MD), for analysis warp
+// sizes below 32 and to report runs with more than 32 records (a lane must
+// repeat).  The ring holds the run: it started at most one piece back.
+template <int F>
+__device__ __noinline__ void walk_run(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
+                                      const RingView R, uint32_t j0, uint32_t nrec, uint64_t c_lo) {
+  if (nrec > 32) { report(A.sc, c_lo + j0, 2); return; }
+  Acc acc{0, 0};
+  const bool bb = (R.meta[ring_slot(j0)] & 3u) == 2u;
+  const uint32_t ws = bb ? A.ws_bd : A.ws_md;
+  for (uint32_t r = 0; r < nrec; ++r) {
+    const uint32_t sr = ring_slot(j0 + r);
+    const uint32_t tr = R.tid[sr], sub = (tr & 31u) >> ws;
+    bool leader = true;
+    for (uint32_t q = 0; q < r && leader; ++q) leader = ((R.tid[ring_slot(j0 + q)] & 31u) >> ws) != sub;
+    if (!leader) continue;
+    uint32_t deg = 0, cnt = 0, mask = 0, maxt = 0;
+    for (uint32_t q = r; q < nrec; ++q) {
+      const uint32_t sq = ring_slot(j0 + q);
+      const uint32_t tq = R.tid[sq];
+      if (((tq & 31u) >> ws) != sub) continue;
+      cnt++;
+      mask |= 1u << (tq & 31u);
+      maxt = max(maxt, tq);
+      if (!bb) {
+        const uint64_t lq = R.addr[sq] >> A.lbs_md;
+        bool first = true;
+        for (uint32_t u = r; u < q && first; ++u) {
+          const uint32_t su = ring_slot(j0 + u);
+          if (((R.tid[su] & 31u) >> ws) == sub && (R.addr[su] >> A.lbs_md) == lq) first = false;
+        }
+        deg += first;
+      }
+    }
+    if ((uint32_t)__popc(mask) != cnt) { report(A.sc, c_lo + j0 + r, 2); continue; }
+    const uint32_t s = A.nsites ? R.site[sr] : 0u;
+    if (bb) finish_bd(A, C, acc, sites_smem, cnt, s, R.cta[sr], tr >> ws, maxt);
+    else finish_md(A, C, whist, sites_smem, R.meta[sr] & 3u, deg, s);
+  }
+  if (acc.bd_exec) { atomicAdd(&C.bd_tot[0], acc.bd_exec); atomicAdd(&C.bd_tot[2], acc.bd_threads); }
+}
+
+// run aggregates packed for the segmented scans: deg | cnt << 10 | viol << 20
+constexpr uint32_t PK_CNT = 10, PK_VIOL = 20, PK_M = 1023;
+
+// Finalizes the queued complete runs (one per lane, the warp converged).  A
+// run is one warp32 instruction of one CTA: with W = 32 it is the group, and
+// when its lines never decrease (viol = 0) deg = the number of line changes.
+template <int F>
+__device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
+                                        const RingView R, const uint32_t* qj, const uint32_t* qu,
+                                        const uint32_t* qm, uint32_t qn, uint64_t c_lo) {
+  constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
+  const uint32_t lane = lane_id();
+  uint32_t exec = 0, thr = 0;
+  for (uint32_t q0 = 0; q0 < qn; q0 += 32) {
+    const uint32_t q = q0 + lane;
+    bool md = false, bd = false;
+    uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0;
+    if (q < qn) {
+      j = qj[q];
+      u = qu[q];
+      m = qm[q];
+      const uint32_t sl = ring_slot(j);
+      kind = R.meta[sl] & 3u;
+      t = R.tid[sl];
+      cta = R.cta[sl];
+      s = A.nsites ? R.site[sl] : 0u;
+      const bool bb = kind == 2u;
+      if (bb ? BD : MD) {
+        const uint32_t cnt = (u >> PK_CNT) & PK_M;
+        if ((u >> PK_VIOL) || (bb ? A.ws_bd : A.ws_md) != 5u || cnt > 32) walk_run<F>(A, C, whist, sites_smem, R, j, cnt, c_lo);
+        else if ((uint32_t)__popc(m) != cnt) report(A.sc, c_lo + j, 2);
+        else if (bb) bd = true;
+        else md = true;
+      }
+    }
+    if (MD && md) finish_md(A, C, whist, sites_smem, kind, u & PK_M, s);
+    if (BD) {
+      const uint32_t cnt = (u >> PK_CNT) & PK_M;
+      if (bd) {
+        exec += 1;
+        thr += cnt;
+        red_max(A.tc + cta, ((t & ~31u) | (31u - __clz(m))) + 1u);
+        if (sites_smem) {
+          if (s < A.nsites) { atomicAdd(&C.bd_sites[3 * s], 1u); atomicAdd(&C.bd_sites[3 * s + 2], cnt); }
+          else *A.site_flag = 1;
+        } else if (A.nsites) {
+          site_add(A, nullptr, A.bd_sites, 3, s, 1, cnt);
+        }
+      }
+      // groups with fewer than 32 active lanes wait for T_c (warp-aggregated append)
+      const bool need = bd && cnt < 32u;
+      const uint32_t dm = __ballot_sync(FULL, need);
+      if (dm) {
+        const uint32_t leader = __ffs(dm) - 1;
+        unsigned long long b = 0;
+        if (lane == leader) b = atomicAdd(A.ndefer, (unsigned long long)__popc(dm));
+        b = __shfl_sync(FULL, b, leader);
+        if (need)
+          A.defer[b + __popc(dm & lanemask_lt())] = make_uint4(cta, t >> 5, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
+      }
+    }
+  }
+  if (BD) {
+    exec = __reduce_add_sync(FULL, exec);
+    thr = __reduce_add_sync(FULL, thr);
+    if (lane == 0 && exec) { atomicAdd(&C.bd_tot[0], exec); atomicAdd(&C.bd_tot[2], thr); }
+  }
+}
+
+// Segmented suffix scans: lane l gets the sum (OR) of lanes l .. h, h the
+// first lane >= l whose head flag is set (h = 31 if none).
+__device__ __forceinline__ void seg_scan2(uint32_t& v, uint32_t& m, uint32_t head) {
+  const uint32_t lane = lane_id();
+  uint32_t h = head;
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    const uint32_t vo = __shfl_down_sync(FULL, v, d), mo = __shfl_down_sync(FULL, m, d),
+                   ho = __shfl_down_sync(FULL, h, d);
+    if (lane + d < 32 && !h) { v += vo; m |= mo; h = ho; }
+  }
+}
+
 template <int F>
 __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
   constexpr bool RD = (F & F_RD) != 0, MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
@@ -204,12 +376,17 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
   uint32_t* sites = (uint32_t*)(smem + NWARP * R_BYTES);
   uint32_t* wh_all = sites + ((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM;
   const bool sites_smem = A.nsites && A.nsites <= NSITE_SMEM;
-  Counters C{s_md_hist, (MD && sites_smem) ? sites : nullptr, s_bd_tot,
-             (BD && sites_smem) ? sites + (MD ? 2 * NSITE_SMEM : 0) : nullptr};
+  const Counters C{s_md_hist, (MD && sites_smem) ? sites : nullptr, s_bd_tot,
+                   (BD && sites_smem) ? sites + (MD ? 2 * NSITE_SMEM : 0) : nullptr};
   for (uint32_t k = tx; k < 2 * 33; k += NTHR) s_md_hist[k] = 0;
   if (tx < 3) s_bd_tot[tx] = 0;
   if (sites_smem)
     for (uint32_t k = tx; k < (uint32_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM; k += NTHR) sites[k] = 0;
+  uint32_t* whist = wh_all + warp * 68;  // warp-private MD histogram [2][33]
+  uint32_t* qj = wh_all + NWARP * 68 + warp * QCAP * 3;  // queue of complete runs: start, aggregate, lanes
+  uint32_t* qu = qj + QCAP;
+  uint32_t* qm = qu + QCAP;
+  for (uint32_t k = lane; k < 68; k += 32) whist[k] = 0;
   __syncthreads();
 
   uint8_t* ring = smem + warp * R_BYTES;
@@ -217,37 +394,29 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
   const uint64_t gw = (uint64_t)blockIdx.x * NWARP + warp;
   const uint64_t c_lo = gw * A.chunk;
   const uint64_t c_hi = c_lo + A.chunk < A.n ? c_lo + A.chunk : A.n;
-  uint32_t kept = 0, ndup = 0, bd_exec = 0, bd_threads = 0;
-  uint32_t* whist = wh_all + warp * 68;  // warp-private MD histogram [2][33]
-  for (uint32_t k = lane; k < 68; k += 32) whist[k] = 0;
-  __syncwarp();
+  uint32_t kept = 0, ndup = 0;
   if (c_lo < A.n) {
     const uint32_t clen = (uint32_t)(c_hi - c_lo);
-    const uint64_t s_end = c_hi + 32 < A.n ? c_hi + 32 : A.n;     // lookahead for the last runs
+    // the chunk's last run may reach 32 records past its end; one more record
+    // decides whether the last kept reuse record is followed by a duplicate
+    const uint64_t s_end = c_hi + 32 < A.n ? c_hi + 32 : A.n;
     const uint32_t slen = (uint32_t)(s_end - c_lo);
     const uint32_t npieces = (slen + KR - 1) / KR;
-    const uint64_t nrel64 = A.n - c_lo;
-    const uint32_t nrel = nrel64 < 0xffffffffull ? (uint32_t)nrel64 : 0xffffffffu;
     if (lane == 0) {
       for (int s = 0; s < KS; ++s) mbar_init(&bar[s], 1);
       fence_barrier_init();
     }
     __syncwarp();
-    uint32_t issued = 0, waited = 0;
     Issuer<F> io;
     io.init(A, ring, bar, c_lo, s_end);
+    uint32_t issued = npieces < 2 ? npieces : 2, waited = 0;
     if (lane == 0)
-      for (; issued < (uint32_t)KS && issued < npieces; ++issued) io.issue(issued);
-    issued = __shfl_sync(FULL, issued, 0);
-    const uint64_t* r_addr = (const uint64_t*)(ring + R_ADDR);
-    const uint32_t* r_cta = (const uint32_t*)(ring + R_CTA);
-    const uint16_t* r_tid = (const uint16_t*)(ring + R_TID);
-    const uint32_t* r_winst = (const uint32_t*)(ring + R_WINST);
-    const uint32_t* r_site = (const uint32_t*)(ring + R_SITE);
-    const uint8_t* r_meta = ring + R_META;
-
-    // previous record (the one before the batch), warp-uniform
-    uint32_t p_cta = 0xffffffffu, p_tm = 3u << 16, p_winst = 0;  // meta 3: "no record"
+      for (uint32_t p = 0; p < issued; ++p) io.issue(p);
+    const RingView R{(const uint64_t*)(ring + R_ADDR), (const uint32_t*)(ring + R_CTA),
+                     (const uint16_t*)(ring + R_TID),  (const uint32_t*)(ring + R_WINST),
+                     (const uint32_t*)(ring + R_SITE), ring + R_META};
+    // the record before the step (warp-uniform); meta 3 = "no record"
+    uint32_t p_cta = 0xffffffffu, p_tm = 3u << 16, p_winst = 0;
     uint64_t p_addr = 0;
     if (c_lo > 0) {
       p_cta = __ldg(A.cta + c_lo - 1);
@@ -258,266 +427,271 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       p_tm = (pm0 << 16) | (NG ? (uint32_t)__ldg(A.tid + c_lo - 1) : 0u);
       if (NG) p_winst = __ldg(A.winst + c_lo - 1);
     }
-    uint32_t p_rk = run_hi(p_tm & 0xffffu, p_tm >> 16);
-    // RD carried state; r_* = the chunk's last record seen by the compression
-    bool pv = false, pst = false, r_mem = false;
-    uint64_t r_line = 0;
-    uint32_t r_scope = 0;
-    uint64_t pline = 0;
-    uint32_t pscope = 0, pw = 0, cstart = 0;  // cstart: chunk-relative index of the current store chain start
+    // the run open at the step end (warp-uniform); owned iff it starts in the chunk
+    bool cr_on = false, cr_own = false;
+    uint32_t cr_v = 0, cr_mask = 0, cr_j = 0;
+    // RD: the last kept record when its compression run reaches the step end
+    bool open_rd = false;
     uint64_t* wbv = A.vout ? A.vout + gw * A.chunk : nullptr;
     uint32_t* wbk = A.kout ? A.kout + gw * A.chunk : nullptr;
-    const uint32_t ws_md = A.ws_md, ws_bd = A.ws_bd;
 
-    uint32_t g = 0;
-    while (g < clen) {
-      // ---- pieces needed for records [g, g + 33)
-      const uint32_t need = (g + 33 < slen) ? g + 33 : slen;
-      while (waited * KR < need) {
-        mbar_wait(&bar[waited % KS], (waited / KS) & 1u);
-        ++waited;
+    for (uint32_t p = 0; p < npieces; ++p) {
+      const uint32_t base = p * KR;
+      if (base >= clen && !(NG && cr_on && cr_own) && !(RD && open_rd)) break;
+      mbar_wait(&bar[p % KS], (p / KS) & 1u);
+      waited = p + 1;
+      // ---- this lane's LPR consecutive records (vector shared-memory loads)
+      const uint32_t j0 = base + lane * LPR;
+      const uint32_t sl = ring_slot(j0);
+      uint32_t c[LPR], tm[LPR], w[LPR], mmx, mmy, tor = 0;
+      uint64_t a[LPR];
+      {
+        const uint4 c0 = *(const uint4*)(R.cta + sl), c1 = *(const uint4*)(R.cta + sl + 4);
+        c[0] = c0.x; c[1] = c0.y; c[2] = c0.z; c[3] = c0.w; c[4] = c1.x; c[5] = c1.y; c[6] = c1.z; c[7] = c1.w;
+        const uint2 mm = *(const uint2*)(R.meta + sl);
+        mmx = mm.x;
+        mmy = mm.y;
+        uint32_t tt[LPR];
+        if (NG) {
+          const uint4 t4 = *(const uint4*)(R.tid + sl);
+          tor = t4.x | t4.y | t4.z | t4.w;
+          tt[0] = t4.x & 0xffffu; tt[1] = t4.x >> 16; tt[2] = t4.y & 0xffffu; tt[3] = t4.y >> 16;
+          tt[4] = t4.z & 0xffffu; tt[5] = t4.z >> 16; tt[6] = t4.w & 0xffffu; tt[7] = t4.w >> 16;
+          const uint4 w0 = *(const uint4*)(R.winst + sl), w1 = *(const uint4*)(R.winst + sl + 4);
+          w[0] = w0.x; w[1] = w0.y; w[2] = w0.z; w[3] = w0.w; w[4] = w1.x; w[5] = w1.y; w[6] = w1.z; w[7] = w1.w;
+        } else {
+#pragma unroll
+          for (int k = 0; k < LPR; ++k) tt[k] = w[k] = 0;
+        }
+#pragma unroll
+        for (int k = 0; k < LPR; ++k) tm[k] = ((((k < 4 ? mm.x : mm.y) >> ((k & 3) * 8)) & 0xffu) << 16) | tt[k];
+        if (NA) {
+#pragma unroll
+          for (int q = 0; q < LPR / 2; ++q) {
+            const uint4 v = *(const uint4*)(R.addr + sl + 2 * q);
+            a[2 * q] = ((uint64_t)v.y << 32) | v.x;
+            a[2 * q + 1] = ((uint64_t)v.w << 32) | v.z;
+          }
+        } else {
+#pragma unroll
+          for (int k = 0; k < LPR; ++k) a[k] = 0;
+        }
       }
-      // ---- this batch's records (tm = tid | meta << 16)
-      const uint32_t j = g + lane;
-      const bool inb = j < slen;
-      const uint32_t slot = ring_slot(j);
-      uint32_t c = 0xfffffffeu, tm = 3u << 16, w = 0;
-      uint64_t a = 0;
-      if (inb) {
-        c = r_cta[slot];
-        tm = ((uint32_t)r_meta[slot] << 16) | (NG ? (uint32_t)r_tid[slot] : 0u);
-        if (NG) w = r_winst[slot];
-        if (NA) a = r_addr[slot];
+      // owned / in-stream records of the lane (all of them except near the chunk end)
+      const uint32_t ownm = j0 >= clen ? 0u : (clen - j0 >= LPR ? 0xffu : (1u << (clen - j0)) - 1u);
+      const uint32_t inbm = j0 >= slen ? 0u : (slen - j0 >= LPR ? 0xffu : (1u << (slen - j0)) - 1u);
+      if (base + KR > slen) {  // the stream's last piece: records past it are "no record"
+#pragma unroll
+        for (int k = 0; k < LPR; ++k)
+          if (!((inbm >> k) & 1u)) { tm[k] = 3u << 16; c[k] = 0xfffffffeu; w[k] = 0; a[k] = 0; }
       }
-      // predecessor record
-      uint32_t pc = __shfl_up_sync(FULL, c, 1), ptm = __shfl_up_sync(FULL, tm, 1), pwi = __shfl_up_sync(FULL, w, 1);
-      const uint32_t rk = run_hi(tm & 0xffffu, tm >> 16);
-      uint32_t prk = __shfl_up_sync(FULL, rk, 1);
-      if (lane == 0) prk = p_rk;
-      uint64_t pa = __shfl_up_sync(FULL, a, 1);
+      // validation: SWAR checks over the lane's 8 records, exact per record only if one fails
+      {
+        uint32_t bad = 0;
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          const uint32_t v = h ? mmy : mmx;
+          const uint32_t lo = v & 0x01010101u, hi = (v >> 1) & 0x01010101u;
+          bad |= (lo & hi) | ((v >> 5) & 0x07070707u) |                              // kind 3, reserved bits
+                 ((v >> 4) & ((v >> 3) | (v >> 2)) & 0x01010101u & ~(hi & ~lo));   // memory size > 16 B
+        }
+        if (NA) {
+#pragma unroll
+          for (int k = 0; k < LPR; ++k) {
+            const uint32_t m = tm[k] >> 16;
+            const uint32_t msk = (1u << ((m >> 2) & 7u)) - 1u;
+            if (!(m & 2u)) bad |= ((uint32_t)a[k] & msk) | ((uint32_t)(a[k] >> 32) & 0xfc000000u);
+          }
+        }
+        if (NG) bad |= tor & 0xfc00fc00u;
+        if (__any_sync(FULL, bad != 0)) {
+#pragma unroll
+          for (int k = 0; k < LPR; ++k) {
+            if (!((ownm >> k) & 1u)) continue;
+            const uint8_t m = (uint8_t)(tm[k] >> 16);
+            bool ok = meta_ok(m);
+            if (NA && ok && is_mem(m)) ok = addr_ok(a[k], m);
+            if (NG && ok) ok = (tm[k] & 0xffffu) < 1024u;
+            if (!ok) {
+              report(A.sc, c_lo + j0 + k, 1);
+              tm[k] = (3u << 16) | (tm[k] & 0xffffu);
+            }
+          }
+        }
+      }
+      // predecessor of record 0: the previous lane's last record (lane 0: the carry)
+      uint32_t pc = __shfl_up_sync(FULL, c[LPR - 1], 1), ptm = __shfl_up_sync(FULL, tm[LPR - 1], 1);
+      uint32_t pwi = NG ? __shfl_up_sync(FULL, w[LPR - 1], 1) : 0u;
+      uint64_t pa = NA ? __shfl_up_sync(FULL, a[LPR - 1], 1) : 0ull;
       if (lane == 0) { pc = p_cta; ptm = p_tm; pwi = p_winst; pa = p_addr; }
-      uint32_t m = tm >> 16;
-      const uint32_t t = tm & 0xffffu, pm = ptm >> 16, pt = ptm & 0xffffu;
-      // ---- run structure (only needed for the divergence analyses)
-      uint32_t adv;
-      uint32_t S = 0, e32 = 1;
-      bool rs = true;
-      if (NG) {
-        rs = !inb || c != pc || w != pwi || rk != prk;
-        S = __ballot_sync(FULL, rs);
-        // does the record after the batch start a new run?
-        const uint32_t j32 = g + 32;
-        const uint32_t c31 = __shfl_sync(FULL, c, 31), rk31 = __shfl_sync(FULL, rk, 31),
-                       w31 = __shfl_sync(FULL, w, 31);
-        if (j32 < nrel) {
-          const uint32_t s32 = ring_slot(j32);
-          const uint32_t c32 = r_cta[s32], tm32 = ((uint32_t)r_meta[s32] << 16) | r_tid[s32], w32 = r_winst[s32];
-          e32 = (c32 != c31 || w32 != w31 || run_hi(tm32 & 0xffffu, tm32 >> 16) != rk31) ? 1u : 0u;
+
+      // ================= R1: run compression of the chunk's records
+      if (RD) {
+        uint32_t keepm = 0, dupm = 0, mrgm = 0, stm = 0;
+        uint64_t line[LPR];
+        uint32_t scope[LPR];
+#pragma unroll
+        for (int k = 0; k < LPR; ++k) {
+          const uint32_t kd = (tm[k] >> 16) & 3u, qk = ((k == 0 ? ptm : tm[k - 1]) >> 16) & 3u;
+          line[k] = a[k] >> A.lbs_rd;
+          scope[k] = A.cta_scope ? c[k] : 0u;
+          const uint64_t ql = (k == 0 ? pa : a[k - 1]) >> A.lbs_rd;
+          const uint32_t qs = A.cta_scope ? (k == 0 ? pc : c[k - 1]) : 0u;
+          const bool same = kd < 2u && qk < 2u && scope[k] == qs && line[k] == ql;
+          const bool dup = same && kd == 0u;                   // a load repeating its predecessor: RD 0
+          const bool mrg = k > 0 && same && kd == 1u && qk == 1u;  // store chains merge inside a lane
+          if (dup) dupm |= 1u << k;
+          if (mrg) mrgm |= 1u << k;
+          if (kd < 2u && !dup && !mrg) keepm |= 1u << k;
+          if (kd == 1u) stm |= 1u << k;
         }
-      }
-      const uint32_t S1 = S | 1u;                                   // lane 0 always opens a (pseudo) run
-      const uint32_t gs = 31u - __clz(S1 & lanemask_le());          // first lane of this lane's run
-      const bool complete = (S1 & ~lanemask_le() & ~((1u << gs) - 1u)) != 0 || e32;
-      const bool real = (S >> gs) & 1u;                             // the run starts inside the batch
-      const bool owned = real && (g + gs) < clen;
-      if (NG) {
-        const uint32_t inc = __ballot_sync(FULL, lane == gs && !complete);
-        if (inc & 1u) {
-          // the batch's first run is longer than 32 records
-          if (lane == 0) report(A.sc, c_lo + g, 2);
-          break;
+        keepm &= ownm;
+        mrgm &= ownm;
+        // has_dup of a run reaching the lane end: the next lane's first record
+        const uint32_t nfd = __shfl_down_sync(FULL, dupm & 1u, 1);
+        if (open_rd && lane == 0 && (dupm & 1u)) wbv[kept - 1] |= 1ull << VB_DUP;  // the previous step's open run
+        const uint32_t nk = __popc(keepm);
+        uint32_t x = nk;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t y = __shfl_up_sync(FULL, x, o);
+          if (lane >= (uint32_t)o) x += y;
         }
-        adv = inc ? (uint32_t)(__ffs(inc) - 1) : 32u;
-        if (g + adv > slen) adv = slen - g;
-      } else {
-        adv = (slen - g) < 32u ? (slen - g) : 32u;
-      }
-      // ---- per-record validity (each record of the chunk once)
-      if (lane < adv && j < clen) {
-        bool ok = meta_ok((uint8_t)m);
-        if (NA && ok && is_mem((uint8_t)m)) ok = addr_ok(a, (uint8_t)m);
-        if (NG && ok) ok = t < 1024u;
-        if (!ok) {
-          report(A.sc, c_lo + j, 1);
-          m = 3;  // treat as "no record" below
+        const uint32_t tot = __shfl_sync(FULL, x, 31);
+        uint32_t pos = kept + x - nk;
+        bool last_open = false;
+#pragma unroll
+        for (int k = 0; k < LPR; ++k) {
+          if (!((keepm >> k) & 1u)) continue;
+          const uint32_t after = ~mrgm & (0xffu << (k + 1)) & 0xffu;   // first record after the merged chain
+          const uint32_t e = after ? (uint32_t)(__ffs(after) - 1) : (uint32_t)LPR;
+          const bool hd = e < LPR ? ((dupm >> e) & 1u) != 0 : (lane < 31 && nfd != 0);
+          last_open = e == LPR && lane == 31;
+          wbv[pos] = line[k] | ((uint64_t)((stm >> k) & 1u) << VB_STORE) | ((uint64_t)hd << VB_DUP) |
+                     ((uint64_t)(e - k - 1) << VB_W);
+          if (wbk) wbk[pos] = scope[k];
+          ++pos;
         }
-      }
-      const bool part = inb && owned && complete;
-      const uint32_t lt = t & 31u, plt = pt & 31u;
-      const bool pmem = part && (m & 3u) < 2u;
-      const bool pbb = part && (m & 3u) == 2u;
-      // ---- M1-M3 memory divergence
-      if (MD && __any_sync(FULL, pmem)) {
-        const uint64_t line = a >> A.lbs_md, pl = pa >> A.lbs_md;
-        const bool gst = rs || ((lt ^ plt) >> ws_md) != 0;
-        const bool bad = pmem && !rs && (lt <= plt || (!gst && line < pl));
-        uint32_t LEAD, deg;
-        if (!__any_sync(FULL, bad)) {
-          const uint32_t SG = __ballot_sync(FULL, gst);
-          const uint32_t nxg = SG & ~lanemask_le();
-          const uint32_t ge = nxg ? (uint32_t)(__ffs(nxg) - 1) : 32u;
-          const uint32_t NL = __ballot_sync(FULL, pmem && (gst || line != pl));
-          deg = __popc(NL & bits_from(lane, ge));
-          LEAD = __ballot_sync(FULL, pmem && gst);
-        } else {
-          const uint32_t sub = lt >> ws_md;
-          const uint32_t tag = pmem ? ((gs << 5) | sub) : (1024u + lane);
-          const uint32_t mt = __match_any_sync(FULL, tag);
-          const uint32_t ml = __match_any_sync(FULL, pmem ? line : (~0ull - lane));
-          const uint32_t fl = __ballot_sync(FULL, pmem && (uint32_t)(__ffs(mt & ml) - 1) == lane);
-          const uint32_t ln = __match_any_sync(FULL, pmem ? ((gs << 5) | lt) : (2048u + lane));
-          if (pmem && __popc(ln) > 1) report(A.sc, c_lo + j, 2);
-          deg = __popc(fl & mt);
-          LEAD = __ballot_sync(FULL, pmem && (uint32_t)(__ffs(mt) - 1) == lane);
-        }
-        const uint32_t s = inb ? r_site[slot] : 0u;
-        // leaders update the counters in parallel (shared-memory atomics)
-        if ((LEAD >> lane) & 1u) {
-          atomicAdd(&whist[(m & 3u) * 33 + deg], 1u);
-          if (sites_smem) {
-            if (s < A.nsites) { atomicAdd(&C.md_sites[2 * s], 1u); atomicAdd(&C.md_sites[2 * s + 1], deg); }
-            else *A.site_flag = 1;
-          } else if (A.nsites) {
-            site_add(A, nullptr, A.md_sites, 2, s, 1, deg);
-          }
-        }
-      }
-      // ---- B1-B3 branch divergence
-      if (BD && __any_sync(FULL, pbb)) {
-        const uint32_t W = 1u << ws_bd;
-        const bool gst = rs || ((lt ^ plt) >> ws_bd) != 0;
-        const bool bad = pbb && !rs && lt <= plt;
-        uint32_t LEAD, cnt;
-        const uint32_t CN = __ballot_sync(FULL, pbb);
-        if (!__any_sync(FULL, bad)) {
-          const uint32_t SG = __ballot_sync(FULL, gst);
-          const uint32_t nxg = SG & ~lanemask_le();
-          const uint32_t ge = nxg ? (uint32_t)(__ffs(nxg) - 1) : 32u;
-          cnt = __popc(CN & bits_from(lane, ge));
-          LEAD = __ballot_sync(FULL, pbb && gst);
-          // the group's last lane holds its largest tid
-          if (pbb && ge == lane + 1u) red_max(A.tc + c, t + 1u);
-        } else {
-          const uint32_t sub = lt >> ws_bd;
-          const uint32_t tag = pbb ? ((gs << 5) | sub) : (1024u + lane);
-          const uint32_t mt = __match_any_sync(FULL, tag);
-          const uint32_t ln = __match_any_sync(FULL, pbb ? ((gs << 5) | lt) : (2048u + lane));
-          if (pbb && __popc(ln) > 1) report(A.sc, c_lo + j, 2);
-          cnt = __popc(mt);
-          LEAD = __ballot_sync(FULL, pbb && (uint32_t)(__ffs(mt) - 1) == lane);
-          if (pbb) red_max(A.tc + c, t + 1u);
-        }
-        bd_exec += __popc(LEAD);
-        bd_threads += __popc(CN);
-        const uint32_t s = inb ? r_site[slot] : 0u;
-        // leaders update the per-site counters (shared-memory atomics, different sites in parallel)
-        const bool lead = (LEAD >> lane) & 1u;
-        if (lead) {
-          if (sites_smem) {
-            if (s < A.nsites) { atomicAdd(&C.bd_sites[3 * s], 1u); atomicAdd(&C.bd_sites[3 * s + 2], cnt); }
-            else *A.site_flag = 1;
-          } else if (A.nsites) {
-            site_add(A, nullptr, A.bd_sites, 3, s, 1, cnt);
-          }
-        }
-        // groups with fewer than W lanes: divergence decided once T_c is known
-        const bool dfr = lead && cnt < W;
-        const uint32_t MDF = __ballot_sync(FULL, dfr);
-        if (MDF) {
-          unsigned long long base = 0;
-          if (lane == 0) base = atomicAdd(A.ndefer, (unsigned long long)__popc(MDF));
-          base = __shfl_sync(FULL, base, 0);
-          if (dfr)
-            A.defer[base + __popc(MDF & lanemask_lt())] =
-                make_uint4(c, t >> ws_bd, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
-        }
-      }
-      // ---- R1 run compression over the consumed records of this chunk
-      const uint32_t rlim = (clen - g) < adv ? (clen - g) : adv;
-      const bool rd_any = RD && __any_sync(FULL, lane < rlim && (m & 3u) < 2u);
-      if (RD && !rd_any) {
-        // no memory record in this batch: close the carried record, forget the predecessor
-        if (pv) {
-          if (lane == 0) {
-            wbv[kept] = pline | ((uint64_t)pst << VB_STORE) | ((uint64_t)(pw - 1) << VB_W);
-            if (wbk) wbk[kept] = pscope;
-          }
-          kept++;
-          pv = false;
-        }
-        if (rlim) r_mem = false;
-      }
-      if (RD && rd_any) {
-        const uint32_t lim = rlim;  // records of this chunk in the batch
-        const bool valid = lane < lim;
-        const bool mem = valid && (m & 3u) < 2u;
-        const bool st = mem && (m & 3u) == 1u;
-        const uint64_t line = a >> A.lbs_rd;
-        const uint32_t scope = A.cta_scope ? c : 0u;
-        const bool q_mem = (pm & 3u) < 2u;
-        const bool q_st = (pm & 3u) == 1u;
-        const uint64_t q_line = pa >> A.lbs_rd;
-        const uint32_t q_scope = A.cta_scope ? pc : 0u;
-        const bool same = mem && q_mem && scope == q_scope && line == q_line;
-        const bool dup = same && !st;
-        const bool elig = same && st && q_st && !(g == 0 && lane == 0);
-        const uint32_t Mnon = __ballot_sync(FULL, st && !elig);
-        const uint32_t below = Mnon & lanemask_le();
-        const uint32_t cs = below ? g + (31u - __clz(below)) : cstart;
-        const bool merged = elig && ((g + lane - cs) & 15u) != 0;
-        const bool keep = mem && !dup && !merged;
-        const uint32_t Mmerged = __ballot_sync(FULL, merged);
-        const uint32_t Mdup = __ballot_sync(FULL, dup);
-        if (Mnon) cstart = g + (31u - __clz(Mnon));
-        if (pv) {
-          // the record carried from the previous batch ends before the first non-merged lane
-          const uint32_t e = __ffs(~Mmerged) - 1;
-          const uint32_t wgt = pw + (pst ? e : 0u);
-          const bool hd = e < lim && ((Mdup >> e) & 1u);
-          if (lane == 0) {
-            wbv[kept] = pline | ((uint64_t)pst << VB_STORE) | ((uint64_t)hd << VB_DUP) | ((uint64_t)(wgt - 1) << VB_W);
-            if (wbk) wbk[kept] = pscope;
-          }
-          kept++;
-          pv = false;
-        }
-        const uint32_t after = ~Mmerged & ~lanemask_le();
-        const uint32_t e_l = st ? (after ? (uint32_t)(__ffs(after) - 1) : 32u) : lane + 1;
-        const bool fin = keep && e_l < lim;
-        const uint32_t Mfin = __ballot_sync(FULL, fin);
-        if (fin) {
-          const uint32_t pos = kept + __popc(Mfin & lanemask_lt());
-          const bool hd = (Mdup >> e_l) & 1u;
-          wbv[pos] = line | ((uint64_t)st << VB_STORE) | ((uint64_t)hd << VB_DUP) | ((uint64_t)(e_l - lane - 1) << VB_W);
-          if (wbk) wbk[pos] = scope;
-        }
-        kept += __popc(Mfin);
-        const uint32_t Mp = __ballot_sync(FULL, keep && e_l >= lim);
-        if (Mp) {
-          const uint32_t pl_ = __ffs(Mp) - 1;
-          pv = true;
-          pline = __shfl_sync(FULL, line, pl_);
-          pscope = __shfl_sync(FULL, scope, pl_);
-          pst = __shfl_sync(FULL, (uint32_t)st, pl_) != 0;
-          pw = pst ? lim - pl_ : 1u;
-        }
-        ndup += __popc(Mdup);
-        if (lim) {
-          r_mem = __shfl_sync(FULL, (uint32_t)mem, lim - 1) != 0;
-          r_line = __shfl_sync(FULL, line, lim - 1);
-          r_scope = __shfl_sync(FULL, scope, lim - 1);
-        }
-      }
-      // ---- carry the last consumed record, advance, recycle fully consumed pieces
-      const uint32_t last = adv - 1;
-      p_cta = __shfl_sync(FULL, c, last);
-      p_tm = __shfl_sync(FULL, (m << 16) | t, last);
-      p_rk = __shfl_sync(FULL, rk, last);
-      p_winst = __shfl_sync(FULL, w, last);
-      p_addr = __shfl_sync(FULL, a, last);
-      g += adv;
-      while (issued < npieces && g >= (issued - KS + 1) * KR) {
+        open_rd = __shfl_sync(FULL, (uint32_t)last_open, 31) != 0;
+        kept += tot;
+        ndup += __popc(dupm & ownm);
         __syncwarp();
+      }
+
+      // ================= M1-M3 / B1-B3: runs = warp-level groups
+      if (NG) {
+        uint32_t rsm = 0, nlm = 0, vim = 0, bits[LPR];
+        uint32_t prk = run_hi(ptm & 0xffffu, ptm >> 16);
+        uint64_t pl = pa >> A.lbs_md;
+#pragma unroll
+        for (int k = 0; k < LPR; ++k) {
+          const uint32_t t = tm[k] & 0xffffu;
+          const uint32_t rk = run_hi(t, tm[k] >> 16);
+          const uint32_t qc = k == 0 ? pc : c[k - 1], qw = k == 0 ? pwi : w[k - 1];
+          const bool rs = c[k] != qc || w[k] != qw || rk != prk;
+          if (rs) rsm |= 1u << k;
+          if (MD) {
+            const uint64_t l = a[k] >> A.lbs_md;
+            if (rs || l != pl) nlm |= 1u << k;
+            if (!rs && l < pl) vim |= 1u << k;
+            pl = l;
+          }
+          bits[k] = 1u << (t & 31u);
+          prk = rk;
+        }
+        rsm |= ~inbm & 0xffu;  // every record past the stream is a run of its own (never finalized)
+        // per-run aggregates inside the lane (backward): u = packed, m = lane bits
+        uint32_t ru[LPR], rm[LPR];
+        uint32_t u = 0, m = 0;
+#pragma unroll
+        for (int k = LPR - 1; k >= 0; --k) {
+          u += ((nlm >> k) & 1u) | (1u << PK_CNT) | (((vim >> k) & 1u) << PK_VIOL);
+          m |= bits[k];
+          ru[k] = u;
+          rm[k] = m;
+          if ((rsm >> k) & 1u) { u = 0; m = 0; }
+        }
+        // u / m now hold the lane's prefix (records before its first run start)
+        const uint32_t head = rsm != 0;
+        seg_scan2(u, m, head);
+        const uint32_t S_next = __shfl_down_sync(FULL, u, 1), M_next = __shfl_down_sync(FULL, m, 1);
+        const uint32_t heads = __ballot_sync(FULL, head);
+        uint32_t qn = 0;
+        // ---- the run carried in from the previous step ends at the first head
+        if (cr_on) {
+          cr_v += __shfl_sync(FULL, u, 0);
+          cr_mask |= __shfl_sync(FULL, m, 0);
+          if (((cr_v >> PK_CNT) & PK_M) > 32) {  // a lane repeats: bad trace (stop counting)
+            if (lane == 0 && cr_own) report(A.sc, c_lo + cr_j, 2);
+            cr_own = false;
+          }
+          if (heads) {
+            if (cr_own) {
+              if (lane == 0) { qj[0] = cr_j; qu[0] = cr_v; qm[0] = cr_mask; }
+              qn = 1;
+            }
+            cr_on = false;
+          }
+        }
+        // ---- runs starting in this lane that end in this step are queued
+        const bool above = (heads & ~lanemask_le()) != 0;
+        const uint32_t lastk = rsm ? 31u - __clz(rsm) : 0u;
+        const uint32_t starts = rsm & inbm;
+        const bool tail_open = !above && ((starts >> lastk) & 1u);  // continues past the step end
+        const uint32_t todo = starts & ownm & ~(tail_open ? 1u << lastk : 0u);
+#pragma unroll
+        for (int k = 0; k < LPR; ++k) {
+          const bool it = (todo >> k) & 1u;
+          const uint32_t im = __ballot_sync(FULL, it);
+          if (im) {
+            if (it) {
+              uint32_t u2 = ru[k], m2 = rm[k];
+              if ((uint32_t)k == lastk) { u2 += S_next; m2 |= M_next; }  // closed by a later lane's head
+              const uint32_t pos = qn + __popc(im & lanemask_lt());
+              qj[pos] = j0 + k;
+              qu[pos] = u2;
+              qm[pos] = m2;
+            }
+            qn += __popc(im);
+          }
+          if (k == LPR / 2 - 1 && qn > QCAP - 32 * LPR / 2) {
+            __syncwarp();
+            flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qn, c_lo);
+            qn = 0;
+            __syncwarp();
+          }
+        }
+        if (qn) {
+          __syncwarp();
+          flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qn, c_lo);
+        }
+        // ---- the last head lane's open run becomes the carry
+        if (heads) {
+          const uint32_t hl = 31u - __clz(heads);
+          uint32_t tu = 0, tmk = 0;
+          if (tail_open) {
+            const uint32_t msk = 0xffu << lastk;
+            tu = __popc(nlm & msk) | ((LPR - lastk) << PK_CNT) | (__popc(vim & msk) << PK_VIOL);
+#pragma unroll
+            for (int k = 0; k < LPR; ++k)
+              if ((uint32_t)k >= lastk) tmk |= bits[k];
+            if (lane < 31) { tu += S_next; tmk |= M_next; }
+          }
+          cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
+          cr_v = __shfl_sync(FULL, tu, hl);
+          cr_mask = __shfl_sync(FULL, tmk, hl);
+          cr_j = __shfl_sync(FULL, j0 + lastk, hl);
+          cr_own = cr_j < clen;
+        }
+        __syncwarp();
+      }
+      // ---- carry the step's last record; recycle piece p - 1 for piece p + 2
+      p_cta = __shfl_sync(FULL, c[LPR - 1], 31);
+      p_tm = __shfl_sync(FULL, tm[LPR - 1], 31);
+      if (NG) p_winst = __shfl_sync(FULL, w[LPR - 1], 31);
+      if (NA) p_addr = __shfl_sync(FULL, a[LPR - 1], 31);
+      __syncwarp();
+      if (p >= 1 && issued < npieces) {
         if (lane == 0) {
           fence_proxy_async();
           io.issue(issued);
@@ -525,36 +699,21 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
         ++issued;
       }
     }
-    // ---- drain the pieces still in flight (their barriers must complete before exit)
-    while (waited < issued) {
-      mbar_wait(&bar[waited % KS], (waited / KS) & 1u);
-      ++waited;
+    // a run open at the end of the stream ends with the trace
+    if (NG && cr_on && cr_own) {
+      if (lane == 0) { qj[0] = cr_j; qu[0] = cr_v; qm[0] = cr_mask; }
+      __syncwarp();
+      flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, 1, c_lo);
     }
-    if (RD && pv) {
-      // the record after the chunk decides has_dup (it is never merged into us)
-      bool hd = false;
-      if (c_hi < A.n) {
-        const uint8_t m2 = __ldg(A.meta + c_hi);
-        if (is_mem(m2) && !is_store(m2) && meta_ok(m2) && r_mem) {
-          const uint64_t a2 = __ldg(A.addr + c_hi);
-          const uint32_t s2 = A.cta_scope ? __ldg(A.cta + c_hi) : 0u;
-          hd = addr_ok(a2, m2) && (a2 >> A.lbs_rd) == r_line && s2 == r_scope;
-        }
-      }
-      if (lane == 0) {
-        wbv[kept] = pline | ((uint64_t)pst << VB_STORE) | ((uint64_t)hd << VB_DUP) | ((uint64_t)(pw - 1) << VB_W);
-        if (wbk) wbk[kept] = pscope;
-      }
-      kept++;
-    }
+    // no bulk copy may still target the ring when the CTA exits
+    for (uint32_t q = waited; q < issued; ++q) mbar_wait(&bar[q % KS], (q / KS) & 1u);
   }
   if (RD && lane == 0) {
     A.wcnt[gw] = kept;
-    if (ndup) atomicAdd((unsigned long long*)A.hist0, (unsigned long long)ndup);
   }
-  if (BD && lane == 0) {
-    if (bd_exec) atomicAdd(&s_bd_tot[0], bd_exec);
-    if (bd_threads) atomicAdd(&s_bd_tot[2], bd_threads);
+  if (RD) {
+    const uint32_t d = __reduce_add_sync(FULL, ndup);
+    if (lane == 0 && d) atomicAdd((unsigned long long*)A.hist0, (unsigned long long)d);
   }
   if (MD) {
     __syncwarp();
@@ -630,7 +789,8 @@ __global__ void __launch_bounds__(256) k_squeeze(const uint32_t* __restrict__ ki
 template <int F>
 size_t scan_smem() {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
-  return (size_t)NWARP * R_BYTES + (size_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + (size_t)NWARP * 68 * 4;
+  return (size_t)NWARP * R_BYTES + (size_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + (size_t)NWARP * 68 * 4 +
+         (size_t)NWARP * QCAP * 12;
 }
 
 int g_scan_ready[8] = {0, 0, 0, 0, 0, 0, 0, 0};
