@@ -55,6 +55,9 @@
  *   the trace and receives the identical global result (DESIGN.md
  *   "Multi-GPU").
  * Errors: functions return a cadv_status; details via cadv_last_error().
+ * Environment (testing only): CADV_SCAN_CTAS=n, read by cadv_create, caps
+ *   the streaming pass at n CTAs so that each warp's contiguous chunk spans
+ *   many 256-record steps even for small traces; results do not change.
  */
 #ifndef CADV_H
 #define CADV_H

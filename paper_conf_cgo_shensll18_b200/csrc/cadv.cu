@@ -1,6 +1,7 @@
 // cadv.cu — the C ABI of libcadv (include/cadv.h): context, trace
 // registration + ingest pass R0, and the synchronous analysis entry points.
 #include <cuda_runtime.h>
+#include <cstdlib>
 #include <stdio.h>
 #include <string.h>
 
@@ -243,6 +244,7 @@ CADV_API cadv_status cadv_create(cadv_ctx** out, int device, void* cuda_stream, 
   c->rank = rank;
   c->nranks = nranks;
   c->num_sms = prop.multiProcessorCount;
+  if (const char* e = getenv("CADV_SCAN_CTAS")) c->scan_ctas = atoi(e);
   if (cudaEventCreate(&c->ev0) != cudaSuccess || cudaEventCreate(&c->ev1) != cudaSuccess) {
     delete c;
     return CADV_ERR_CUDA;

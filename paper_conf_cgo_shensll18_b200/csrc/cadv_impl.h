@@ -48,6 +48,7 @@ struct cadv_ctx {
   int rank = 0, nranks = 1;
   void* comm = nullptr;  // ncclComm_t when nranks > 1
   int num_sms = 148;
+  int scan_ctas = 0;     // CADV_SCAN_CTAS (testing): cap on the scan grid, 0 = one CTA per SM
   // registered trace (device pointers)
   bool loaded = false;
   cadv_trace_desc t{};

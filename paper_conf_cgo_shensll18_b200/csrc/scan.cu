@@ -365,7 +365,7 @@ __device__ __forceinline__ void seg_scan2(uint32_t& v, uint32_t& m, uint32_t hea
 }
 
 template <int F>
-__global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
+__global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanArgs A) {
   constexpr bool RD = (F & F_RD) != 0, MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
   extern __shared__ __align__(128) uint8_t smem[];
@@ -526,8 +526,12 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
       if (lane == 0) { pc = p_cta; ptm = p_tm; pwi = p_winst; pa = p_addr; }
 
       // ================= R1: run compression of the chunk's records
+      // dup  : a load repeating its predecessor's (scope, line): RD 0, never kept;
+      // chain: consecutive stores to one (scope, line); every 16th one is kept
+      //        with the weight of the chain piece it heads.  Chains are cut at
+      //        step starts and at the chunk end (both only split a piece).
       if (RD) {
-        uint32_t keepm = 0, dupm = 0, mrgm = 0, stm = 0;
+        uint32_t memm = 0, dupm = 0, contm = 0, stm = 0;
         uint64_t line[LPR];
         uint32_t scope[LPR];
 #pragma unroll
@@ -538,18 +542,31 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
           const uint64_t ql = (k == 0 ? pa : a[k - 1]) >> A.lbs_rd;
           const uint32_t qs = A.cta_scope ? (k == 0 ? pc : c[k - 1]) : 0u;
           const bool same = kd < 2u && qk < 2u && scope[k] == qs && line[k] == ql;
-          const bool dup = same && kd == 0u;                   // a load repeating its predecessor: RD 0
-          const bool mrg = k > 0 && same && kd == 1u && qk == 1u;  // store chains merge inside a lane
-          if (dup) dupm |= 1u << k;
-          if (mrg) mrgm |= 1u << k;
-          if (kd < 2u && !dup && !mrg) keepm |= 1u << k;
+          if (kd < 2u) memm |= 1u << k;
+          if (same && kd == 0u) dupm |= 1u << k;
+          if (same && kd == 1u && qk == 1u) contm |= 1u << k;
           if (kd == 1u) stm |= 1u << k;
         }
+        if (lane == 0) contm &= ~1u;
+        // breaks: records that do not continue a store chain (the chunk end is one)
+        const uint32_t brk = (~contm | ~ownm) & 0xffu;
+        const uint32_t sb = lane * LPR;
+        const uint32_t hb = __ballot_sync(FULL, brk != 0);
+        const uint32_t lt = hb & lanemask_lt(), gt = hb & ~lanemask_le();
+        const uint32_t lastb = brk ? sb + 31u - __clz(brk) : 0u;
+        const uint32_t fb = brk ? (uint32_t)(__ffs(brk) - 1) : 0u;
+        const uint32_t sv = __shfl_sync(FULL, lastb, lt ? 31u - __clz(lt) : 0u);
+        const uint32_t nv = __shfl_sync(FULL, (sb + fb) | (((dupm >> fb) & 1u) << 16), gt ? (uint32_t)(__ffs(gt) - 1) : 0u);
+        const uint32_t nb_l = gt ? (nv & 0xffffu) : (uint32_t)KR;  // first break after the lane
+        const bool nd_l = gt && (nv >> 16);
+        uint32_t start = lt ? sv : 0u, keepm = memm & ~dupm & brk;
+#pragma unroll
+        for (int k = 0; k < LPR; ++k) {
+          if ((brk >> k) & 1u) start = sb + k;
+          else if (((sb + k - start) & 15u) == 0u) keepm |= 1u << k;  // every 16th chain store
+        }
         keepm &= ownm;
-        mrgm &= ownm;
-        // has_dup of a run reaching the lane end: the next lane's first record
-        const uint32_t nfd = __shfl_down_sync(FULL, dupm & 1u, 1);
-        if (open_rd && lane == 0 && (dupm & 1u)) wbv[kept - 1] |= 1ull << VB_DUP;  // the previous step's open run
+        if (open_rd && lane == 0 && (dupm & 1u)) wbv[kept - 1] |= 1ull << VB_DUP;  // the previous step's open piece
         const uint32_t nk = __popc(keepm);
         uint32_t x = nk;
 #pragma unroll
@@ -563,16 +580,20 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(ScanArgs A) {
 #pragma unroll
         for (int k = 0; k < LPR; ++k) {
           if (!((keepm >> k) & 1u)) continue;
-          const uint32_t after = ~mrgm & (0xffu << (k + 1)) & 0xffu;   // first record after the merged chain
-          const uint32_t e = after ? (uint32_t)(__ffs(after) - 1) : (uint32_t)LPR;
-          const bool hd = e < LPR ? ((dupm >> e) & 1u) != 0 : (lane < 31 && nfd != 0);
-          last_open = e == LPR && lane == 31;
+          const uint32_t after = brk & (0xffu << (k + 1)) & 0xffu;
+          const uint32_t ab = after ? (uint32_t)(__ffs(after) - 1) : 0u;
+          const uint32_t nb = after ? sb + ab : nb_l;   // the first break after record k
+          const bool nd = after ? ((dupm >> ab) & 1u) != 0 : nd_l;
+          uint32_t wgt = nb - (sb + k);
+          bool hd = nd;
+          if (wgt > 16u) { wgt = 16u; hd = false; }      // the chain goes on with another kept store
+          else last_open = nb == (uint32_t)KR;           // decided by the next step's first record
           wbv[pos] = line[k] | ((uint64_t)((stm >> k) & 1u) << VB_STORE) | ((uint64_t)hd << VB_DUP) |
-                     ((uint64_t)(e - k - 1) << VB_W);
+                     ((uint64_t)(wgt - 1u) << VB_W);
           if (wbk) wbk[pos] = scope[k];
           ++pos;
         }
-        open_rd = __shfl_sync(FULL, (uint32_t)last_open, 31) != 0;
+        open_rd = __ballot_sync(FULL, last_open) != 0;
         kept += tot;
         ndup += __popc(dupm & ownm);
         __syncwarp();
@@ -814,6 +835,7 @@ cudaError_t launch_scan_t(cadv_ctx* c, const ScanArgs& A, uint64_t grid) {
 // One CTA per SM; every warp a contiguous chunk whose length is a multiple of KR.
 void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nwarps, uint64_t* chunk) {
   uint64_t g = (uint64_t)c->num_sms;
+  if (c->scan_ctas > 0 && (uint64_t)c->scan_ctas < g) g = (uint64_t)c->scan_ctas;
   const uint64_t tw = g * NWARP;
   uint64_t ch = (n + tw - 1) / tw;
   ch = ((ch + KR - 1) / KR) * KR;

@@ -334,3 +334,81 @@ def test_c2_sgemm_full(ctx, cadv):
     t = tg.generate("sgemm", n=256)
     assert t.n == 35782656
     full_check(ctx, cadv, t, lbs=(32, 128), scopes=(0,))
+
+
+# ----------------------------------------------------------------- store chains / long warp chunks
+
+def _chain_trace(seed, n_chains=400, max_len=300):
+    """Store chains of random length (1 .. max_len, also >16 and across lanes,
+    steps and chunks), each followed by 0-3 loads of the same line (duplicates,
+    RD 0) and a few unrelated loads, over a handful of CTAs."""
+    rng = np.random.default_rng(seed)
+    addr, cta, meta = [], [], []
+    for _ in range(n_chains):
+        line = int(rng.integers(0, 64))
+        c = int(rng.integers(0, 3))
+        L = int(rng.choice([1, 2, 15, 16, 17, 31, 32, 33, 255, 256, 257, int(rng.integers(1, max_len))]))
+        base = 0x7F0000000000 + 128 * line
+        addr += [base + 4 * int(o) for o in rng.integers(0, 32, L)]
+        cta += [c] * L
+        meta += [(2 << 2) | 1] * L
+        nd = int(rng.integers(0, 4))
+        addr += [base] * nd
+        cta += [c] * nd
+        meta += [2 << 2] * nd
+        no = int(rng.integers(0, 4))
+        addr += [0x7F0000000000 + 128 * int(x) for x in rng.integers(0, 64, no)]
+        cta += [c] * no
+        meta += [2 << 2] * no
+    n = len(addr)
+    return _mk(np.array(addr, np.uint64), np.array(cta), meta=np.array(meta))
+
+
+@pytest.mark.parametrize("seed", [11, 12, 13])
+def test_store_chains(ctx, cadv, seed):
+    t = _chain_trace(seed)
+    full_check(ctx, cadv, t, lbs=(4, 128), W=(32,))
+
+
+@pytest.fixture(scope="module")
+def ctx_long(cadv):
+    """A context whose streaming pass uses 1 CTA: warp chunks of many 256-record steps."""
+    import os
+    old = os.environ.get("CADV_SCAN_CTAS")
+    os.environ["CADV_SCAN_CTAS"] = "1"
+    try:
+        c = cadv.create(0)
+    finally:
+        if old is None:
+            del os.environ["CADV_SCAN_CTAS"]
+        else:
+            os.environ["CADV_SCAN_CTAS"] = old
+    yield c
+    c.destroy()
+
+
+LONG_CASES = [
+    ("chains", dict(seed=21)),
+    ("rand", dict(seed=4, ctas=8, threads=96, instrs=20, lines=40, pbb=0.5)),
+    ("rand", dict(seed=5, ctas=5, threads=33, instrs=50, lines=3, pstore=0.5)),
+    ("rand", dict(seed=6, ctas=2, threads=1024, instrs=30, lines=200, pstore=0.3)),
+    ("srad", dict(rows=128, cols=128, iters=2)),
+    ("bfs", dict(nodes=20000, seed=3)),
+    ("nw", dict(ctas=3)),
+]
+
+
+@pytest.mark.parametrize("case", range(len(LONG_CASES)))
+def test_long_chunks(ctx_long, cadv, case):
+    name, kw = LONG_CASES[case]
+    t = _chain_trace(kw["seed"]) if name == "chains" else tg.generate(name, **kw)
+    full_check(ctx_long, cadv, t, lbs=(4, 128), W=(32, 8))
+    out = ctx_long.analyze(rd=(128, 1, 0, 66), md=(32, 32), bd=32, nsites=t.nsites)
+    assert (out["reuse"][0] == orc.reuse(t, 128, 1, 0, 66)[0]).all()
+    assert (out["mem_div"][0] == orc.mem_div(t, 32, 32)[0]).all()
+    assert (out["branch_div"][1] == orc.branch_div(t, 32)[1]).all()
+
+
+def test_long_chunks_non_contiguous(ctx_long, cadv):
+    t = tg.generate("rand", seed=7, ctas=6, threads=128, instrs=15, lines=30, scramble=1, scramble_seed=7)
+    full_check(ctx_long, cadv, t, lbs=(32,), contiguous=False, W=(32, 16))
