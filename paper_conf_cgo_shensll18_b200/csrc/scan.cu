@@ -104,6 +104,11 @@ __device__ __forceinline__ void red_max(uint32_t* p, uint32_t v) {
   asm volatile("red.relaxed.gpu.global.max.u32 [%0], %1;" ::"l"(p), "r"(v) : "memory");
 }
 
+// bit 0 of each byte of v -> bits 0..3
+__device__ __forceinline__ uint32_t gather4(uint32_t v) { return ((v & 0x01010101u) * 0x10204080u) >> 28; }
+// bit 0 of each of the 8 bytes (x: bytes 0-3, y: bytes 4-7) -> bits 0..7
+__device__ __forceinline__ uint32_t gather8(uint32_t x, uint32_t y) { return gather4(x) | (gather4(y) << 4); }
+
 // bits [a, e) of a lane mask, 0 <= a < e <= 32
 __device__ __forceinline__ uint32_t bits_from(uint32_t a, uint32_t e) {
   const uint32_t hi = e >= 32 ? FULL : ((1u << e) - 1u);
@@ -416,7 +421,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
                      (const uint16_t*)(ring + R_TID),  (const uint32_t*)(ring + R_WINST),
                      (const uint32_t*)(ring + R_SITE), ring + R_META};
     // the record before the step (warp-uniform); meta 3 = "no record"
-    uint32_t p_cta = 0xffffffffu, p_tm = 3u << 16, p_winst = 0;
+    // p_kb: kind bits of that record (bit 0 memory, 1 store, 2 BB; 0 = invalid / none)
+    uint32_t p_cta = 0xffffffffu, p_t = 0, p_kb = 0, p_winst = 0;
     uint64_t p_addr = 0;
     if (c_lo > 0) {
       p_cta = __ldg(A.cta + c_lo - 1);
@@ -424,7 +430,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       if (NA) p_addr = __ldg(A.addr + c_lo - 1);
       // an invalid record never continues a run of compressible accesses
       if (!meta_ok((uint8_t)pm0) || (NA && is_mem((uint8_t)pm0) && !addr_ok(p_addr, (uint8_t)pm0))) pm0 = 3;
-      p_tm = (pm0 << 16) | (NG ? (uint32_t)__ldg(A.tid + c_lo - 1) : 0u);
+      p_kb = (pm0 & 3u) < 2u ? (1u | ((pm0 & 1u) << 1)) : ((pm0 & 3u) == 2u ? 4u : 0u);
+      if (NG) p_t = __ldg(A.tid + c_lo - 1);
       if (NG) p_winst = __ldg(A.winst + c_lo - 1);
     }
     // the run open at the step end (warp-uniform); owned iff it starts in the chunk
@@ -443,7 +450,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       // ---- this lane's LPR consecutive records (vector shared-memory loads)
       const uint32_t j0 = base + lane * LPR;
       const uint32_t sl = ring_slot(j0);
-      uint32_t c[LPR], tm[LPR], w[LPR], mmx, mmy, tor = 0;
+      uint32_t c[LPR], t[LPR], w[LPR], mmx, mmy, tor = 0;
       uint64_t a[LPR];
       {
         const uint4 c0 = *(const uint4*)(R.cta + sl), c1 = *(const uint4*)(R.cta + sl + 4);
@@ -451,20 +458,17 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         const uint2 mm = *(const uint2*)(R.meta + sl);
         mmx = mm.x;
         mmy = mm.y;
-        uint32_t tt[LPR];
         if (NG) {
           const uint4 t4 = *(const uint4*)(R.tid + sl);
           tor = t4.x | t4.y | t4.z | t4.w;
-          tt[0] = t4.x & 0xffffu; tt[1] = t4.x >> 16; tt[2] = t4.y & 0xffffu; tt[3] = t4.y >> 16;
-          tt[4] = t4.z & 0xffffu; tt[5] = t4.z >> 16; tt[6] = t4.w & 0xffffu; tt[7] = t4.w >> 16;
+          t[0] = t4.x & 0xffffu; t[1] = t4.x >> 16; t[2] = t4.y & 0xffffu; t[3] = t4.y >> 16;
+          t[4] = t4.z & 0xffffu; t[5] = t4.z >> 16; t[6] = t4.w & 0xffffu; t[7] = t4.w >> 16;
           const uint4 w0 = *(const uint4*)(R.winst + sl), w1 = *(const uint4*)(R.winst + sl + 4);
           w[0] = w0.x; w[1] = w0.y; w[2] = w0.z; w[3] = w0.w; w[4] = w1.x; w[5] = w1.y; w[6] = w1.z; w[7] = w1.w;
         } else {
 #pragma unroll
-          for (int k = 0; k < LPR; ++k) tt[k] = w[k] = 0;
+          for (int k = 0; k < LPR; ++k) t[k] = w[k] = 0;
         }
-#pragma unroll
-        for (int k = 0; k < LPR; ++k) tm[k] = ((((k < 4 ? mm.x : mm.y) >> ((k & 3) * 8)) & 0xffu) << 16) | tt[k];
         if (NA) {
 #pragma unroll
           for (int q = 0; q < LPR / 2; ++q) {
@@ -480,50 +484,50 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       // owned / in-stream records of the lane (all of them except near the chunk end)
       const uint32_t ownm = j0 >= clen ? 0u : (clen - j0 >= LPR ? 0xffu : (1u << (clen - j0)) - 1u);
       const uint32_t inbm = j0 >= slen ? 0u : (slen - j0 >= LPR ? 0xffu : (1u << (slen - j0)) - 1u);
-      if (base + KR > slen) {  // the stream's last piece: records past it are "no record"
-#pragma unroll
-        for (int k = 0; k < LPR; ++k)
-          if (!((inbm >> k) & 1u)) { tm[k] = 3u << 16; c[k] = 0xfffffffeu; w[k] = 0; a[k] = 0; }
-      }
-      // validation: SWAR checks over the lane's 8 records, exact per record only if one fails
+      // kind masks (bit k = record k) from the meta bytes
+      const uint32_t glo = gather8(mmx, mmy), ghi = gather8(mmx >> 1, mmy >> 1);
+      uint32_t okm = inbm;
       {
-        uint32_t bad = 0;
+        // validation: SWAR checks over the lane's records, exact per record only if one fails
+        uint32_t badm = 0;
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
           const uint32_t v = h ? mmy : mmx;
           const uint32_t lo = v & 0x01010101u, hi = (v >> 1) & 0x01010101u;
-          bad |= (lo & hi) | ((v >> 5) & 0x07070707u) |                              // kind 3, reserved bits
-                 ((v >> 4) & ((v >> 3) | (v >> 2)) & 0x01010101u & ~(hi & ~lo));   // memory size > 16 B
+          const uint32_t b = (lo & hi) | (((v >> 5) | (v >> 6) | (v >> 7)) & 0x01010101u) |  // kind 3, reserved bits
+                             ((v >> 4) & ((v >> 3) | (v >> 2)) & ~hi & 0x01010101u);        // memory size > 16 B
+          badm |= gather4(b) << (4 * h);
         }
         if (NA) {
 #pragma unroll
           for (int k = 0; k < LPR; ++k) {
-            const uint32_t m = tm[k] >> 16;
-            const uint32_t msk = (1u << ((m >> 2) & 7u)) - 1u;
-            if (!(m & 2u)) bad |= ((uint32_t)a[k] & msk) | ((uint32_t)(a[k] >> 32) & 0xfc000000u);
+            const uint32_t msk = (1u << ((((k < 4 ? mmx : mmy) >> (8 * (k & 3))) >> 2) & 7u)) - 1u;
+            if (!((ghi >> k) & 1u) && (((uint32_t)a[k] & msk) | ((uint32_t)(a[k] >> 32) & 0xfc000000u))) badm |= 1u << k;
           }
         }
-        if (NG) bad |= tor & 0xfc00fc00u;
-        if (__any_sync(FULL, bad != 0)) {
+        badm &= ownm;
+        if (__any_sync(FULL, badm != 0 || (NG && (tor & 0xfc00fc00u)))) {
 #pragma unroll
           for (int k = 0; k < LPR; ++k) {
             if (!((ownm >> k) & 1u)) continue;
-            const uint8_t m = (uint8_t)(tm[k] >> 16);
+            const uint8_t m = (uint8_t)(((k < 4 ? mmx : mmy) >> (8 * (k & 3))) & 0xffu);
             bool ok = meta_ok(m);
             if (NA && ok && is_mem(m)) ok = addr_ok(a[k], m);
-            if (NG && ok) ok = (tm[k] & 0xffffu) < 1024u;
+            if (NG && ok) ok = t[k] < 1024u;
             if (!ok) {
               report(A.sc, c_lo + j0 + k, 1);
-              tm[k] = (3u << 16) | (tm[k] & 0xffffu);
+              okm &= ~(1u << k);
             }
           }
         }
       }
+      const uint32_t memm = ~ghi & okm, stm = glo & ~ghi & okm, bbm = ~glo & ghi & okm;
       // predecessor of record 0: the previous lane's last record (lane 0: the carry)
-      uint32_t pc = __shfl_up_sync(FULL, c[LPR - 1], 1), ptm = __shfl_up_sync(FULL, tm[LPR - 1], 1);
-      uint32_t pwi = NG ? __shfl_up_sync(FULL, w[LPR - 1], 1) : 0u;
+      uint32_t pc = __shfl_up_sync(FULL, c[LPR - 1], 1);
+      uint32_t pkb = __shfl_up_sync(FULL, ((memm >> 7) & 1u) | ((stm >> 6) & 2u) | ((bbm >> 5) & 4u), 1);
+      uint32_t pt = NG ? __shfl_up_sync(FULL, t[LPR - 1], 1) : 0u, pwi = NG ? __shfl_up_sync(FULL, w[LPR - 1], 1) : 0u;
       uint64_t pa = NA ? __shfl_up_sync(FULL, a[LPR - 1], 1) : 0ull;
-      if (lane == 0) { pc = p_cta; ptm = p_tm; pwi = p_winst; pa = p_addr; }
+      if (lane == 0) { pc = p_cta; pkb = p_kb; pt = p_t; pwi = p_winst; pa = p_addr; }
 
       // ================= R1: run compression of the chunk's records
       // dup  : a load repeating its predecessor's (scope, line): RD 0, never kept;
@@ -531,40 +535,31 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       //        with the weight of the chain piece it heads.  Chains are cut at
       //        step starts and at the chunk end (both only split a piece).
       if (RD) {
-        uint32_t memm = 0, dupm = 0, contm = 0, stm = 0;
-        uint64_t line[LPR];
-        uint32_t scope[LPR];
+        uint32_t eqm = 0;
+        const uint64_t lim = 1ull << A.lbs_rd;
 #pragma unroll
         for (int k = 0; k < LPR; ++k) {
-          const uint32_t kd = (tm[k] >> 16) & 3u, qk = ((k == 0 ? ptm : tm[k - 1]) >> 16) & 3u;
-          line[k] = a[k] >> A.lbs_rd;
-          scope[k] = A.cta_scope ? c[k] : 0u;
-          const uint64_t ql = (k == 0 ? pa : a[k - 1]) >> A.lbs_rd;
-          const uint32_t qs = A.cta_scope ? (k == 0 ? pc : c[k - 1]) : 0u;
-          const bool same = kd < 2u && qk < 2u && scope[k] == qs && line[k] == ql;
-          if (kd < 2u) memm |= 1u << k;
-          if (same && kd == 0u) dupm |= 1u << k;
-          if (same && kd == 1u && qk == 1u) contm |= 1u << k;
-          if (kd == 1u) stm |= 1u << k;
+          const bool e = (a[k] ^ (k == 0 ? pa : a[k - 1])) < lim && (!A.cta_scope || c[k] == (k == 0 ? pc : c[k - 1]));
+          eqm |= (uint32_t)e << k;
         }
-        if (lane == 0) contm &= ~1u;
+        const uint32_t pm = ((memm << 1) | (pkb & 1u)) & 0xffu, ps = ((stm << 1) | ((pkb >> 1) & 1u)) & 0xffu;
+        const uint32_t dupm = eqm & memm & ~stm & pm;
+        const uint32_t contm = eqm & stm & ps & (lane == 0 ? 0xfeu : 0xffu);
         // breaks: records that do not continue a store chain (the chunk end is one)
         const uint32_t brk = (~contm | ~ownm) & 0xffu;
         const uint32_t sb = lane * LPR;
         const uint32_t hb = __ballot_sync(FULL, brk != 0);
         const uint32_t lt = hb & lanemask_lt(), gt = hb & ~lanemask_le();
+        const uint32_t fbk = brk ? (uint32_t)(__ffs(brk) - 1) : (uint32_t)LPR;
         const uint32_t lastb = brk ? sb + 31u - __clz(brk) : 0u;
-        const uint32_t fb = brk ? (uint32_t)(__ffs(brk) - 1) : 0u;
         const uint32_t sv = __shfl_sync(FULL, lastb, lt ? 31u - __clz(lt) : 0u);
-        const uint32_t nv = __shfl_sync(FULL, (sb + fb) | (((dupm >> fb) & 1u) << 16), gt ? (uint32_t)(__ffs(gt) - 1) : 0u);
+        const uint32_t nv = __shfl_sync(FULL, (sb + fbk) | (((dupm >> fbk) & 1u) << 16), gt ? (uint32_t)(__ffs(gt) - 1) : 0u);
         const uint32_t nb_l = gt ? (nv & 0xffffu) : (uint32_t)KR;  // first break after the lane
         const bool nd_l = gt && (nv >> 16);
-        uint32_t start = lt ? sv : 0u, keepm = memm & ~dupm & brk;
-#pragma unroll
-        for (int k = 0; k < LPR; ++k) {
-          if ((brk >> k) & 1u) start = sb + k;
-          else if (((sb + k - start) & 15u) == 0u) keepm |= 1u << k;  // every 16th chain store
-        }
+        // chain records before the lane's first break continue a chain started at
+        // sv: the one at chain position 16 m (if any) is kept
+        const uint32_t k0 = ((lt ? sv : 0u) - sb) & 15u;
+        uint32_t keepm = (memm & ~dupm & brk) | (k0 < fbk ? (1u << k0) : 0u);
         keepm &= ownm;
         if (open_rd && lane == 0 && (dupm & 1u)) wbv[kept - 1] |= 1ull << VB_DUP;  // the previous step's open piece
         const uint32_t nk = __popc(keepm);
@@ -588,9 +583,9 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           bool hd = nd;
           if (wgt > 16u) { wgt = 16u; hd = false; }      // the chain goes on with another kept store
           else last_open = nb == (uint32_t)KR;           // decided by the next step's first record
-          wbv[pos] = line[k] | ((uint64_t)((stm >> k) & 1u) << VB_STORE) | ((uint64_t)hd << VB_DUP) |
+          wbv[pos] = (a[k] >> A.lbs_rd) | ((uint64_t)((stm >> k) & 1u) << VB_STORE) | ((uint64_t)hd << VB_DUP) |
                      ((uint64_t)(wgt - 1u) << VB_W);
-          if (wbk) wbk[pos] = scope[k];
+          if (wbk) wbk[pos] = A.cta_scope ? c[k] : 0u;
           ++pos;
         }
         open_rd = __ballot_sync(FULL, last_open) != 0;
@@ -602,37 +597,36 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       // ================= M1-M3 / B1-B3: runs = warp-level groups
       if (NG) {
         uint32_t rsm = 0, nlm = 0, vim = 0, bits[LPR];
-        uint32_t prk = run_hi(ptm & 0xffffu, ptm >> 16);
-        uint64_t pl = pa >> A.lbs_md;
+        const uint64_t lim = 1ull << A.lbs_md;
 #pragma unroll
         for (int k = 0; k < LPR; ++k) {
-          const uint32_t t = tm[k] & 0xffffu;
-          const uint32_t rk = run_hi(t, tm[k] >> 16);
-          const uint32_t qc = k == 0 ? pc : c[k - 1], qw = k == 0 ? pwi : w[k - 1];
-          const bool rs = c[k] != qc || w[k] != qw || rk != prk;
-          if (rs) rsm |= 1u << k;
+          const uint32_t qc = k == 0 ? pc : c[k - 1], qw = k == 0 ? pwi : w[k - 1], qt = k == 0 ? pt : t[k - 1];
+          rsm |= (uint32_t)(c[k] != qc || w[k] != qw || (t[k] ^ qt) >= 32u) << k;
           if (MD) {
-            const uint64_t l = a[k] >> A.lbs_md;
-            if (rs || l != pl) nlm |= 1u << k;
-            if (!rs && l < pl) vim |= 1u << k;
-            pl = l;
+            const uint64_t qa = k == 0 ? pa : a[k - 1];
+            const bool ne = (a[k] ^ qa) >= lim;
+            nlm |= (uint32_t)ne << k;
+            vim |= (uint32_t)(ne && a[k] < qa) << k;
           }
-          bits[k] = 1u << (t & 31u);
-          prk = rk;
+          bits[k] = 1u << (t[k] & 31u);
         }
+        rsm |= (bbm ^ ((bbm << 1) | ((pkb >> 2) & 1u))) & 0xffu;  // BB and memory records never share a run
         rsm |= ~inbm & 0xffu;  // every record past the stream is a run of its own (never finalized)
-        // per-run aggregates inside the lane (backward): u = packed, m = lane bits
-        uint32_t ru[LPR], rm[LPR];
-        uint32_t u = 0, m = 0;
+        nlm |= rsm;
+        vim &= ~rsm;
+        // lane bits of each in-lane run piece (backward)
+        uint32_t rm[LPR];
+        uint32_t m = 0;
 #pragma unroll
         for (int k = LPR - 1; k >= 0; --k) {
-          u += ((nlm >> k) & 1u) | (1u << PK_CNT) | (((vim >> k) & 1u) << PK_VIOL);
           m |= bits[k];
-          ru[k] = u;
           rm[k] = m;
-          if ((rsm >> k) & 1u) { u = 0; m = 0; }
+          if ((rsm >> k) & 1u) m = 0;
         }
-        // u / m now hold the lane's prefix (records before its first run start)
+        // the lane's prefix (records before its first run start)
+        const uint32_t fr = rsm ? (uint32_t)(__ffs(rsm) - 1) : (uint32_t)LPR;
+        const uint32_t pre = (1u << fr) - 1u;
+        uint32_t u = __popc(nlm & pre) | (fr << PK_CNT) | (__popc(vim & pre) << PK_VIOL);
         const uint32_t head = rsm != 0;
         seg_scan2(u, m, head);
         const uint32_t S_next = __shfl_down_sync(FULL, u, 1), M_next = __shfl_down_sync(FULL, m, 1);
@@ -666,7 +660,10 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           const uint32_t im = __ballot_sync(FULL, it);
           if (im) {
             if (it) {
-              uint32_t u2 = ru[k], m2 = rm[k];
+              const uint32_t nxt = rsm & (0xfeu << k) & 0xffu;
+              const uint32_t seg = (nxt ? (nxt & (0u - nxt)) - 1u : 0xffu) & (0xffu << k);
+              uint32_t u2 = __popc(nlm & seg) | (__popc(seg) << PK_CNT) | (__popc(vim & seg) << PK_VIOL);
+              uint32_t m2 = rm[k];
               if ((uint32_t)k == lastk) { u2 += S_next; m2 |= M_next; }  // closed by a later lane's head
               const uint32_t pos = qn + __popc(im & lanemask_lt());
               qj[pos] = j0 + k;
@@ -695,7 +692,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             tu = __popc(nlm & msk) | ((LPR - lastk) << PK_CNT) | (__popc(vim & msk) << PK_VIOL);
 #pragma unroll
             for (int k = 0; k < LPR; ++k)
-              if ((uint32_t)k >= lastk) tmk |= bits[k];
+              if ((uint32_t)k == lastk) tmk = rm[k];
             if (lane < 31) { tu += S_next; tmk |= M_next; }
           }
           cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
@@ -708,7 +705,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       }
       // ---- carry the step's last record; recycle piece p - 1 for piece p + 2
       p_cta = __shfl_sync(FULL, c[LPR - 1], 31);
-      p_tm = __shfl_sync(FULL, tm[LPR - 1], 31);
+      p_kb = __shfl_sync(FULL, ((memm >> 7) & 1u) | ((stm >> 6) & 2u) | ((bbm >> 5) & 4u), 31);
+      if (NG) p_t = __shfl_sync(FULL, t[LPR - 1], 31);
       if (NG) p_winst = __shfl_sync(FULL, w[LPR - 1], 31);
       if (NA) p_addr = __shfl_sync(FULL, a[LPR - 1], 31);
       __syncwarp();
