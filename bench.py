@@ -147,13 +147,32 @@ def algorithmic_bytes(kname, st):
         "k_scan<2>": 23 * n,                        # addr, cta, tid, winst, site, meta
         "k_scan<4>": 15 * n,                        # cta, tid, winst, site, meta
         "k_ingest": 5 * n,                          # cta 4 + meta 1
-        "k_rd_compact": 13 * n + 12 * kept,         # read addr 8 + cta 4 + meta 1; write key 4 + value 8 per kept
-        "k_divergence<0>": 19 * n + 4 * mgroups,    # addr 8 + cta 4 + tid 2 + winst 4 + meta 1; site per group
-        "k_cta_maxtid": 7 * n,                      # cta 4 + tid 2 + meta 1
-        "k_divergence<1>": 11 * n + 4 * bgroups,    # cta 4 + tid 2 + winst 4 + meta 1; site per group
-        "k_rd_tile": 12 * kept,                     # key 4 + value 8 per kept record
+        "k_rd_tile<false>": 12 * kept,              # key 4 + value 8 per kept record
+        "k_squeeze": 24 * kept,                     # kept records read and written once
     }
     return table.get(kname)
+
+
+def ncu_traffic(kname):
+    """DRAM bytes (read + write) per launch of `kname` from the committed
+    `ncu --set full` summary of this bench's workload, or None."""
+    import csv
+    p = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "ncu_full_latest.csv")
+    try:
+        with open(p) as f:
+            rows = list(csv.reader(f))
+    except OSError:
+        return None
+    hdr, units = rows[0], rows[1]
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+    for r in rows[2:]:
+        if r[0] == kname:
+            tot = 0.0
+            for m in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+                i = hdr.index(m)
+                tot += float(r[i]) * scale.get(units[i], 1)
+            return int(tot)
+    return None
 
 
 # ----------------------------------------------------------------- CPU oracle (baseline / reference arm)
@@ -283,7 +302,8 @@ def main():
         if per is not None:
             gbs = per / (avg_ms / 1e3) / 1e9
             roof = {"bound": "hbm", "kernel": dom, "achieved": round(gbs, 1), "peak": peak, "unit": "GB/s",
-                    "frac": round(gbs / peak, 4), "traffic": None, "peak_source": peak_src,
+                    "frac": round(gbs / peak, 4), "traffic": ncu_traffic(dom), "peak_source": peak_src,
+                    "traffic_source": "profiles/ncu_full_latest.csv (dram read+write bytes per launch, ncu --set full)",
                     "avg_launch_ms": round(avg_ms, 4), "algorithmic_bytes_per_launch": per,
                     "share_of_step": round(tot_ms / (ms * 1.0), 4)}
     kernels = {k: {"launches": v[1], "total_ms": round(v[0], 3)} for k, v in sorted(agg.items(), key=lambda kv: -kv[1][0])}

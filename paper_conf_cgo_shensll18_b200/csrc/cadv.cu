@@ -80,8 +80,17 @@ static void prof_collect(cadv_ctx* c) {
     std::string src = c->prof_src[k] ? c->prof_src[k] : "";
     size_t a = src.find("<<<");
     std::string nm = src.substr(0, a);
-    size_t sp = nm.find_last_of(" (,");
-    if (sp != std::string::npos) nm = nm.substr(sp + 1);
+    // the launched name: the identifier (with its template arguments) before "<<<"
+    int depth = 0;
+    size_t i = nm.size();
+    while (i > 0) {
+      const char ch = nm[i - 1];
+      if (ch == '>') depth++;
+      else if (ch == '<') depth--;
+      else if (depth == 0 && (ch == ' ' || ch == '(' || ch == ',' || ch == ';')) break;
+      --i;
+    }
+    nm = nm.substr(i);
     c->prof_name[k] = nm;
   }
 }
