@@ -111,14 +111,36 @@ typedef struct { uint64_t exec, divergent, threads; } cadv_site_branch;     /* p
 
 /* Creates a context on `device` (must be an sm_100 GPU).  `cuda_stream` is a
  * cudaStream_t (NULL = default stream).  nccl_unique_id: NULL for one GPU, or
- * the 128-byte ncclUniqueId shared by all ranks (rank in [0, nranks)). */
+ * the 128-byte ncclUniqueId shared by all ranks (rank in [0, nranks), one
+ * process per GPU; cadv_create is then collective).  libnccl.so.2 is opened
+ * at run time (the copy the process already loaded, else the default search
+ * path or $CADV_NCCL_LIB); CADV_ERR_NCCL if that or ncclCommInitRank fails. */
 CADV_API cadv_status cadv_create(cadv_ctx **out, int device, void *cuda_stream,
                                  const void *nccl_unique_id, int rank, int nranks);
+
+/* Writes a fresh 128-byte ncclUniqueId to out128 (call on rank 0, broadcast
+ * it to the other ranks, e.g. with torch.distributed, before cadv_create). */
+CADV_API cadv_status cadv_nccl_unique_id(void *out128);
+
+/* In-process multi-rank contexts for testing on one GPU: a group of nranks
+ * ranks that exchange data through host staging instead of NCCL.  Each rank
+ * is a thread of the calling process holding its own context (created with
+ * cadv_create_loopback(.., group, rank)); every collective call blocks until
+ * all ranks of the group made it.  The group must outlive its contexts. */
+CADV_API void *cadv_loopback_group_create(int nranks);
+CADV_API cadv_status cadv_loopback_group_destroy(void *group);
+CADV_API cadv_status cadv_create_loopback(cadv_ctx **out, int device, void *cuda_stream, void *group, int rank);
 
 /* Registers the trace (or this rank's shard of it).  global_offset = trace
  * position of this shard's first record (0 for one GPU).  Runs the ingest
  * pass R0 (record counts per kind, CTA id range) on the device.  Does not
- * validate records; each analysis validates what it reads. */
+ * validate records; each analysis validates what it reads.
+ * Multi-rank: shards are consecutive position ranges in rank order (rank r's
+ * records precede rank r+1's in the trace; empty shards allowed).  The call
+ * is collective (global CTA-id range; shard-edge group keys).  Divergence
+ * analyses then need warp_contiguous shards whose boundaries do not split a
+ * warp-level group (else CADV_ERR_UNSUPPORTED / CADV_ERR_BAD_TRACE); reuse
+ * distance accepts any position split. */
 CADV_API cadv_status cadv_load_trace(cadv_ctx *ctx, const cadv_trace_desc *desc, uint64_t global_offset);
 
 /* Reuse-distance histogram over the load/store records (number of

@@ -94,6 +94,14 @@ def lib():
     L.cadv_last_count.argtypes = [P, i32]
     L.cadv_last_count.restype = u64
     L.cadv_version.restype = ctypes.c_char_p
+    L.cadv_nccl_unique_id.argtypes = [P]
+    L.cadv_nccl_unique_id.restype = i32
+    L.cadv_loopback_group_create.argtypes = [i32]
+    L.cadv_loopback_group_create.restype = P
+    L.cadv_loopback_group_destroy.argtypes = [P]
+    L.cadv_loopback_group_destroy.restype = i32
+    L.cadv_create_loopback.argtypes = [ctypes.POINTER(P), i32, P, P, i32]
+    L.cadv_create_loopback.restype = i32
     _lib = L
     return L
 
@@ -119,15 +127,24 @@ def _ptr_and_kind(a, name):
 class Context:
     """One analysis context (one per GPU / rank): cadv_create ... cadv_destroy."""
 
-    def __init__(self, device: int = 0, stream=None):
+    def __init__(self, device: int = 0, stream=None, nccl_id: bytes | None = None, rank: int = 0, nranks: int = 1,
+                 loopback=None):
         L = lib()
         h = ctypes.c_void_p()
-        s = L.cadv_create(ctypes.byref(h), int(device), ctypes.c_void_p(stream or 0), None, 0, 1)
+        if loopback is not None:
+            s = L.cadv_create_loopback(ctypes.byref(h), int(device), ctypes.c_void_p(stream or 0), loopback.handle,
+                                       int(rank))
+            nranks = loopback.nranks
+        else:
+            idbuf = ctypes.create_string_buffer(bytes(nccl_id), 128) if nccl_id is not None else None
+            s = L.cadv_create(ctypes.byref(h), int(device), ctypes.c_void_p(stream or 0), idbuf, int(rank),
+                              int(nranks))
         if s != CADV_OK:
-            raise CadvError(s, "cadv_create failed (needs an sm_100 GPU and the CUDA driver)")
+            raise CadvError(s, "cadv_create failed (needs an sm_100 GPU and the CUDA driver; NCCL for nranks > 1)")
         self._h = h
         self._keep = None
         self.device = device
+        self.rank, self.nranks = rank, nranks
 
     # -- helpers
     def _check(self, s):
@@ -248,8 +265,37 @@ class Context:
         self.destroy()
 
 
-def create(device: int = 0, stream=None) -> Context:
-    return Context(device, stream)
+def create(device: int = 0, stream=None, nccl_id: bytes | None = None, rank: int = 0, nranks: int = 1) -> Context:
+    """cadv_create.  nranks > 1: one process per GPU, all ranks pass the same
+    nccl_id (from nccl_unique_id() on rank 0)."""
+    return Context(device, stream, nccl_id, rank, nranks)
+
+
+def nccl_unique_id() -> bytes:
+    """cadv_nccl_unique_id: 128 bytes to broadcast to every rank."""
+    buf = ctypes.create_string_buffer(128)
+    s = lib().cadv_nccl_unique_id(buf)
+    if s != CADV_OK:
+        raise CadvError(s, "cadv_nccl_unique_id failed")
+    return buf.raw
+
+
+class LoopbackGroup:
+    """cadv_loopback_group_create: N in-process ranks on one GPU (tests)."""
+
+    def __init__(self, nranks: int):
+        self.nranks = nranks
+        self.handle = lib().cadv_loopback_group_create(int(nranks))
+        if not self.handle:
+            raise CadvError(CADV_ERR_INVALID_ARG, "bad loopback group size")
+
+    def context(self, rank: int, device: int = 0, stream=None) -> Context:
+        return Context(device, stream, rank=rank, loopback=self)
+
+    def destroy(self):
+        if self.handle:
+            lib().cadv_loopback_group_destroy(self.handle)
+            self.handle = None
 
 
 def version() -> str:

@@ -146,6 +146,13 @@ __global__ void __launch_bounds__(256) k_ingest(const uint32_t* __restrict__ cta
   }
 }
 
+__global__ void k_agree_flags(const Scalars* s, const uint64_t* f1, const uint64_t* f2, uint32_t* out) {
+  if (threadIdx.x == 0) {
+    out[0] = s->err_code;
+    out[1] = ((f1 && *f1) || (f2 && *f2)) ? 1u : 0u;
+  }
+}
+
 cudaError_t launch_ingest(cadv_ctx* c) {
   uint64_t n = c->t.n;
   if (n == 0) return cudaSuccess;
@@ -226,18 +233,68 @@ cadv_status end_call(cadv_ctx* c, const void* d_out, size_t nout, void** h_out) 
   return CADV_OK;
 }
 
+// Multi-rank load: the global max CTA id (all-reduce max) and the run keys
+// (cta, tid / 32, winst, family) of every shard's first and last record, so
+// that a shard boundary splitting a warp-level group is detected.
+cadv_status load_trace_collective(cadv_ctx* c) {
+  const int G = c->nranks;
+  void* p;
+  CK(ensure(c, B_COMM, 64 + (size_t)G * 64 + 64, &p), "workspace");
+  uint32_t* d = (uint32_t*)p;
+  uint32_t h[16] = {0};
+  h[0] = c->t.n ? c->max_cta : 0;
+  if (c->t.n) {
+    const uint64_t at[2] = {0, c->t.n - 1};
+    for (int k = 0; k < 2; ++k) {
+      uint32_t cta, winst;
+      uint16_t tid;
+      uint8_t meta;
+      CK(cudaMemcpy(&cta, c->t.cta + at[k], 4, cudaMemcpyDeviceToHost), "D2H");
+      CK(cudaMemcpy(&winst, c->t.winst + at[k], 4, cudaMemcpyDeviceToHost), "D2H");
+      CK(cudaMemcpy(&tid, c->t.tid + at[k], 2, cudaMemcpyDeviceToHost), "D2H");
+      CK(cudaMemcpy(&meta, c->t.meta + at[k], 1, cudaMemcpyDeviceToHost), "D2H");
+      h[1 + 4 * k] = 1;
+      h[2 + 4 * k] = cta;
+      h[3 + 4 * k] = ((uint32_t)tid >> 5) | (((meta & 3u) == 2u) ? 0x10000u : 0u);
+      h[4 + 4 * k] = winst;
+    }
+  }
+  CK(cudaMemcpyAsync(d, h, 64, cudaMemcpyHostToDevice, c->stream), "H2D");
+  if (c->comm->allgather(d, d + 16, 64, c->stream)) return fail(c, CADV_ERR_NCCL, c->comm->err);
+  std::vector<uint32_t> all((size_t)G * 16);
+  CK(cudaMemcpyAsync(all.data(), d + 16, (size_t)G * 64, cudaMemcpyDeviceToHost, c->stream), "D2H");
+  CK(cudaStreamSynchronize(c->stream), "collective");
+  uint32_t mx = 0;
+  c->split_group = false;
+  const uint32_t* prev_last = nullptr;
+  for (int r = 0; r < G; ++r) {
+    const uint32_t* e = all.data() + (size_t)r * 16;
+    mx = e[0] > mx ? e[0] : mx;
+    if (!e[1]) continue;  // empty shard
+    if (prev_last && prev_last[0] && prev_last[1] == e[2] && prev_last[2] == e[3] && prev_last[3] == e[4])
+      c->split_group = true;
+    prev_last = e + 5;
+  }
+  c->max_cta = mx;
+  return CADV_OK;
+}
+
 }  // namespace
 
 extern "C" {
 
 CADV_API const char* cadv_version(void) { return "cadv 0.1 (sm_100a)"; }
 
-CADV_API cadv_status cadv_create(cadv_ctx** out, int device, void* cuda_stream, const void* nccl_unique_id, int rank,
-                                 int nranks) {
+}  // extern "C"
+
+namespace {
+
+cadv_status create_ctx(cadv_ctx** out, int device, void* cuda_stream, const void* nccl_unique_id,
+                       LoopbackGroup* group, int rank, int nranks) {
   if (!out) return CADV_ERR_INVALID_ARG;
   *out = nullptr;
   if (nranks < 1 || rank < 0 || rank >= nranks) return CADV_ERR_INVALID_ARG;
-  if (nranks > 1 && !nccl_unique_id) return CADV_ERR_INVALID_ARG;
+  if (nranks > 1 && !nccl_unique_id && !group) return CADV_ERR_INVALID_ARG;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
     cudaGetLastError();
@@ -258,13 +315,54 @@ CADV_API cadv_status cadv_create(cadv_ctx** out, int device, void* cuda_stream, 
     delete c;
     return CADV_ERR_CUDA;
   }
-  if (nranks > 1) {
-    c->err = "multi-rank contexts are not available in this build";
-    delete c;
-    return CADV_ERR_UNSUPPORTED;
+  if (group) {
+    c->comm = make_loopback_comm(group, rank);
+  } else if (nranks > 1) {
+    std::string err;
+    c->comm = make_nccl_comm(nccl_unique_id, rank, nranks, &err);
+    if (!c->comm) {
+      fprintf(stderr, "cadv_create: %s\n", err.c_str());
+      cudaEventDestroy(c->ev0);
+      cudaEventDestroy(c->ev1);
+      delete c;
+      return CADV_ERR_NCCL;
+    }
   }
   *out = c;
   return CADV_OK;
+}
+
+}  // namespace
+
+extern "C" {
+
+CADV_API cadv_status cadv_create(cadv_ctx** out, int device, void* cuda_stream, const void* nccl_unique_id, int rank,
+                                 int nranks) {
+  return create_ctx(out, device, cuda_stream, nccl_unique_id, nullptr, rank, nranks);
+}
+
+CADV_API cadv_status cadv_nccl_unique_id(void* out128) {
+  if (!out128) return CADV_ERR_INVALID_ARG;
+  std::string err;
+  if (nccl_unique_id(out128, &err)) {
+    fprintf(stderr, "cadv_nccl_unique_id: %s\n", err.c_str());
+    return CADV_ERR_NCCL;
+  }
+  return CADV_OK;
+}
+
+CADV_API void* cadv_loopback_group_create(int nranks) { return nranks >= 1 ? loopback_group_new(nranks) : nullptr; }
+
+CADV_API cadv_status cadv_loopback_group_destroy(void* group) {
+  if (!group) return CADV_ERR_INVALID_ARG;
+  loopback_group_delete((LoopbackGroup*)group);
+  return CADV_OK;
+}
+
+CADV_API cadv_status cadv_create_loopback(cadv_ctx** out, int device, void* cuda_stream, void* group, int rank) {
+  if (!group) return CADV_ERR_INVALID_ARG;
+  int n = loopback_group_size((LoopbackGroup*)group);
+  return create_ctx(out, device, cuda_stream, nullptr, (LoopbackGroup*)group, rank, n);
 }
 
 CADV_API cadv_status cadv_destroy(cadv_ctx* c) {
@@ -277,6 +375,7 @@ CADV_API cadv_status cadv_destroy(cadv_ctx* c) {
   if (c->ev0) cudaEventDestroy(c->ev0);
   if (c->ev1) cudaEventDestroy(c->ev1);
   for (auto e : c->prof_ev) cudaEventDestroy(e);
+  delete c->comm;
   delete c;
   return CADV_OK;
 }
@@ -343,6 +442,10 @@ CADV_API cadv_status cadv_load_trace(cadv_ctx* c, const cadv_trace_desc* d, uint
   Scalars* hs = (Scalars*)c->host_pinned;
   c->max_cta = (uint32_t)hs->max_cta;
   for (int k = 0; k < 4; ++k) c->n_kind[k] = hs->n_kind[k];
+  if (c->nranks > 1) {
+    s = load_trace_collective(c);
+    if (s != CADV_OK) return s;
+  }
   c->loaded = true;
   return CADV_OK;
 }
@@ -375,7 +478,14 @@ cadv_status check_args(cadv_ctx* c, uint32_t line_bytes, uint32_t warp_size, boo
 cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_stats* rd_stats, uint64_t* md_hist,
                          cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites) {
   if (!c->loaded) return fail(c, CADV_ERR_NO_TRACE, "no trace loaded");
-  if (q.bd && c->t.n && c->max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
+  const bool multi = c->nranks > 1;
+  if (q.bd && (c->t.n || multi) && c->max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
+  if (multi && (q.md || q.bd)) {
+    if (!c->t.warp_contiguous)
+      return fail(c, CADV_ERR_UNSUPPORTED, "multi-rank divergence analyses need warp-contiguous shards");
+    if (c->split_group)
+      return fail(c, CADV_ERR_BAD_TRACE, "a shard boundary splits a warp-level group (cta, warp, winst)");
+  }
   CK(cudaSetDevice(c->device), "cudaSetDevice");
   cadv_status s = begin_call(c);
   if (s != CADV_OK) return s;
@@ -411,7 +521,7 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
   P.t = t;
   int flags = 0;
   RdState rs;
-  if (q.rd && t.n) {
+  if (q.rd && (t.n || multi)) {
     CK(rd_begin(c, q.scope, &rs), "reuse workspace");
     flags |= F_RD;
     P.lbs_rd = q.rd_lbs;
@@ -430,7 +540,7 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
   }
   void* tc = nullptr;
   void* defer = nullptr;
-  if (q.bd && t.n) {
+  if (q.bd && (t.n || multi)) {
     flags |= F_BD;
     uint32_t ncta = c->max_cta + 1;
     CK(ensure(c, B_TC, 4ull * ncta, &tc), "workspace");
@@ -446,9 +556,37 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
   P.nsites = (q.md_sites || q.bd_sites) ? q.nsites : 0;
   // one flag word for both site checks
   P.site_flag = d + (q.md ? o_mdf : o_bdf);
-  if (flags) CK(launch_scan(c, flags, P), "scan launch");
-  if (q.rd && t.n) CK(rd_finish(c, rs, q.log2bins, q.nbins, d + o_rdh, d + o_rds), "reuse");
-  if (q.bd && t.n) {
+  if (flags && t.n) CK(launch_scan(c, flags, P), "scan launch");
+  if (multi) {
+    // every rank learns whether any rank found a bad record / site id before
+    // the exchanges (a failing rank must not leave the others in a collective)
+    void* fb;
+    CK(ensure(c, B_COMM, 64, &fb), "workspace");
+    uint32_t* df = (uint32_t*)fb;
+    CADV_LAUNCH(c, k_agree_flags<<<1, 32, 0, c->stream>>>(scalars(c), q.md ? d + o_mdf : nullptr,
+                                                          q.bd ? d + o_bdf : nullptr, df));
+    if (c->comm->allreduce_max_u32(df, 2, c->stream)) return fail(c, CADV_ERR_NCCL, c->comm->err);
+    uint32_t hf[2];
+    CK(cudaMemcpyAsync(hf, df, 8, cudaMemcpyDeviceToHost, c->stream), "D2H");
+    CK(cudaStreamSynchronize(c->stream), "scan");
+    if (hf[0] || hf[1]) {
+      void* h0;
+      s = end_call(c, nullptr, 0, &h0);  // reports this rank's own bad record, if it has one
+      if (s != CADV_OK) return s;
+      if (hf[0]) return fail(c, CADV_ERR_BAD_TRACE, "invalid record or warp-level group on another rank");
+      return fail(c, CADV_ERR_INVALID_ARG, "a record's site id is >= nsites (on some rank)");
+    }
+  }
+  if (q.rd && (t.n || multi)) {
+    cudaError_t e = rd_finish(c, rs, q.log2bins, q.nbins, d + o_rdh, d + o_rds);
+    if (e != cudaSuccess) {
+      if (multi && !c->comm->err.empty()) return fail(c, CADV_ERR_NCCL, c->comm->err);
+      return cuda_fail(c, e, "reuse");
+    }
+  }
+  if (q.bd && (t.n || multi)) {
+    if (multi && c->comm->allreduce_max_u32((uint32_t*)tc, c->max_cta + 1, c->stream))
+      return fail(c, CADV_ERR_NCCL, c->comm->err);
     unsigned long long m = 0;
     CK(cudaMemcpyAsync(&m, P.ndefer, 8, cudaMemcpyDeviceToHost, c->stream), "D2H");
     CK(cudaStreamSynchronize(c->stream), "scan");
@@ -456,6 +594,7 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
                          q.bd_sites ? q.nsites : 0),
        "bd resolve");
   }
+  if (multi && c->comm->allreduce_sum_u64(d, total, c->stream)) return fail(c, CADV_ERR_NCCL, c->comm->err);
   void* h;
   s = end_call(c, d, total * 8, &h);
   if (s != CADV_OK) return s;

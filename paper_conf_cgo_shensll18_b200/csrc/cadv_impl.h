@@ -7,6 +7,7 @@
 #include <vector>
 
 #include "../../include/cadv.h"
+#include "cadv_comm.h"
 
 namespace cadv {
 
@@ -37,6 +38,7 @@ enum BufId {
   B_RD_KEY, B_RD_VAL, B_RD_TILESTAT, B_RD_TILEW, B_RD_TILEQ, B_RD_ENT, B_RD_ENT_KEY0, B_RD_ENT_KEY1,
   B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP, B_DEFER, B_OUT2,
   B_ALIGN0, B_ALIGN1, B_ALIGN2, B_ALIGN3, B_ALIGN4, B_ALIGN5,
+  B_XCH_K0, B_XCH_K1, B_XCH_V0, B_XCH_V1, B_XCH_CNT, B_COMM,
   B_COUNT
 };
 
@@ -46,7 +48,9 @@ struct cadv_ctx {
   int device = 0;
   cudaStream_t stream = nullptr;
   int rank = 0, nranks = 1;
-  void* comm = nullptr;  // ncclComm_t when nranks > 1
+  cadv::Comm* comm = nullptr;            // collectives when nranks > 1 (NCCL or loopback)
+  cadv::LoopbackGroup* loopback = nullptr;
+  bool split_group = false;              // a shard boundary splits a warp-level group (load_trace)
   int num_sms = 148;
   int scan_ctas = 0;     // CADV_SCAN_CTAS (testing): cap on the scan grid, 0 = one CTA per SM
   // registered trace (device pointers)

@@ -1,0 +1,254 @@
+// comm.cpp — the collectives of a multi-rank context.
+//
+// Two backends behind one small interface:
+//   NCCL      one process per GPU (the product path).  libnccl is opened with
+//             dlopen at cadv_create time, preferring the copy the process has
+//             already loaded (torch's), so libcadv has no link-time NCCL
+//             dependency and there is one NCCL per process.
+//   loopback  N ranks = N threads of one process (tests on a single GPU):
+//             buffers are exchanged through host staging under a
+//             barrier.  Same call sequence as NCCL, so the analysis code that
+//             drives the collectives is the one the NCCL path runs.
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+#include <nccl.h>
+#include <string.h>
+
+#include <condition_variable>
+#include <mutex>
+#include <string>
+#include <vector>
+
+#include "cadv_comm.h"
+
+namespace cadv {
+
+// ------------------------------------------------------------------ NCCL
+namespace {
+
+struct NcclApi {
+  void* lib = nullptr;
+  ncclResult_t (*GetUniqueId)(ncclUniqueId*) = nullptr;
+  ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int) = nullptr;
+  ncclResult_t (*CommDestroy)(ncclComm_t) = nullptr;
+  ncclResult_t (*AllReduce)(const void*, void*, size_t, ncclDataType_t, ncclRedOp_t, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*AllGather)(const void*, void*, size_t, ncclDataType_t, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Send)(const void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*Recv)(void*, size_t, ncclDataType_t, int, ncclComm_t, cudaStream_t) = nullptr;
+  ncclResult_t (*GroupStart)() = nullptr;
+  ncclResult_t (*GroupEnd)() = nullptr;
+  const char* (*GetErrorString)(ncclResult_t) = nullptr;
+};
+
+std::mutex g_nccl_mu;
+NcclApi g_nccl;
+
+bool load_nccl(std::string* err) {
+  std::lock_guard<std::mutex> lk(g_nccl_mu);
+  if (g_nccl.lib) return true;
+  void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_NOLOAD);  // the process's NCCL (e.g. torch's)
+  if (!h) {
+    const char* p = getenv("CADV_NCCL_LIB");
+    h = dlopen(p ? p : "libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+  }
+  if (!h) {
+    *err = std::string("cannot load libnccl.so.2: ") + dlerror();
+    return false;
+  }
+  NcclApi a;
+  a.lib = h;
+#define SYM(f, name)                                                  \
+  *(void**)&a.f = dlsym(h, name);                                     \
+  if (!a.f) {                                                         \
+    *err = std::string("libnccl lacks ") + name;                      \
+    return false;                                                     \
+  }
+  SYM(GetUniqueId, "ncclGetUniqueId");
+  SYM(CommInitRank, "ncclCommInitRank");
+  SYM(CommDestroy, "ncclCommDestroy");
+  SYM(AllReduce, "ncclAllReduce");
+  SYM(AllGather, "ncclAllGather");
+  SYM(Send, "ncclSend");
+  SYM(Recv, "ncclRecv");
+  SYM(GroupStart, "ncclGroupStart");
+  SYM(GroupEnd, "ncclGroupEnd");
+  SYM(GetErrorString, "ncclGetErrorString");
+#undef SYM
+  g_nccl = a;
+  return true;
+}
+
+class NcclComm : public Comm {
+ public:
+  NcclComm(int rank, int nranks, ncclComm_t c) : Comm(rank, nranks), comm_(c) {}
+  ~NcclComm() override {
+    if (comm_) g_nccl.CommDestroy(comm_);
+  }
+  int allreduce_sum_u64(uint64_t* d, size_t n, cudaStream_t s) override {
+    return ck(g_nccl.AllReduce(d, d, n, ncclUint64, ncclSum, comm_, s));
+  }
+  int allreduce_max_u32(uint32_t* d, size_t n, cudaStream_t s) override {
+    return ck(g_nccl.AllReduce(d, d, n, ncclUint32, ncclMax, comm_, s));
+  }
+  int allgather(const void* send, void* recv, size_t bytes, cudaStream_t s) override {
+    return ck(g_nccl.AllGather(send, recv, bytes, ncclUint8, comm_, s));
+  }
+  int alltoallv(const void* send, const uint64_t* soff, const uint64_t* scnt, void* recv, const uint64_t* roff,
+                const uint64_t* rcnt, cudaStream_t s) override {
+    int e = ck(g_nccl.GroupStart());
+    if (e) return e;
+    for (int p = 0; p < nranks; ++p) {
+      if (scnt[p]) e |= ck(g_nccl.Send((const uint8_t*)send + soff[p], scnt[p], ncclUint8, p, comm_, s));
+      if (rcnt[p]) e |= ck(g_nccl.Recv((uint8_t*)recv + roff[p], rcnt[p], ncclUint8, p, comm_, s));
+    }
+    e |= ck(g_nccl.GroupEnd());
+    return e;
+  }
+
+ private:
+  int ck(ncclResult_t r) {
+    if (r == ncclSuccess) return 0;
+    err = std::string("NCCL: ") + g_nccl.GetErrorString(r);
+    return 1;
+  }
+  ncclComm_t comm_;
+};
+
+}  // namespace
+
+int nccl_unique_id(void* out128, std::string* err) {
+  if (!load_nccl(err)) return 1;
+  ncclUniqueId id;
+  ncclResult_t r = g_nccl.GetUniqueId(&id);
+  if (r != ncclSuccess) {
+    *err = std::string("ncclGetUniqueId: ") + g_nccl.GetErrorString(r);
+    return 1;
+  }
+  memcpy(out128, &id, sizeof id);
+  return 0;
+}
+
+Comm* make_nccl_comm(const void* id128, int rank, int nranks, std::string* err) {
+  if (!load_nccl(err)) return nullptr;
+  ncclUniqueId id;
+  memcpy(&id, id128, sizeof id);
+  ncclComm_t c = nullptr;
+  ncclResult_t r = g_nccl.CommInitRank(&c, nranks, id, rank);
+  if (r != ncclSuccess) {
+    *err = std::string("ncclCommInitRank: ") + g_nccl.GetErrorString(r);
+    return nullptr;
+  }
+  return new NcclComm(rank, nranks, c);
+}
+
+// ------------------------------------------------------------------ loopback
+struct LoopbackGroup {
+  explicit LoopbackGroup(int n) : n(n), slot(n), soff(n), scnt(n) {}
+  int n;
+  std::mutex mu;
+  std::condition_variable cv;
+  int arrived = 0;
+  uint64_t generation = 0;
+  std::vector<std::vector<uint8_t>> slot;  // per-rank host staging of the contribution
+  std::vector<std::vector<uint64_t>> soff, scnt;
+  void barrier() {
+    std::unique_lock<std::mutex> lk(mu);
+    const uint64_t g = generation;
+    if (++arrived == n) {
+      arrived = 0;
+      ++generation;
+      cv.notify_all();
+    } else {
+      cv.wait(lk, [&] { return generation != g; });
+    }
+  }
+};
+
+LoopbackGroup* loopback_group_new(int nranks) { return nranks >= 1 ? new LoopbackGroup(nranks) : nullptr; }
+void loopback_group_delete(LoopbackGroup* g) { delete g; }
+int loopback_group_size(const LoopbackGroup* g) { return g->n; }
+
+namespace {
+
+class LoopbackComm : public Comm {
+ public:
+  LoopbackComm(LoopbackGroup* g, int rank) : Comm(rank, g->n), g_(g) {}
+  int allreduce_sum_u64(uint64_t* d, size_t n, cudaStream_t s) override { return reduce(d, n * 8, s, true); }
+  int allreduce_max_u32(uint32_t* d, size_t n, cudaStream_t s) override { return reduce(d, n * 4, s, false); }
+  int allgather(const void* send, void* recv, size_t bytes, cudaStream_t s) override {
+    const int e0 = publish(send, bytes, s);
+    g_->barrier();
+    if (e0) return finish(1);
+    for (int p = 0; p < nranks; ++p)
+      if (bytes && cuda(cudaMemcpyAsync((uint8_t*)recv + (size_t)p * bytes, g_->slot[p].data(), bytes,
+                                        cudaMemcpyHostToDevice, s)))
+        return finish(1);
+    return finish(cuda(cudaStreamSynchronize(s)));
+  }
+  int alltoallv(const void* send, const uint64_t* soff, const uint64_t* scnt, void* recv, const uint64_t* roff,
+                const uint64_t* rcnt, cudaStream_t s) override {
+    uint64_t end = 0;
+    for (int p = 0; p < nranks; ++p) end = soff[p] + scnt[p] > end ? soff[p] + scnt[p] : end;
+    const int e0 = publish(send, end, s);
+    g_->soff[rank].assign(soff, soff + nranks);
+    g_->scnt[rank].assign(scnt, scnt + nranks);
+    g_->barrier();
+    if (e0) return finish(1);
+    for (int p = 0; p < nranks; ++p) {
+      if (g_->scnt[p][rank] != rcnt[p]) {
+        err = "loopback alltoallv: send / receive counts disagree";
+        return finish(1);
+      }
+      if (rcnt[p] && cuda(cudaMemcpyAsync((uint8_t*)recv + roff[p], g_->slot[p].data() + g_->soff[p][rank], rcnt[p],
+                                          cudaMemcpyHostToDevice, s)))
+        return finish(1);
+    }
+    return finish(cuda(cudaStreamSynchronize(s)));
+  }
+
+ private:
+  int cuda(cudaError_t e) {
+    if (e == cudaSuccess) return 0;
+    err = std::string("loopback: ") + cudaGetErrorString(e);
+    return 1;
+  }
+  // the rank's contribution -> its host slot
+  int publish(const void* d, size_t bytes, cudaStream_t s) {
+    g_->slot[rank].resize(bytes);
+    if (bytes && cuda(cudaMemcpyAsync(g_->slot[rank].data(), d, bytes, cudaMemcpyDeviceToHost, s))) return 1;
+    return cuda(cudaStreamSynchronize(s));
+  }
+  // second barrier: nobody rewrites a slot before every rank has read it.
+  // A rank that failed still takes part in both barriers (no deadlock).
+  int finish(int e) {
+    g_->barrier();
+    return e;
+  }
+  int reduce(void* d, size_t bytes, cudaStream_t s, bool sum64) {
+    const int e0 = publish(d, bytes, s);
+    g_->barrier();
+    if (e0) return finish(1);
+    std::vector<uint8_t> acc(g_->slot[0]);
+    for (int p = 1; p < nranks; ++p) {
+      if (sum64) {
+        uint64_t* a = (uint64_t*)acc.data();
+        const uint64_t* b = (const uint64_t*)g_->slot[p].data();
+        for (size_t i = 0; i < bytes / 8; ++i) a[i] += b[i];
+      } else {
+        uint32_t* a = (uint32_t*)acc.data();
+        const uint32_t* b = (const uint32_t*)g_->slot[p].data();
+        for (size_t i = 0; i < bytes / 4; ++i) a[i] = a[i] > b[i] ? a[i] : b[i];
+      }
+    }
+    int e = bytes ? cuda(cudaMemcpyAsync(d, acc.data(), bytes, cudaMemcpyHostToDevice, s)) : 0;
+    if (!e) e = cuda(cudaStreamSynchronize(s));
+    return finish(e);
+  }
+  LoopbackGroup* g_;
+};
+
+}  // namespace
+
+Comm* make_loopback_comm(LoopbackGroup* g, int rank) { return new LoopbackComm(g, rank); }
+
+}  // namespace cadv

@@ -32,6 +32,8 @@
 #include <cuda_runtime.h>
 #include <stdio.h>
 
+#include <vector>
+
 #include "cadv_impl.h"
 #include "common.cuh"
 
@@ -732,6 +734,30 @@ __global__ void k_iota(uint32_t* p, uint64_t n) {
     p[i] = (uint32_t)i;
 }
 
+// ---- multi-rank exchange helpers
+__global__ void k_bucket_count(const uint32_t* __restrict__ key, uint64_t K, int shift, unsigned long long* cnt) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < K; i += (uint64_t)gridDim.x * blockDim.x) {
+    // keys are sorted: one atomic per run of equal buckets inside a warp
+    const uint32_t b = __ldg(key + i) >> shift;
+    const uint32_t peers = __match_any_sync(__activemask(), b);
+    if ((lane_id()) == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&cnt[b], (unsigned long long)__popc(peers));
+  }
+}
+
+// out[r] = first position whose bucket >= bnd[r], r < m (keys sorted)
+__global__ void k_lower_bounds(const uint32_t* __restrict__ key, uint64_t K, int shift, const uint64_t* bnd, int m,
+                               uint64_t* out) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= m) return;
+  uint64_t lo = 0, hi = K;
+  while (lo < hi) {
+    const uint64_t md = (lo + hi) >> 1;
+    if ((uint64_t)(key[md] >> shift) < bnd[r]) lo = md + 1;
+    else hi = md;
+  }
+  out[r] = lo;
+}
+
 int bits_for(uint64_t maxv) {
   int b = 0;
   while (b < 64 && (maxv >> b)) ++b;
@@ -770,38 +796,143 @@ cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st) {
   return cudaSuccess;
 }
 
+// Multi-rank contexts: every rank's kept records (CTA-major after the local
+// sort) are redistributed so that each scope lives on one rank: CTA ranges
+// balanced by kept-record counts (CTA scope), or everything to rank 0
+// (kernel scope: one scope).  A scope's records arrive from the ranks in rank
+// order = trace order, and a stable sort by scope restores the global
+// CTA-major order exactly.  Collective: every rank calls it.
+cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const uint64_t** val, uint64_t* K) {
+  cudaError_t e;
+  const int G = c->nranks, me = c->rank;
+  Comm* cm = c->comm;
+  std::vector<uint64_t> scnt(G, 0), soff(G, 0), rcnt(G, 0), roff(G, 0);
+  void* cb;
+  if ((e = ensure(c, B_COMM, (size_t)(G + 2) * 8 + (size_t)G * G * 8 + 64, &cb))) return e;
+  uint64_t* d_send = (uint64_t*)cb;
+  uint64_t* d_mat = d_send + G + 2;
+  const uint64_t Kl = *K;
+  if (!cta_scope) {
+    scnt[0] = Kl;
+  } else {
+    const int cbits = bits_for(c->max_cta);
+    const int shift = cbits > 20 ? cbits - 20 : 0;
+    const uint64_t nb = ((uint64_t)c->max_cta >> shift) + 1;
+    void* cntb;
+    if ((e = ensure(c, B_XCH_CNT, (nb + 2 * G + 4) * 8 + 64, &cntb))) return e;
+    unsigned long long* cnt = (unsigned long long*)cntb;
+    uint64_t* d_bnd = (uint64_t*)(cnt + nb);
+    if ((e = cudaMemsetAsync(cnt, 0, nb * 8, c->stream))) return e;
+    if (Kl) CADV_LAUNCH(c, k_bucket_count<<<c->num_sms * 4, 256, 0, c->stream>>>(*key, Kl, shift, cnt));
+    if (cm->allreduce_sum_u64((uint64_t*)cnt, nb, c->stream)) return cudaErrorUnknown;
+    std::vector<uint64_t> h(nb);
+    if ((e = cudaMemcpyAsync(h.data(), cnt, nb * 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+    if ((e = cudaStreamSynchronize(c->stream))) return e;
+    // rank r owns buckets [bnd[r], bnd[r+1]): equal shares of the global kept count
+    uint64_t total = 0;
+    for (uint64_t b = 0; b < nb; ++b) total += h[b];
+    std::vector<uint64_t> bnd(G + 1, nb);
+    bnd[0] = 0;
+    uint64_t acc = 0, b = 0;
+    for (int r = 1; r < G; ++r) {
+      const uint64_t target = (uint64_t)((unsigned __int128)total * r / G);
+      while (b < nb && acc + h[b] <= target) acc += h[b++];
+      bnd[r] = b;
+    }
+    std::vector<uint64_t> pos(G + 1, 0);
+    pos[G] = Kl;
+    if (Kl && G > 1) {
+      if ((e = cudaMemcpyAsync(d_bnd, bnd.data() + 1, (G - 1) * 8, cudaMemcpyHostToDevice, c->stream))) return e;
+      CADV_LAUNCH(c, k_lower_bounds<<<1, 32, 0, c->stream>>>(*key, Kl, shift, d_bnd, G - 1, d_bnd + G));
+      if ((e = cudaMemcpyAsync(pos.data() + 1, d_bnd + G, (G - 1) * 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+      if ((e = cudaStreamSynchronize(c->stream))) return e;
+    } else {
+      for (int r = 1; r < G; ++r) pos[r] = 0;
+    }
+    for (int r = 0; r < G; ++r) {
+      soff[r] = pos[r];
+      scnt[r] = pos[r + 1] - pos[r];
+    }
+  }
+  // the G x G count matrix: row p = what rank p sends to each rank
+  std::vector<uint64_t> mat((size_t)G * G);
+  if ((e = cudaMemcpyAsync(d_send, scnt.data(), G * 8, cudaMemcpyHostToDevice, c->stream))) return e;
+  if (cm->allgather(d_send, d_mat, G * 8, c->stream)) return cudaErrorUnknown;
+  if ((e = cudaMemcpyAsync(mat.data(), d_mat, (size_t)G * G * 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  uint64_t Kn = 0;
+  for (int p = 0; p < G; ++p) {
+    rcnt[p] = mat[(size_t)p * G + me];
+    roff[p] = Kn;
+    Kn += rcnt[p];
+  }
+  if (Kn >= 0xffffffffull) return cudaErrorNotSupported;  // kept positions are u32
+  void *rk0, *rk1 = nullptr, *rv0, *rv1;
+  if ((e = ensure(c, B_XCH_V0, Kn * 8 + 16, &rv0)) || (e = ensure(c, B_XCH_V1, Kn * 8 + 16, &rv1))) return e;
+  if (cta_scope &&
+      ((e = ensure(c, B_XCH_K0, Kn * 4 + 16, &rk0)) || (e = ensure(c, B_XCH_K1, Kn * 4 + 16, &rk1))))
+    return e;
+  auto scaled = [&](const std::vector<uint64_t>& v, uint64_t f) {
+    std::vector<uint64_t> o(v);
+    for (auto& x : o) x *= f;
+    return o;
+  };
+  if (cta_scope && cm->alltoallv(*key, scaled(soff, 4).data(), scaled(scnt, 4).data(), rk0, scaled(roff, 4).data(),
+                                 scaled(rcnt, 4).data(), c->stream))
+    return cudaErrorUnknown;
+  if (cm->alltoallv(*val, scaled(soff, 8).data(), scaled(scnt, 8).data(), rv0, scaled(roff, 8).data(),
+                    scaled(rcnt, 8).data(), c->stream))
+    return cudaErrorUnknown;
+  *K = Kn;
+  *val = (const uint64_t*)rv0;
+  *key = nullptr;
+  if (cta_scope && Kn) {
+    int res, bits = bits_for(c->max_cta);
+    if (bits == 0) bits = 1;
+    if ((e = radix_sort_pairs<uint32_t, uint64_t>(c, (uint32_t*)rk0, (uint64_t*)rv0, (uint32_t*)rk1, (uint64_t*)rv1,
+                                                  Kn, 0, bits, &res)))
+      return e;
+    *key = res ? (const uint32_t*)rk1 : (const uint32_t*)rk0;
+    *val = res ? (const uint64_t*)rv1 : (const uint64_t*)rv0;
+  }
+  return cudaSuccess;
+}
+
 cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbins, uint64_t* d_hist,
                       uint64_t* d_stats) {
   cudaError_t e;
   const int cta_scope = S.cta_scope;
   const int grid_ls = c->num_sms * 4;
   Scalars* sc = scalars(c);
-  if (S.grid == 0) return cudaSuccess;
-  void *k0 = S.k0, *k1 = S.k1, *v0 = S.v0, *v1 = S.v1;
-  // pack the per-block regions: offsets = exclusive scan of the block counts
-  uint64_t* off = S.blkcnt + S.grid + 4;
-  if ((e = exclusive_scan_u64(c, S.blkcnt, off, S.grid + 1))) return e;
-  uint64_t K;
-  if ((e = cudaMemcpyAsync(&K, off + S.grid, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
-  if ((e = launch_squeeze(c, (const uint32_t*)k1, (const uint64_t*)v1, (uint32_t*)k0, (uint64_t*)v0, S.blkcnt, off,
-                          S.grid, S.chunk_cap)))
-    return e;
-  if ((e = cudaStreamSynchronize(c->stream))) return e;
-  c->counts[0] = K;
-  if (K == 0) return cudaSuccess;
-  // ---- R1b regroup by CTA (stable)
+  uint64_t K = 0;
   const uint32_t* key = nullptr;
-  const uint64_t* val = (const uint64_t*)v0;
-  if (cta_scope) {
-    int res;
-    int bits = bits_for(c->max_cta);
-    if (bits == 0) bits = 1;
-    if ((e = radix_sort_pairs<uint32_t, uint64_t>(c, (uint32_t*)k0, (uint64_t*)v0, (uint32_t*)k1, (uint64_t*)v1, K, 0,
-                                                  bits, &res)))
+  const uint64_t* val = nullptr;
+  if (S.grid) {
+    void *k0 = S.k0, *k1 = S.k1, *v0 = S.v0, *v1 = S.v1;
+    // pack the per-block regions: offsets = exclusive scan of the block counts
+    uint64_t* off = S.blkcnt + S.grid + 4;
+    if ((e = exclusive_scan_u64(c, S.blkcnt, off, S.grid + 1))) return e;
+    if ((e = cudaMemcpyAsync(&K, off + S.grid, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+    if ((e = launch_squeeze(c, (const uint32_t*)k1, (const uint64_t*)v1, (uint32_t*)k0, (uint64_t*)v0, S.blkcnt, off,
+                            S.grid, S.chunk_cap)))
       return e;
-    key = res ? (const uint32_t*)k1 : (const uint32_t*)k0;
-    val = res ? (const uint64_t*)v1 : (const uint64_t*)v0;
+    if ((e = cudaStreamSynchronize(c->stream))) return e;
+    c->counts[0] = K;
+    // ---- R1b regroup by CTA (stable)
+    val = (const uint64_t*)v0;
+    if (cta_scope && K) {
+      int res;
+      int bits = bits_for(c->max_cta);
+      if (bits == 0) bits = 1;
+      if ((e = radix_sort_pairs<uint32_t, uint64_t>(c, (uint32_t*)k0, (uint64_t*)v0, (uint32_t*)k1, (uint64_t*)v1, K,
+                                                    0, bits, &res)))
+        return e;
+      key = res ? (const uint32_t*)k1 : (const uint32_t*)k0;
+      val = res ? (const uint64_t*)v1 : (const uint64_t*)v0;
+    }
   }
+  if (c->nranks > 1 && (e = rd_exchange(c, cta_scope, &key, &val, &K))) return e;
+  if (K == 0) return cudaSuccess;
   // ---- tiles
   uint64_t ntiles = (K + TL_NOM - 1) / TL_NOM;
   c->counts[3] = ntiles;

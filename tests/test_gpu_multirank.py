@@ -1,0 +1,163 @@
+"""Multi-rank parity on one GPU: G loopback ranks (threads of this process,
+each with its own context and stream) analyse consecutive position-range
+shards of one trace; every rank must return the oracle's whole-trace result,
+bit-exact.  The loopback group drives the same collective
+call sequence the NCCL path runs (include/cadv.h cadv_create_loopback).
+"""
+import threading
+
+import numpy as np
+import pytest
+
+import oracle as orc
+import tracegen as tg
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def cadv():
+    import paper_conf_cgo_shensll18_b200 as m
+    return m
+
+
+def run_ranks(cadv, t, cuts, fn):
+    """fn(ctx) on every rank r with shard [cuts[r], cuts[r+1]); returns per-rank results."""
+    import torch
+    G = len(cuts) - 1
+    grp = cadv.LoopbackGroup(G)
+    out, err = [None] * G, [None] * G
+
+    def work(r):
+        try:
+            stream = torch.cuda.Stream()
+            lo, hi = cuts[r], cuts[r + 1]
+            cols = {k: torch.from_numpy(np.ascontiguousarray(t.cols[k][lo:hi])).cuda() for k in cadv.COLUMNS}
+            torch.cuda.synchronize()
+            ctx = grp.context(r, stream=stream.cuda_stream)
+            try:
+                ctx.load_trace(cols, global_offset=lo)
+                out[r] = fn(ctx)
+            finally:
+                ctx.destroy()
+        except Exception as e:  # noqa: BLE001 - re-raised in the main thread
+            err[r] = e
+
+    th = [threading.Thread(target=work, args=(r,)) for r in range(G)]
+    for x in th:
+        x.start()
+    for x in th:
+        x.join(timeout=300)
+    assert not any(x.is_alive() for x in th), "a rank hung in a collective"
+    grp.destroy()
+    return out, err
+
+
+def random_cuts(n, G, seed, empty=False):
+    rng = np.random.default_rng(seed)
+    inner = sorted(int(x) for x in rng.integers(0, n + 1, G - 1))
+    if empty and G > 2:
+        inner[1] = inner[0]  # one empty shard
+    return [0] + inner + [n]
+
+
+def snapped_cuts(t, G, seed):
+    return tg.snap_cuts(t.cols, random_cuts(t.n, G, seed))
+
+
+def check_all_equal(out, ref):
+    for r, o in enumerate(out):
+        assert o is not None, f"rank {r} returned nothing"
+        for a, b in zip(o, ref):
+            assert np.array_equal(np.asarray(a), np.asarray(b)), (r, a, b)
+
+
+TRACES = {
+    "rand_stores": lambda: tg.generate("rand", seed=3, ctas=9, threads=96, instrs=25, lines=40, pstore=0.3, pbb=0.3),
+    "rand_bigcta": lambda: tg.generate("rand", seed=4, ctas=2, threads=1024, instrs=30, lines=300, pstore=0.2),
+    "srad": lambda: tg.generate("srad", rows=128, cols=128, iters=2),
+    "bfs": lambda: tg.generate("bfs", nodes=20000, seed=3),
+}
+
+
+@pytest.mark.parametrize("name", sorted(TRACES))
+@pytest.mark.parametrize("G", [2, 3, 4])
+@pytest.mark.parametrize("scope", [0, 1])
+def test_reuse_position_shards(cadv, name, G, scope):
+    """Reuse distance on arbitrary (unsnapped) position splits, CTA and kernel scope."""
+    t = TRACES[name]()
+    cuts = random_cuts(t.n, G, seed=G * 7 + scope, empty=(G == 4))
+    h_ref, s_ref = orc.reuse(t, 128, scope, 0, 66)
+    out, err = run_ranks(cadv, t, cuts, lambda c: c.reuse_histogram(128, scope, 0, 66))
+    assert not any(err), err
+    for h, s in out:
+        assert (h == h_ref).all(), (np.nonzero(h != h_ref), h, h_ref)
+        assert s == s_ref
+
+
+@pytest.mark.parametrize("name", sorted(TRACES))
+@pytest.mark.parametrize("G", [2, 4])
+def test_fused_snapped_shards(cadv, name, G):
+    """All three analyses in one call on group-snapped shards."""
+    t = TRACES[name]()
+    cuts = snapped_cuts(t, G, seed=G)
+    ref_rd = orc.reuse(t, 32, 0, 1, 20)
+    ref_md = orc.mem_div(t, 128, 32)
+    ref_bd = orc.branch_div(t, 32)
+
+    def fn(c):
+        o = c.analyze(rd=(32, 0, 1, 20), md=(128, 32), bd=32, nsites=t.nsites)
+        return o["reuse"][0], o["reuse"][1]["streaming"], o["mem_div"][0], o["mem_div"][1], \
+            o["branch_div"][0], o["branch_div"][1]
+
+    out, err = run_ranks(cadv, t, cuts, fn)
+    assert not any(err), err
+    check_all_equal(out, (ref_rd[0], ref_rd[1]["streaming"], ref_md[0], ref_md[1], ref_bd[0], ref_bd[1]))
+
+
+def test_divergence_subwarp_shards(cadv):
+    t = TRACES["rand_stores"]()
+    cuts = snapped_cuts(t, 3, seed=1)
+    out, err = run_ranks(cadv, t, cuts, lambda c: (c.mem_divergence(32, 8, t.nsites)[0],
+                                                  c.branch_divergence(16, t.nsites)[1]))
+    assert not any(err), err
+    check_all_equal(out, (orc.mem_div(t, 32, 8)[0], orc.branch_div(t, 16)[1]))
+
+
+def test_split_group_rejected(cadv):
+    """A shard boundary inside a warp-level group: divergence is refused on
+    every rank (BAD_TRACE), reuse distance is still exact."""
+    t = TRACES["srad"]()
+    gs = tg.group_starts(t.cols["cta"], t.cols["tid"], t.cols["winst"], t.cols["meta"])
+    mid = int(np.flatnonzero(~gs[t.n // 2:])[0]) + t.n // 2  # inside a group
+    cuts = [0, mid, t.n]
+
+    def fn(c):
+        with pytest.raises(cadv.CadvError) as e:
+            c.mem_divergence(128, 32, t.nsites)
+        assert e.value.status == cadv.CADV_ERR_BAD_TRACE
+        return c.reuse_histogram(128, 0, 0, 66)
+
+    out, err = run_ranks(cadv, t, cuts, fn)
+    assert not any(err), err
+    h_ref, _ = orc.reuse(t, 128, 0, 0, 66)
+    for h, _ in out:
+        assert (h == h_ref).all()
+
+
+def test_bad_record_on_one_rank(cadv):
+    """A bad record on rank 1 fails the call on every rank (no rank hangs)."""
+    t = TRACES["rand_stores"]()
+    cols = {k: v.copy() for k, v in t.cols.items()}
+    cuts = snapped_cuts(t, 3, seed=5)
+    cols["meta"][cuts[1] + 3] = 3
+    t2 = tg.from_arrays(*(cols[k] for k, _ in tg.COLUMNS), nsites=t.nsites)
+
+    def fn(c):
+        with pytest.raises(cadv.CadvError) as e:
+            c.analyze(rd=(128, 0, 0, 66), md=(128, 32), bd=32, nsites=t.nsites)
+        return e.value.status
+
+    out, err = run_ranks(cadv, t2, cuts, fn)
+    assert not any(err), err
+    assert all(s == cadv.CADV_ERR_BAD_TRACE for s in out), out

@@ -116,6 +116,53 @@ def shard_bounds(workload: str, rank: int, world: int, **params):
     return cut[rank], cut[rank + 1]
 
 
+def group_starts(cta, tid, winst, meta) -> np.ndarray:
+    """Boolean mask of records that start a warp-level group run: the first
+    record, or one whose (cta, tid // 32, winst, BB-or-memory) differs from
+    its predecessor's.  Sharding plumbing (where a position split may fall
+    without cutting a group), not analysis arithmetic."""
+    n = len(cta)
+    m = np.ones(n, dtype=bool)
+    if n > 1:
+        fam = (np.asarray(meta) & 3) == 2
+        w = np.asarray(tid).astype(np.uint32) >> 5
+        m[1:] = ((cta[1:] != cta[:-1]) | (w[1:] != w[:-1]) | (winst[1:] != winst[:-1]) | (fam[1:] != fam[:-1]))
+    return m
+
+
+def snap_cuts(cols, cuts):
+    """Moves every interior cut point forward to the next group start."""
+    gs = group_starts(cols["cta"], cols["tid"], cols["winst"], cols["meta"])
+    idx = np.flatnonzero(gs)
+    out = []
+    for c in cuts:
+        k = np.searchsorted(idx, c)
+        out.append(int(idx[k]) if k < len(idx) else len(gs))
+    return out
+
+
+def position_bounds(workload: str, world: int, snap: bool = True, **params):
+    """world + 1 cut points of equal position-range shards of the whole trace
+    (SURVEY.md 8(e)); with snap, each interior cut moves to the next group
+    start (found in a 64-record window generated around it), so divergence
+    groups are never split.  Deterministic: every rank computes the same."""
+    h, n, *_ = plan(workload, **params)
+    _load().tg_free(h)
+    cuts = [0]
+    for r in range(1, world):
+        c = r * n // world
+        if snap and 0 < c < n:
+            lo, hi = max(0, c - 64), min(n, c + 64)
+            w = generate(workload, lo, hi, **params)
+            gs = group_starts(w.cols["cta"], w.cols["tid"], w.cols["winst"], w.cols["meta"])
+            gs[0] = lo == 0
+            k = np.flatnonzero(gs[c - lo:])
+            c = c + int(k[0]) if len(k) else hi
+        cuts.append(max(cuts[-1], c))
+    cuts.append(n)
+    return cuts
+
+
 def generate(workload: str, lo: int | None = None, hi: int | None = None, alloc=None, **params) -> Trace:
     """Generates records [lo, hi) (default: all) of a workload.
 
