@@ -10,10 +10,14 @@ divergence), whole job, plus the dominant kernel's HBM roofline fraction.
 
 Workload (N=1): config 4, Rodinia-shaped SRAD 2048x2048, 6 iterations, with
 its basic-block trace (tracegen "srad"); 478,150,656 memory records.
-N>1 (torchrun, one rank per GPU): weak scaling, every rank analyses its own
-SRAD trace of the same size (seed = 42 + rank); histograms are summed over
-ranks with one NCCL all-reduce per step (ranks share no other data: CTA
-scope and divergence never cross kernel instances).
+N>1 (torchrun, one rank per GPU), --sharding position (default): weak
+scaling over ONE global trace N times the N=1 workload (SRAD: 6N
+iterations), cut into N equal position ranges snapped to warp-level group
+boundaries; each rank holds one shard and the library's
+NCCL context does the exchange (kept records redistributed by CTA range,
+T_c max-reduce, histogram all-reduce), so every rank gets the global
+result.  --sharding independent: every rank its own trace (seed 42 + rank),
+histograms summed with torch.distributed.
 
 --impl reference: the CPU oracle (oracle/) as it stands, on this host's
 cores, on a bounded sample of the same workload.
@@ -39,6 +43,8 @@ WORKLOADS = {
     "c3_bfs": ("bfs", dict(nodes=1000000, seed=42)),
     "c4_backprop": ("backprop", {"in": 4194304}),
 }
+# how a workload grows with N for position-range weak scaling (param, factor per GPU)
+SCALE = {"c4_srad": "iters", "c4_backprop": "in"}
 METRIC = "trace records analysed/sec (reuse+divergence)"
 UNIT = "records/s"
 
@@ -55,6 +61,8 @@ def parse():
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--profile-run", action="store_true", help="short run for ncu (no clocks / baselines)")
+    ap.add_argument("--sharding", default="position", choices=["position", "independent"],
+                    help="N>1: shards of one global trace (library NCCL exchange) or one trace per rank")
     ap.add_argument("--separate", action="store_true",
                     help="one library call per analysis (three passes) instead of the fused cadv_analyze")
     return ap.parse_args()
@@ -117,14 +125,25 @@ def peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def make_trace(workload, rank, pinned):
-    import tracegen as tg
+def workload_params(workload, world, sharding):
+    """(generator, params) of the global trace analysed by `world` GPUs."""
     name, params = WORKLOADS[workload]
     params = dict(params)
-    if rank and "seed" in params:
-        params["seed"] = params["seed"] + rank
-    elif rank:
-        params["seed"] = 42 + rank
+    if world > 1 and sharding == "position" and workload in SCALE:
+        params[SCALE[workload]] = params[SCALE[workload]] * world
+    return name, params
+
+
+def make_trace(workload, rank, world, sharding, pinned):
+    """This rank's trace: its position-range shard of the global trace, or
+    (independent / unscalable workloads) a whole trace of its own.  Returns
+    (trace, global_offset, global_records, mode)."""
+    import tracegen as tg
+    name, params = workload_params(workload, world, sharding)
+    mode = "position" if (world > 1 and sharding == "position" and workload in SCALE) else (
+        "independent" if world > 1 else "single")
+    if mode == "independent" and rank:
+        params["seed"] = params.get("seed", 42) + rank
     alloc = None
     if pinned:
         import torch
@@ -133,9 +152,16 @@ def make_trace(workload, rank, pinned):
         def alloc(n, dt):
             return torch.empty(n, dtype=tmap[dt], pin_memory=True).numpy()
     t0 = time.time()
-    t = tg.generate(name, alloc=alloc, **params)
-    log(f"[bench] rank {rank}: generated {workload} ({name} {params}): {t.n:,} records in {time.time() - t0:.1f}s")
-    return t
+    if mode == "position":
+        cuts = tg.position_bounds(name, world, snap=True, **params)
+        t = tg.generate(name, cuts[rank], cuts[rank + 1], alloc=alloc, **params)
+        off, total = cuts[rank], cuts[-1]
+    else:
+        t = tg.generate(name, alloc=alloc, **params)
+        off, total = 0, t.n * world
+    log(f"[bench] rank {rank}: generated {workload} ({name} {params}) [{off:,}, {off + t.n:,}) of {total:,} "
+        f"records in {time.time() - t0:.1f}s")
+    return t, off, total, mode
 
 
 # Algorithmic bytes per launch of each kernel.
@@ -212,20 +238,26 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    t = make_trace(args.workload, rank, pinned=True)
+    t, goff, gtotal, mode = make_trace(args.workload, rank, world, args.sharding, pinned=True)
     n = t.n
     nsites = t.nsites
     dev = {k: torch.from_numpy(t.cols[k]).to(f"cuda:{local}", non_blocking=True) for k in cadv.COLUMNS}
     torch.cuda.synchronize()
     stream = torch.cuda.current_stream()
-    ctx = cadv.create(local, stream.cuda_stream)
+    if mode == "position":
+        # one NCCL communicator inside the library; rank 0's id broadcast over torch.distributed
+        obj = [cadv.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        ctx = cadv.create(local, stream.cuda_stream, nccl_id=obj[0], rank=rank, nranks=world)
+    else:
+        ctx = cadv.create(local, stream.cuda_stream)
     lb = args.line_bytes
     NB = 66
 
     def step(cols, allreduce=True):
         launches = 0
         ktimes = []
-        ctx.load_trace(cols)
+        ctx.load_trace(cols, global_offset=goff)
         launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
         if args.separate:
             h, st = ctx.reuse_histogram(lb, cadv.SCOPE_CTA, cadv.BINS_LINEAR, NB)
@@ -242,7 +274,7 @@ def main():
             h, st = out["reuse"]
             hm, _ = out["mem_div"]
             _, tot = out["branch_div"]
-        if world > 1 and allreduce:
+        if mode == "independent" and allreduce:
             r = torch.from_numpy(np.concatenate([h, hm.ravel(), tot]).astype(np.int64)).cuda()
             dist.all_reduce(r)
             launches += 1
@@ -351,7 +383,12 @@ def main():
                        "analyses": ("load_trace + reuse + mem_div + branch_div (three calls)" if args.separate else
                                     "load_trace + cadv_analyze(reuse, mem_div, branch_div: one fused pass)"),
                        "l2": "inputs larger than L2 (trace >> 126 MB), no flush needed",
-                       "parallelism": f"dp{world} (independent trace per GPU, histograms all-reduced)"},
+                       "global_records": gtotal, "sharding": mode,
+                       "parallelism": (f"position-range shards of one trace over {world} GPUs (library NCCL: "
+                                       "kept records exchanged by CTA range, T_c max, histograms all-reduced)"
+                                       if mode == "position" else
+                                       f"dp{world} (independent trace per GPU, histograms all-reduced)"
+                                       if world > 1 else "single GPU")},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
             "clocks": ck, "kernels": kernels,
         }
@@ -370,7 +407,7 @@ def run_reference(args, rank, world):
     name, params = WORKLOADS[args.workload]
     lb = args.line_bytes
     # a bounded sample: the first launch's worth of records, capped
-    t = make_trace(args.workload, 0, pinned=False)
+    t = make_trace(args.workload, 0, 1, args.sharding, pinned=False)[0]
     nsamp, dt_probe, cores, desc = oracle_sample(t, max(args.cpu_seconds / 2, 2.0), lb)
     sub = tg.from_arrays(*(t.cols[k][:nsamp] for k, _ in tg.COLUMNS), nsites=t.nsites)
 

@@ -114,7 +114,9 @@ typedef struct { uint64_t exec, divergent, threads; } cadv_site_branch;     /* p
  * the 128-byte ncclUniqueId shared by all ranks (rank in [0, nranks), one
  * process per GPU; cadv_create is then collective).  libnccl.so.2 is opened
  * at run time (the copy the process already loaded, else the default search
- * path or $CADV_NCCL_LIB); CADV_ERR_NCCL if that or ncclCommInitRank fails. */
+ * path or $CADV_NCCL_LIB); CADV_ERR_NCCL if that or ncclCommInitRank fails.
+ * A non-NULL id with nranks = 1 builds a one-rank communicator that runs the
+ * multi-rank code path (exchange included) against itself. */
 CADV_API cadv_status cadv_create(cadv_ctx **out, int device, void *cuda_stream,
                                  const void *nccl_unique_id, int rank, int nranks);
 

@@ -317,7 +317,7 @@ cadv_status create_ctx(cadv_ctx** out, int device, void* cuda_stream, const void
   }
   if (group) {
     c->comm = make_loopback_comm(group, rank);
-  } else if (nranks > 1) {
+  } else if (nccl_unique_id) {
     std::string err;
     c->comm = make_nccl_comm(nccl_unique_id, rank, nranks, &err);
     if (!c->comm) {
@@ -442,7 +442,7 @@ CADV_API cadv_status cadv_load_trace(cadv_ctx* c, const cadv_trace_desc* d, uint
   Scalars* hs = (Scalars*)c->host_pinned;
   c->max_cta = (uint32_t)hs->max_cta;
   for (int k = 0; k < 4; ++k) c->n_kind[k] = hs->n_kind[k];
-  if (c->nranks > 1) {
+  if (c->comm) {
     s = load_trace_collective(c);
     if (s != CADV_OK) return s;
   }
@@ -478,7 +478,7 @@ cadv_status check_args(cadv_ctx* c, uint32_t line_bytes, uint32_t warp_size, boo
 cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_stats* rd_stats, uint64_t* md_hist,
                          cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites) {
   if (!c->loaded) return fail(c, CADV_ERR_NO_TRACE, "no trace loaded");
-  const bool multi = c->nranks > 1;
+  const bool multi = c->comm != nullptr;  // also a 1-rank NCCL / loopback context (plumbing tests)
   if (q.bd && (c->t.n || multi) && c->max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
   if (multi && (q.md || q.bd)) {
     if (!c->t.warp_contiguous)

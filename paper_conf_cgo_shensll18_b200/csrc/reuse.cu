@@ -931,7 +931,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
       val = res ? (const uint64_t*)v1 : (const uint64_t*)v0;
     }
   }
-  if (c->nranks > 1 && (e = rd_exchange(c, cta_scope, &key, &val, &K))) return e;
+  if (c->comm && (e = rd_exchange(c, cta_scope, &key, &val, &K))) return e;
   if (K == 0) return cudaSuccess;
   // ---- tiles
   uint64_t ntiles = (K + TL_NOM - 1) / TL_NOM;

@@ -9,7 +9,13 @@ decomposition the multi-GPU path relies on:
     per CTA) -- checked with the oracle on each rank;
   * bench.py's weak-scaling combination: two independent traces (different
     seeds) analysed on two ranks sum to the analysis of their concatenation
-    with disjoint CTA ids.
+    with disjoint CTA ids;
+  * bench.py's position-range sharding (the N>1 default): every rank derives
+    the same cut points of the N-times-larger global trace, the shards tile
+    it exactly, every cut falls on a warp-level group start, and the shard
+    contents equal the corresponding slices of the global trace.  (The
+    library's cross-rank exchange itself is covered on one GPU by
+    tests/test_gpu_multirank.py with in-process loopback ranks.)
 """
 import os
 import socket
@@ -56,6 +62,30 @@ def _worker(rank, world, port, mode, q):
             ctas[np.unique(t.cta).astype(np.int64)] = 1
             dist.all_reduce(ctas)
             assert int(ctas.max()) <= 1
+        elif mode == "position":
+            import bench
+            bench.WORKLOADS["t_srad"] = ("srad", dict(rows=64, cols=64, iters=1, bb=1))
+            bench.SCALE["t_srad"] = "iters"
+            name, params = bench.workload_params("t_srad", world, "position")
+            assert params["iters"] == world
+            t, off, total, mode2 = bench.make_trace("t_srad", rank, world, "position", pinned=False)
+            assert mode2 == "position"
+            cuts = torch.tensor(tg.position_bounds(name, world, snap=True, **params), dtype=torch.int64)
+            allc = [torch.zeros_like(cuts) for _ in range(world)]
+            dist.all_gather(allc, cuts)
+            assert all((c == cuts).all() for c in allc)
+            assert off == int(cuts[rank]) and off + t.n == int(cuts[rank + 1]) and total == int(cuts[-1])
+            whole = tg.generate(name, **params)
+            assert total == whole.n
+            for k, _ in tg.COLUMNS:
+                assert (t.cols[k] == whole.cols[k][off:off + t.n]).all()
+            gs = tg.group_starts(whole.cta, whole.tid, whole.winst, whole.meta)
+            assert gs[off] or off == 0
+            v = torch.tensor([t.n], dtype=torch.int64)
+            dist.all_reduce(v)
+            if rank == 0:
+                q.put(np.array([int(v[0]), total]))
+            return
         else:
             t = tg.generate("rand", seed=10 + rank, ctas=5, threads=96, instrs=25, lines=40, launches=2)
         v = torch.from_numpy(_analyse(t, 32))
@@ -111,3 +141,8 @@ def test_weak_scaling_combination():
     cat = tg.from_arrays(*(cols[k] for k, _ in tg.COLUMNS), nsites=max(a.nsites, b.nsites))
     want = _analyse(cat, 32)
     assert (got == want).all()
+
+
+def test_bench_position_sharding():
+    got = _run("position")
+    assert got[0] == got[1]

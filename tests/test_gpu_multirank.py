@@ -161,3 +161,23 @@ def test_bad_record_on_one_rank(cadv):
     out, err = run_ranks(cadv, t2, cuts, fn)
     assert not any(err), err
     assert all(s == cadv.CADV_ERR_BAD_TRACE for s in out), out
+
+
+def test_nccl_single_rank_context(cadv):
+    """The NCCL backend itself (dlopen, ncclCommInitRank, all-reduce,
+    all-gather, grouped send/recv to self) on a one-rank communicator, which
+    runs the whole multi-rank code path on this one GPU."""
+    import torch
+    t = TRACES["rand_stores"]()
+    ctx = cadv.create(0, torch.cuda.current_stream().cuda_stream, nccl_id=cadv.nccl_unique_id(), rank=0, nranks=1)
+    try:
+        ctx.load_trace(cadv.to_device(t))
+        o = ctx.analyze(rd=(128, 0, 0, 66), md=(128, 32), bd=32, nsites=t.nsites)
+        h_ref, s_ref = orc.reuse(t, 128, 0, 0, 66)
+        assert (o["reuse"][0] == h_ref).all() and o["reuse"][1] == s_ref
+        assert (o["mem_div"][0] == orc.mem_div(t, 128, 32)[0]).all()
+        assert (o["branch_div"][1] == orc.branch_div(t, 32)[1]).all()
+        h, _ = ctx.reuse_histogram(32, 1, 1, 20)
+        assert (h == orc.reuse(t, 32, 1, 1, 20)[0]).all()
+    finally:
+        ctx.destroy()
