@@ -39,7 +39,7 @@ namespace {
 
 constexpr int LPR = 8;                 // consecutive records per lane in one warp step
 constexpr int KR = 32 * LPR;           // records per piece = one warp step
-constexpr int KS = 3;                  // ring stages per warp (pieces p - 1, p, p + 1)
+constexpr int KS = 3;                  // ring stages per warp (piece p and two in flight)
 constexpr int RING = KR * KS;          // ring slots: record j lives in stage (j / KR) % KS
 constexpr int NWARP = 11;              // warps per CTA (one CTA per SM)
 constexpr int NTHR = NWARP * 32;
@@ -247,42 +247,38 @@ struct RingView {
 // sub-warp group's distinct lines (MD) / lanes (BD) by pairwise comparison.
 // Used for runs whose lines are not non-decreasing (MD), for analysis warp
 // sizes below 32 and to report runs with more than 32 records (a lane must
-// repeat).  The ring holds the run: it started at most one piece back.
+// repeat).  Reads the run from global memory (rare path).
 template <int F>
 __device__ __noinline__ void walk_run(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
-                                      const RingView R, uint32_t j0, uint32_t nrec, uint64_t c_lo) {
-  if (nrec > 32) { report(A.sc, c_lo + j0, 2); return; }
+                                      uint64_t g0, uint32_t nrec) {
+  if (nrec > 32) { report(A.sc, g0, 2); return; }
   Acc acc{0, 0};
-  const bool bb = (R.meta[ring_slot(j0)] & 3u) == 2u;
+  const bool bb = (__ldg(A.meta + g0) & 3u) == 2u;
   const uint32_t ws = bb ? A.ws_bd : A.ws_md;
   for (uint32_t r = 0; r < nrec; ++r) {
-    const uint32_t sr = ring_slot(j0 + r);
-    const uint32_t tr = R.tid[sr], sub = (tr & 31u) >> ws;
+    const uint32_t tr = __ldg(A.tid + g0 + r), sub = (tr & 31u) >> ws;
     bool leader = true;
-    for (uint32_t q = 0; q < r && leader; ++q) leader = ((R.tid[ring_slot(j0 + q)] & 31u) >> ws) != sub;
+    for (uint32_t q = 0; q < r && leader; ++q) leader = ((__ldg(A.tid + g0 + q) & 31u) >> ws) != sub;
     if (!leader) continue;
     uint32_t deg = 0, cnt = 0, mask = 0, maxt = 0;
     for (uint32_t q = r; q < nrec; ++q) {
-      const uint32_t sq = ring_slot(j0 + q);
-      const uint32_t tq = R.tid[sq];
+      const uint32_t tq = __ldg(A.tid + g0 + q);
       if (((tq & 31u) >> ws) != sub) continue;
       cnt++;
       mask |= 1u << (tq & 31u);
       maxt = max(maxt, tq);
       if (!bb) {
-        const uint64_t lq = R.addr[sq] >> A.lbs_md;
+        const uint64_t lq = __ldg(A.addr + g0 + q) >> A.lbs_md;
         bool first = true;
-        for (uint32_t u = r; u < q && first; ++u) {
-          const uint32_t su = ring_slot(j0 + u);
-          if (((R.tid[su] & 31u) >> ws) == sub && (R.addr[su] >> A.lbs_md) == lq) first = false;
-        }
+        for (uint32_t u = r; u < q && first; ++u)
+          if (((__ldg(A.tid + g0 + u) & 31u) >> ws) == sub && (__ldg(A.addr + g0 + u) >> A.lbs_md) == lq) first = false;
         deg += first;
       }
     }
-    if ((uint32_t)__popc(mask) != cnt) { report(A.sc, c_lo + j0 + r, 2); continue; }
-    const uint32_t s = A.nsites ? R.site[sr] : 0u;
-    if (bb) finish_bd(A, C, acc, sites_smem, cnt, s, R.cta[sr], tr >> ws, maxt);
-    else finish_md(A, C, whist, sites_smem, R.meta[sr] & 3u, deg, s);
+    if ((uint32_t)__popc(mask) != cnt) { report(A.sc, g0 + r, 2); continue; }
+    const uint32_t s = A.nsites ? __ldg(A.site + g0 + r) : 0u;
+    if (bb) finish_bd(A, C, acc, sites_smem, cnt, s, __ldg(A.cta + g0 + r), tr >> ws, maxt);
+    else finish_md(A, C, whist, sites_smem, __ldg(A.meta + g0 + r) & 3u, deg, s);
   }
   if (acc.bd_exec) { atomicAdd(&C.bd_tot[0], acc.bd_exec); atomicAdd(&C.bd_tot[2], acc.bd_threads); }
 }
@@ -296,7 +292,7 @@ constexpr uint32_t PK_CNT = 10, PK_VIOL = 20, PK_M = 1023;
 template <int F>
 __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
                                         const RingView R, const uint32_t* qj, const uint32_t* qu,
-                                        const uint32_t* qm, uint32_t qn, uint64_t c_lo) {
+                                        const uint32_t* qm, const uint32_t* qc, uint32_t qn, uint64_t c_lo) {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   const uint32_t lane = lane_id();
   uint32_t exec = 0, thr = 0;
@@ -308,15 +304,23 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
       j = qj[q];
       u = qu[q];
       m = qm[q];
-      const uint32_t sl = ring_slot(j);
-      kind = R.meta[sl] & 3u;
-      t = R.tid[sl];
-      cta = R.cta[sl];
-      s = A.nsites ? R.site[sl] : 0u;
+      if (j >> 31) {  // the carried run: its first record's fields were saved (its piece may be gone)
+        j &= 0x7fffffffu;
+        kind = qc[0] & 3u;
+        t = qc[1];
+        cta = qc[2];
+        s = qc[3];
+      } else {
+        const uint32_t sl = ring_slot(j);
+        kind = R.meta[sl] & 3u;
+        t = R.tid[sl];
+        cta = R.cta[sl];
+        s = A.nsites ? R.site[sl] : 0u;
+      }
       const bool bb = kind == 2u;
       if (bb ? BD : MD) {
         const uint32_t cnt = (u >> PK_CNT) & PK_M;
-        if ((u >> PK_VIOL) || (bb ? A.ws_bd : A.ws_md) != 5u || cnt > 32) walk_run<F>(A, C, whist, sites_smem, R, j, cnt, c_lo);
+        if ((u >> PK_VIOL) || (bb ? A.ws_bd : A.ws_md) != 5u || cnt > 32) walk_run<F>(A, C, whist, sites_smem, c_lo + j, cnt);
         else if ((uint32_t)__popc(m) != cnt) report(A.sc, c_lo + j, 2);
         else if (bb) bd = true;
         else md = true;
@@ -388,9 +392,10 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   if (sites_smem)
     for (uint32_t k = tx; k < (uint32_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM; k += NTHR) sites[k] = 0;
   uint32_t* whist = wh_all + warp * 68;  // warp-private MD histogram [2][33]
-  uint32_t* qj = wh_all + NWARP * 68 + warp * QCAP * 3;  // queue of complete runs: start, aggregate, lanes
+  uint32_t* qj = wh_all + NWARP * 68 + warp * (QCAP * 3 + 4);  // queue of complete runs: start, aggregate, lanes
   uint32_t* qu = qj + QCAP;
   uint32_t* qm = qu + QCAP;
+  uint32_t* qc = qm + QCAP;  // the carried run's first record: kind, tid, cta, site
   for (uint32_t k = lane; k < 68; k += 32) whist[k] = 0;
   __syncthreads();
 
@@ -414,7 +419,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     __syncwarp();
     Issuer<F> io;
     io.init(A, ring, bar, c_lo, s_end);
-    uint32_t issued = npieces < 2 ? npieces : 2, waited = 0;
+    uint32_t issued = npieces < (uint32_t)KS ? npieces : (uint32_t)KS, waited = 0;
     if (lane == 0)
       for (uint32_t p = 0; p < issued; ++p) io.issue(p);
     const RingView R{(const uint64_t*)(ring + R_ADDR), (const uint32_t*)(ring + R_CTA),
@@ -445,6 +450,14 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     for (uint32_t p = 0; p < npieces; ++p) {
       const uint32_t base = p * KR;
       if (base >= clen && !(NG && cr_on && cr_own) && !(RD && open_rd)) break;
+      // piece p + 2 goes into the stage of piece p - 1 (consumed): two pieces in flight
+      if (p >= 1 && issued < npieces) {
+        if (lane == 0) {
+          fence_proxy_async();
+          io.issue(issued);
+        }
+        ++issued;
+      }
       mbar_wait(&bar[p % KS], (p / KS) & 1u);
       waited = p + 1;
       // ---- this lane's LPR consecutive records (vector shared-memory loads)
@@ -642,7 +655,11 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           }
           if (heads) {
             if (cr_own) {
-              if (lane == 0) { qj[0] = cr_j; qu[0] = cr_v; qm[0] = cr_mask; }
+              if (lane == 0) {
+                qj[0] = cr_j | 0x80000000u;
+                qu[0] = cr_v;
+                qm[0] = cr_mask;
+              }
               qn = 1;
             }
             cr_on = false;
@@ -674,14 +691,14 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           }
           if (k == LPR / 2 - 1 && qn > QCAP - 32 * LPR / 2) {
             __syncwarp();
-            flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qn, c_lo);
+            flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qc, qn, c_lo);
             qn = 0;
             __syncwarp();
           }
         }
         if (qn) {
           __syncwarp();
-          flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qn, c_lo);
+          flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qc, qn, c_lo);
         }
         // ---- the last head lane's open run becomes the carry
         if (heads) {
@@ -690,16 +707,25 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           if (tail_open) {
             const uint32_t msk = 0xffu << lastk;
             tu = __popc(nlm & msk) | ((LPR - lastk) << PK_CNT) | (__popc(vim & msk) << PK_VIOL);
+            uint32_t tt = 0, tc = 0;
 #pragma unroll
             for (int k = 0; k < LPR; ++k)
-              if ((uint32_t)k == lastk) tmk = rm[k];
+              if ((uint32_t)k == lastk) { tmk = rm[k]; tt = t[k]; tc = c[k]; }
             if (lane < 31) { tu += S_next; tmk |= M_next; }
+            if (lane == hl) {  // the carried run's first record (its piece is recycled before the run closes)
+              const uint32_t sl0 = ring_slot(j0 + lastk);
+              qc[0] = R.meta[sl0] & 3u;
+              qc[1] = tt;
+              qc[2] = tc;
+              qc[3] = A.nsites ? R.site[sl0] : 0u;
+            }
           }
           cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
           cr_v = __shfl_sync(FULL, tu, hl);
           cr_mask = __shfl_sync(FULL, tmk, hl);
           cr_j = __shfl_sync(FULL, j0 + lastk, hl);
           cr_own = cr_j < clen;
+
         }
         __syncwarp();
       }
@@ -710,19 +736,16 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       if (NG) p_winst = __shfl_sync(FULL, w[LPR - 1], 31);
       if (NA) p_addr = __shfl_sync(FULL, a[LPR - 1], 31);
       __syncwarp();
-      if (p >= 1 && issued < npieces) {
-        if (lane == 0) {
-          fence_proxy_async();
-          io.issue(issued);
-        }
-        ++issued;
-      }
     }
     // a run open at the end of the stream ends with the trace
     if (NG && cr_on && cr_own) {
-      if (lane == 0) { qj[0] = cr_j; qu[0] = cr_v; qm[0] = cr_mask; }
+      if (lane == 0) {
+        qj[0] = cr_j | 0x80000000u;
+        qu[0] = cr_v;
+        qm[0] = cr_mask;
+      }
       __syncwarp();
-      flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, 1, c_lo);
+      flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qc, 1, c_lo);
     }
     // no bulk copy may still target the ring when the CTA exits
     for (uint32_t q = waited; q < issued; ++q) mbar_wait(&bar[q % KS], (q / KS) & 1u);
@@ -809,7 +832,7 @@ template <int F>
 size_t scan_smem() {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   return (size_t)NWARP * R_BYTES + (size_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + (size_t)NWARP * 68 * 4 +
-         (size_t)NWARP * QCAP * 12;
+         (size_t)NWARP * (QCAP * 12 + 16);
 }
 
 int g_scan_ready[8] = {0, 0, 0, 0, 0, 0, 0, 0};
