@@ -57,6 +57,8 @@ def parse():
     ap.add_argument("--impl", default="cadv", choices=["cadv", "reference"])
     ap.add_argument("--workload", default="c4_srad", choices=sorted(WORKLOADS))
     ap.add_argument("--line-bytes", type=int, default=128)
+    ap.add_argument("--rd-scope", default="cta", choices=["cta", "kernel"],
+                    help="reuse-distance scope (kernel = whole trace, SURVEY.md NEXT-1)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--cpu-seconds", type=float, default=12.0, help="target CPU time of the oracle sample")
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -253,6 +255,7 @@ def main():
         ctx = cadv.create(local, stream.cuda_stream)
     lb = args.line_bytes
     NB = 66
+    SC = cadv.SCOPE_CTA if args.rd_scope == "cta" else cadv.SCOPE_KERNEL
 
     def step(cols, allreduce=True):
         launches = 0
@@ -260,7 +263,7 @@ def main():
         ctx.load_trace(cols, global_offset=goff)
         launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
         if args.separate:
-            h, st = ctx.reuse_histogram(lb, cadv.SCOPE_CTA, cadv.BINS_LINEAR, NB)
+            h, st = ctx.reuse_histogram(lb, SC, cadv.BINS_LINEAR, NB)
             launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
             kept = ctx.last_count(0)
             hm, _ = ctx.mem_divergence(lb, 32, nsites)
@@ -268,7 +271,7 @@ def main():
             _, tot = ctx.branch_divergence(32, nsites)
             launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
         else:
-            out = ctx.analyze(rd=(lb, cadv.SCOPE_CTA, cadv.BINS_LINEAR, NB), md=(lb, 32), bd=32, nsites=nsites)
+            out = ctx.analyze(rd=(lb, SC, cadv.BINS_LINEAR, NB), md=(lb, 32), bd=32, nsites=nsites)
             launches += ctx.last_launches(); ktimes += ctx.last_kernel_times()
             kept = ctx.last_count(0)
             h, st = out["reuse"]
@@ -379,7 +382,7 @@ def main():
             "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
             "config": {"workload": args.workload, "generator": name, "params": params,
                        "records_per_gpu": n, "mem_records_per_gpu": int(((t.meta & 3) < 2).sum()),
-                       "line_bytes": lb, "warp_size": 32, "rd_scope": "cta", "rd_bins": "linear 66",
+                       "line_bytes": lb, "warp_size": 32, "rd_scope": args.rd_scope, "rd_bins": "linear 66",
                        "analyses": ("load_trace + reuse + mem_div + branch_div (three calls)" if args.separate else
                                     "load_trace + cadv_analyze(reuse, mem_div, branch_div: one fused pass)"),
                        "l2": "inputs larger than L2 (trace >> 126 MB), no flush needed",

@@ -702,6 +702,38 @@ __global__ void k_merge_count(const uint32_t* __restrict__ kin, const uint32_t* 
   }
 }
 
+// The first 12 levels of that merge sort in shared memory: block b sorts the
+// 4096 items [4096 b, 4096 b + 4096) by key (keys are distinct previous-use
+// positions), adding to cnt[id] the number of earlier items in the block
+// with a larger key.  Global k_merge_count levels continue from w = 4096.
+constexpr int MC_BLOCK = 4096;
+struct MergeBlockSmem {
+  uint64_t ka[MC_BLOCK], kb[MC_BLOCK];
+  uint16_t c[MC_BLOCK];
+};
+__global__ void __launch_bounds__(512) k_merge_count_block(const uint32_t* __restrict__ kin,
+                                                           const uint32_t* __restrict__ iin,
+                                                           uint32_t* __restrict__ kout, uint32_t* __restrict__ iout,
+                                                           uint64_t M, uint32_t* __restrict__ cnt) {
+  extern __shared__ __align__(16) uint8_t mc_raw[];
+  MergeBlockSmem& S = *reinterpret_cast<MergeBlockSmem*>(mc_raw);
+  const uint64_t base = (uint64_t)blockIdx.x * MC_BLOCK;
+  const uint32_t n = (uint32_t)(M - base < MC_BLOCK ? M - base : MC_BLOCK);
+  for (uint32_t i = threadIdx.x; i < MC_BLOCK; i += blockDim.x) {
+    S.ka[swz<uint64_t>(i)] = i < n ? ((uint64_t)kin[base + i] << 12) | i : ~0ull;
+    S.c[i] = 0;
+  }
+  __syncthreads();
+  const int res = block_sort_keys<512, uint64_t, true>(S.ka, S.kb, S.c, ~0ull, MC_BLOCK);
+  const uint64_t* src = res ? S.kb : S.ka;
+  for (uint32_t i = threadIdx.x; i < n; i += blockDim.x) {
+    const uint64_t v = src[swz<uint64_t>(i)];
+    kout[base + i] = (uint32_t)(v >> 12);
+    iout[base + i] = iin[base + (v & 0xfffu)];
+    if (S.c[i]) cnt[iin[base + i]] += S.c[i];
+  }
+}
+
 __global__ void k_iota_gather(const uint32_t* __restrict__ order, const uint32_t* __restrict__ xq, uint64_t M,
                               uint32_t* __restrict__ k, uint32_t* __restrict__ id, uint32_t* __restrict__ cnt) {
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
@@ -712,16 +744,34 @@ __global__ void k_iota_gather(const uint32_t* __restrict__ order, const uint32_t
   }
 }
 
-__global__ void k_cross_final(const int64_t* __restrict__ part, const uint32_t* __restrict__ cnt, uint64_t M,
-                              int log2bins, uint32_t nbins, uint64_t* g_hist, Scalars* sc) {
+constexpr uint32_t XF_SMEM_BINS = 4096;
+__global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__ part,
+                                                     const uint32_t* __restrict__ cnt, uint64_t M, int log2bins,
+                                                     uint32_t nbins, uint64_t* g_hist, Scalars* sc) {
+  __shared__ uint32_t h[XF_SMEM_BINS];
+  const bool sm = nbins <= XF_SMEM_BINS;
+  if (sm)
+    for (uint32_t k = threadIdx.x; k < nbins; k += blockDim.x) h[k] = 0;
+  __syncthreads();
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
     int64_t rd = part[i] - (int64_t)cnt[i];
     if (rd < 0) {
       atomicMax(&sc->err_code, 3u);
       rd = 0;
     }
-    atomicAdd((unsigned long long*)&g_hist[rd_bin((uint64_t)rd, log2bins, nbins)], 1ull);
+    const uint32_t b = rd_bin((uint64_t)rd, log2bins, nbins);
+    if (sm) {
+      // warp-aggregated: one shared-memory atomic per distinct bin in the warp
+      const uint32_t peers = __match_any_sync(__activemask(), b);
+      if (lane_id() == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&h[b], (uint32_t)__popc(peers));
+    } else {
+      atomicAdd((unsigned long long*)&g_hist[b], 1ull);
+    }
   }
+  __syncthreads();
+  if (sm)
+    for (uint32_t k = threadIdx.x; k < nbins; k += blockDim.x)
+      if (h[k]) atomicAdd((unsigned long long*)&g_hist[k], (unsigned long long)h[k]);
 }
 
 __global__ void k_widen(const uint32_t* a, unsigned long long* o, uint64_t nvalid, uint64_t n) {
@@ -765,6 +815,7 @@ int bits_for(uint64_t maxv) {
 }
 
 int g_tile_smem_set = 0;
+int g_mc_smem_set = 0;
 
 }  // namespace
 
@@ -1088,7 +1139,17 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   ka = (uint32_t*)ek0;
   kb = ka + M;
   CADV_LAUNCH(c, k_iota_gather<<<grid_ls, 256, 0, c->stream>>>(ord, X.xq, M, ka, ia, cnt));
-  for (uint64_t w = 1; w < M; w <<= 1) {
+  if (!g_mc_smem_set) {
+    if ((e = cudaFuncSetAttribute(k_merge_count_block, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)sizeof(MergeBlockSmem))))
+      return e;
+    g_mc_smem_set = 1;
+  }
+  CADV_LAUNCH(c, k_merge_count_block<<<(unsigned)((M + MC_BLOCK - 1) / MC_BLOCK), 512, sizeof(MergeBlockSmem),
+                                       c->stream>>>(ka, ia, kb, ib, M, cnt));
+  std::swap(ka, kb);
+  std::swap(ia, ib);
+  for (uint64_t w = MC_BLOCK; w < M; w <<= 1) {
     CADV_LAUNCH(c, k_merge_count<<<grid_ls, 256, 0, c->stream>>>(ka, ia, kb, ib, M, w, cnt));
     std::swap(ka, kb);
     std::swap(ia, ib);

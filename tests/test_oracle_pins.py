@@ -345,3 +345,16 @@ def test_bad_trace_rejected():
     with pytest.raises(orc.OracleError) as e:
         orc.reuse(literal(["A"]), line_bytes=48)
     assert e.value.code == 1
+
+
+def test_kernel_scope_properties_match_oracle():
+    """The size-free properties used by the full-size GPU tests (mass, ∞ =
+    first use of every renamed element, streaming = elements used once)
+    equal the LRU oracle's on random traces with stores, both line models."""
+    from props import kernel_scope_properties
+    for seed in range(4):
+        t = tg.generate("rand", seed=seed, ctas=4, threads=64, instrs=20, lines=30, pstore=0.3)
+        for lb in (1, 4, 128):
+            for scope in (1,):
+                h, s = orc.reuse(t, lb, scope, 0, 40)
+                assert kernel_scope_properties(t, lb) == (int(h.sum()), int(h[-1]), s["streaming"])
