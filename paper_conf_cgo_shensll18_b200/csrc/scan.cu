@@ -39,9 +39,9 @@ namespace {
 
 constexpr int LPR = 8;                 // consecutive records per lane in one warp step
 constexpr int KR = 32 * LPR;           // records per piece = one warp step
-constexpr int KS = 3;                  // ring stages per warp (piece p and two in flight)
+constexpr int KS = 2;                  // ring stages per warp (piece p and piece p + 1 in flight)
 constexpr int RING = KR * KS;          // ring slots: record j lives in stage (j / KR) % KS
-constexpr int NWARP = 11;              // warps per CTA (one CTA per SM)
+constexpr int NWARP = 12;              // warps per CTA (one CTA per SM; 3 per SM sub-partition)
 constexpr int NTHR = NWARP * 32;
 constexpr int NSITE_SMEM = 512;        // per-site counters kept in shared memory up to this many sites
 constexpr int QCAP = 160;              // per-warp queue of complete runs awaiting finalization
@@ -289,10 +289,15 @@ constexpr uint32_t PK_CNT = 10, PK_VIOL = 20, PK_M = 1023;
 // Finalizes the queued complete runs (one per lane, the warp converged).  A
 // run is one warp32 instruction of one CTA: with W = 32 it is the group, and
 // when its lines never decrease (viol = 0) deg = the number of line changes.
+// Entries are self-contained (run start j, aggregate u, lane bits m, kind |
+// tid, CTA and site of the first record), so flushes are batched across steps.
+struct RunQueue {
+  uint32_t *j, *u, *m, *kt, *cta, *site;
+};
+
 template <int F>
 __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
-                                        const RingView R, const uint32_t* qj, const uint32_t* qu,
-                                        const uint32_t* qm, const uint32_t* qc, uint32_t qn, uint64_t c_lo) {
+                                        const RunQueue Q, uint32_t qn, uint64_t c_lo) {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   const uint32_t lane = lane_id();
   uint32_t exec = 0, thr = 0;
@@ -301,23 +306,15 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
     bool md = false, bd = false;
     uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0;
     if (q < qn) {
-      j = qj[q];
-      u = qu[q];
-      m = qm[q];
-      if (j >> 31) {  // the carried run: its first record's fields were saved (its piece may be gone)
-        j &= 0x7fffffffu;
-        kind = qc[0] & 3u;
-        t = qc[1];
-        cta = qc[2];
-        s = qc[3];
-      } else {
-        const uint32_t sl = ring_slot(j);
-        kind = R.meta[sl] & 3u;
-        t = R.tid[sl];
-        cta = R.cta[sl];
-        s = A.nsites ? R.site[sl] : 0u;
-      }
-      const bool bb = kind == 2u;
+      j = Q.j[q];
+      u = Q.u[q];
+      m = Q.m[q];
+      const uint32_t kt = Q.kt[q];
+      kind = kt >> 16;
+      t = kt & 0xffffu;
+      cta = Q.cta[q];
+      s = Q.site[q];
+    const bool bb = kind == 2u;
       if (bb ? BD : MD) {
         const uint32_t cnt = (u >> PK_CNT) & PK_M;
         if ((u >> PK_VIOL) || (bb ? A.ws_bd : A.ws_md) != 5u || cnt > 32) walk_run<F>(A, C, whist, sites_smem, c_lo + j, cnt);
@@ -392,10 +389,9 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   if (sites_smem)
     for (uint32_t k = tx; k < (uint32_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM; k += NTHR) sites[k] = 0;
   uint32_t* whist = wh_all + warp * 68;  // warp-private MD histogram [2][33]
-  uint32_t* qj = wh_all + NWARP * 68 + warp * (QCAP * 3 + 4);  // queue of complete runs: start, aggregate, lanes
-  uint32_t* qu = qj + QCAP;
-  uint32_t* qm = qu + QCAP;
-  uint32_t* qc = qm + QCAP;  // the carried run's first record: kind, tid, cta, site
+  uint32_t* qbase = wh_all + NWARP * 68 + warp * (QCAP * 6 + 4);
+  const RunQueue Q{qbase, qbase + QCAP, qbase + 2 * QCAP, qbase + 3 * QCAP, qbase + 4 * QCAP, qbase + 5 * QCAP};
+  uint32_t* qc = qbase + 6 * QCAP;  // the carried run's first record: kind << 16 | tid, cta, site
   for (uint32_t k = lane; k < 68; k += 32) whist[k] = 0;
   __syncthreads();
 
@@ -442,6 +438,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     // the run open at the step end (warp-uniform); owned iff it starts in the chunk
     bool cr_on = false, cr_own = false;
     uint32_t cr_v = 0, cr_mask = 0, cr_j = 0;
+    uint32_t qn = 0;  // queued complete runs (warp-uniform)
     // RD: the last kept record when its compression run reaches the step end
     bool open_rd = false;
     uint64_t* wbv = A.vout ? A.vout + gw * A.chunk : nullptr;
@@ -450,7 +447,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     for (uint32_t p = 0; p < npieces; ++p) {
       const uint32_t base = p * KR;
       if (base >= clen && !(NG && cr_on && cr_own) && !(RD && open_rd)) break;
-      // piece p + 2 goes into the stage of piece p - 1 (consumed): two pieces in flight
+      // piece p + 1 goes into the stage of piece p - 1 (consumed)
       if (p >= 1 && issued < npieces) {
         if (lane == 0) {
           fence_proxy_async();
@@ -644,7 +641,6 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         seg_scan2(u, m, head);
         const uint32_t S_next = __shfl_down_sync(FULL, u, 1), M_next = __shfl_down_sync(FULL, m, 1);
         const uint32_t heads = __ballot_sync(FULL, head);
-        uint32_t qn = 0;
         // ---- the run carried in from the previous step ends at the first head
         if (cr_on) {
           cr_v += __shfl_sync(FULL, u, 0);
@@ -656,11 +652,14 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           if (heads) {
             if (cr_own) {
               if (lane == 0) {
-                qj[0] = cr_j | 0x80000000u;
-                qu[0] = cr_v;
-                qm[0] = cr_mask;
+                Q.j[qn] = cr_j;
+                Q.u[qn] = cr_v;
+                Q.m[qn] = cr_mask;
+                Q.kt[qn] = qc[0];
+                Q.cta[qn] = qc[1];
+                Q.site[qn] = qc[2];
               }
-              qn = 1;
+              ++qn;
             }
             cr_on = false;
           }
@@ -683,22 +682,27 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
               uint32_t m2 = rm[k];
               if ((uint32_t)k == lastk) { u2 += S_next; m2 |= M_next; }  // closed by a later lane's head
               const uint32_t pos = qn + __popc(im & lanemask_lt());
-              qj[pos] = j0 + k;
-              qu[pos] = u2;
-              qm[pos] = m2;
+              Q.j[pos] = j0 + k;
+              Q.u[pos] = u2;
+              Q.m[pos] = m2;
+              Q.kt[pos] = ((((k < 4 ? mmx : mmy) >> (8 * (k & 3))) & 3u) << 16) | t[k];
+              Q.cta[pos] = c[k];
+              Q.site[pos] = A.nsites ? R.site[ring_slot(j0 + k)] : 0u;
             }
             qn += __popc(im);
           }
-          if (k == LPR / 2 - 1 && qn > QCAP - 32 * LPR / 2) {
+          // flushes are batched (>= 32 runs), always leaving room for half a step
+          if (k == LPR / 2 - 1 && qn > QCAP - 32 * LPR / 2 - 1) {
             __syncwarp();
-            flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qc, qn, c_lo);
+            flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
             qn = 0;
             __syncwarp();
           }
         }
-        if (qn) {
+        if (qn >= 32) {
           __syncwarp();
-          flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qc, qn, c_lo);
+          flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
+          qn = 0;
         }
         // ---- the last head lane's open run becomes the carry
         if (heads) {
@@ -713,11 +717,9 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
               if ((uint32_t)k == lastk) { tmk = rm[k]; tt = t[k]; tc = c[k]; }
             if (lane < 31) { tu += S_next; tmk |= M_next; }
             if (lane == hl) {  // the carried run's first record (its piece is recycled before the run closes)
-              const uint32_t sl0 = ring_slot(j0 + lastk);
-              qc[0] = R.meta[sl0] & 3u;
-              qc[1] = tt;
-              qc[2] = tc;
-              qc[3] = A.nsites ? R.site[sl0] : 0u;
+              qc[0] = ((((lastk < 4 ? mmx : mmy) >> (8 * (lastk & 3u))) & 3u) << 16) | tt;
+              qc[1] = tc;
+              qc[2] = A.nsites ? R.site[ring_slot(j0 + lastk)] : 0u;
             }
           }
           cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
@@ -737,15 +739,21 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       if (NA) p_addr = __shfl_sync(FULL, a[LPR - 1], 31);
       __syncwarp();
     }
-    // a run open at the end of the stream ends with the trace
+    // a run open at the end of the stream ends with the trace; then the rest of the queue
     if (NG && cr_on && cr_own) {
       if (lane == 0) {
-        qj[0] = cr_j | 0x80000000u;
-        qu[0] = cr_v;
-        qm[0] = cr_mask;
+        Q.j[qn] = cr_j;
+        Q.u[qn] = cr_v;
+        Q.m[qn] = cr_mask;
+        Q.kt[qn] = qc[0];
+        Q.cta[qn] = qc[1];
+        Q.site[qn] = qc[2];
       }
+      ++qn;
+    }
+    if (NG && qn) {
       __syncwarp();
-      flush_runs<F>(A, C, whist, sites_smem, R, qj, qu, qm, qc, 1, c_lo);
+      flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
     }
     // no bulk copy may still target the ring when the CTA exits
     for (uint32_t q = waited; q < issued; ++q) mbar_wait(&bar[q % KS], (q / KS) & 1u);
@@ -832,7 +840,7 @@ template <int F>
 size_t scan_smem() {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   return (size_t)NWARP * R_BYTES + (size_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + (size_t)NWARP * 68 * 4 +
-         (size_t)NWARP * (QCAP * 12 + 16);
+         (size_t)NWARP * (QCAP * 24 + 16);
 }
 
 int g_scan_ready[8] = {0, 0, 0, 0, 0, 0, 0, 0};
