@@ -204,7 +204,8 @@ __device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key, uint32_t 
 #pragma unroll
     for (int j = 0; j < IPT; ++j) ka[swz<K>(t * IPT + j)] = k[j];
   }
-  __syncthreads();
+  // levels whose merges stay inside one warp's 32 * IPT items sync the warp only
+  __syncwarp();
   K* ks = ka;
   K* kd = kb;
   int res = 0;
@@ -238,12 +239,14 @@ __device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key, uint32_t 
       }
     }
     }
-    __syncthreads();
+    if (4 * w <= 32 * IPT) __syncwarp();
+    else __syncthreads();
     K* tk = ks;
     ks = kd;
     kd = tk;
     res ^= 1;
   }
+  if (N <= 16u * IPT) __syncthreads();  // the last level synced one warp only: callers read everything
   return res;
 }
 
