@@ -124,6 +124,7 @@ constexpr int RS_IPT = 16;
 constexpr int RS_TILE = RS_NT * RS_IPT;  // 4096
 constexpr int RS_WARPS = RS_NT / 32;
 constexpr int RS_PER_WARP = RS_TILE / RS_WARPS;  // 512 = 16 rounds of 32
+constexpr int RS_MAXB = 9;                        // digit bits per pass (<= 512 buckets)
 
 template <typename K>
 __device__ __forceinline__ uint32_t digit(K k, int shift, uint32_t mask) {
@@ -133,7 +134,7 @@ __device__ __forceinline__ uint32_t digit(K k, int shift, uint32_t mask) {
 template <typename K>
 __global__ void __launch_bounds__(RS_NT) k_rs_upsweep(const K* __restrict__ keys, uint64_t n, int shift, int bits,
                                                       uint32_t* __restrict__ counts, uint64_t ntiles) {
-  __shared__ uint32_t h[256];
+  __shared__ uint32_t h[1 << RS_MAXB];
   const uint32_t radix = 1u << bits, mask = radix - 1;
   for (uint32_t k = threadIdx.x; k < radix; k += RS_NT) h[k] = 0;
   __syncthreads();
@@ -155,7 +156,7 @@ __global__ void __launch_bounds__(RS_NT) k_rs_scatter(const K* __restrict__ kin,
                                                       K* __restrict__ kout, V* __restrict__ vout, uint64_t n,
                                                       int shift, int bits, const uint32_t* __restrict__ offs,
                                                       uint64_t ntiles) {
-  __shared__ uint32_t wc[RS_WARPS][256];
+  __shared__ uint32_t wc[RS_WARPS][1 << RS_MAXB];
   const uint32_t radix = 1u << bits, mask = radix - 1;
   const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
   for (uint32_t k = lane; k < radix; k += 32) wc[warp][k] = 0;
@@ -240,9 +241,9 @@ cudaError_t radix_sort_pairs(cadv_ctx* c, K* k0, V* v0, K* k1, V* v1, uint64_t n
   if (n <= 1 || bit_hi <= bit_lo) return cudaSuccess;
   uint64_t ntiles = (n + RS_TILE - 1) / RS_TILE;
   void* hist;
-  cudaError_t e = ensure(c, B_SORT_HIST, 256ull * ntiles * 4 + 64, &hist);
+  cudaError_t e = ensure(c, B_SORT_HIST, (1ull << RS_MAXB) * ntiles * 4 + 64, &hist);
   if (e != cudaSuccess) return e;
-  int passes = (bit_hi - bit_lo + 7) / 8;
+  int passes = (bit_hi - bit_lo + RS_MAXB - 1) / RS_MAXB;
   int per = (bit_hi - bit_lo + passes - 1) / passes;
   K* ki = k0; V* vi = v0; K* ko = k1; V* vo = v1;
   for (int shift = bit_lo; shift < bit_hi; shift += per) {
