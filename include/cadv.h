@@ -134,9 +134,10 @@ CADV_API cadv_status cadv_loopback_group_destroy(void *group);
 CADV_API cadv_status cadv_create_loopback(cadv_ctx **out, int device, void *cuda_stream, void *group, int rank);
 
 /* Registers the trace (or this rank's shard of it).  global_offset = trace
- * position of this shard's first record (0 for one GPU).  Runs the ingest
- * pass R0 (record counts per kind, CTA id range) on the device.  Does not
- * validate records; each analysis validates what it reads.
+ * position of this shard's first record (0 for one GPU).  Host columns are
+ * copied to the device here; device columns are only registered.  R0 (record
+ * validation, CTA-id range) runs inside each analysis' streaming pass; each
+ * analysis validates the columns it reads.
  * Multi-rank: shards are consecutive position ranges in rank order (rank r's
  * records precede rank r+1's in the trace; empty shards allowed).  The call
  * is collective (global CTA-id range; shard-edge group keys).  Divergence

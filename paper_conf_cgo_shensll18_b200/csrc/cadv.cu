@@ -1,5 +1,5 @@
 // cadv.cu — the C ABI of libcadv (include/cadv.h): context, trace
-// registration + ingest pass R0, and the synchronous analysis entry points.
+// registration, and the synchronous analysis entry points.
 #include <cuda_runtime.h>
 #include <cstdlib>
 #include <stdio.h>
@@ -95,71 +95,12 @@ static void prof_collect(cadv_ctx* c) {
   }
 }
 
-// ------------------------------------------------------------------ R0 ingest
-// One streaming pass over (cta, meta): max CTA id and record count per kind.
-// 16 records per thread and step: four 16-byte loads of cta, one of meta.
-__device__ __forceinline__ void ingest_one(uint32_t c, uint32_t m, uint32_t& mx, uint32_t (&cnt)[4]) {
-  mx = max(mx, c);
-  const uint32_t k = m & 3u;
-  cnt[0] += k == 0;
-  cnt[1] += k == 1;
-  cnt[2] += k == 2;
-  cnt[3] += k == 3;
-}
-
-__global__ void __launch_bounds__(256) k_ingest(const uint32_t* __restrict__ cta, const uint8_t* __restrict__ meta,
-                                                uint64_t n, Scalars* s) {
-  uint32_t mx = 0;
-  uint32_t cnt[4] = {0, 0, 0, 0};
-  const bool vec = (((uintptr_t)cta | (uintptr_t)meta) & 15) == 0;
-  const uint64_t tid = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x, nth = (uint64_t)gridDim.x * blockDim.x;
-  uint64_t done = 0;
-  if (vec) {
-    const uint64_t ng = n / 16;
-    const uint4* c4 = (const uint4*)cta;
-    const uint4* m4 = (const uint4*)meta;
-    for (uint64_t gi = tid; gi < ng; gi += nth) {
-      const uint4 mm = __ldg(m4 + gi);
-      uint4 cc[4];
-#pragma unroll
-      for (int k = 0; k < 4; ++k) cc[k] = __ldg(c4 + 4 * gi + k);
-      const uint32_t mw[4] = {mm.x, mm.y, mm.z, mm.w};
-#pragma unroll
-      for (int k = 0; k < 4; ++k) {
-        ingest_one(cc[k].x, mw[k] & 0xffu, mx, cnt);
-        ingest_one(cc[k].y, (mw[k] >> 8) & 0xffu, mx, cnt);
-        ingest_one(cc[k].z, (mw[k] >> 16) & 0xffu, mx, cnt);
-        ingest_one(cc[k].w, mw[k] >> 24, mx, cnt);
-      }
-    }
-    done = ng * 16;
-  }
-  for (uint64_t i = done + tid; i < n; i += nth) ingest_one(__ldg(cta + i), __ldg(meta + i), mx, cnt);
-  mx = __reduce_max_sync(FULL, mx);
-#pragma unroll
-  for (int k = 0; k < 4; ++k) cnt[k] = __reduce_add_sync(FULL, cnt[k]);
-  if (lane_id() == 0) {
-    atomicMax(&s->max_cta, (unsigned long long)mx);
-#pragma unroll
-    for (int k = 0; k < 4; ++k)
-      if (cnt[k]) atomicAdd(&s->n_kind[k], (unsigned long long)cnt[k]);
-  }
-}
-
 __global__ void k_agree_flags(const Scalars* s, const uint64_t* f1, const uint64_t* f2, uint32_t* out) {
   if (threadIdx.x == 0) {
     out[0] = s->err_code;
     out[1] = ((f1 && *f1) || (f2 && *f2)) ? 1u : 0u;
+    out[2] = (uint32_t)s->max_cta;
   }
-}
-
-cudaError_t launch_ingest(cadv_ctx* c) {
-  uint64_t n = c->t.n;
-  if (n == 0) return cudaSuccess;
-  uint64_t want = (n / 16 + 255) / 256 + 1;
-  int grid = (int)(want < (uint64_t)c->num_sms * 8 ? want : (uint64_t)c->num_sms * 8);
-  CADV_LAUNCH(c, k_ingest<<<grid, 256, 0, c->stream>>>(c->t.cta, c->t.meta, n, scalars(c)));
-  return cudaGetLastError();
 }
 
 }  // namespace cadv
@@ -233,7 +174,7 @@ cadv_status end_call(cadv_ctx* c, const void* d_out, size_t nout, void** h_out) 
   return CADV_OK;
 }
 
-// Multi-rank load: the global max CTA id (all-reduce max) and the run keys
+// Multi-rank load: the run keys
 // (cta, tid / 32, winst, family) of every shard's first and last record, so
 // that a shard boundary splitting a warp-level group is detected.
 cadv_status load_trace_collective(cadv_ctx* c) {
@@ -242,7 +183,6 @@ cadv_status load_trace_collective(cadv_ctx* c) {
   CK(ensure(c, B_COMM, 64 + (size_t)G * 64 + 64, &p), "workspace");
   uint32_t* d = (uint32_t*)p;
   uint32_t h[16] = {0};
-  h[0] = c->t.n ? c->max_cta : 0;
   if (c->t.n) {
     const uint64_t at[2] = {0, c->t.n - 1};
     for (int k = 0; k < 2; ++k) {
@@ -264,18 +204,15 @@ cadv_status load_trace_collective(cadv_ctx* c) {
   std::vector<uint32_t> all((size_t)G * 16);
   CK(cudaMemcpyAsync(all.data(), d + 16, (size_t)G * 64, cudaMemcpyDeviceToHost, c->stream), "D2H");
   CK(cudaStreamSynchronize(c->stream), "collective");
-  uint32_t mx = 0;
   c->split_group = false;
   const uint32_t* prev_last = nullptr;
   for (int r = 0; r < G; ++r) {
     const uint32_t* e = all.data() + (size_t)r * 16;
-    mx = e[0] > mx ? e[0] : mx;
     if (!e[1]) continue;  // empty shard
     if (prev_last && prev_last[0] && prev_last[1] == e[2] && prev_last[2] == e[3] && prev_last[3] == e[4])
       c->split_group = true;
     prev_last = e + 5;
   }
-  c->max_cta = mx;
   return CADV_OK;
 }
 
@@ -375,6 +312,7 @@ CADV_API cadv_status cadv_destroy(cadv_ctx* c) {
   if (c->ev0) cudaEventDestroy(c->ev0);
   if (c->ev1) cudaEventDestroy(c->ev1);
   for (auto e : c->prof_ev) cudaEventDestroy(e);
+  if (c->tc_buf) cudaFree(c->tc_buf);
   delete c->comm;
   delete c;
   return CADV_OK;
@@ -435,13 +373,10 @@ CADV_API cadv_status cadv_load_trace(cadv_ctx* c, const cadv_trace_desc* d, uint
     c->t.winst = (const uint32_t*)dst[4];
     c->t.meta = (const uint8_t*)dst[5];
   }
-  CK(launch_ingest(c), "ingest launch");
   void* h;
   s = end_call(c, nullptr, 0, &h);
   if (s != CADV_OK) return s;
-  Scalars* hs = (Scalars*)c->host_pinned;
-  c->max_cta = (uint32_t)hs->max_cta;
-  for (int k = 0; k < 4; ++k) c->n_kind[k] = hs->n_kind[k];
+  c->max_cta = 0;  // R0's CTA-id range comes out of each analysis' streaming pass
   if (c->comm) {
     s = load_trace_collective(c);
     if (s != CADV_OK) return s;
@@ -475,11 +410,47 @@ cadv_status check_args(cadv_ctx* c, uint32_t line_bytes, uint32_t warp_size, boo
 // branch-divergence resolution.  Device output layout in B_OUT2:
 //   [rd hist nbins][rd stats 4][md hist 2(W+1)][md sites 2 nsites][md flag]
 //   [bd totals 3][bd flag][bd sites 3 nsites]
+constexpr cadv_status RETRY = (cadv_status)100;  // internal: workspace grown, run the call again
+
+// (re)allocates the T_c table with `cap` entries; keep = entries to preserve
+cudaError_t tc_resize(cadv_ctx* c, uint32_t cap, uint32_t keep) {
+  uint32_t* nb = nullptr;
+  cudaError_t e = cudaMalloc(&nb, 4ull * cap);
+  if (e != cudaSuccess) return e;
+  if ((e = cudaMemsetAsync(nb, 0, 4ull * cap, c->stream))) return e;
+  if (keep && c->tc_buf &&
+      (e = cudaMemcpyAsync(nb, c->tc_buf, 4ull * keep, cudaMemcpyDeviceToDevice, c->stream)))
+    return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  if (c->tc_buf) cudaFree(c->tc_buf);
+  c->tc_buf = nb;
+  c->tc_cap = cap;
+  return cudaSuccess;
+}
+
+cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_stats* rd_stats, uint64_t* md_hist,
+                     cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites);
+
 cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_stats* rd_stats, uint64_t* md_hist,
                          cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites) {
   if (!c->loaded) return fail(c, CADV_ERR_NO_TRACE, "no trace loaded");
+  if (q.bd) {
+    // one T_c generation per call (identical on every rank: calls run in lockstep)
+    if (++c->tc_gen >= (1u << 21)) {
+      c->tc_gen = 1;
+      if (c->tc_buf) CK(cudaMemsetAsync(c->tc_buf, 0, 4ull * c->tc_cap, c->stream), "memset");
+    }
+  }
+  for (int attempt = 0;; ++attempt) {
+    cadv_status s = run_once(c, q, rd_hist, rd_stats, md_hist, md_sites, bd_tot, bd_sites);
+    if (s != RETRY) return s;
+    if (attempt > 4) return fail(c, CADV_ERR_OOM, "workspace did not converge");
+  }
+}
+
+cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_stats* rd_stats, uint64_t* md_hist,
+                     cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites) {
   const bool multi = c->comm != nullptr;  // also a 1-rank NCCL / loopback context (plumbing tests)
-  if (q.bd && (c->t.n || multi) && c->max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
   if (multi && (q.md || q.bd)) {
     if (!c->t.warp_contiguous)
       return fail(c, CADV_ERR_UNSUPPORTED, "multi-rank divergence analyses need warp-contiguous shards");
@@ -538,16 +509,17 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
     P.md_hist = d + o_mdh;
     P.md_sites = q.md_sites ? d + o_mds : nullptr;
   }
-  void* tc = nullptr;
   void* defer = nullptr;
   if (q.bd && (t.n || multi)) {
     flags |= F_BD;
-    uint32_t ncta = c->max_cta + 1;
-    CK(ensure(c, B_TC, 4ull * ncta, &tc), "workspace");
-    CK(cudaMemsetAsync(tc, 0, 4ull * ncta, c->stream), "memset");
-    CK(ensure(c, B_DEFER, 16ull * (c->n_kind[2] + 1), &defer), "workspace");
+    if (!c->tc_buf) CK(tc_resize(c, 1u << 16, 0), "workspace");
+    if (!c->defer_cap) c->defer_cap = t.n / 8 + 4096;
+    CK(ensure(c, B_DEFER, 16ull * c->defer_cap, &defer), "workspace");
     P.ws_bd = q.bd_ws;
-    P.tc = (uint32_t*)tc;
+    P.tc = c->tc_buf;
+    P.tc_cap = c->tc_cap;
+    P.tc_gen = c->tc_gen;
+    P.defer_cap = c->defer_cap;
     P.bd_tot = d + o_bdt;
     P.bd_sites = q.bd_sites ? d + o_bds : nullptr;
     P.defer = defer;
@@ -557,6 +529,28 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
   // one flag word for both site checks
   P.site_flag = d + (q.md ? o_mdf : o_bdf);
   if (flags && t.n) CK(launch_scan(c, flags, P), "scan launch");
+  // R0 results of the pass: CTA-id range, T_c / deferred-group capacity
+  {
+    Scalars hs;
+    CK(cudaMemcpyAsync(&hs, scalars(c), sizeof hs, cudaMemcpyDeviceToHost, c->stream), "D2H");
+    CK(cudaStreamSynchronize(c->stream), "scan");
+    c->max_cta = (uint32_t)hs.max_cta;
+    if (q.bd && t.n) {
+      if (hs.max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
+      bool again = false;
+      if (hs.tc_overflow) {
+        uint64_t cap = (uint64_t)c->tc_cap * 2;
+        if (cap < hs.max_cta + 1) cap = hs.max_cta + 1;
+        CK(tc_resize(c, (uint32_t)cap, 0), "workspace");
+        again = true;
+      }
+      if (hs.ndefer > c->defer_cap) {
+        c->defer_cap = hs.ndefer + hs.ndefer / 4 + 4096;
+        again = true;
+      }
+      if (again && !hs.err_code) return RETRY;
+    }
+  }
   if (multi) {
     // every rank learns whether any rank found a bad record / site id before
     // the exchanges (a failing rank must not leave the others in a collective)
@@ -565,10 +559,11 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
     uint32_t* df = (uint32_t*)fb;
     CADV_LAUNCH(c, k_agree_flags<<<1, 32, 0, c->stream>>>(scalars(c), q.md ? d + o_mdf : nullptr,
                                                           q.bd ? d + o_bdf : nullptr, df));
-    if (c->comm->allreduce_max_u32(df, 2, c->stream)) return fail(c, CADV_ERR_NCCL, c->comm->err);
-    uint32_t hf[2];
-    CK(cudaMemcpyAsync(hf, df, 8, cudaMemcpyDeviceToHost, c->stream), "D2H");
+    if (c->comm->allreduce_max_u32(df, 3, c->stream)) return fail(c, CADV_ERR_NCCL, c->comm->err);
+    uint32_t hf[3];
+    CK(cudaMemcpyAsync(hf, df, 12, cudaMemcpyDeviceToHost, c->stream), "D2H");
     CK(cudaStreamSynchronize(c->stream), "scan");
+    c->max_cta = hf[2];  // global CTA-id range
     if (hf[0] || hf[1]) {
       void* h0;
       s = end_call(c, nullptr, 0, &h0);  // reports this rank's own bad record, if it has one
@@ -585,12 +580,16 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
     }
   }
   if (q.bd && (t.n || multi)) {
-    if (multi && c->comm->allreduce_max_u32((uint32_t*)tc, c->max_cta + 1, c->stream))
-      return fail(c, CADV_ERR_NCCL, c->comm->err);
+    if (multi) {
+      if (c->max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
+      if (c->tc_cap < c->max_cta + 1) CK(tc_resize(c, c->max_cta + 1, c->tc_cap), "workspace");
+      if (c->comm->allreduce_max_u32(c->tc_buf, c->max_cta + 1, c->stream))
+        return fail(c, CADV_ERR_NCCL, c->comm->err);
+    }
     unsigned long long m = 0;
     CK(cudaMemcpyAsync(&m, P.ndefer, 8, cudaMemcpyDeviceToHost, c->stream), "D2H");
     CK(cudaStreamSynchronize(c->stream), "scan");
-    CK(launch_bd_resolve(c, defer, m, (const uint32_t*)tc, q.bd_ws, d + o_bdt, q.bd_sites ? d + o_bds : nullptr,
+    CK(launch_bd_resolve(c, defer, m, c->tc_buf, c->tc_gen, q.bd_ws, d + o_bdt, q.bd_sites ? d + o_bds : nullptr,
                          q.bd_sites ? q.nsites : 0),
        "bd resolve");
   }

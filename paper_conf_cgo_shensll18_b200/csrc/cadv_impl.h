@@ -24,8 +24,9 @@ struct Scalars {
   unsigned int err_code;         // 1 = bad record, 2 = run longer than 32 / duplicate lane
   unsigned int tile_counter;     // dynamic tile assignment
   unsigned long long count[8];   // generic counters (kept records, entries, ...)
-  unsigned long long max_cta;    // ingest: max CTA id
-  unsigned long long n_kind[4];  // ingest: records per kind
+  unsigned long long max_cta;    // scan: max CTA id of the trace (shard)
+  unsigned long long n_kind[4];  // (unused)
+  unsigned long long tc_overflow;  // scan: a CTA id >= the T_c capacity was seen
   unsigned long long ndefer;     // branch divergence: deferred partial groups
   unsigned long long rd_line_min, rd_line_max;  // reuse cross-tile phase: entry line range
 };
@@ -57,9 +58,14 @@ struct cadv_ctx {
   bool loaded = false;
   cadv_trace_desc t{};
   uint64_t global_offset = 0;
-  // ingest results (R0)
-  uint32_t max_cta = 0;
-  uint64_t n_kind[4] = {0, 0, 0, 0};
+  // R0 results (from the streaming pass of the last analysis)
+  uint32_t max_cta = 0;               // of the current trace (shard; global after a multi-rank scan)
+  uint64_t n_kind[4] = {0, 0, 0, 0};  // (unused)
+  // B2 T_c table, kept across calls: entry = generation << 11 | T_c, so a new
+  // call needs no clearing; capacity and the deferred-group buffer grow on demand
+  uint32_t* tc_buf = nullptr;
+  uint32_t tc_cap = 0, tc_gen = 0;
+  uint64_t defer_cap = 0;
   // bookkeeping
   std::string err;
   float elapsed_ms = 0.f;
@@ -88,7 +94,6 @@ Scalars* scalars(cadv_ctx* c);
 
 // ---- launchers (each returns cudaSuccess or the launch error; they add the
 // number of kernels they launched to c->launches)
-cudaError_t launch_ingest(cadv_ctx* c);
 // Stable (cta, tid/32) ordering of a non-warp-contiguous trace: fills `out`
 // with device copies of every column in that order.
 cudaError_t regroup_by_warp(cadv_ctx* c, cadv_trace_desc* out);
@@ -111,6 +116,8 @@ struct ScanParams {
   // branch divergence
   uint32_t ws_bd = 5;
   uint32_t* tc = nullptr;
+  uint32_t tc_cap = 0, tc_gen = 0;
+  uint64_t defer_cap = 0;
   uint64_t* bd_tot = nullptr;
   uint64_t* bd_sites = nullptr;
   void* defer = nullptr;
@@ -123,8 +130,8 @@ void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nwarps, ui
 cudaError_t launch_squeeze(cadv_ctx* c, const uint32_t* kin, const uint64_t* vin, uint32_t* kout, uint64_t* vout,
                            const uint64_t* cnt, const uint64_t* off, uint64_t nblocks, uint64_t chunk_cap);
 cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P);
-cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const uint32_t* tc, uint32_t ws,
-                              uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites);
+cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const uint32_t* tc, uint32_t tc_gen,
+                              uint32_t ws, uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites);
 
 // ---- reuse distance around the scan (reuse.cu)
 struct RdState {

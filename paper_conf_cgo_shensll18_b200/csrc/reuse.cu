@@ -825,7 +825,7 @@ int g_mc_smem_set = 0;
 cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st) {
   cudaError_t e;
   const uint64_t n = c->t.n;
-  const uint64_t nmem = c->n_kind[0] + c->n_kind[1];
+  const uint64_t nmem = n;  // memory records <= records (R0 counts now come out of the scan)
   st->cta_scope = scope == CADV_SCOPE_CTA;
   uint64_t grid, nw, chunk;
   scan_geometry(c, n, &grid, &nw, &chunk);
@@ -866,6 +866,16 @@ cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const 
   uint64_t* d_send = (uint64_t*)cb;
   uint64_t* d_mat = d_send + G + 2;
   const uint64_t Kl = *K;
+  {
+    // every rank's CTA-id range of its kept records -> the global range
+    uint32_t* dm = (uint32_t*)d_mat;
+    if ((e = cudaMemcpyAsync(dm, &c->max_cta, 4, cudaMemcpyHostToDevice, c->stream))) return e;
+    if (cm->allreduce_max_u32(dm, 1, c->stream)) return cudaErrorUnknown;
+    uint32_t gm = 0;
+    if ((e = cudaMemcpyAsync(&gm, dm, 4, cudaMemcpyDeviceToHost, c->stream))) return e;
+    if ((e = cudaStreamSynchronize(c->stream))) return e;
+    c->max_cta = gm;
+  }
   if (!cta_scope) {
     scnt[0] = Kl;
   } else {
@@ -970,7 +980,10 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     if ((e = launch_squeeze(c, (const uint32_t*)k1, (const uint64_t*)v1, (uint32_t*)k0, (uint64_t*)v0, S.blkcnt, off,
                             S.grid, S.chunk_cap)))
       return e;
+    unsigned long long mxc = 0;  // CTA-id range of the kept records (and BB groups), from the scan / squeeze
+    if ((e = cudaMemcpyAsync(&mxc, &scalars(c)->max_cta, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
     if ((e = cudaStreamSynchronize(c->stream))) return e;
+    if (mxc > c->max_cta) c->max_cta = (uint32_t)mxc;
     c->counts[0] = K;
     // ---- R1b regroup by CTA (stable)
     val = (const uint64_t*)v0;

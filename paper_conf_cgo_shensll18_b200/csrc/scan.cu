@@ -85,7 +85,9 @@ struct ScanArgs {
   uint64_t* md_sites;    // [nsites][2] or null
   // BD
   uint32_t ws_bd;
-  uint32_t* tc;          // T_c per CTA id (RED.MAX)
+  uint32_t* tc;          // T_c per CTA id (RED.MAX of gen << 11 | T_c)
+  uint32_t tc_cap, tc_gen;
+  uint64_t defer_cap;
   uint64_t* bd_tot;      // [3] exec, divergent, threads
   uint64_t* bd_sites;    // [nsites][3] or null
   uint4* defer;          // deferred partial groups
@@ -113,6 +115,17 @@ __device__ __forceinline__ uint32_t gather8(uint32_t x, uint32_t y) { return gat
 __device__ __forceinline__ uint32_t bits_from(uint32_t a, uint32_t e) {
   const uint32_t hi = e >= 32 ? FULL : ((1u << e) - 1u);
   return hi & ~((1u << a) - 1u);
+}
+
+// T_c candidate of one BB group (RED.MAX, tagged with the call's generation);
+// a CTA id beyond the table's capacity makes the host grow it and rerun.
+__device__ __forceinline__ void tc_update(const ScanArgs& A, uint32_t cta, uint32_t maxtid) {
+  if (cta < A.tc_cap) {
+    red_max(A.tc + cta, (A.tc_gen << 11) | (maxtid + 1u));
+  } else {
+    A.sc->tc_overflow = 1;
+    atomicMax(&A.sc->max_cta, (unsigned long long)cta);
+  }
 }
 
 struct Counters {        // block-level shared-memory accumulators
@@ -221,7 +234,8 @@ __device__ __forceinline__ void finish_bd(const ScanArgs& A, const Counters& C, 
                                           uint32_t cnt, uint32_t s, uint32_t cta, uint32_t wsub, uint32_t maxtid) {
   acc.bd_exec += 1;
   acc.bd_threads += cnt;
-  red_max(A.tc + cta, maxtid + 1u);
+  tc_update(A, cta, maxtid);
+  atomicMax(&A.sc->max_cta, (unsigned long long)cta);  // rare (exact walk) path
   if (sites_smem) {
     if (s < A.nsites) { atomicAdd(&C.bd_sites[3 * s], 1u); atomicAdd(&C.bd_sites[3 * s + 2], cnt); }
     else *A.site_flag = 1;
@@ -230,7 +244,7 @@ __device__ __forceinline__ void finish_bd(const ScanArgs& A, const Counters& C, 
   }
   if (cnt < (1u << A.ws_bd)) {
     const unsigned long long k = atomicAdd(A.ndefer, 1ull);
-    A.defer[k] = make_uint4(cta, wsub, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
+    if (k < A.defer_cap) A.defer[k] = make_uint4(cta, wsub, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
   }
 }
 
@@ -300,7 +314,7 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
                                         const RunQueue Q, uint32_t qn, uint64_t c_lo) {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   const uint32_t lane = lane_id();
-  uint32_t exec = 0, thr = 0;
+  uint32_t exec = 0, thr = 0, mxc = 0;
   for (uint32_t q0 = 0; q0 < qn; q0 += 32) {
     const uint32_t q = q0 + lane;
     bool md = false, bd = false;
@@ -329,7 +343,8 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
       if (bd) {
         exec += 1;
         thr += cnt;
-        red_max(A.tc + cta, ((t & ~31u) | (31u - __clz(m))) + 1u);
+        mxc = max(mxc, cta);
+        tc_update(A, cta, (t & ~31u) | (31u - __clz(m)));
         if (sites_smem) {
           if (s < A.nsites) { atomicAdd(&C.bd_sites[3 * s], 1u); atomicAdd(&C.bd_sites[3 * s + 2], cnt); }
           else *A.site_flag = 1;
@@ -345,15 +360,21 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
         unsigned long long b = 0;
         if (lane == leader) b = atomicAdd(A.ndefer, (unsigned long long)__popc(dm));
         b = __shfl_sync(FULL, b, leader);
-        if (need)
-          A.defer[b + __popc(dm & lanemask_lt())] = make_uint4(cta, t >> 5, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
+        const unsigned long long slot = b + __popc(dm & lanemask_lt());
+        if (need && slot < A.defer_cap)
+          A.defer[slot] = make_uint4(cta, t >> 5, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
       }
     }
   }
   if (BD) {
     exec = __reduce_add_sync(FULL, exec);
     thr = __reduce_add_sync(FULL, thr);
-    if (lane == 0 && exec) { atomicAdd(&C.bd_tot[0], exec); atomicAdd(&C.bd_tot[2], thr); }
+    mxc = __reduce_max_sync(FULL, mxc);  // the CTA-id range of the BB groups (T_c table size)
+    if (lane == 0 && exec) {
+      atomicAdd(&C.bd_tot[0], exec);
+      atomicAdd(&C.bd_tot[2], thr);
+      atomicMax(&A.sc->max_cta, (unsigned long long)mxc);
+    }
   }
 }
 
@@ -532,6 +553,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         }
       }
       const uint32_t memm = ~ghi & okm, stm = glo & ~ghi & okm, bbm = ~glo & ghi & okm;
+
       // predecessor of record 0: the previous lane's last record (lane 0: the carry)
       uint32_t pc = __shfl_up_sync(FULL, c[LPR - 1], 1);
       uint32_t pkb = __shfl_up_sync(FULL, ((memm >> 7) & 1u) | ((stm >> 6) & 2u) | ((bbm >> 5) & 4u), 1);
@@ -761,6 +783,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   if (RD && lane == 0) {
     A.wcnt[gw] = kept;
   }
+
   if (RD) {
     const uint32_t d = __reduce_add_sync(FULL, ndup);
     if (lane == 0 && d) atomicAdd((unsigned long long*)A.hist0, (unsigned long long)d);
@@ -793,7 +816,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
 
 // Deferred BD groups: divergent iff active < clamp(T_c - w*W, 0, W).
 __global__ void __launch_bounds__(256) k_bd_resolve(const uint4* __restrict__ defer, uint64_t m,
-                                                    const uint32_t* __restrict__ tc, uint32_t ws,
+                                                    const uint32_t* __restrict__ tc, uint32_t gen, uint32_t ws,
                                                     uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites) {
   __shared__ uint32_t s_div[NSITE_SMEM];
   const bool sm = nsites && nsites <= NSITE_SMEM;
@@ -804,7 +827,9 @@ __global__ void __launch_bounds__(256) k_bd_resolve(const uint4* __restrict__ de
   const uint32_t W = 1u << ws;
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < m; i += (uint64_t)gridDim.x * blockDim.x) {
     const uint4 d = defer[i];
-    int64_t live = (int64_t)__ldg(tc + d.x) - (int64_t)d.y * W;
+    const uint32_t v = __ldg(tc + d.x);
+    const uint32_t tcv = (v >> 11) == gen ? (v & 0x7ffu) : 0u;  // 1 + max tid of the CTA's BB records
+    int64_t live = (int64_t)tcv - (int64_t)d.y * W;
     live = live < 0 ? 0 : (live > (int64_t)W ? (int64_t)W : live);
     if ((int64_t)d.z < live) {
       tot++;
@@ -824,16 +849,24 @@ __global__ void __launch_bounds__(256) k_bd_resolve(const uint4* __restrict__ de
 
 // Packs every warp's kept records from its gapped region to their final
 // (exclusive-scan) offsets: one CTA per warp chunk.
+// Also R0's CTA-id range of the kept records (the radix sort's key bits).
 __global__ void __launch_bounds__(256) k_squeeze(const uint32_t* __restrict__ kin, const uint64_t* __restrict__ vin,
                                                  uint32_t* __restrict__ kout, uint64_t* __restrict__ vout,
                                                  const uint64_t* __restrict__ cnt, const uint64_t* __restrict__ off,
-                                                 uint64_t chunk) {
+                                                 uint64_t chunk, Scalars* sc) {
   const uint64_t b = blockIdx.x, m = cnt[b], o = off[b];
   const uint64_t src = b * chunk;
+  uint32_t mx = 0;
   for (uint64_t k = threadIdx.x; k < m; k += blockDim.x) {
     vout[o + k] = vin[src + k];
-    if (kin) kout[o + k] = kin[src + k];
+    if (kin) {
+      const uint32_t key = kin[src + k];
+      kout[o + k] = key;
+      mx = max(mx, key);
+    }
   }
+  mx = __reduce_max_sync(FULL, mx);
+  if (lane_id() == 0 && mx) atomicMax(&sc->max_cta, (unsigned long long)mx);
 }
 
 template <int F>
@@ -880,7 +913,7 @@ void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nwarps, ui
 cudaError_t launch_squeeze(cadv_ctx* c, const uint32_t* kin, const uint64_t* vin, uint32_t* kout, uint64_t* vout,
                            const uint64_t* cnt, const uint64_t* off, uint64_t nchunks, uint64_t chunk) {
   if (nchunks == 0) return cudaSuccess;
-  CADV_LAUNCH(c, k_squeeze<<<(unsigned)nchunks, 256, 0, c->stream>>>(kin, vin, kout, vout, cnt, off, chunk));
+  CADV_LAUNCH(c, k_squeeze<<<(unsigned)nchunks, 256, 0, c->stream>>>(kin, vin, kout, vout, cnt, off, chunk, scalars(c)));
   return cudaGetLastError();
 }
 
@@ -895,7 +928,8 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
   A.lbs_rd = P.lbs_rd; A.cta_scope = P.cta_scope; A.kout = P.kout; A.vout = P.vout; A.wcnt = P.blkcnt;
   A.hist0 = P.hist0;
   A.lbs_md = P.lbs_md; A.ws_md = P.ws_md; A.md_hist = P.md_hist; A.md_sites = P.md_sites;
-  A.ws_bd = P.ws_bd; A.tc = P.tc; A.bd_tot = P.bd_tot; A.bd_sites = P.bd_sites; A.defer = (uint4*)P.defer;
+  A.ws_bd = P.ws_bd; A.tc = P.tc; A.tc_cap = P.tc_cap; A.tc_gen = P.tc_gen; A.defer_cap = P.defer_cap;
+  A.bd_tot = P.bd_tot; A.bd_sites = P.bd_sites; A.defer = (uint4*)P.defer;
   A.ndefer = P.ndefer;
   A.nsites = P.nsites; A.site_flag = P.site_flag; A.sc = scalars(c);
   switch (flags) {
@@ -910,12 +944,12 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
   }
 }
 
-cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const uint32_t* tc, uint32_t ws,
-                              uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites) {
+cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const uint32_t* tc, uint32_t tc_gen,
+                              uint32_t ws, uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites) {
   if (m == 0) return cudaSuccess;
   const uint64_t want = (m + 255) / 256;
   const int grid = (int)(want < (uint64_t)c->num_sms * 4 ? want : (uint64_t)c->num_sms * 4);
-  CADV_LAUNCH(c, k_bd_resolve<<<grid, 256, 0, c->stream>>>((const uint4*)defer, m, tc, ws, bd_tot, bd_sites, nsites));
+  CADV_LAUNCH(c, k_bd_resolve<<<grid, 256, 0, c->stream>>>((const uint4*)defer, m, tc, tc_gen, ws, bd_tot, bd_sites, nsites));
   return cudaGetLastError();
 }
 

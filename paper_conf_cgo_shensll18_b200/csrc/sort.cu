@@ -279,8 +279,7 @@ cudaError_t regroup_by_warp(cadv_ctx* c, cadv_trace_desc* out) {
     return e;
   int grid = c->num_sms * 8;
   CADV_LAUNCH(c, k_warp_keys<<<grid, 256, 0, c->stream>>>(t.cta, t.tid, n, (uint64_t*)k0, (uint32_t*)v0));
-  int bits = 5;
-  while (bits < 64 && ((uint64_t)c->max_cta << 5) >> bits) ++bits;
+  const int bits = 37;  // (cta << 5 | warp): the CTA-id range is not known before the scan
   int res;
   e = radix_sort_pairs<uint64_t, uint32_t>(c, (uint64_t*)k0, (uint32_t*)v0, (uint64_t*)k1, (uint32_t*)v1, n, 0, bits,
                                            &res);
