@@ -149,63 +149,43 @@ __device__ __forceinline__ void site_add(const ScanArgs& A, uint32_t* smem_tab, 
   }
 }
 
-// Per-warp TMA issuer: global column pointers at the chunk start, ring
-// shared-memory addresses, and the byte count of a full piece, computed once.
+// Per-warp TMA issue of piece p (records [c_lo + p KR, ...) of the warp's
+// stream) into ring stage p % KS: one 1-D bulk copy per column, completion
+// counted on the stage's mbarrier.  Stateless: column pointers come from the
+// kernel parameters (constant bank), so no lane holds them in registers.
 template <int F>
-struct Issuer {
-  static constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
-  static constexpr uint32_t FULL_BYTES = KR * (4 + 1 + (NA ? 8 : 0) + (NG ? 2 + 4 + 4 : 0));
-  const uint8_t *ga, *gc, *gt, *gw, *gs, *gm;  // column bytes at record c_lo
-  uint32_t sa, sc, st, sw, ss, sm, sbar;       // shared addresses of stage 0 / barrier 0
-  uint64_t c_lo, s_end;
-  __device__ __forceinline__ void init(const ScanArgs& A, uint8_t* ring, uint64_t* bar, uint64_t lo, uint64_t end) {
-    c_lo = lo;
-    s_end = end;
-    ga = (const uint8_t*)(A.addr + lo); gc = (const uint8_t*)(A.cta + lo); gt = (const uint8_t*)(A.tid + lo);
-    gw = (const uint8_t*)(A.winst + lo); gs = (const uint8_t*)(A.site + lo); gm = (const uint8_t*)(A.meta + lo);
-    const uint32_t r = smem_u32(ring);
-    sa = r + R_ADDR; sc = r + R_CTA; st = r + R_TID; sw = r + R_WINST; ss = r + R_SITE; sm = r + R_META;
-    sbar = smem_u32(bar);
+__device__ __forceinline__ void bulk_cp(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
+               "l"(src), "r"(bytes), "r"(bar)
+               : "memory");
+}
+template <int F>
+__device__ __forceinline__ void issue_piece(const ScanArgs& A, uint32_t ring, uint32_t bar0, uint64_t c_lo,
+                                            uint64_t s_end, uint32_t p) {
+  constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
+  constexpr uint32_t FULL_BYTES = KR * (4 + 1 + (NA ? 8 : 0) + (NG ? 2 + 4 + 4 : 0));
+  const uint32_t stg = p % KS, bar = bar0 + stg * 8;
+  const uint64_t q0 = c_lo + (uint64_t)p * KR;
+  const bool full = q0 + KR <= s_end;
+  const uint32_t cnt = full ? (uint32_t)KR : (uint32_t)(s_end - q0);
+  // partial last piece: sizes rounded up to 16 bytes (sources stay in the padded columns)
+  auto r16 = [](uint32_t b_) { return (b_ + 15u) & ~15u; };
+  uint32_t bytes = FULL_BYTES;
+  if (!full) {
+    bytes = r16(cnt * 4) + r16(cnt);
+    if (NA) bytes += r16(cnt * 8);
+    if (NG) bytes += r16(cnt * 2) + 2 * r16(cnt * 4);
   }
-  __device__ __forceinline__ static void cp(uint32_t dst, const uint8_t* src, uint32_t bytes, uint32_t bar) {
-    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-                 "l"(src), "r"(bytes), "r"(bar)
-                 : "memory");
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+  if (NA) bulk_cp<F>(ring + R_ADDR + stg * KR * 8, A.addr + q0, r16(cnt * 8), bar);
+  bulk_cp<F>(ring + R_CTA + stg * KR * 4, A.cta + q0, r16(cnt * 4), bar);
+  if (NG) {
+    bulk_cp<F>(ring + R_TID + stg * KR * 2, A.tid + q0, r16(cnt * 2), bar);
+    bulk_cp<F>(ring + R_WINST + stg * KR * 4, A.winst + q0, r16(cnt * 4), bar);
+    bulk_cp<F>(ring + R_SITE + stg * KR * 4, A.site + q0, r16(cnt * 4), bar);
   }
-  // piece p -> stage p % KS
-  __device__ __forceinline__ void issue(uint32_t p) const {
-    const uint32_t stg = p % KS, bar = sbar + stg * 8;
-    const uint64_t q0 = c_lo + (uint64_t)p * KR;
-    const uint32_t off = p * KR;
-    if (q0 + KR <= s_end) {
-      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(FULL_BYTES) : "memory");
-      if (NA) cp(sa + stg * KR * 8, ga + (size_t)off * 8, KR * 8, bar);
-      cp(sc + stg * KR * 4, gc + (size_t)off * 4, KR * 4, bar);
-      if (NG) {
-        cp(st + stg * KR * 2, gt + (size_t)off * 2, KR * 2, bar);
-        cp(sw + stg * KR * 4, gw + (size_t)off * 4, KR * 4, bar);
-        cp(ss + stg * KR * 4, gs + (size_t)off * 4, KR * 4, bar);
-      }
-      cp(sm + stg * KR, gm + off, KR, bar);
-    } else {
-      // the last (partial) piece: sizes rounded up to 16 bytes
-      const uint32_t cnt = (uint32_t)(s_end - q0);
-      auto r16 = [](uint32_t b) { return (b + 15u) & ~15u; };
-      uint32_t bytes = r16(cnt * 4) + r16(cnt);
-      if (NA) bytes += r16(cnt * 8);
-      if (NG) bytes += r16(cnt * 2) + 2 * r16(cnt * 4);
-      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
-      if (NA) cp(sa + stg * KR * 8, ga + (size_t)off * 8, r16(cnt * 8), bar);
-      cp(sc + stg * KR * 4, gc + (size_t)off * 4, r16(cnt * 4), bar);
-      if (NG) {
-        cp(st + stg * KR * 2, gt + (size_t)off * 2, r16(cnt * 2), bar);
-        cp(sw + stg * KR * 4, gw + (size_t)off * 4, r16(cnt * 4), bar);
-        cp(ss + stg * KR * 4, gs + (size_t)off * 4, r16(cnt * 4), bar);
-      }
-      cp(sm + stg * KR, gm + off, r16(cnt), bar);
-    }
-  }
-};
+  bulk_cp<F>(ring + R_META + stg * KR, A.meta + q0, r16(cnt), bar);
+}
 
 // run identity: (cta, warp32, winst, family)
 __device__ __forceinline__ uint32_t run_hi(uint32_t tid, uint32_t meta) {
@@ -434,11 +414,10 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       fence_barrier_init();
     }
     __syncwarp();
-    Issuer<F> io;
-    io.init(A, ring, bar, c_lo, s_end);
+    const uint32_t ring_s = smem_u32(ring), bar_s = smem_u32(bar);
     uint32_t issued = npieces < (uint32_t)KS ? npieces : (uint32_t)KS, waited = 0;
     if (lane == 0)
-      for (uint32_t p = 0; p < issued; ++p) io.issue(p);
+      for (uint32_t p = 0; p < issued; ++p) issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, p);
     const RingView R{(const uint64_t*)(ring + R_ADDR), (const uint32_t*)(ring + R_CTA),
                      (const uint16_t*)(ring + R_TID),  (const uint32_t*)(ring + R_WINST),
                      (const uint32_t*)(ring + R_SITE), ring + R_META};
@@ -472,7 +451,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       if (p >= 1 && issued < npieces) {
         if (lane == 0) {
           fence_proxy_async();
-          io.issue(issued);
+          issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, issued);
         }
         ++issued;
       }
