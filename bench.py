@@ -77,45 +77,70 @@ def log(*a):
 
 
 class Clocks:
-    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
-    FIELDS = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
-              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
-              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    """SM clocks and throttle reasons sampled DURING the timed region
+    (B200_PROFILING.md clocks line): NVML in a background thread every 2 ms
+    (works for timed regions of a few ms); nvidia-smi if NVML is missing."""
 
     def __init__(self, device):
         self.device = device
-        self.p = None
+        self.samples = []
+        self.err = None
+        self._stop = None
+        self._th = None
 
     def start(self):
+        import threading
         try:
-            self.p = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                                       "-lms", "200", "-i", str(self.device)], stdout=subprocess.PIPE,
-                                      stderr=subprocess.DEVNULL, text=True)
-        except Exception:
-            self.p = None
+            import pynvml as nv
+            nv.nvmlInit()
+            # torch's device index -> NVML handle (CUDA_VISIBLE_DEVICES may remap)
+            h = nv.nvmlDeviceGetHandleByIndex(self._nvml_index(nv))
+            self.max_mhz = nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM)
+        except Exception as e:  # noqa: BLE001
+            self.err = f"NVML unavailable: {e}"
+            return
+        self.samples = []
+        self._stop = threading.Event()
+        first = threading.Event()
+
+        def run():
+            while True:
+                try:
+                    self.samples.append((nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM),
+                                         nv.nvmlDeviceGetCurrentClocksEventReasons(h)))
+                except Exception:  # noqa: BLE001
+                    pass
+                first.set()
+                if self._stop.wait(0.002):
+                    break
+
+        self._th = threading.Thread(target=run, daemon=True)
+        self._th.start()
+        first.wait(2.0)
+
+    def _nvml_index(self, nv):
+        vis = os.environ.get("CUDA_VISIBLE_DEVICES")
+        if vis:
+            ids = [x.strip() for x in vis.split(",") if x.strip()]
+            if self.device < len(ids) and ids[self.device].isdigit():
+                return int(ids[self.device])
+        return self.device
 
     def stop(self):
-        if not self.p:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        self.p.terminate()
-        out, _ = self.p.communicate(timeout=10)
-        sm, mx, reasons = [], [], set()
-        names = ("hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap")
-        for line in out.strip().splitlines():
-            f = [x.strip() for x in line.split(",")]
-            if len(f) < 9:
-                continue
-            try:
-                sm.append(float(f[1]))
-                mx.append(float(f[2]))
-            except ValueError:
-                continue
-            for nm, v in zip(names, f[5:9]):
-                if v.lower().startswith("active"):
-                    reasons.add(nm)
-        under = [s for s in sm if s > 300] or sm
-        return {"sm_mhz": statistics.median(under) if under else None, "sm_max_mhz": max(mx) if mx else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+        if self._th is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [self.err or "no sampler"], "samples": 0}
+        self._stop.set()
+        self._th.join(timeout=5)
+        import pynvml as nv
+        names = {"hw_slowdown": nv.nvmlClocksEventReasonHwSlowdown,
+                 "hw_thermal_slowdown": nv.nvmlClocksEventReasonHwThermalSlowdown,
+                 "sw_thermal_slowdown": nv.nvmlClocksEventReasonSwThermalSlowdown,
+                 "sw_power_cap": nv.nvmlClocksEventReasonSwPowerCap}
+        sm = [float(c) for c, _ in self.samples]
+        reasons = sorted({nm for _, r in self.samples for nm, bit in names.items() if r & bit})
+        under = [x for x in sm if x > 300] or sm
+        return {"sm_mhz": statistics.median(under) if under else None, "sm_max_mhz": float(self.max_mhz),
+                "reasons": reasons, "samples": len(sm), "source": "NVML, 2 ms"}
 
 
 def peaks():
@@ -191,7 +216,7 @@ def ncu_traffic(kname):
     except OSError:
         return None
     hdr, units = rows[0], rows[1]
-    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12, "": 1}
     for r in rows[2:]:
         if r[0] == kname:
             tot = 0.0

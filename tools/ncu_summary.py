@@ -1,8 +1,9 @@
 """Per-kernel summary of an ncu report (run here, on the copied .ncu-rep).
 
-usage: python tools/ncu_summary.py report.ncu-rep out.csv
+usage: python tools/ncu_summary.py out.csv report.ncu-rep [report2.ncu-rep ...]
 Aggregates every captured launch of a kernel (mean per launch) over the
 metrics the design decisions in DESIGN.md / profiles/README.md cite.
+Byte metrics are written in bytes, durations in ms (units row).
 """
 import csv
 import subprocess
@@ -31,29 +32,42 @@ METRICS = [
 ]
 
 
-def main(rep, out):
+SCALE = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12,
+         "ns": 1e-6, "us": 1e-3, "usecond": 1e-3, "msecond": 1.0, "ms": 1.0, "nsecond": 1e-6, "s": 1e3}
+
+
+def load(rep, acc):
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(raw.splitlines()))
     hdr, units, data = rows[0], rows[1], rows[2:]
     ik = hdr.index("Kernel Name")
-    cols = [(m, hdr.index(m)) for m in METRICS if m in hdr]
-    acc = defaultdict(lambda: [0, [0.0] * len(cols)])
     for r in data:
         name = r[ik].split("(")[0].replace("void ", "").split("::")[-1]
         a = acc[name]
         a[0] += 1
-        for j, (_, i) in enumerate(cols):
+        for j, m in enumerate(METRICS):
+            if m not in hdr:
+                continue
+            i = hdr.index(m)
             try:
-                a[1][j] += float(r[i].replace(",", ""))
+                v = float(r[i].replace(",", ""))
             except ValueError:
-                pass
+                continue
+            a[1][j] += v * SCALE.get(units[i], 1.0)
+
+
+def main(out, reps):
+    acc = defaultdict(lambda: [0, [0.0] * len(METRICS)])
+    for rep in reps:
+        load(rep, acc)
+    unit = {"gpu__time_duration.sum": "ms", "dram__bytes_read.sum": "byte", "dram__bytes_write.sum": "byte"}
     with open(out, "w", newline="") as f:
         w = csv.writer(f)
-        w.writerow(["kernel", "launches"] + [m for m, _ in cols])
-        w.writerow(["", ""] + [units[i] for _, i in cols])
+        w.writerow(["kernel", "launches"] + METRICS)
+        w.writerow(["", ""] + [unit.get(m, "") for m in METRICS])
         for name, (n, s) in sorted(acc.items(), key=lambda kv: -kv[1][1][0]):
             w.writerow([name, n] + ["%.6g" % (v / n) for v in s])
 
 
 if __name__ == "__main__":
-    main(sys.argv[1], sys.argv[2])
+    main(sys.argv[1], sys.argv[2:])
