@@ -546,12 +546,16 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       //        with the weight of the chain piece it heads.  Chains are cut at
       //        step starts and at the chunk end (both only split a piece).
       if (RD) {
+        // same (scope, line) as the predecessor: 32-bit halves, line bits only (lbs <= 12)
         uint32_t eqm = 0;
-        const uint64_t lim = 1ull << A.lbs_rd;
+        const uint32_t mlo = ~((1u << A.lbs_rd) - 1u), msc = A.cta_scope ? 0xffffffffu : 0u;
 #pragma unroll
         for (int k = 0; k < LPR; ++k) {
-          const bool e = (a[k] ^ (k == 0 ? pa : a[k - 1])) < lim && (!A.cta_scope || c[k] == (k == 0 ? pc : c[k - 1]));
-          eqm |= (uint32_t)e << k;
+          const uint64_t q = k == 0 ? pa : a[k - 1];
+          const uint32_t qs = k == 0 ? pc : c[k - 1];
+          const uint32_t x = (((uint32_t)a[k] ^ (uint32_t)q) & mlo) | ((uint32_t)(a[k] >> 32) ^ (uint32_t)(q >> 32)) |
+                             ((c[k] ^ qs) & msc);
+          eqm |= (uint32_t)(x == 0u) << k;
         }
         const uint32_t pm = ((memm << 1) | (pkb & 1u)) & 0xffu, ps = ((stm << 1) | ((pkb >> 1) & 1u)) & 0xffu;
         const uint32_t dupm = eqm & memm & ~stm & pm;
@@ -608,19 +612,21 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       // ================= M1-M3 / B1-B3: runs = warp-level groups
       if (NG) {
         uint32_t rsm = 0, nlm = 0, vim = 0, bits[LPR];
-        const uint64_t lim = 1ull << A.lbs_md;
+        const uint32_t mlo = ~((1u << A.lbs_md) - 1u);
 #pragma unroll
         for (int k = 0; k < LPR; ++k) {
           const uint32_t qc = k == 0 ? pc : c[k - 1], qw = k == 0 ? pwi : w[k - 1], qt = k == 0 ? pt : t[k - 1];
-          rsm |= (uint32_t)(c[k] != qc || w[k] != qw || (t[k] ^ qt) >= 32u) << k;
+          const uint32_t x = (c[k] ^ qc) | (w[k] ^ qw) | ((t[k] ^ qt) & ~31u);  // (cta, winst, warp32) differ
+          rsm |= (uint32_t)(x != 0u) << k;
           if (MD) {
             const uint64_t qa = k == 0 ? pa : a[k - 1];
-            const bool ne = (a[k] ^ qa) >= lim;
-            nlm |= (uint32_t)ne << k;
-            vim |= (uint32_t)(ne && a[k] < qa) << k;
+            const uint32_t y = (((uint32_t)a[k] ^ (uint32_t)qa) & mlo) | ((uint32_t)(a[k] >> 32) ^ (uint32_t)(qa >> 32));
+            nlm |= (uint32_t)(y != 0u) << k;
+            vim |= (uint32_t)(a[k] < qa) << k;  // only where the line changes (masked below)
           }
           bits[k] = 1u << (t[k] & 31u);
         }
+        vim &= nlm;
         rsm |= (bbm ^ ((bbm << 1) | ((pkb >> 2) & 1u))) & 0xffu;  // BB and memory records never share a run
         rsm |= ~inbm & 0xffu;  // every record past the stream is a run of its own (never finalized)
         nlm |= rsm;
