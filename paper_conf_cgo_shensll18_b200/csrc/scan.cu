@@ -508,15 +508,18 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
                              ((v >> 4) & ((v >> 3) | (v >> 2)) & ~hi & 0x01010101u);        // memory size > 16 B
           badm |= gather4(b) << (4 * h);
         }
+        uint32_t abad = 0;  // memory records: address bits below the access size, or >= 2^58 (lane-level)
         if (NA) {
+          const uint32_t memk = ~ghi & ownm;
 #pragma unroll
           for (int k = 0; k < LPR; ++k) {
             const uint32_t msk = (1u << ((((k < 4 ? mmx : mmy) >> (8 * (k & 3))) >> 2) & 7u)) - 1u;
-            if (!((ghi >> k) & 1u) && (((uint32_t)a[k] & msk) | ((uint32_t)(a[k] >> 32) & 0xfc000000u))) badm |= 1u << k;
+            const uint32_t v = ((uint32_t)a[k] & msk) | ((uint32_t)(a[k] >> 32) & 0xfc000000u);
+            abad |= (memk >> k) & 1u ? v : 0u;
           }
         }
         badm &= ownm;
-        if (__any_sync(FULL, badm != 0 || (NG && (tor & 0xfc00fc00u)))) {
+        if (__any_sync(FULL, (badm | abad) != 0 || (NG && (tor & 0xfc00fc00u)))) {
 #pragma unroll
           for (int k = 0; k < LPR; ++k) {
             if (!((ownm >> k) & 1u)) continue;
@@ -718,15 +721,18 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           if (tail_open) {
             const uint32_t msk = 0xffu << lastk;
             tu = __popc(nlm & msk) | ((LPR - lastk) << PK_CNT) | (__popc(vim & msk) << PK_VIOL);
-            uint32_t tt = 0, tc = 0;
-#pragma unroll
-            for (int k = 0; k < LPR; ++k)
-              if ((uint32_t)k == lastk) { tmk = rm[k]; tt = t[k]; tc = c[k]; }
+            {  // rm[lastk] by a 3-level select on the bits of lastk
+              const bool b0 = lastk & 1u, b1 = lastk & 2u, b2 = lastk & 4u;
+              const uint32_t x01 = b0 ? rm[1] : rm[0], x23 = b0 ? rm[3] : rm[2];
+              const uint32_t x45 = b0 ? rm[5] : rm[4], x67 = b0 ? rm[7] : rm[6];
+              tmk = b2 ? (b1 ? x67 : x45) : (b1 ? x23 : x01);
+            }
             if (lane < 31) { tu += S_next; tmk |= M_next; }
-            if (lane == hl) {  // the carried run's first record (its piece is recycled before the run closes)
-              qc[0] = ((((lastk < 4 ? mmx : mmy) >> (8 * (lastk & 3u))) & 3u) << 16) | tt;
-              qc[1] = tc;
-              qc[2] = A.nsites ? R.site[ring_slot(j0 + lastk)] : 0u;
+            {  // the carried run's first record (its piece is recycled before the run closes)
+              const uint32_t sl0 = ring_slot(j0 + lastk);
+              qc[0] = ((R.meta[sl0] & 3u) << 16) | R.tid[sl0];
+              qc[1] = R.cta[sl0];
+              qc[2] = A.nsites ? R.site[sl0] : 0u;
             }
           }
           cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
