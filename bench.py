@@ -199,7 +199,7 @@ def algorithmic_bytes(kname, st):
         "k_scan<1>": 13 * n + 12 * kept,            # addr, cta, meta + kept records
         "k_scan<2>": 23 * n,                        # addr, cta, tid, winst, site, meta
         "k_scan<4>": 15 * n,                        # cta, tid, winst, site, meta
-        "k_rd_tile<false>": 12 * kept,              # key 4 + value 8 per kept record
+        "k_rd_tile<0>": 12 * kept,                  # key 4 + value 8 per kept record
         "k_squeeze": 24 * kept,                     # kept records read and written once
     }
     return table.get(kname)

@@ -298,10 +298,14 @@ struct EntryCols {
 // scope) inside the tile; pieces cut by the tile's start (head) or end
 // (tail) are "partial" and emit one entry per distinct line for the
 // cross-tile phase.
-// WIDE = 0: tiles whose line range fits 52 bits (the others are counted in
-// sc->count[3] / listed in wide_list and handled by the WIDE = 1 instance).
-template <bool WIDE>
-__global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
+// MODE (by the tile's line range R = max - min line):
+//   0  R < 2^20: packed u32 sort keys (line - min) << 12 | position (every
+//      tile of the paper-shaped workloads at 128 B lines);
+//   1  R < 2^52: packed u64 keys;  2: lines and positions in separate arrays.
+// The MODE 0 launch covers all tiles and lists the others (sc->count[4] /
+// tile_list + ntiles, sc->count[3] / wide_list) for the MODE 1 / 2 launches.
+template <int MODE>
+__global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     k_rd_tile(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val, uint64_t K,
               const uint32_t* __restrict__ bounds, uint32_t ntiles, int log2bins, uint32_t nbins,
               uint64_t* __restrict__ g_hist, uint64_t* __restrict__ g_stream, uint32_t* __restrict__ tile_w,
@@ -309,7 +313,8 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
   extern __shared__ __align__(128) uint8_t smem_raw[];
   TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
   const uint32_t tx = threadIdx.x;
-  const uint32_t tile = WIDE ? wide_list[blockIdx.x] : blockIdx.x;
+  constexpr bool WIDE = MODE == 2;
+  const uint32_t tile = MODE == 0 ? blockIdx.x : MODE == 1 ? wide_list[ntiles + 2 + blockIdx.x] : wide_list[blockIdx.x];
   const uint64_t b = bounds[tile], e = bounds[tile + 1];
   const uint32_t m = (uint32_t)(e - b);
   const bool smem_hist = nbins <= TL_SMEM_BINS;
@@ -339,11 +344,16 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
   }
   __syncthreads();
   const uint64_t lmin = m ? S.lmin : 0;
-  if (!WIDE && m && ((S.lmax - lmin) >> 52)) {
-    // handled by the WIDE instance
+  if (MODE == 0 && m && ((S.lmax - lmin) >> 20)) {
+    // handled by the MODE 1 / MODE 2 instances
     if (tx == 0) {
-      unsigned long long k = atomicAdd((unsigned long long*)&sc->count[3], 1ull);
-      wide_list[k] = tile;
+      if ((S.lmax - lmin) >> 52) {
+        const unsigned long long k = atomicAdd((unsigned long long*)&sc->count[3], 1ull);
+        wide_list[k] = tile;
+      } else {
+        const unsigned long long k = atomicAdd((unsigned long long*)&sc->count[4], 1ull);
+        wide_list[ntiles + 2 + k] = tile;
+      }
     }
     return;
   }
@@ -351,15 +361,19 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
     for (uint32_t k = tx; k < nbins; k += TL_NT) S.hist[k] = 0;
   // ---- load (striped)
   uint16_t* PSW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[0] : nullptr;
+  uint32_t* const K32a = reinterpret_cast<uint32_t*>(S.key[0]);
+  uint32_t* const K32b = reinterpret_cast<uint32_t*>(S.key[1]);
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) {
     if (x < m) {
       uint64_t v = __ldg(val + b + x);
       uint64_t l = v & LINE_MASK;
-      S.key[0][WIDE ? x : swz<uint64_t>(x)] = WIDE ? l : (((l - lmin) << 12) | x);
+      if (MODE == 0) K32a[swz<uint32_t>(x)] = (uint32_t)(((l - lmin) << 12) | x);
+      else S.key[0][WIDE ? x : swz<uint64_t>(x)] = WIDE ? l : (((l - lmin) << 12) | x);
       uint32_t w = (uint32_t)(v >> VB_W) + 1u;
       S.sdw[x] = (uint8_t)(((v >> VB_STORE) & 1u) | (((v >> VB_DUP) & 1u) << 1) | (w << 2));
     } else {
-      S.key[0][WIDE ? x : swz<uint64_t>(x)] = ~0ull;
+      if (MODE == 0) K32a[swz<uint32_t>(x)] = 0xffffffffu;
+      else S.key[0][WIDE ? x : swz<uint64_t>(x)] = ~0ull;
       S.sdw[x] = 0;
     }
     if (WIDE) PSW[x] = (uint16_t)x;
@@ -406,13 +420,20 @@ __global__ void __launch_bounds__(TL_NT, WIDE ? 1 : 2)
     TileSmemWide& SW = *reinterpret_cast<TileSmemWide*>(smem_raw);
     r = block_merge_sort<TL_NT, IPT, uint64_t, uint16_t, false>(S.key[0], SW.ps[0], S.key[1], SW.ps[1], nullptr,
                                                                 ~0ull);
-  } else {
+  } else if (MODE == 1) {
     r = block_sort_keys<TL_NT, uint64_t, false>(S.key[0], S.key[1], nullptr, ~0ull);
+  } else {
+    r = block_sort_keys<TL_NT, uint32_t, false>(K32a, K32b, nullptr, 0xffffffffu);
   }
   const uint64_t* KS = S.key[r];
+  const uint32_t* KS32 = r ? K32b : K32a;
   const uint16_t* PW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[r] : nullptr;
-  auto POS = [&](uint32_t s_) -> uint32_t { return WIDE ? PW[s_] : (uint32_t)(KS[swz<uint64_t>(s_)] & 0xfffu); };
-  auto LN = [&](uint32_t s_) -> uint64_t { return WIDE ? KS[s_] : (KS[swz<uint64_t>(s_)] >> 12); };
+  auto POS = [&](uint32_t s_) -> uint32_t {
+    return WIDE ? PW[s_] : MODE == 0 ? (KS32[swz<uint32_t>(s_)] & 0xfffu) : (uint32_t)(KS[swz<uint64_t>(s_)] & 0xfffu);
+  };
+  auto LN = [&](uint32_t s_) -> uint64_t {
+    return WIDE ? KS[s_] : MODE == 0 ? (uint64_t)(KS32[swz<uint32_t>(s_)] >> 12) : (KS[swz<uint64_t>(s_)] >> 12);
+  };
   // ---- previous local use; first / last use of the line in its piece
   uint32_t isent = 0, nent = 0;
 #pragma unroll
@@ -1004,7 +1025,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   uint64_t ntiles = (K + TL_NOM - 1) / TL_NOM;
   c->counts[3] = ntiles;
   void *bnd, *tw, *tq;
-  if ((e = ensure(c, B_RD_XTMP, (2 * ntiles + 4) * 4 + 64, &bnd))) return e;  // bounds + wide-tile list
+  if ((e = ensure(c, B_RD_XTMP, (3 * ntiles + 8) * 4 + 64, &bnd))) return e;  // bounds + MODE 2 / MODE 1 lists
   if ((e = ensure(c, B_RD_TILEW, (ntiles + 2) * 8 * 2, &tw))) return e;
   if ((e = ensure(c, B_RD_TILEQ, (ntiles + 2) * 8 * 2, &tq))) return e;
   CADV_LAUNCH(c, k_tile_bounds<<<(unsigned)((ntiles + 1 + 7) / 8), 256, 0, c->stream>>>(key, K, (uint32_t*)bnd,
@@ -1030,9 +1051,9 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     En.lf = (uint8_t*)take(K);
   }
   if (!g_tile_smem_set) {
-    if ((e = cudaFuncSetAttribute(k_rd_tile<false>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)sizeof(TileSmem))) ||
-        (e = cudaFuncSetAttribute(k_rd_tile<true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    if ((e = cudaFuncSetAttribute(k_rd_tile<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))) ||
+        (e = cudaFuncSetAttribute(k_rd_tile<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))) ||
+        (e = cudaFuncSetAttribute(k_rd_tile<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   (int)sizeof(TileSmemWide))))
       return e;
     g_tile_smem_set = 1;
@@ -1040,15 +1061,21 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   uint32_t* tile_w = (uint32_t*)tw;
   uint32_t* tile_q = (uint32_t*)tq;
   uint32_t* wide_list = (uint32_t*)bnd + (ntiles + 2);
-  CADV_LAUNCH(c, k_rd_tile<false><<<(unsigned)ntiles, TL_NT, sizeof(TileSmem), c->stream>>>(
+  CADV_LAUNCH(c, k_rd_tile<0><<<(unsigned)ntiles, TL_NT, sizeof(TileSmem), c->stream>>>(
                      key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
                      tile_q, En, sc, wide_list));
   if ((e = cudaGetLastError())) return e;
-  unsigned long long cnt13[3];
-  if ((e = cudaMemcpyAsync(cnt13, &sc->count[1], 24, cudaMemcpyDeviceToHost, c->stream))) return e;
+  unsigned long long cnt14[4];  // count[1..4]: entries, cross queries, MODE 2 tiles, MODE 1 tiles
+  if ((e = cudaMemcpyAsync(cnt14, &sc->count[1], 32, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
-  if (cnt13[2]) {
-    CADV_LAUNCH(c, k_rd_tile<true><<<(unsigned)cnt13[2], TL_NT, sizeof(TileSmemWide), c->stream>>>(
+  if (cnt14[3]) {
+    CADV_LAUNCH(c, k_rd_tile<1><<<(unsigned)cnt14[3], TL_NT, sizeof(TileSmem), c->stream>>>(
+                       key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
+                       tile_q, En, sc, wide_list));
+    if ((e = cudaGetLastError())) return e;
+  }
+  if (cnt14[2]) {
+    CADV_LAUNCH(c, k_rd_tile<2><<<(unsigned)cnt14[2], TL_NT, sizeof(TileSmemWide), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
                        tile_q, En, sc, wide_list));
     if ((e = cudaGetLastError())) return e;

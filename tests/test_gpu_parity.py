@@ -412,3 +412,17 @@ def test_long_chunks(ctx_long, cadv, case):
 def test_long_chunks_non_contiguous(ctx_long, cadv):
     t = tg.generate("rand", seed=7, ctas=6, threads=128, instrs=15, lines=30, scramble=1, scramble_seed=7)
     full_check(ctx_long, cadv, t, lbs=(32,), contiguous=False, W=(32, 16))
+
+
+@pytest.mark.parametrize("spread", [40, 57])
+def test_tile_key_widths(ctx, cadv, spread):
+    """Tiles whose line range needs 64-bit packed sort keys (2^20 <= range <
+    2^52 lines) or separate line / position arrays (>= 2^52, 1-byte lines):
+    addresses spread over 2^spread bytes, with repeats so reuses exist."""
+    rng = np.random.default_rng(spread)
+    n = 30000
+    base = rng.integers(0, 1 << spread, 500, dtype=np.uint64) & ~np.uint64(15)
+    addr = base[rng.integers(0, 500, n)]
+    meta = np.where(rng.random(n) < 0.2, (2 << 2) | 1, 2 << 2)
+    t = _mk(addr, rng.integers(0, 3, n), meta=meta)
+    full_check(ctx, cadv, t, lbs=(1, 128), W=(32,))
