@@ -11,7 +11,7 @@ CADV_HDR  := $(wildcard $(PKG)/csrc/*.cuh) $(wildcard $(PKG)/csrc/*.h) include/c
 NVFLAGS   := -ccbin $(HOSTCXX) $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -fvisibility=hidden \
              -Iinclude --expt-relaxed-constexpr -Xptxas -v
 
-all: tracegen/libtracegen.so oracle/liboracle.so $(PKG)/libcadv.so
+all: tracegen/libtracegen.so oracle/liboracle.so $(PKG)/libcadv.so $(PKG)/producer/libcadv_demo.so
 
 tracegen/libtracegen.so: tracegen/tracegen.cpp
 	$(HOSTCXX) -O2 -std=c++17 -fopenmp -shared -fPIC -o $@ $<
@@ -22,7 +22,11 @@ oracle/liboracle.so: oracle/oracle.cpp
 $(PKG)/libcadv.so: $(CADV_SRC) $(CADV_HDR)
 	$(NVCC) $(NVFLAGS) -shared -o $@ $(CADV_SRC) -ldl 2> $(PKG)/ptxas.log || (cat $(PKG)/ptxas.log; exit 1)
 
+# hand-instrumented demo kernels (device-side trace producer, include/cadv_record.cuh)
+$(PKG)/producer/libcadv_demo.so: $(PKG)/producer/demo_kernels.cu include/cadv_record.cuh
+	$(NVCC) $(NVFLAGS) -shared -o $@ $< 2> $(PKG)/producer/ptxas.log || (cat $(PKG)/producer/ptxas.log; exit 1)
+
 clean:
-	rm -f tracegen/libtracegen.so oracle/liboracle.so $(PKG)/libcadv.so
+	rm -f tracegen/libtracegen.so oracle/liboracle.so $(PKG)/libcadv.so $(PKG)/producer/libcadv_demo.so
 
 .PHONY: all clean
