@@ -72,10 +72,10 @@ def reuse(t, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66):
     """Returns (hist[nbins] u64, stats dict)."""
     lib = _load()
     hist = np.zeros(nbins, np.uint64)
-    st = np.zeros(4, np.uint64)
+    st = np.zeros(5, np.uint64)
     _check(lib.oracle_reuse(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.meta), t.n, line_bytes, scope, binning,
                             nbins, _p(hist), _p(st)))
-    return hist, dict(zip(("accesses", "inf", "streaming", "overflow"), map(int, st)))
+    return hist, dict(zip(("accesses", "inf", "streaming", "overflow", "finite_sum"), map(int, st)))
 
 
 def reuse_rd(t, line_bytes=128, scope=SCOPE_CTA):
@@ -90,11 +90,11 @@ def reuse_brute(t, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=6
     """O(n^2) literal definition; returns (hist, stats, rd per record)."""
     lib = _load()
     hist = np.zeros(nbins, np.uint64)
-    st = np.zeros(4, np.uint64)
+    st = np.zeros(5, np.uint64)
     rd = np.zeros(t.n, np.int64)
     _check(lib.oracle_reuse_brute(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.meta), t.n, line_bytes, scope, binning,
                                   nbins, _p(hist), _p(st), _p(rd)))
-    return hist, dict(zip(("accesses", "inf", "streaming", "overflow"), map(int, st))), rd
+    return hist, dict(zip(("accesses", "inf", "streaming", "overflow", "finite_sum"), map(int, st))), rd
 
 
 def mem_div(t, line_bytes=128, warp_size=32, nsites=None, per_site=True):

@@ -157,8 +157,9 @@ void lru_scope(const std::vector<uint64_t>& idx, const uint64_t* addr, const uin
 
 extern "C" {
 
-// Reuse-distance histogram (LRU-stack oracle).  hist[nbins]; stats[4] =
-// {accesses, inf, streaming, overflow}.  Returns 0 / 1 (invalid arg) / 2 (bad trace).
+// Reuse-distance histogram (LRU-stack oracle).  hist[nbins]; stats[5] =
+// {accesses, inf, streaming, overflow, sum of the finite distances} (the last
+// gives Eq. (1)'s average reuse distance).  Returns 0 / 1 (invalid arg) / 2 (bad trace).
 int oracle_reuse(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid, const uint8_t* meta, uint64_t n,
                  uint32_t line_bytes, int scope, int binning, uint32_t nbins, uint64_t* hist, uint64_t* stats) {
   int rc = check_reuse_args(line_bytes, scope, binning, nbins);
@@ -166,23 +167,27 @@ int oracle_reuse(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid,
   if (!check_all(addr, nullptr, meta, n)) return BAD_TRACE;
   auto sc = scopes_of(cta, meta, n, scope);
   std::vector<uint64_t> h(nbins, 0);
-  uint64_t streaming = 0;
+  uint64_t streaming = 0, fsum = 0;
 #pragma omp parallel
   {
     std::vector<uint64_t> hl(nbins, 0);
-    uint64_t sl = 0;
+    uint64_t sl = 0, fl = 0;
     std::vector<int64_t> rd;
 #pragma omp for schedule(dynamic, 1)
     for (int64_t s = 0; s < (int64_t)sc.size(); ++s) {
       uint64_t st = 0;
       lru_scope(sc[s], addr, meta, line_bytes, rd, st);
       sl += st;
-      for (int64_t d : rd) hl[d < 0 ? nbins - 1 : bin_of((uint64_t)d, binning, nbins)]++;
+      for (int64_t d : rd) {
+        hl[d < 0 ? nbins - 1 : bin_of((uint64_t)d, binning, nbins)]++;
+        if (d > 0) fl += (uint64_t)d;
+      }
     }
 #pragma omp critical
     {
       for (uint32_t b = 0; b < nbins; ++b) h[b] += hl[b];
       streaming += sl;
+      fsum += fl;
     }
   }
   uint64_t acc = 0;
@@ -191,6 +196,7 @@ int oracle_reuse(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid,
   stats[1] = h[nbins - 1];
   stats[2] = streaming;
   stats[3] = h[nbins - 2];
+  stats[4] = fsum;
   return OK;
 }
 
@@ -239,6 +245,7 @@ int oracle_reuse_brute(const uint64_t* addr, const uint32_t* cta, const uint16_t
     key[i] = std::make_tuple(s, line, stores);
   }
   std::vector<uint64_t> h(nbins, 0);
+  uint64_t fsum = 0;
   for (uint64_t i = 0; i < n; ++i) {
     if (!mem[i]) { if (rd_out) rd_out[i] = -2; continue; }
     int64_t rd = -1;
@@ -255,6 +262,7 @@ int oracle_reuse_brute(const uint64_t* addr, const uint32_t* cta, const uint16_t
     }
     if (rd_out) rd_out[i] = rd;
     h[rd < 0 ? nbins - 1 : bin_of((uint64_t)rd, binning, nbins)]++;
+    if (rd > 0) fsum += (uint64_t)rd;
   }
   uint64_t streaming = 0;
   for (uint64_t i = 0; i < n; ++i) {
@@ -265,7 +273,7 @@ int oracle_reuse_brute(const uint64_t* addr, const uint32_t* cta, const uint16_t
   }
   uint64_t acc = 0;
   for (uint32_t b = 0; b < nbins; ++b) { hist[b] = h[b]; acc += h[b]; }
-  stats[0] = acc; stats[1] = h[nbins - 1]; stats[2] = streaming; stats[3] = h[nbins - 2];
+  stats[0] = acc; stats[1] = h[nbins - 1]; stats[2] = streaming; stats[3] = h[nbins - 2]; stats[4] = fsum;
   return OK;
 }
 

@@ -57,6 +57,8 @@ def test_paper_worked_example(golden_dir):
     assert list(rd) == [-1, -1, -1, 0, -1, -1, -1, 5, 0, 0, 5]
     h, st = orc.reuse(t, line_bytes=4, nbins=8)
     assert h[0] == 3 and h[5] == 2 and h[7] == 6 and h.sum() == 11
+    # Eq. (1)'s average reuse distance over the finite distances: 10 / 5
+    assert st["finite_sum"] == 10 and st["finite_sum"] / (st["accesses"] - st["inf"]) == 2.0
 
 
 @pytest.mark.parametrize("K,R", [(1, 5), (3, 4), (7, 3), (40, 2), (130, 3)])
@@ -69,6 +71,7 @@ def test_cyclic_closed_form(K, R):
     assert h[K - 1] == K * (R - 1)
     assert h.sum() == K * R
     assert st["streaming"] == (K if R == 1 else 0)
+    assert st["finite_sum"] == K * (R - 1) * (K - 1)
 
 
 def test_write_rule_restarts_counting():
