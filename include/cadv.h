@@ -104,6 +104,9 @@ typedef struct {
   uint64_t inf;       /* accesses with no reuse (∞ bin) */
   uint64_t streaming; /* accesses to elements "never reused by the same CTA" */
   uint64_t overflow;  /* finite distances beyond the last exact bin */
+  uint64_t finite_sum; /* sum of all finite distances (exact, overflow included): the
+                          average reuse distance of Eq. (1), is
+                          finite_sum / (accesses - inf) */
 } cadv_reuse_stats;
 
 typedef struct { uint64_t groups, sum_deg; } cadv_site_mem;                 /* per memory site */

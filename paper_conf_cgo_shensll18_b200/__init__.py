@@ -56,7 +56,7 @@ class Analysis(ctypes.Structure):
 
 class ReuseStats(ctypes.Structure):
     _fields_ = [("accesses", ctypes.c_uint64), ("inf", ctypes.c_uint64), ("streaming", ctypes.c_uint64),
-                ("overflow", ctypes.c_uint64)]
+                ("overflow", ctypes.c_uint64), ("finite_sum", ctypes.c_uint64)]
 
 
 _lib = None
@@ -202,7 +202,8 @@ class Context:
         st = ReuseStats()
         self._check(lib().cadv_reuse_histogram(self._h, line_bytes, scope, binning, hist.ctypes.data, nbins,
                                                ctypes.byref(st)))
-        return hist, {"accesses": st.accesses, "inf": st.inf, "streaming": st.streaming, "overflow": st.overflow}
+        return hist, {"accesses": st.accesses, "inf": st.inf, "streaming": st.streaming, "overflow": st.overflow,
+                      "finite_sum": st.finite_sum}
 
     # -- cadv_mem_divergence
     def mem_divergence(self, line_bytes=128, warp_size=32, nsites=0):
@@ -238,7 +239,7 @@ class Context:
                                        p(ms), p(bt), p(bs)))
         if rd:
             out["reuse"] = (rh, {"accesses": st.accesses, "inf": st.inf, "streaming": st.streaming,
-                                 "overflow": st.overflow})
+                                 "overflow": st.overflow, "finite_sum": st.finite_sum})
         if md:
             out["mem_div"] = (mh, ms)
         if bd:

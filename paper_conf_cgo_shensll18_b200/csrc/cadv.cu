@@ -609,6 +609,7 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
       rd_stats->inf = hr[o_rdh + q.nbins - 1];
       rd_stats->overflow = hr[o_rdh + q.nbins - 2];
       rd_stats->streaming = hr[o_rds];
+      rd_stats->finite_sum = hr[o_rds + 1];
     }
   }
   if (q.md) {

@@ -538,6 +538,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   const uint32_t* QS = r2 ? QK2 : QK;
   // ---- R4: bin the local accesses
   uint32_t stream = 0;
+  unsigned long long rdsum = 0;  // finite distances (Eq. (1)'s average reuse distance)
 #pragma unroll
   for (int j = 0; j < IPT; ++j) {
     const uint32_t x = tx * IPT + j;
@@ -551,6 +552,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       const uint32_t p = S.pl[x] - 1u;
       const uint32_t rd = (WP[x] - WP[p] - (uint32_t)(S.sdw[p] >> 2)) - CNT[x];
       bin = rd_bin(rd, log2bins, nbins);
+      rdsum += rd;
     } else if (st) {
       bin = nbins - 1;
       cntb = w;
@@ -598,6 +600,9 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   // ---- flush
   stream = __reduce_add_sync(FULL, stream);
   if (lane_id() == 0 && stream) atomicAdd((unsigned long long*)g_stream, (unsigned long long)stream);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) rdsum += __shfl_xor_sync(FULL, rdsum, o);
+  if (lane_id() == 0 && rdsum) atomicAdd((unsigned long long*)g_stream + 1, rdsum);
   if (tx == 0) {
     tile_w[tile] = WT;
     tile_q[tile] = Q;
@@ -771,7 +776,9 @@ __global__ void k_iota_gather(const uint32_t* __restrict__ order, const uint32_t
 constexpr uint32_t XF_SMEM_BINS = 4096;
 __global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__ part,
                                                      const uint32_t* __restrict__ cnt, uint64_t M, int log2bins,
-                                                     uint32_t nbins, uint64_t* g_hist, Scalars* sc) {
+                                                     uint32_t nbins, uint64_t* g_hist, uint64_t* g_stats,
+                                                     Scalars* sc) {
+  unsigned long long rdsum = 0;
   __shared__ uint32_t h[XF_SMEM_BINS];
   const bool sm = nbins <= XF_SMEM_BINS;
   if (sm)
@@ -784,6 +791,7 @@ __global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__
       rd = 0;
     }
     const uint32_t b = rd_bin((uint64_t)rd, log2bins, nbins);
+    rdsum += (unsigned long long)rd;
     if (sm) {
       // warp-aggregated: one shared-memory atomic per distinct bin in the warp
       const uint32_t peers = __match_any_sync(__activemask(), b);
@@ -792,6 +800,9 @@ __global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__
       atomicAdd((unsigned long long*)&g_hist[b], 1ull);
     }
   }
+#pragma unroll
+  for (int o = 16; o; o >>= 1) rdsum += __shfl_xor_sync(FULL, rdsum, o);
+  if (lane_id() == 0 && rdsum) atomicAdd((unsigned long long*)g_stats + 1, rdsum);
   __syncthreads();
   if (sm)
     for (uint32_t k = threadIdx.x; k < nbins; k += blockDim.x)
@@ -1197,7 +1208,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     std::swap(ka, kb);
     std::swap(ia, ib);
   }
-  CADV_LAUNCH(c, k_cross_final<<<grid_ls, 256, 0, c->stream>>>(X.part, cnt, M, log2bins, nbins, d_hist, sc));
+  CADV_LAUNCH(c, k_cross_final<<<grid_ls, 256, 0, c->stream>>>(X.part, cnt, M, log2bins, nbins, d_hist, d_stats, sc));
   return cudaGetLastError();
 }
 

@@ -426,3 +426,18 @@ def test_tile_key_widths(ctx, cadv, spread):
     meta = np.where(rng.random(n) < 0.2, (2 << 2) | 1, 2 << 2)
     t = _mk(addr, rng.integers(0, 3, n), meta=meta)
     full_check(ctx, cadv, t, lbs=(1, 128), W=(32,))
+
+
+def test_eq1_from_gpu_outputs(ctx, cadv):
+    """NEXT-4: Eq. (1) from the library's outputs equals the
+    same metric from the oracle's (R.D. from the exact finite-distance sum)."""
+    from paper_conf_cgo_shensll18_b200 import metrics as M
+    t = tg.generate("srad", rows=128, cols=128, iters=2)
+    load(ctx, cadv, t)
+    o = ctx.analyze(rd=(128, 0, 0, 20), md=(128, 32), bd=None, nsites=t.nsites)
+    h_ref, s_ref = orc.reuse(t, 128, 0, 0, 20)
+    assert o["reuse"][1] == s_ref and s_ref["overflow"] > 0   # the mean needs the exact sum, not the bins
+    rd, md = M.mean_reuse_distance(o["reuse"][1]), M.md_degree(o["mem_div"][0])
+    assert rd == M.mean_reuse_distance(s_ref) and md == M.md_degree(orc.mem_div(t, 128)[0])
+    assert M.opt_num_warps(16384, rd, 128, md, 4) == M.opt_num_warps(16384, M.mean_reuse_distance(s_ref), 128,
+                                                                       orc.md_degree(orc.mem_div(t, 128)[0]), 4)

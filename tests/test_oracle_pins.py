@@ -10,6 +10,7 @@ Each pin cites the PAPER.md passage or the closed form it checks (DESIGN.md
   - wrong binning index                        -> explicit bin-boundary cases
 """
 import json
+import math
 import os
 
 import numpy as np
@@ -361,3 +362,21 @@ def test_kernel_scope_properties_match_oracle():
             for scope in (1,):
                 h, s = orc.reuse(t, lb, scope, 0, 40)
                 assert kernel_scope_properties(t, lb) == (int(h.sum()), int(h[-1]), s["streaming"])
+
+
+def test_eq1_bypass_warps_arithmetic():
+    """PAPER.md L363 Eq. (1): floor(L1 / (R.D. * line * M.D. * CTAs/SM)),
+    with R.D. and M.D. from the analyses' outputs (here the oracle's)."""
+    from paper_conf_cgo_shensll18_b200 import metrics as M
+    assert M.opt_num_warps(16 * 1024, 2.0, 128, 2.0, 1) == 32
+    assert M.opt_num_warps(48 * 1024, 3.0, 128, 4.0, 2) == 16
+    assert M.opt_num_warps(24 * 1024, 0.0, 128, 2.0, 1) == -1
+    t = literal(list("ABCCDEFAAAB"))
+    _, st = orc.reuse(t, line_bytes=4, nbins=8)
+    assert M.mean_reuse_distance(st) == 2.0
+    h = np.zeros((2, 33), np.uint64)
+    h[0, 1] = 3
+    h[1, 32] = 1
+    assert M.md_degree(h) == pytest.approx(orc.md_degree(h)) == pytest.approx(35 / 4)
+    s = M.instance_stats([1.0, 2.0, 3.0, 6.0])
+    assert s["mean"] == 3.0 and s["min"] == 1.0 and s["max"] == 6.0 and s["stddev"] == pytest.approx(math.sqrt(3.5))
