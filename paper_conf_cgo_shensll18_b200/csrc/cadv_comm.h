@@ -21,6 +21,14 @@ class Comm {
   // them at its roff[me]; rcnt[p] = what p sends here (host arrays of nranks)
   virtual int alltoallv(const void* send, const uint64_t* soff, const uint64_t* scnt, void* recv,
                         const uint64_t* roff, const uint64_t* rcnt, cudaStream_t s) = 0;
+  // Peer memory: every rank passes the base of one of its device allocations
+  // (slot = which of the caller's buffers); peers[p] = rank p's allocation
+  // mapped into this process (CUDA IPC over NVLink for NCCL contexts, plain
+  // pointers for in-process loopback ranks), so kernels can store into it.
+  // Mappings are cached per (slot, peer) and reopened when a peer reallocates.
+  virtual int map_peers(int slot, void* local, void** peers, cudaStream_t s) = 0;
+  // All ranks reach this point with their queued work complete.
+  virtual int barrier(cudaStream_t s) = 0;
   const int rank, nranks;
   std::string err;
 };

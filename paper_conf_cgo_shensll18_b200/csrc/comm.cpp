@@ -82,6 +82,10 @@ class NcclComm : public Comm {
  public:
   NcclComm(int rank, int nranks, ncclComm_t c) : Comm(rank, nranks), comm_(c) {}
   ~NcclComm() override {
+    for (auto& v : cache_)
+      for (auto& m : v)
+        if (m.ptr) cudaIpcCloseMemHandle(m.ptr);
+    if (dev_) cudaFree(dev_);
     if (comm_) g_nccl.CommDestroy(comm_);
   }
   int allreduce_sum_u64(uint64_t* d, size_t n, cudaStream_t s) override {
@@ -104,8 +108,50 @@ class NcclComm : public Comm {
     e |= ck(g_nccl.GroupEnd());
     return e;
   }
+  int map_peers(int slot, void* local, void** peers, cudaStream_t s) override {
+    cudaIpcMemHandle_t h;
+    if (cu(cudaIpcGetMemHandle(&h, local))) return 1;
+    if (!dev_) {
+      if (cu(cudaMalloc(&dev_, (size_t)(nranks + 1) * sizeof h))) return 1;
+    }
+    uint8_t* d = (uint8_t*)dev_;
+    if (cu(cudaMemcpyAsync(d, &h, sizeof h, cudaMemcpyHostToDevice, s))) return 1;
+    if (ck(g_nccl.AllGather(d, d + sizeof h, sizeof h, ncclUint8, comm_, s))) return 1;
+    std::vector<cudaIpcMemHandle_t> all(nranks);
+    if (cu(cudaMemcpyAsync(all.data(), d + sizeof h, nranks * sizeof h, cudaMemcpyDeviceToHost, s))) return 1;
+    if (cu(cudaStreamSynchronize(s))) return 1;
+    if ((int)cache_.size() <= slot) cache_.resize(slot + 1, std::vector<Mapped>(nranks));
+    for (int p = 0; p < nranks; ++p) {
+      if (p == rank) { peers[p] = local; continue; }
+      Mapped& m = cache_[slot][p];
+      if (!m.ptr || memcmp(&m.h, &all[p], sizeof h)) {
+        if (m.ptr) cudaIpcCloseMemHandle(m.ptr);
+        m.ptr = nullptr;
+        if (cu(cudaIpcOpenMemHandle(&m.ptr, all[p], cudaIpcMemLazyEnablePeerAccess))) return 1;
+        m.h = all[p];
+      }
+      peers[p] = m.ptr;
+    }
+    return 0;
+  }
+  int barrier(cudaStream_t s) override {
+    if (!dev_ && cu(cudaMalloc(&dev_, (size_t)(nranks + 1) * sizeof(cudaIpcMemHandle_t)))) return 1;
+    if (ck(g_nccl.AllReduce(dev_, dev_, 1, ncclUint32, ncclMax, comm_, s))) return 1;
+    return cu(cudaStreamSynchronize(s));
+  }
 
  private:
+  struct Mapped {
+    cudaIpcMemHandle_t h;
+    void* ptr = nullptr;
+  };
+  std::vector<std::vector<Mapped>> cache_;
+  void* dev_ = nullptr;
+  int cu(cudaError_t e) {
+    if (e == cudaSuccess) return 0;
+    err = std::string("CUDA IPC: ") + cudaGetErrorString(e);
+    return 1;
+  }
   int ck(ncclResult_t r) {
     if (r == ncclSuccess) return 0;
     err = std::string("NCCL: ") + g_nccl.GetErrorString(r);
@@ -143,7 +189,7 @@ Comm* make_nccl_comm(const void* id128, int rank, int nranks, std::string* err) 
 
 // ------------------------------------------------------------------ loopback
 struct LoopbackGroup {
-  explicit LoopbackGroup(int n) : n(n), slot(n), soff(n), scnt(n) {}
+  explicit LoopbackGroup(int n) : n(n), slot(n), soff(n), scnt(n), ptr(n, nullptr) {}
   int n;
   std::mutex mu;
   std::condition_variable cv;
@@ -151,6 +197,7 @@ struct LoopbackGroup {
   uint64_t generation = 0;
   std::vector<std::vector<uint8_t>> slot;  // per-rank host staging of the contribution
   std::vector<std::vector<uint64_t>> soff, scnt;
+  std::vector<void*> ptr;  // map_peers: the ranks' device buffers (one process, one address space)
   void barrier() {
     std::unique_lock<std::mutex> lk(mu);
     const uint64_t g = generation;
@@ -204,6 +251,18 @@ class LoopbackComm : public Comm {
         return finish(1);
     }
     return finish(cuda(cudaStreamSynchronize(s)));
+  }
+  int map_peers(int slot, void* local, void** peers, cudaStream_t s) override {
+    (void)slot;
+    const int e0 = cuda(cudaStreamSynchronize(s));
+    g_->ptr[rank] = local;
+    g_->barrier();
+    for (int p = 0; p < nranks; ++p) peers[p] = g_->ptr[p];
+    return finish(e0);
+  }
+  int barrier(cudaStream_t s) override {
+    const int e0 = cuda(cudaStreamSynchronize(s));
+    return finish(e0);
   }
 
  private:

@@ -31,6 +31,8 @@
 //                    inversion count on the compacted cross-tile set.
 #include <cuda_runtime.h>
 #include <stdio.h>
+#include <stdlib.h>
+#include <string.h>
 
 #include <vector>
 
@@ -843,6 +845,30 @@ __global__ void k_lower_bounds(const uint32_t* __restrict__ key, uint64_t K, int
   out[r] = lo;
 }
 
+// Exchange over peer memory: every rank stores its slice for rank r straight
+// into r's receive buffers (CUDA IPC mappings over NVLink / NVSwitch, or the
+// in-process loopback ranks' buffers), one launch for all destinations.
+constexpr int MAX_RANKS = 64;
+struct PushArgs {
+  const uint32_t* key;
+  const uint64_t* val;
+  uint32_t* pk[MAX_RANKS];
+  uint64_t* pv[MAX_RANKS];
+  uint64_t soff[MAX_RANKS], scnt[MAX_RANKS], doff[MAX_RANKS];
+};
+__global__ void __launch_bounds__(256) k_push(const __grid_constant__ PushArgs P) {
+  const int r = blockIdx.y;
+  const uint64_t n = P.scnt[r];
+  const uint32_t* ks = P.key ? P.key + P.soff[r] : nullptr;
+  const uint64_t* vs = P.val + P.soff[r];
+  uint32_t* kd = P.key ? P.pk[r] + P.doff[r] : nullptr;
+  uint64_t* vd = P.pv[r] + P.doff[r];
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    if (ks) kd[i] = __ldg(ks + i);
+    vd[i] = __ldg(vs + i);
+  }
+}
+
 int bits_for(uint64_t maxv) {
   int b = 0;
   while (b < 64 && (maxv >> b)) ++b;
@@ -973,12 +999,43 @@ cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const 
     for (auto& x : o) x *= f;
     return o;
   };
-  if (cta_scope && cm->alltoallv(*key, scaled(soff, 4).data(), scaled(scnt, 4).data(), rk0, scaled(roff, 4).data(),
-                                 scaled(rcnt, 4).data(), c->stream))
-    return cudaErrorUnknown;
-  if (cm->alltoallv(*val, scaled(soff, 8).data(), scaled(scnt, 8).data(), rv0, scaled(roff, 8).data(),
-                    scaled(rcnt, 8).data(), c->stream))
-    return cudaErrorUnknown;
+  const bool via_nccl = getenv("CADV_EXCHANGE") && !strcmp(getenv("CADV_EXCHANGE"), "nccl");
+  if (via_nccl || G > MAX_RANKS) {
+    // baseline: NCCL grouped send / receive
+    if (cta_scope && cm->alltoallv(*key, scaled(soff, 4).data(), scaled(scnt, 4).data(), rk0,
+                                   scaled(roff, 4).data(), scaled(rcnt, 4).data(), c->stream))
+      return cudaErrorUnknown;
+    if (cm->alltoallv(*val, scaled(soff, 8).data(), scaled(scnt, 8).data(), rv0, scaled(roff, 8).data(),
+                      scaled(rcnt, 8).data(), c->stream))
+      return cudaErrorUnknown;
+  } else {
+    // peer memory: map the receive buffers of every rank, store the slices directly
+    PushArgs P{};
+    void* pk[MAX_RANKS];
+    void* pv[MAX_RANKS];
+    if (cta_scope && cm->map_peers(0, rk0, pk, c->stream)) return cudaErrorUnknown;
+    if (cm->map_peers(1, rv0, pv, c->stream)) return cudaErrorUnknown;
+    P.key = cta_scope ? *key : nullptr;
+    P.val = *val;
+    uint64_t maxc = 0;
+    for (int r = 0; r < G; ++r) {
+      P.pk[r] = cta_scope ? (uint32_t*)pk[r] : nullptr;
+      P.pv[r] = (uint64_t*)pv[r];
+      P.soff[r] = soff[r];
+      P.scnt[r] = scnt[r];
+      uint64_t d = 0;  // where my slice starts in rank r's buffer: what ranks < me send to r
+      for (int p = 0; p < me; ++p) d += mat[(size_t)p * G + r];
+      P.doff[r] = d;
+      maxc = scnt[r] > maxc ? scnt[r] : maxc;
+    }
+    if (maxc) {
+      const uint64_t want = (maxc + 255) / 256;
+      const dim3 grid((unsigned)(want < (uint64_t)c->num_sms * 4 ? want : (uint64_t)c->num_sms * 4), G);
+      CADV_LAUNCH(c, k_push<<<grid, 256, 0, c->stream>>>(P));
+      if ((e = cudaGetLastError())) return e;
+    }
+    if (cm->barrier(c->stream)) return cudaErrorUnknown;  // every slice has landed
+  }
   *K = Kn;
   *val = (const uint64_t*)rv0;
   *key = nullptr;

@@ -181,3 +181,18 @@ def test_nccl_single_rank_context(cadv):
         assert (h == orc.reuse(t, 32, 1, 1, 20)[0]).all()
     finally:
         ctx.destroy()
+
+
+@pytest.mark.parametrize("scope", [0, 1])
+def test_exchange_collective_baseline(cadv, monkeypatch, scope):
+    """CADV_EXCHANGE=nccl: the kept-record exchange through the communicator's
+    all-to-all (NCCL send / recv) instead of the peer-memory store kernel;
+    same result."""
+    monkeypatch.setenv("CADV_EXCHANGE", "nccl")
+    t = TRACES["rand_bigcta"]()
+    cuts = random_cuts(t.n, 3, seed=99)
+    h_ref, s_ref = orc.reuse(t, 32, scope, 0, 66)
+    out, err = run_ranks(cadv, t, cuts, lambda c: c.reuse_histogram(32, scope, 0, 66))
+    assert not any(err), err
+    for h, s in out:
+        assert (h == h_ref).all() and s == s_ref
