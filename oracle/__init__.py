@@ -10,6 +10,7 @@ Functions follow PAPER.md (see oracle.cpp header for the passages):
   reuse_brute(trace, ...)  O(n^2) literal definition
   mem_div(trace, ...)      unique lines per warp instruction
   branch_div(trace, ...)   divergent warp-level block executions
+  data_centric(trace, objects, ...)  per-data-object RD / MD histograms
 Every function is pinned in tests/test_oracle_pins.py.
 """
 from __future__ import annotations
@@ -48,8 +49,9 @@ def _load():
     lib.oracle_reuse_brute.argtypes = [P, P, P, P, u64, u32, i32, i32, u32, P, P, P]
     lib.oracle_mem_div.argtypes = [P, P, P, P, P, P, u64, u32, u32, u32, P, P]
     lib.oracle_branch_div.argtypes = [P, P, P, P, P, u64, u32, u32, P, P]
+    lib.oracle_data_centric.argtypes = [P, P, P, P, P, u64, P, P, u32, u32, i32, i32, u32, u32, P, P]
     for f in ("oracle_reuse", "oracle_reuse_rd", "oracle_reuse_brute", "oracle_mem_div",
-              "oracle_branch_div", "oracle_num_threads"):
+              "oracle_branch_div", "oracle_data_centric", "oracle_num_threads"):
         getattr(lib, f).restype = ctypes.c_int
     _lib = lib
     return lib
@@ -117,6 +119,21 @@ def branch_div(t, warp_size=32, nsites=None, per_site=True):
     _check(lib.oracle_branch_div(_p(t.cta), _p(t.tid), _p(t.winst), _p(t.site), _p(t.meta), t.n, warp_size,
                                  nsites, _p(ps), _p(tot)))
     return ps, tot
+
+
+def data_centric(t, objects, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66, warp_size=32,
+                 rd=True, md=True):
+    """objects = (base u64[k], bytes u64[k]).  Returns (rd_hist[k+1][nbins] or
+    None, md_hist[k+1][2][W+1] or None); row k = unattributed lines."""
+    lib = _load()
+    base = np.ascontiguousarray(objects[0], dtype=np.uint64)
+    nb = np.ascontiguousarray(objects[1], dtype=np.uint64)
+    k = len(base)
+    rh = np.zeros((k + 1, nbins), np.uint64) if rd else None
+    mh = np.zeros((k + 1, 2, warp_size + 1), np.uint64) if md else None
+    _check(lib.oracle_data_centric(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.winst), _p(t.meta), t.n, _p(base), _p(nb),
+                                   k, line_bytes, scope, binning, nbins, warp_size, _p(rh), _p(mh)))
+    return rh, mh
 
 
 def md_degree(hist):

@@ -409,6 +409,99 @@ int oracle_branch_div(const uint32_t* cta, const uint16_t* tid, const uint32_t* 
   return OK;
 }
 
+// Data-centric attribution (the profiler "associates the memory
+// accesses in GPU kernels with the data allocation ... utilizes this
+// effective address to associate the memory access with data object"),
+// applied to the two memory analyses (reading R18):
+//   objects: nobj allocations [base[k], base[k] + bytes[k]), bytes > 0, in
+//     ascending order; at line granularity a line belongs to the object whose
+//     byte range it intersects, and no line may intersect two objects (else
+//     INVALID_ARG).  Lines in no object belong to row nobj ("unattributed").
+//   rd_hist[(nobj + 1) * nbins] (nullable): every memory access's reuse
+//     distance exactly as oracle_reuse (same scope / binning), counted in the
+//     row of the object of the access's line.
+//   md_hist[(nobj + 1) * 2 * (W + 1)] (nullable): every group (cta, tid / W,
+//     winst) exactly as oracle_mem_div, counted in the row of the object of
+//     its first record's line.
+// Rows are found by a linear scan over the table (the definition).
+int oracle_data_centric(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid, const uint32_t* winst,
+                        const uint8_t* meta, uint64_t n, const uint64_t* obj_base, const uint64_t* obj_bytes,
+                        uint32_t nobj, uint32_t line_bytes, int scope, int binning, uint32_t nbins,
+                        uint32_t warp_size, uint64_t* rd_hist, uint64_t* md_hist) {
+  if (!rd_hist && !md_hist) return INVALID_ARG;
+  int rc = check_reuse_args(line_bytes, scope, binning, rd_hist ? nbins : 3);
+  if (rc) return rc;
+  if (md_hist && (!pow2(warp_size) || warp_size > 32)) return INVALID_ARG;
+  const uint64_t L = line_bytes;
+  for (uint32_t k = 0; k < nobj; ++k) {
+    if (obj_bytes[k] == 0 || obj_base[k] + obj_bytes[k] < obj_base[k]) return INVALID_ARG;
+    // the last line of object k-1 must lie strictly before the first line of object k
+    if (k > 0 && (obj_base[k - 1] + obj_bytes[k - 1] - 1) / L >= obj_base[k] / L) return INVALID_ARG;
+  }
+  if (!check_all(addr, md_hist ? tid : nullptr, meta, n)) return BAD_TRACE;
+  auto row_of_line = [&](uint64_t line) -> uint32_t {
+    const uint64_t lo = line * L, hi = lo + L;  // the line's bytes [lo, hi)
+    for (uint32_t k = 0; k < nobj; ++k)
+      if (lo < obj_base[k] + obj_bytes[k] && obj_base[k] < hi) return k;
+    return nobj;
+  };
+  const uint64_t R = (uint64_t)nobj + 1;
+  if (rd_hist) {
+    std::vector<int64_t> rd(n);
+    rc = oracle_reuse_rd(addr, cta, tid, meta, n, line_bytes, scope, rd.data());
+    if (rc) return rc;
+    std::vector<uint64_t> h(R * nbins, 0);
+    for (uint64_t i = 0; i < n; ++i) {
+      if (rd[i] == -2) continue;  // not a memory record
+      const uint32_t b = rd[i] < 0 ? nbins - 1 : bin_of((uint64_t)rd[i], binning, nbins);
+      h[row_of_line(addr[i] / L) * nbins + b]++;
+    }
+    std::memcpy(rd_hist, h.data(), h.size() * 8);
+  }
+  if (md_hist) {
+    const uint32_t W = warp_size;
+    std::map<uint32_t, std::vector<uint64_t>> by_cta;
+    for (uint64_t i = 0; i < n; ++i)
+      if ((meta[i] & 3u) != KIND_BB) by_cta[cta[i]].push_back(i);
+    std::vector<const std::vector<uint64_t>*> lists;
+    for (auto& kv : by_cta) lists.push_back(&kv.second);
+    std::vector<uint64_t> H(R * 2 * (W + 1), 0);
+    int bad = 0;
+#pragma omp parallel
+    {
+      std::vector<uint64_t> Hl(H.size(), 0);
+#pragma omp for schedule(dynamic, 4)
+      for (int64_t c = 0; c < (int64_t)lists.size(); ++c) {
+        struct Group { uint64_t first; std::set<uint64_t> lines; std::set<uint32_t> lanes; uint64_t count = 0; };
+        std::map<std::pair<uint32_t, uint32_t>, Group> groups;  // (tid / W, winst)
+        for (uint64_t i : *lists[c]) {
+          auto key = std::make_pair((uint32_t)(tid[i] / W), winst[i]);
+          auto it = groups.find(key);
+          if (it == groups.end()) { it = groups.emplace(key, Group()).first; it->second.first = i; }
+          it->second.lines.insert(addr[i] / L);
+          it->second.lanes.insert(tid[i] % W);
+          it->second.count++;
+        }
+        for (auto& kv : groups) {
+          const Group& g = kv.second;
+          if (g.lanes.size() != g.count) {
+#pragma omp atomic write
+            bad = 1;
+            continue;
+          }
+          const uint32_t kind = meta[g.first] & 3u;
+          Hl[(row_of_line(addr[g.first] / L) * 2 + kind) * (W + 1) + g.lines.size()]++;
+        }
+      }
+#pragma omp critical
+      for (size_t k = 0; k < H.size(); ++k) H[k] += Hl[k];
+    }
+    if (bad) return BAD_TRACE;
+    std::memcpy(md_hist, H.data(), H.size() * 8);
+  }
+  return OK;
+}
+
 int oracle_num_threads(void) {
 #ifdef _OPENMP
   return omp_get_max_threads();

@@ -380,3 +380,151 @@ def test_eq1_bypass_warps_arithmetic():
     assert M.md_degree(h) == pytest.approx(orc.md_degree(h)) == pytest.approx(35 / 4)
     s = M.instance_stats([1.0, 2.0, 3.0, 6.0])
     assert s["mean"] == 3.0 and s["min"] == 1.0 and s["max"] == 6.0 and s["stddev"] == pytest.approx(math.sqrt(3.5))
+
+
+# ----------------------------------------------------------------- data-centric attribution (NEXT-3)
+# each access is associated with the data object whose range
+# holds its effective address; reading R18 fixes line granularity.
+
+def _brute_rd_py(t, L, scope):
+    """Literal P:L248 in pure Python loops (tiny traces): distinct renamed
+    elements strictly between an access and the previous use of its element."""
+    n = t.n
+    key = [None] * n
+    for i in range(n):
+        if (int(t.meta[i]) & 3) == BB:
+            continue
+        s = int(t.cta[i]) if scope == orc.SCOPE_CTA else 0
+        line = int(t.addr[i]) // L
+        stores = sum(1 for j in range(i + 1) if (int(t.meta[j]) & 3) == ST and key_line(t, j, L, scope) == (s, line))
+        key[i] = (s, line, stores)
+    rd = [None] * n
+    for i in range(n):
+        if key[i] is None:
+            continue
+        rd[i] = -1
+        if (int(t.meta[i]) & 3) == LD:
+            for j in range(i - 1, -1, -1):
+                if key[j] == key[i]:
+                    rd[i] = len({key[m] for m in range(j + 1, i) if key[m] is not None and key[m][0] == key[i][0]})
+                    break
+    return rd
+
+
+def key_line(t, j, L, scope):
+    return (int(t.cta[j]) if scope == orc.SCOPE_CTA else 0, int(t.addr[j]) // L)
+
+
+def _row_py(line, L, objs):
+    lo, hi = line * L, line * L + L
+    for k, (b, nb) in enumerate(zip(*objs)):
+        if lo < int(b) + int(nb) and int(b) < hi:
+            return k
+    return len(objs[0])
+
+
+def _bin_py(d, nbins):
+    return nbins - 1 if d < 0 else min(d, nbins - 2)
+
+
+@pytest.mark.parametrize("L", [128, 32])
+def test_data_centric_vecadd_closed_form(L):
+    """vecAdd (C1): c[i] = a[i] + b[i], N = 683 fp32, arrays 4 KiB aligned.
+    Per object: a and b are read once per element, so each of their
+    ceil(4N / L) lines is first touched once (∞) and every other load is a
+    reuse at distance 0; every store to c opens a new element (∞).
+    MD: every warp instruction touches one object; 22 per array, all
+    coalesced (1 line at 128 B; at 32 B 4 lines, the 11-lane tail 2 lines)."""
+    N = 683
+    t = tg.generate("vecadd")
+    objs = tg.objects("vecadd")
+    assert len(objs[0]) == 3 and all(int(b) % 4096 == 0 for b in objs[0])
+    rh, mh = orc.data_centric(t, objs, L, nbins=66)
+    lines = -(-4 * N // L)
+    for k in (0, 1):
+        assert rh[k, 0] == N - lines and rh[k, 65] == lines and rh[k].sum() == N
+    assert rh[2, 65] == N and rh[2].sum() == N
+    assert rh[3].sum() == 0
+    for k, kind in ((0, LD), (1, LD), (2, ST)):
+        row = mh[k, kind]
+        if L == 128:
+            assert row[1] == 22 and row.sum() == 22
+        else:
+            assert row[4] == 21 and row[2] == 1 and row.sum() == 22
+        assert mh[k, 1 - kind].sum() == 0
+
+
+@pytest.mark.parametrize("seed", range(10))
+def test_data_centric_equals_python_brute_force(seed):
+    """Per-object RD and MD vs a pure-Python literal computation on tiny
+    random traces, with random object tables (gaps, unattributed lines)."""
+    rng = np.random.default_rng(1000 + seed)
+    L = int(rng.choice([1, 4, 16, 32, 128]))
+    scope = int(rng.integers(0, 2))
+    n = int(rng.integers(20, 120))
+    ncta = int(rng.integers(1, 4))
+    nelem = int(rng.integers(2, 40))
+    base0 = 0x7F0000000000
+    addr = base0 + 4 * rng.integers(0, nelem, n)
+    kinds = np.where(rng.random(n) < 0.25, ST, LD)
+    cta = rng.integers(0, ncta, n)
+    tid = rng.integers(0, 64, n)
+    # winst per (cta, warp): every record its own warp instruction, except a few shared
+    t = tg.from_arrays(addr, cta, tid, np.zeros(n), np.arange(n), [meta(k) for k in kinds], nsites=1)
+    # object table: random line-disjoint ranges over [base0, base0 + 4 nelem),
+    # each trimmed inside its first / last line (so partial lines occur)
+    nlines = 4 * nelem // L + 2
+    cuts = sorted(set(int(x) for x in rng.integers(0, nlines, 6)))
+    objs_b, objs_n = [], []
+    for a, b in zip(cuts[::2], cuts[1::2]):
+        lo = base0 + a * L + int(rng.integers(0, max(1, L // 2)))
+        hi = base0 + b * L - int(rng.integers(0, max(1, L // 2)))
+        if hi > lo and (not objs_b or (objs_b[-1] + objs_n[-1] - 1) // L < lo // L):
+            objs_b.append(lo)
+            objs_n.append(hi - lo)
+    assert seed % 5 or objs_b  # most seeds have objects (checked on a subset)
+    objs = (np.array(objs_b, np.uint64), np.array(objs_n, np.uint64))
+    nb = 10
+    rh, mh = orc.data_centric(t, objs, L, scope=scope, nbins=nb, warp_size=32)
+    rd = _brute_rd_py(t, L, scope)
+    want = np.zeros((len(objs_b) + 1, nb), np.uint64)
+    for i in range(n):
+        want[_row_py(int(addr[i]) // L, L, objs), _bin_py(rd[i], nb)] += 1
+    assert (rh == want).all()
+    # MD: every record is its own group (distinct winst) -> degree 1 in its object's row
+    wm = np.zeros((len(objs_b) + 1, 2, 33), np.uint64)
+    for i in range(n):
+        wm[_row_py(int(addr[i]) // L, L, objs), kinds[i], 1] += 1
+    assert (mh == wm).all()
+
+
+def test_data_centric_rows_partition_the_analyses():
+    """Rows partition the whole-trace histograms (every access / group lands
+    in exactly one row), on a generated trace with stores, both scopes."""
+    t = tg.generate("rand", seed=3, ctas=5, threads=128, instrs=30, lines=200, pstore=0.2, pbb=0.2)
+    base = int(t.addr[(t.meta & 3) != BB].min()) // 4096 * 4096
+    objs = (np.array([base, base + 8192, base + 40960], np.uint64), np.array([4096, 8192, 1 << 20], np.uint64))
+    for L, scope in ((128, 0), (32, 1), (4, 0)):
+        rh, mh = orc.data_centric(t, objs, L, scope=scope, nbins=40)
+        h, _ = orc.reuse(t, L, scope, 0, 40)
+        assert (rh.sum(axis=0) == h).all()
+        hm, _ = orc.mem_div(t, L, 32)
+        assert (mh.sum(axis=0) == hm).all()
+    # no objects: everything is unattributed
+    rh, mh = orc.data_centric(t, (np.zeros(0, np.uint64), np.zeros(0, np.uint64)), 128, nbins=40)
+    assert rh.shape == (1, 40) and (rh[0] == orc.reuse(t, 128, 0, 0, 40)[0]).all()
+
+
+def test_data_centric_rejects_bad_tables():
+    t = tg.generate("vecadd")
+    b = 0x7F0000000000
+    bad = [
+        ([b, b + 64], [64, 64]),       # both objects share line b at 128 B
+        ([b + 4096, b], [64, 64]),     # not ascending
+        ([b], [0]),                    # empty object
+    ]
+    for base, nb in bad:
+        with pytest.raises(orc.OracleError):
+            orc.data_centric(t, (np.array(base, np.uint64), np.array(nb, np.uint64)), 128)
+    # the same pair is fine at 64 B lines (no line intersects both)
+    orc.data_centric(t, (np.array([b, b + 64], np.uint64), np.array([64, 64], np.uint64)), 64)

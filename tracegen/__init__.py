@@ -47,6 +47,8 @@ def _load():
     lib.tg_launch_offsets.argtypes = [P, P]
     lib.tg_free.restype = None
     lib.tg_free.argtypes = [P]
+    lib.tg_objects.restype = u32
+    lib.tg_objects.argtypes = [P, P, P]
     _lib = lib
     return lib
 
@@ -98,6 +100,22 @@ def launch_offsets(workload: str, **params) -> np.ndarray:
         out = np.zeros(nl + 1, np.uint64)
         lib.tg_launch_offsets(h, out.ctypes.data)
         return out
+    finally:
+        lib.tg_free(h)
+
+
+def objects(workload: str, **params):
+    """The workload's data objects (its allocated arrays): (base, bytes) as
+    two uint64 arrays, ascending base (the allocation map of P:L131; input
+    description, not analysis arithmetic)."""
+    lib = _load()
+    h, *_ = plan(workload, **params)
+    try:
+        k = int(lib.tg_objects(h, None, None))
+        base, nbytes = np.zeros(k, np.uint64), np.zeros(k, np.uint64)
+        if k:
+            lib.tg_objects(h, base.ctypes.data, nbytes.ctypes.data)
+        return base, nbytes
     finally:
         lib.tg_free(h)
 

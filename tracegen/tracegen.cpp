@@ -97,10 +97,16 @@ struct Launch {
   uint64_t count = 0, offset = 0;
 };
 
+// Bump allocator of the synthetic kernel's arrays; every allocation is
+// recorded as a data object [base, base + bytes) (the allocation map the
+// paper's data-centric profiler builds from the malloc family).
 struct Alloc {
   uint64_t next = VA_BASE;
+  std::vector<std::pair<uint64_t, uint64_t>>* objs = nullptr;
+  explicit Alloc(std::vector<std::pair<uint64_t, uint64_t>>* o = nullptr) : objs(o) {}
   uint64_t get(uint64_t bytes) {
     uint64_t a = next;
+    if (objs) objs->push_back({a, bytes});
     next += (bytes + 4095) & ~4095ull;
     next += 4096;  // guard page between arrays
     return a;
@@ -118,6 +124,7 @@ struct Trace {
   uint32_t nsites = 0;
   uint32_t nctas = 0;
   uint64_t n = 0;
+  std::vector<std::pair<uint64_t, uint64_t>> objs;  // allocated arrays (base, bytes), ascending
   // state shared by the generator closures
   std::vector<std::shared_ptr<void>> keep;
   int scramble = 0;
@@ -259,7 +266,7 @@ struct Params {
 void wl_vecadd(Trace& T, const Params& P) {
   uint32_t N = (uint32_t)P.i("n", 683), NT = (uint32_t)P.i("threads", 64);
   int bb = (int)P.i("bb", 1);
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t a = A.get(N * 4ull), b = A.get(N * 4ull), c = A.get(N * 4ull);
   enum { S_ENTRY, S_HDR, S_BODY, S_EXIT, S_LDA, S_LDB, S_STC, S_N };
   T.nsites = S_N;
@@ -292,7 +299,7 @@ void wl_sgemm(Trace& T, const Params& P) {
   uint32_t n = (uint32_t)P.i("n", 256);
   const uint32_t TS = 16;
   int naive = (int)P.i("naive", 1), tiled = (int)P.i("tiled", 1), bb = (int)P.i("bb", 0);
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t a = A.get(4ull * n * n), b = A.get(4ull * n * n), c = A.get(4ull * n * n);
   uint32_t g = n / TS;
   uint32_t site = 0;
@@ -347,7 +354,7 @@ void wl_sgemm(Trace& T, const Params& P) {
 void wl_bicg(Trace& T, const Params& P) {
   uint32_t nx = (uint32_t)P.i("nx", 1024), ny = (uint32_t)P.i("ny", 1024), NT = 256;
   int final_store = (int)P.i("store", 0);
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t a = A.get(4ull * nx * ny), r = A.get(4ull * nx), p_ = A.get(4ull * ny);
   uint64_t s = A.get(4ull * ny), q = A.get(4ull * nx);
   enum { S_K1_A, S_K1_R, S_K1_S, S_K2_A, S_K2_P, S_K2_Q, S_N };
@@ -383,7 +390,7 @@ void wl_bicg(Trace& T, const Params& P) {
 void wl_syrk(Trace& T, const Params& P, bool two) {
   uint32_t ni = (uint32_t)P.i("ni", 8), nj = (uint32_t)P.i("nj", 32), M = (uint32_t)P.i("m", 1024);
   uint32_t N = (uint32_t)std::max(ni, nj);
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t a = A.get(4ull * N * M), b = A.get(4ull * N * M), c = A.get(4ull * N * N);
   enum { S_AI, S_BJ, S_BI, S_AJ, S_C, S_N };
   T.nsites = S_N;
@@ -451,7 +458,7 @@ void wl_bfs(Trace& T, const Params& P) {
       if (upd[v]) { mask[v] = 1; vis[v] = 1; over = true; upd[v] = 0; }
     if (!over) break;
   }
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t nodes = A.get(8ull * N), edges = A.get(4ull * tot), gmask = A.get(N), gupd = A.get(N);
   uint64_t gvis = A.get(N), cost = A.get(4ull * N), overp = A.get(4);
   enum {
@@ -543,7 +550,7 @@ void wl_srad(Trace& T, const Params& P) {
   uint64_t seed = (uint64_t)P.i("seed", 42);
   const uint32_t TS = 16;
   uint32_t gx = (C + TS - 1) / TS, gy = (R + TS - 1) / TS;
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t sz = 4ull * R * C;
   uint64_t J = A.get(sz), Cc = A.get(sz), dN = A.get(sz), dS = A.get(sz), dW = A.get(sz), dE = A.get(sz);
   enum {
@@ -612,7 +619,7 @@ void wl_backprop(Trace& T, const Params& P) {
   uint32_t in = (uint32_t)P.i("in", 65536), hid = 16;
   int bb = (int)P.i("bb", 1);
   const uint32_t TS = 16;
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t inp = A.get(4ull * (in + 1)), w = A.get(4ull * (in + 1) * (hid + 1));
   uint64_t part = A.get(4ull * (in / TS) * hid), delta = A.get(4ull * (hid + 1)), oldw = A.get(4ull * (in + 1) * (hid + 1));
   enum { F_ENTRY, F_TX0, F_RED, F_RED_IF, F_TAIL, F_LD_IN, F_LD_W, F_ST_W, F_ST_PART,
@@ -710,7 +717,7 @@ void wl_rand(Trace& T, const Params& P) {
   uint64_t seed = (uint64_t)P.i("seed", 1);
   uint32_t nmsite = 16, nbsite = 8;
   T.nsites = nmsite + nbsite;
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t pool = A.get(128ull * lines + 4096);
   uint64_t pool2 = A.get(128ull * lines * 64 + 4096);
   for (uint32_t li = 0; li < nlaunch; ++li) {
@@ -768,7 +775,7 @@ void wl_literal(Trace& T, const Params& P) {
   }
   uint32_t elem = (uint32_t)P.i("elem", 4);
   T.nsites = 2;
-  Alloc A;
+  Alloc A(&T.objs);
   uint64_t base = A.get(1 << 20);
   Launch L; L.ncta = 1; L.nthreads = 1;
   L.gen = [=](uint32_t, uint32_t, Prog& p) {
@@ -872,6 +879,18 @@ void tg_launch_offsets(const tg_trace* t, uint64_t* out) {
   const Trace* T = reinterpret_cast<const Trace*>(t);
   for (size_t k = 0; k < T->launches.size(); ++k) out[k] = T->launches[k].offset;
   out[T->launches.size()] = T->n;
+}
+
+// Data objects of the workload (its allocated arrays, ascending base):
+// returns their number; fills base[] / bytes[] when non-NULL.  The mixed
+// workload reuses the address range per sub-workload and reports none.
+uint32_t tg_objects(const tg_trace* t, uint64_t* base, uint64_t* bytes) {
+  const Trace* T = reinterpret_cast<const Trace*>(t);
+  for (size_t k = 0; k < T->objs.size(); ++k) {
+    if (base) base[k] = T->objs[k].first;
+    if (bytes) bytes[k] = T->objs[k].second;
+  }
+  return (uint32_t)T->objs.size();
 }
 
 // Writes records [lo, hi) of the trace into the caller's arrays (indexed from 0).
