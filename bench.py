@@ -65,6 +65,7 @@ def parse():
     ap.add_argument("--profile-run", action="store_true", help="short run for ncu (no clocks / baselines)")
     ap.add_argument("--sharding", default="position", choices=["position", "independent"],
                     help="N>1: shards of one global trace (library NCCL exchange) or one trace per rank")
+    ap.add_argument("--no-data-centric", action="store_true", help="skip the data-centric attribution leg")
     ap.add_argument("--separate", action="store_true",
                     help="one library call per analysis (three passes) instead of the fused cadv_analyze")
     return ap.parse_args()
@@ -199,6 +200,7 @@ def algorithmic_bytes(kname, st):
         "k_scan<1>": 13 * n + 12 * kept,            # addr, cta, meta + kept records
         "k_scan<2>": 23 * n,                        # addr, cta, tid, winst, site, meta
         "k_scan<4>": 15 * n,                        # cta, tid, winst, site, meta
+        "k_scan<11>": 19 * n + 12 * kept,           # data-centric: addr, cta, tid, winst, meta + kept records
         "k_rd_tile<0>": 12 * kept,                  # key 4 + value 8 per kept record
         "k_squeeze": 24 * kept,                     # kept records read and written once
     }
@@ -367,6 +369,48 @@ def main():
                     "share_of_step": round(tot_ms / (ms * 1.0), 4)}
     kernels = {k: {"launches": v[1], "total_ms": round(v[0], 3)} for k, v in sorted(agg.items(), key=lambda kv: -kv[1][0])}
 
+    # ---- data-centric attribution: the same trace, per-object
+    # RD + MD rows over the workload's allocation table (one fused pass)
+    dcen = None
+    if world == 1 and not args.profile_run and not args.no_data_centric:
+        import tracegen as tg
+        gname, gparams = WORKLOADS[args.workload]
+        objs = tg.objects(gname, **gparams)
+        if len(objs[0]):
+            def dstep():
+                ctx.data_centric(objs, lb, SC, cadv.BINS_LINEAR, NB, 32)
+                return ctx.last_launches(), ctx.last_kernel_times(), ctx.last_count(0)
+            for _ in range(2):
+                dstep()
+            ctx.set_profiling(True)
+            torch.cuda.synchronize()
+            g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            g0.record(stream)
+            dk, dl, dkept = [], 0, 0
+            for _ in range(args.steps):
+                L_, k_, dkept = dstep()
+                dl += L_
+                dk += k_
+            g1.record(stream)
+            torch.cuda.synchronize()
+            ctx.set_profiling(False)
+            dms = g0.elapsed_time(g1) / max(args.steps, 1)
+            dagg = {}
+            for name_, t_ms in dk:
+                a = dagg.setdefault(name_, [0.0, 0])
+                a[0] += t_ms
+                a[1] += 1
+            ddom = max(dagg.items(), key=lambda kv: kv[1][0])[0]
+            per = algorithmic_bytes(ddom, dict(n=n, kept=dkept, md_groups=0, bd_groups=0))
+            davg = dagg[ddom][0] / dagg[ddom][1]
+            dcen = {"value": round(n / (dms / 1e3), 1), "unit": UNIT, "ms_per_step": round(dms, 3),
+                    "objects": int(len(objs[0])), "call": "cadv_data_centric(rd + md rows per object)",
+                    "gpu_launches": dl,
+                    "roofline": ({"bound": "hbm", "kernel": ddom, "achieved": round(per / (davg / 1e3) / 1e9, 1),
+                                  "peak": peak, "unit": "GB/s", "frac": round(per / (davg / 1e3) / 1e9 / peak, 4),
+                                  "avg_launch_ms": round(davg, 4), "algorithmic_bytes_per_launch": per}
+                                 if per else None)}
+
     # ---- e2e: the same step through the C ABI with HOST buffers (H2D inside the timed region)
     e2e = None
     if args.e2e_steps > 0 and not args.profile_run:
@@ -417,7 +461,7 @@ def main():
                                        f"dp{world} (independent trace per GPU, histograms all-reduced)"
                                        if world > 1 else "single GPU")},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-            "clocks": ck, "kernels": kernels,
+            "clocks": ck, "kernels": kernels, "data_centric": dcen,
         }
         print(json.dumps(line), flush=True)
     ctx.destroy()

@@ -204,6 +204,32 @@ CADV_API cadv_status cadv_analyze(cadv_ctx *ctx, const cadv_analysis *a, uint64_
                                   cadv_reuse_stats *rd_stats, uint64_t *md_hist, cadv_site_mem *md_sites,
                                   uint64_t *bd_totals, cadv_site_branch *bd_sites);
 
+/* One data object (an allocation): bytes [base, base + bytes). */
+typedef struct { uint64_t base, bytes; } cadv_object;
+
+/* Data-centric attribution (the profiler "associates the memory
+ * accesses in GPU kernels with the data allocation ... utilizes this
+ * effective address to associate the memory access with data object"):
+ * the reuse-distance and memory-divergence histograms split per data object
+ * (reading R18).
+ *   objs[nobj]: ascending, non-empty byte ranges; at line granularity
+ *       (line_bytes) a line belongs to the object whose range it
+ *       intersects, and no line may intersect two objects (else
+ *       CADV_ERR_INVALID_ARG).  Lines in no object form the extra row nobj
+ *       ("unattributed").  nobj = 0 is allowed (one row).  The table is
+ *       copied; objs is not retained.
+ *   rd_hist[(nobj + 1) * nbins] (nullable): row k = the reuse distances
+ *       (as cadv_reuse_histogram with line_bytes, scope, binning, nbins) of
+ *       the accesses whose line belongs to object k.
+ *   md_hist[(nobj + 1) * 2 * (warp_size + 1)] (nullable): row k = the
+ *       memory-divergence histogram (as cadv_mem_divergence) of the groups
+ *       whose FIRST record's line belongs to object k.
+ * At least one of rd_hist / md_hist must be non-NULL.  One streaming pass
+ * computes both; multi-rank contexts return the global rows on every rank. */
+CADV_API cadv_status cadv_data_centric(cadv_ctx *ctx, const cadv_object *objs, uint32_t nobj, uint32_t line_bytes,
+                                       int scope, int binning, uint32_t nbins, uint32_t warp_size,
+                                       uint64_t *rd_hist, uint64_t *md_hist);
+
 /* Releases the context and all its device workspace. */
 CADV_API cadv_status cadv_destroy(cadv_ctx *ctx);
 

@@ -77,9 +77,10 @@ def lib():
     L.cadv_mem_divergence.argtypes = [P, u32, u32, P, P, u32]
     L.cadv_branch_divergence.argtypes = [P, u32, P, u32, P]
     L.cadv_analyze.argtypes = [P, ctypes.POINTER(Analysis), P, ctypes.POINTER(ReuseStats), P, P, P, P]
+    L.cadv_data_centric.argtypes = [P, P, u32, u32, i32, i32, u32, u32, P, P]
     L.cadv_destroy.argtypes = [P]
     for f in ("cadv_create", "cadv_load_trace", "cadv_reuse_histogram", "cadv_mem_divergence",
-              "cadv_branch_divergence", "cadv_analyze", "cadv_destroy"):
+              "cadv_branch_divergence", "cadv_analyze", "cadv_data_centric", "cadv_destroy"):
         getattr(L, f).restype = i32
     L.cadv_last_error.argtypes = [P]
     L.cadv_last_error.restype = ctypes.c_char_p
@@ -245,6 +246,22 @@ class Context:
         if bd:
             out["branch_div"] = (bs, bt)
         return out
+
+    # -- cadv_data_centric
+    def data_centric(self, objects, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66, warp_size=32,
+                     rd=True, md=True):
+        """objects = (base, bytes) arrays (ascending).  Returns (rd_hist[k+1][nbins]
+        or None, md_hist[k+1][2][W+1] or None); row k = unattributed lines."""
+        base = np.asarray(objects[0], dtype=np.uint64)
+        nb = np.asarray(objects[1], dtype=np.uint64)
+        k = len(base)
+        tab = np.ascontiguousarray(np.stack([base, nb], axis=1)) if k else np.zeros((0, 2), np.uint64)
+        rh = np.zeros((k + 1, nbins), np.uint64) if rd else None
+        mh = np.zeros((k + 1, 2, warp_size + 1), np.uint64) if md else None
+        p = lambda x: x.ctypes.data if x is not None else None
+        self._check(lib().cadv_data_centric(self._h, tab.ctypes.data if k else None, k, line_bytes, scope, binning,
+                                            nbins, warp_size, p(rh), p(mh)))
+        return rh, mh
 
     # -- cadv_destroy
     def destroy(self):

@@ -395,6 +395,11 @@ struct Req {
   int scope = CADV_SCOPE_CTA, log2bins = 0;
   uint32_t nbins = 66, nsites = 0;
   bool md_sites = false, bd_sites = false;
+  // data-centric attribution (cadv_data_centric): nobj > 0 object line extents
+  // on the device; the RD / MD histograms get one row per object + 1
+  uint32_t nobj = 0;
+  const uint64_t* obj_lo = nullptr;
+  const uint64_t* obj_hi = nullptr;
 };
 
 cadv_status check_args(cadv_ctx* c, uint32_t line_bytes, uint32_t warp_size, bool check_line, bool check_warp) {
@@ -461,8 +466,9 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
   cadv_status s = begin_call(c);
   if (s != CADV_OK) return s;
   const uint32_t mdW = 1u << q.md_ws;
-  const size_t o_rdh = 0, o_rds = o_rdh + (q.rd ? q.nbins : 0), o_mdh = o_rds + (q.rd ? 4 : 0);
-  const size_t o_mds = o_mdh + (q.md ? 2 * (mdW + 1) : 0);
+  const size_t rows = (size_t)q.nobj + 1;
+  const size_t o_rdh = 0, o_rds = o_rdh + (q.rd ? rows * q.nbins : 0), o_mdh = o_rds + (q.rd ? 4 : 0);
+  const size_t o_mds = o_mdh + (q.md ? rows * 2 * (mdW + 1) : 0);
   const size_t o_mdf = o_mds + (q.md && q.md_sites ? 2ull * q.nsites : 0);
   const size_t o_bdt = o_mdf + (q.md ? 1 : 0);
   const size_t o_bdf = o_bdt + 3;
@@ -526,6 +532,13 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
     P.ndefer = &scalars(c)->ndefer;
   }
   P.nsites = (q.md_sites || q.bd_sites) ? q.nsites : 0;
+  if (q.nobj) {
+    flags |= F_OBJ;
+    P.obj_lo = q.obj_lo;
+    P.obj_hi = q.obj_hi;
+    P.nobj = q.nobj;
+    P.rd_nbins = q.nbins;
+  }
   // one flag word for both site checks
   P.site_flag = d + (q.md ? o_mdf : o_bdf);
   if (flags && t.n) CK(launch_scan(c, flags, P), "scan launch");
@@ -573,7 +586,8 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
     }
   }
   if (q.rd && (t.n || multi)) {
-    cudaError_t e = rd_finish(c, rs, q.log2bins, q.nbins, d + o_rdh, d + o_rds);
+    const ObjTab ot{q.obj_lo, q.obj_hi, q.nobj};
+    cudaError_t e = rd_finish(c, rs, q.log2bins, q.nbins, d + o_rdh, d + o_rds, &ot);
     if (e != cudaSuccess) {
       if (multi && !c->comm->err.empty()) return fail(c, CADV_ERR_NCCL, c->comm->err);
       return cuda_fail(c, e, "reuse");
@@ -601,8 +615,8 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
   if ((q.md && hr[o_mdf]) || (q.bd && hr[o_bdf]))
     return fail(c, CADV_ERR_INVALID_ARG, "a record's site id is >= nsites");
   if (q.rd) {
-    memcpy(rd_hist, hr + o_rdh, q.nbins * 8);
-    if (rd_stats) {
+    memcpy(rd_hist, hr + o_rdh, rows * q.nbins * 8);
+    if (rd_stats) {  // (single row: not a data-centric call)
       uint64_t acc = 0;
       for (uint32_t b = 0; b < q.nbins; ++b) acc += hr[o_rdh + b];
       rd_stats->accesses = acc;
@@ -613,7 +627,7 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
     }
   }
   if (q.md) {
-    memcpy(md_hist, hr + o_mdh, 2ull * (mdW + 1) * 8);
+    memcpy(md_hist, hr + o_mdh, rows * 2 * (mdW + 1) * 8);
     if (q.md_sites) memcpy(md_sites, hr + o_mds, 2ull * q.nsites * 8);
   }
   if (q.bd) {
@@ -714,6 +728,57 @@ CADV_API cadv_status cadv_analyze(cadv_ctx* c, const cadv_analysis* a, uint64_t*
   }
   q.nsites = a->nsites;
   return run_analyses(c, q, rd_hist, rd_stats, md_hist, md_sites, bd_totals, bd_sites);
+}
+
+CADV_API cadv_status cadv_data_centric(cadv_ctx* c, const cadv_object* objs, uint32_t nobj, uint32_t line_bytes,
+                                       int scope, int binning, uint32_t nbins, uint32_t warp_size, uint64_t* rd_hist,
+                                       uint64_t* md_hist) {
+  if (!c) return CADV_ERR_INVALID_ARG;
+  c->err.clear();
+  if (!rd_hist && !md_hist) return fail(c, CADV_ERR_INVALID_ARG, "no analysis requested");
+  cadv_status s = check_args(c, line_bytes, md_hist ? warp_size : 32, true, md_hist != nullptr);
+  if (s != CADV_OK) return s;
+  if (nobj && !objs) return fail(c, CADV_ERR_INVALID_ARG, "objs is NULL");
+  if (nobj > (1u << 24)) return fail(c, CADV_ERR_INVALID_ARG, "more than 2^24 objects");
+  Req q;
+  if (rd_hist) {
+    if (scope != CADV_SCOPE_CTA && scope != CADV_SCOPE_KERNEL) return fail(c, CADV_ERR_INVALID_ARG, "bad scope");
+    if (binning != CADV_BINS_LINEAR && binning != CADV_BINS_LOG2) return fail(c, CADV_ERR_INVALID_ARG, "bad binning");
+    if (nbins < 3) return fail(c, CADV_ERR_INVALID_ARG, "nbins must be >= 3");
+    q.rd = true;
+    q.rd_lbs = ilog2(line_bytes);
+    q.scope = scope;
+    q.log2bins = binning == CADV_BINS_LOG2;
+    q.nbins = nbins;
+  }
+  if (md_hist) {
+    q.md = true;
+    q.md_lbs = ilog2(line_bytes);
+    q.md_ws = ilog2(warp_size);
+  }
+  // line extents: [base / L, ceil((base + bytes) / L)), ascending and disjoint
+  const uint32_t lbs = ilog2(line_bytes);
+  std::vector<uint64_t> ext(2ull * nobj);
+  for (uint32_t k = 0; k < nobj; ++k) {
+    const uint64_t b = objs[k].base, nb = objs[k].bytes;
+    if (nb == 0 || b + nb < b) return fail(c, CADV_ERR_INVALID_ARG, "object " + std::to_string(k) + ": empty or wraps");
+    ext[k] = b >> lbs;
+    ext[nobj + k] = ((b + nb - 1) >> lbs) + 1;
+    if (k && ext[nobj + k - 1] > ext[k])
+      return fail(c, CADV_ERR_INVALID_ARG,
+                  "objects " + std::to_string(k - 1) + " and " + std::to_string(k) + " are not ascending / share a line");
+  }
+  if (nobj) {
+    void* dv;
+    CK(cudaSetDevice(c->device), "cudaSetDevice");
+    CK(ensure(c, B_OBJ, ext.size() * 8, &dv), "workspace");
+    CK(cudaMemcpyAsync(dv, ext.data(), ext.size() * 8, cudaMemcpyHostToDevice, c->stream), "H2D");
+    CK(cudaStreamSynchronize(c->stream), "H2D");
+    q.nobj = nobj;
+    q.obj_lo = (const uint64_t*)dv;
+    q.obj_hi = (const uint64_t*)dv + nobj;
+  }
+  return run_analyses(c, q, rd_hist, nullptr, md_hist, nullptr, nullptr, nullptr);
 }
 
 }  // extern "C"

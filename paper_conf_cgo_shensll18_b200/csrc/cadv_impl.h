@@ -39,7 +39,7 @@ enum BufId {
   B_RD_KEY, B_RD_VAL, B_RD_TILESTAT, B_RD_TILEW, B_RD_TILEQ, B_RD_ENT, B_RD_ENT_KEY0, B_RD_ENT_KEY1,
   B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP, B_DEFER, B_OUT2,
   B_ALIGN0, B_ALIGN1, B_ALIGN2, B_ALIGN3, B_ALIGN4, B_ALIGN5,
-  B_XCH_K0, B_XCH_K1, B_XCH_V0, B_XCH_V1, B_XCH_CNT, B_COMM,
+  B_XCH_K0, B_XCH_K1, B_XCH_V0, B_XCH_V1, B_XCH_CNT, B_COMM, B_OBJ,
   B_COUNT
 };
 
@@ -99,7 +99,9 @@ Scalars* scalars(cadv_ctx* c);
 cudaError_t regroup_by_warp(cadv_ctx* c, cadv_trace_desc* out);
 
 // ---- the fused streaming pass (scan.cu)
-enum { F_RD = 1, F_MD = 2, F_BD = 4 };
+// F_OBJ: data-centric attribution (cadv_data_centric): the RD bin-0 counts
+// of dropped duplicate loads and the MD groups go to the row of their object.
+enum { F_RD = 1, F_MD = 2, F_BD = 4, F_OBJ = 8 };
 struct ScanParams {
   cadv_trace_desc t;
   // reuse distance: run compression output
@@ -124,6 +126,11 @@ struct ScanParams {
   unsigned long long* ndefer = nullptr;
   uint32_t nsites = 0;
   uint64_t* site_flag = nullptr;
+  // data objects (F_OBJ): line extents, rows of rd_nbins (RD) / 2 (W + 1) (MD) bins
+  const uint64_t* obj_lo = nullptr;
+  const uint64_t* obj_hi = nullptr;
+  uint32_t nobj = 0;
+  uint32_t rd_nbins = 0;
 };
 uint64_t scan_tiles(uint64_t n);
 void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nwarps, uint64_t* chunk);
@@ -146,8 +153,10 @@ struct RdState {
 // workspace for the run-compression output of the scan
 cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st);
 // CTA regroup, tiles, cross-tile phase after the scan wrote the kept records
+// obj (n = 0: off): d_hist holds (obj.n + 1) rows of nbins, one per object + unattributed
+struct ObjTab;
 cudaError_t rd_finish(cadv_ctx* c, const RdState& st, int log2bins, uint32_t nbins, uint64_t* d_hist,
-                      uint64_t* d_stats);
+                      uint64_t* d_stats, const ObjTab* obj = nullptr);
 
 // ---- device-wide primitives (sort.cu)
 // Stable LSD radix sort of (key, value) pairs on bits [bit_lo, bit_hi) of the

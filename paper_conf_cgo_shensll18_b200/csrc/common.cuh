@@ -33,6 +33,27 @@ __device__ __forceinline__ bool addr_ok(uint64_t a, uint8_t m) {
   return (a & (bytes - 1)) == 0 && (a >> 58) == 0;
 }
 
+// ------------------------------------------------------------------ data objects
+// Data-centric attribution (cadv_data_centric): n line-granular
+// object extents [lo[k], hi[k]) in ascending, disjoint order (the host builds
+// them from the byte ranges).  Row of a line = the extent holding it, or n
+// (unattributed).  Binary search; lo / hi may live in global or shared memory.
+struct ObjTab {
+  const uint64_t* lo;
+  const uint64_t* hi;
+  uint32_t n;
+};
+__device__ __forceinline__ uint32_t obj_row(const uint64_t* lo, const uint64_t* hi, uint32_t n, uint64_t line) {
+  uint32_t a = 0, b = n;  // a = number of extents starting at or before the line
+  while (a < b) {
+    const uint32_t m = (a + b) >> 1;
+    if (lo[m] <= line) a = m + 1;
+    else b = m;
+  }
+  return (a && line < hi[a - 1]) ? a - 1 : n;
+}
+__device__ __forceinline__ uint32_t obj_row(const ObjTab& O, uint64_t line) { return obj_row(O.lo, O.hi, O.n, line); }
+
 // ------------------------------------------------------------------ lane helpers
 __device__ __forceinline__ uint32_t lane_id() { return threadIdx.x & 31u; }
 __device__ __forceinline__ uint32_t lanemask_lt() {

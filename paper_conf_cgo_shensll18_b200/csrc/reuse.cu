@@ -311,7 +311,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     k_rd_tile(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val, uint64_t K,
               const uint32_t* __restrict__ bounds, uint32_t ntiles, int log2bins, uint32_t nbins,
               uint64_t* __restrict__ g_hist, uint64_t* __restrict__ g_stream, uint32_t* __restrict__ tile_w,
-              uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc, uint32_t* wide_list) {
+              uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc, uint32_t* wide_list, ObjTab O) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
   const uint32_t tx = threadIdx.x;
@@ -319,7 +319,9 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   const uint32_t tile = MODE == 0 ? blockIdx.x : MODE == 1 ? wide_list[ntiles + 2 + blockIdx.x] : wide_list[blockIdx.x];
   const uint64_t b = bounds[tile], e = bounds[tile + 1];
   const uint32_t m = (uint32_t)(e - b);
-  const bool smem_hist = nbins <= TL_SMEM_BINS;
+  // data-centric attribution: one row of nbins per object + 1 (O.n = 0: one row)
+  const uint32_t hbins = (O.n + 1) * nbins;
+  const bool smem_hist = hbins <= TL_SMEM_BINS;
   // ---- line range of the tile (packed keys need < 2^52)
   if (tx == 0) {
     S.lmin = ~0ull;
@@ -360,7 +362,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     return;
   }
   if (smem_hist)
-    for (uint32_t k = tx; k < nbins; k += TL_NT) S.hist[k] = 0;
+    for (uint32_t k = tx; k < hbins; k += TL_NT) S.hist[k] = 0;
   // ---- load (striped)
   uint16_t* PSW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[0] : nullptr;
   uint32_t* const K32a = reinterpret_cast<uint32_t*>(S.key[0]);
@@ -562,6 +564,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       bin = nbins - 1;
     }
     if (bin != 0xffffffffu) {
+      if (O.n) bin += obj_row(O, __ldg(val + b + x) & LINE_MASK) * nbins;
       if (smem_hist) atomicAdd(&S.hist[bin], cntb);
       else atomicAdd((unsigned long long*)&g_hist[bin], (unsigned long long)cntb);
     }
@@ -611,7 +614,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   }
   __syncthreads();
   if (smem_hist)
-    for (uint32_t k = tx; k < nbins; k += TL_NT)
+    for (uint32_t k = tx; k < hbins; k += TL_NT)
       if (S.hist[k]) atomicAdd((unsigned long long*)&g_hist[k], (unsigned long long)S.hist[k]);
 }
 
@@ -657,7 +660,7 @@ struct CrossOut {
 
 __global__ void k_link(const uint32_t* __restrict__ order, uint64_t E, EntryCols En,
                        const unsigned long long* __restrict__ tile_wb, const unsigned long long* __restrict__ tile_qb,
-                       uint32_t nbins, uint64_t* g_hist, uint64_t* g_stream, CrossOut X, Scalars* sc) {
+                       uint32_t nbins, uint64_t* g_hist, uint64_t* g_stream, CrossOut X, Scalars* sc, ObjTab O) {
   uint32_t stream = 0;
   for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < E; k += (uint64_t)gridDim.x * blockDim.x) {
     uint32_t e = order[k];
@@ -689,7 +692,8 @@ __global__ void k_link(const uint32_t* __restrict__ order, uint64_t E, EntryCols
         X.xq[slot] = En.l[p];
         X.part[slot] = part;
       } else {
-        atomicAdd((unsigned long long*)&g_hist[nbins - 1], 1ull);
+        const uint32_t row = O.n ? obj_row(O, En.line[e]) : 0u;
+        atomicAdd((unsigned long long*)&g_hist[(uint64_t)row * nbins + nbins - 1], 1ull);
       }
     }
     // streaming of the deferred first / last uses
@@ -776,15 +780,19 @@ __global__ void k_iota_gather(const uint32_t* __restrict__ order, const uint32_t
 }
 
 constexpr uint32_t XF_SMEM_BINS = 4096;
+// O.n > 0 (data-centric attribution): the query's row comes from its line,
+// val[xpos[i]] (the CTA-major kept records)
 __global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__ part,
                                                      const uint32_t* __restrict__ cnt, uint64_t M, int log2bins,
                                                      uint32_t nbins, uint64_t* g_hist, uint64_t* g_stats,
-                                                     Scalars* sc) {
+                                                     Scalars* sc, ObjTab O, const uint32_t* __restrict__ xpos,
+                                                     const uint64_t* __restrict__ val) {
   unsigned long long rdsum = 0;
   __shared__ uint32_t h[XF_SMEM_BINS];
-  const bool sm = nbins <= XF_SMEM_BINS;
+  const uint32_t hbins = (O.n + 1) * nbins;
+  const bool sm = hbins <= XF_SMEM_BINS;
   if (sm)
-    for (uint32_t k = threadIdx.x; k < nbins; k += blockDim.x) h[k] = 0;
+    for (uint32_t k = threadIdx.x; k < hbins; k += blockDim.x) h[k] = 0;
   __syncthreads();
   for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
     int64_t rd = part[i] - (int64_t)cnt[i];
@@ -792,7 +800,8 @@ __global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__
       atomicMax(&sc->err_code, 3u);
       rd = 0;
     }
-    const uint32_t b = rd_bin((uint64_t)rd, log2bins, nbins);
+    uint32_t b = rd_bin((uint64_t)rd, log2bins, nbins);
+    if (O.n) b += obj_row(O, __ldg(val + xpos[i]) & LINE_MASK) * nbins;
     rdsum += (unsigned long long)rd;
     if (sm) {
       // warp-aggregated: one shared-memory atomic per distinct bin in the warp
@@ -807,7 +816,7 @@ __global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__
   if (lane_id() == 0 && rdsum) atomicAdd((unsigned long long*)g_stats + 1, rdsum);
   __syncthreads();
   if (sm)
-    for (uint32_t k = threadIdx.x; k < nbins; k += blockDim.x)
+    for (uint32_t k = threadIdx.x; k < hbins; k += blockDim.x)
       if (h[k]) atomicAdd((unsigned long long*)&g_hist[k], (unsigned long long)h[k]);
 }
 
@@ -1052,8 +1061,9 @@ cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const 
 }
 
 cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbins, uint64_t* d_hist,
-                      uint64_t* d_stats) {
+                      uint64_t* d_stats, const ObjTab* obj) {
   cudaError_t e;
+  const ObjTab O = obj ? *obj : ObjTab{nullptr, nullptr, 0u};
   const int cta_scope = S.cta_scope;
   const int grid_ls = c->num_sms * 4;
   Scalars* sc = scalars(c);
@@ -1131,7 +1141,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   uint32_t* wide_list = (uint32_t*)bnd + (ntiles + 2);
   CADV_LAUNCH(c, k_rd_tile<0><<<(unsigned)ntiles, TL_NT, sizeof(TileSmem), c->stream>>>(
                      key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
-                     tile_q, En, sc, wide_list));
+                     tile_q, En, sc, wide_list, O));
   if ((e = cudaGetLastError())) return e;
   unsigned long long cnt14[4];  // count[1..4]: entries, cross queries, MODE 2 tiles, MODE 1 tiles
   if ((e = cudaMemcpyAsync(cnt14, &sc->count[1], 32, cudaMemcpyDeviceToHost, c->stream))) return e;
@@ -1139,13 +1149,13 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   if (cnt14[3]) {
     CADV_LAUNCH(c, k_rd_tile<1><<<(unsigned)cnt14[3], TL_NT, sizeof(TileSmem), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
-                       tile_q, En, sc, wide_list));
+                       tile_q, En, sc, wide_list, O));
     if ((e = cudaGetLastError())) return e;
   }
   if (cnt14[2]) {
     CADV_LAUNCH(c, k_rd_tile<2><<<(unsigned)cnt14[2], TL_NT, sizeof(TileSmemWide), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
-                       tile_q, En, sc, wide_list));
+                       tile_q, En, sc, wide_list, O));
     if ((e = cudaGetLastError())) return e;
   }
   unsigned long long nent;
@@ -1220,7 +1230,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   X.xpos = (uint32_t*)xq;
   X.xq = X.xpos + nent;
   X.part = (int64_t*)(((uintptr_t)(X.xq + nent) + 15) & ~(uintptr_t)15);
-  CADV_LAUNCH(c, k_link<<<grid_ls, 256, 0, c->stream>>>(order, nent, En, twb, tqb, nbins, d_hist, d_stats, X, sc));
+  CADV_LAUNCH(c, k_link<<<grid_ls, 256, 0, c->stream>>>(order, nent, En, twb, tqb, nbins, d_hist, d_stats, X, sc, O));
   unsigned long long M;
   if ((e = cudaMemcpyAsync(&M, &sc->count[2], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
@@ -1265,7 +1275,8 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     std::swap(ka, kb);
     std::swap(ia, ib);
   }
-  CADV_LAUNCH(c, k_cross_final<<<grid_ls, 256, 0, c->stream>>>(X.part, cnt, M, log2bins, nbins, d_hist, d_stats, sc));
+  CADV_LAUNCH(c, k_cross_final<<<grid_ls, 256, 0, c->stream>>>(X.part, cnt, M, log2bins, nbins, d_hist, d_stats, sc, O,
+                                                                      X.xpos, val));
   return cudaGetLastError();
 }
 

@@ -45,6 +45,7 @@ constexpr int NWARP = 12;              // warps per CTA (one CTA per SM; 3 per S
 constexpr int NTHR = NWARP * 32;
 constexpr int NSITE_SMEM = 512;        // per-site counters kept in shared memory up to this many sites
 constexpr int QCAP = 160;              // per-warp queue of complete runs awaiting finalization
+constexpr int OBJ_SMEM = 64;           // F_OBJ: object rows (objects + 1) kept in shared memory up to this many
 
 __device__ __forceinline__ uint32_t ring_slot(uint32_t j) {  // chunk-relative record -> ring slot
   const uint32_t p = j / KR;
@@ -95,6 +96,10 @@ struct ScanArgs {
   uint32_t nsites;
   uint64_t* site_flag;
   Scalars* sc;
+  // F_OBJ: line extents of the data objects; hist0 / md_hist hold one row per object + 1
+  const uint64_t* obj_lo;
+  const uint64_t* obj_hi;
+  uint32_t nobj, rd_nbins;
 };
 
 __device__ __forceinline__ void report(Scalars* sc, uint64_t i, uint32_t code) {
@@ -133,7 +138,17 @@ struct Counters {        // block-level shared-memory accumulators
   uint32_t* md_sites;    // [NSITE_SMEM][2] or null
   uint32_t* bd_tot;      // [3]
   uint32_t* bd_sites;    // [NSITE_SMEM][3] or null
+  // F_OBJ with at most OBJ_SMEM rows (else null: global tables and atomics)
+  const uint64_t* olo;   // [OBJ_SMEM] object line extents
+  const uint64_t* ohi;
+  uint32_t* mdo;         // [rows][2][33] MD histogram per object row
+  uint32_t* dup;         // [rows] dropped duplicate loads (RD 0) per object row
 };
+
+// row of a line among the data objects (F_OBJ)
+__device__ __forceinline__ uint32_t row_of(const ScanArgs& A, const Counters& C, uint64_t line) {
+  return C.olo ? obj_row(C.olo, C.ohi, A.nobj, line) : obj_row(A.obj_lo, A.obj_hi, A.nobj, line);
+}
 
 // Per-site counter update: shared-memory counters when the site table fits,
 // global counters otherwise; an out-of-range site raises the site flag.
@@ -197,9 +212,16 @@ struct Acc {              // per-lane BD accumulators, reduced at the end
   uint32_t bd_exec, bd_threads;
 };
 
+// row (F_OBJ): the object row of the group's first record
+template <int F>
 __device__ __forceinline__ void finish_md(const ScanArgs& A, const Counters& C, uint32_t* whist, bool sites_smem,
-                                          uint32_t kind, uint32_t deg, uint32_t s) {
-  atomicAdd(&whist[kind * 33 + deg], 1u);
+                                          uint32_t kind, uint32_t deg, uint32_t s, uint32_t row) {
+  if (F & F_OBJ) {
+    if (C.mdo) atomicAdd(&C.mdo[row * 66 + kind * 33 + deg], 1u);
+    else atomicAdd((unsigned long long*)&A.md_hist[(row * 2 + kind) * ((1u << A.ws_md) + 1) + deg], 1ull);
+  } else {
+    atomicAdd(&whist[kind * 33 + deg], 1u);
+  }
   if (sites_smem) {
     if (s < A.nsites) { atomicAdd(&C.md_sites[2 * s], 1u); atomicAdd(&C.md_sites[2 * s + 1], deg); }
     else *A.site_flag = 1;
@@ -272,7 +294,8 @@ __device__ __noinline__ void walk_run(const ScanArgs& A, const Counters C, uint3
     if ((uint32_t)__popc(mask) != cnt) { report(A.sc, g0 + r, 2); continue; }
     const uint32_t s = A.nsites ? __ldg(A.site + g0 + r) : 0u;
     if (bb) finish_bd(A, C, acc, sites_smem, cnt, s, __ldg(A.cta + g0 + r), tr >> ws, maxt);
-    else finish_md(A, C, whist, sites_smem, __ldg(A.meta + g0 + r) & 3u, deg, s);
+    else finish_md<F>(A, C, whist, sites_smem, __ldg(A.meta + g0 + r) & 3u, deg, s,
+                      (F & F_OBJ) ? row_of(A, C, __ldg(A.addr + g0 + r) >> A.lbs_md) : 0u);
   }
   if (acc.bd_exec) { atomicAdd(&C.bd_tot[0], acc.bd_exec); atomicAdd(&C.bd_tot[2], acc.bd_threads); }
 }
@@ -317,7 +340,7 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
         else md = true;
       }
     }
-    if (MD && md) finish_md(A, C, whist, sites_smem, kind, u & PK_M, s);
+    if (MD && md) finish_md<F>(A, C, whist, sites_smem, kind, u & PK_M, s, s);  // F_OBJ: s holds the row
     if (BD) {
       const uint32_t cnt = (u >> PK_CNT) & PK_M;
       if (bd) {
@@ -375,6 +398,7 @@ template <int F>
 __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanArgs A) {
   constexpr bool RD = (F & F_RD) != 0, MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
+  constexpr bool OBJ = (F & F_OBJ) != 0;
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ uint64_t bars[NWARP][KS];
   __shared__ uint32_t s_md_hist[2 * 33];
@@ -383,8 +407,24 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   uint32_t* sites = (uint32_t*)(smem + NWARP * R_BYTES);
   uint32_t* wh_all = sites + ((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM;
   const bool sites_smem = A.nsites && A.nsites <= NSITE_SMEM;
+  // F_OBJ tables after the run queues (scan_smem)
+  uint8_t* objm = smem + NWARP * R_BYTES + ((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + NWARP * 68 * 4 +
+                  NWARP * (QCAP * 24 + 16);
+  const bool obj_sm = OBJ && A.nobj < OBJ_SMEM;
+  uint64_t* s_olo = (uint64_t*)objm;
+  uint64_t* s_ohi = s_olo + OBJ_SMEM;
+  uint32_t* s_dup = (uint32_t*)(s_ohi + OBJ_SMEM);
+  uint32_t* s_mdo = s_dup + OBJ_SMEM;
   const Counters C{s_md_hist, (MD && sites_smem) ? sites : nullptr, s_bd_tot,
-                   (BD && sites_smem) ? sites + (MD ? 2 * NSITE_SMEM : 0) : nullptr};
+                   (BD && sites_smem) ? sites + (MD ? 2 * NSITE_SMEM : 0) : nullptr,
+                   obj_sm ? s_olo : nullptr, obj_sm ? s_ohi : nullptr, (obj_sm && MD) ? s_mdo : nullptr,
+                   obj_sm ? s_dup : nullptr};
+  if (obj_sm) {
+    for (uint32_t k = tx; k < A.nobj; k += NTHR) { s_olo[k] = A.obj_lo[k]; s_ohi[k] = A.obj_hi[k]; }
+    for (uint32_t k = tx; k < OBJ_SMEM; k += NTHR) s_dup[k] = 0;
+    if (MD)
+      for (uint32_t k = tx; k < (A.nobj + 1) * 66; k += NTHR) s_mdo[k] = 0;
+  }
   for (uint32_t k = tx; k < 2 * 33; k += NTHR) s_md_hist[k] = 0;
   if (tx < 3) s_bd_tot[tx] = 0;
   if (sites_smem)
@@ -402,6 +442,16 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   const uint64_t c_lo = gw * A.chunk;
   const uint64_t c_hi = c_lo + A.chunk < A.n ? c_lo + A.chunk : A.n;
   uint32_t kept = 0, ndup = 0;
+  // F_OBJ: duplicate loads counted per object row (run of one line per lane)
+  uint64_t dc_line = ~0ull;
+  uint32_t dc_row = 0, dc_cnt = 0;
+  auto dc_flush = [&]() {
+    if (dc_cnt) {
+      if (C.dup) atomicAdd(&C.dup[dc_row], dc_cnt);
+      else atomicAdd((unsigned long long*)&A.hist0[(uint64_t)dc_row * A.rd_nbins], (unsigned long long)dc_cnt);
+      dc_cnt = 0;
+    }
+  };
   if (c_lo < A.n) {
     const uint32_t clen = (uint32_t)(c_hi - c_lo);
     // the chunk's last run may reach 32 records past its end; one more record
@@ -608,7 +658,24 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         }
         open_rd = __ballot_sync(FULL, last_open) != 0;
         kept += tot;
-        ndup += __popc(dupm & ownm);
+        if (OBJ) {
+          const uint32_t dm = dupm & ownm;
+          if (dm) {
+#pragma unroll
+            for (int k = 0; k < LPR; ++k) {
+              if (!((dm >> k) & 1u)) continue;
+              const uint64_t ln = a[k] >> A.lbs_rd;
+              if (ln != dc_line) {
+                dc_flush();
+                dc_line = ln;
+                dc_row = row_of(A, C, ln);
+              }
+              ++dc_cnt;
+            }
+          }
+        } else {
+          ndup += __popc(dupm & ownm);
+        }
         __syncwarp();
       }
 
@@ -697,7 +764,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
               Q.m[pos] = m2;
               Q.kt[pos] = ((((k < 4 ? mmx : mmy) >> (8 * (k & 3))) & 3u) << 16) | t[k];
               Q.cta[pos] = c[k];
-              Q.site[pos] = A.nsites ? R.site[ring_slot(j0 + k)] : 0u;
+              // F_OBJ (no per-site counters): the slot carries the group's object row
+              Q.site[pos] = OBJ ? row_of(A, C, a[k] >> A.lbs_md) : (A.nsites ? R.site[ring_slot(j0 + k)] : 0u);
             }
             qn += __popc(im);
           }
@@ -732,7 +800,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
               const uint32_t sl0 = ring_slot(j0 + lastk);
               qc[0] = ((R.meta[sl0] & 3u) << 16) | R.tid[sl0];
               qc[1] = R.cta[sl0];
-              qc[2] = A.nsites ? R.site[sl0] : 0u;
+              qc[2] = OBJ ? row_of(A, C, R.addr[sl0] >> A.lbs_md) : (A.nsites ? R.site[sl0] : 0u);
             }
           }
           cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
@@ -775,18 +843,30 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     A.wcnt[gw] = kept;
   }
 
-  if (RD) {
+  if (RD && !OBJ) {
     const uint32_t d = __reduce_add_sync(FULL, ndup);
     if (lane == 0 && d) atomicAdd((unsigned long long*)A.hist0, (unsigned long long)d);
   }
-  if (MD) {
+  if (RD && OBJ) dc_flush();
+  if (MD && !OBJ) {
     __syncwarp();
     for (uint32_t k = lane; k < 66; k += 32)
       if (whist[k]) atomicAdd(&s_md_hist[k], whist[k]);
   }
   // ---- flush block-level counters
   __syncthreads();
-  if (MD) {
+  if (RD && obj_sm)
+    for (uint32_t k = tx; k <= A.nobj; k += NTHR)
+      if (s_dup[k]) atomicAdd((unsigned long long*)&A.hist0[(uint64_t)k * A.rd_nbins], (unsigned long long)s_dup[k]);
+  if (MD && obj_sm) {
+    const uint32_t W = 1u << A.ws_md;
+    for (uint32_t k = tx; k < (A.nobj + 1) * 66; k += NTHR) {
+      const uint32_t row = k / 66, kind = (k % 66) / 33, deg = k % 33;
+      if (s_mdo[k] && deg <= W)
+        atomicAdd((unsigned long long*)&A.md_hist[(row * 2 + kind) * (W + 1) + deg], (unsigned long long)s_mdo[k]);
+    }
+  }
+  if (MD && !OBJ) {
     const uint32_t W = 1u << A.ws_md;
     for (uint32_t k = tx; k < 2 * 33; k += NTHR) {
       const uint32_t kind = k / 33, deg = k % 33;
@@ -862,14 +942,15 @@ __global__ void __launch_bounds__(256) k_squeeze(const uint32_t* __restrict__ ki
 
 template <int F>
 size_t scan_smem() {
-  constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
+  constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0, OBJ = (F & F_OBJ) != 0;
   return (size_t)NWARP * R_BYTES + (size_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + (size_t)NWARP * 68 * 4 +
-         (size_t)NWARP * (QCAP * 24 + 16);
+         (size_t)NWARP * (QCAP * 24 + 16) + (OBJ ? (size_t)OBJ_SMEM * (16 + 4 + (MD ? 66 * 4 : 0)) : 0);
 }
 
-int g_scan_ready[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-const char* const kScanName[8] = {"k_scan<0>", "k_scan<1>", "k_scan<2>", "k_scan<3>",
-                                  "k_scan<4>", "k_scan<5>", "k_scan<6>", "k_scan<7>"};
+int g_scan_ready[16] = {0};
+const char* const kScanName[16] = {"k_scan<0>", "k_scan<1>", "k_scan<2>", "k_scan<3>", "k_scan<4>", "k_scan<5>",
+                                   "k_scan<6>", "k_scan<7>", "k_scan<8>", "k_scan<9>", "k_scan<10>", "k_scan<11>",
+                                   "k_scan<12>", "k_scan<13>", "k_scan<14>", "k_scan<15>"};
 
 template <int F>
 cudaError_t launch_scan_t(cadv_ctx* c, const ScanArgs& A, uint64_t grid) {
@@ -923,6 +1004,7 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
   A.bd_tot = P.bd_tot; A.bd_sites = P.bd_sites; A.defer = (uint4*)P.defer;
   A.ndefer = P.ndefer;
   A.nsites = P.nsites; A.site_flag = P.site_flag; A.sc = scalars(c);
+  A.obj_lo = P.obj_lo; A.obj_hi = P.obj_hi; A.nobj = P.nobj; A.rd_nbins = P.rd_nbins;
   switch (flags) {
     case 1: return launch_scan_t<1>(c, A, grid);
     case 2: return launch_scan_t<2>(c, A, grid);
@@ -931,6 +1013,10 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
     case 5: return launch_scan_t<5>(c, A, grid);
     case 6: return launch_scan_t<6>(c, A, grid);
     case 7: return launch_scan_t<7>(c, A, grid);
+    // data-centric attribution (cadv_data_centric): reuse and / or memory divergence per object
+    case F_OBJ | 1: return launch_scan_t<F_OBJ | 1>(c, A, grid);
+    case F_OBJ | 2: return launch_scan_t<F_OBJ | 2>(c, A, grid);
+    case F_OBJ | 3: return launch_scan_t<F_OBJ | 3>(c, A, grid);
     default: return cudaErrorInvalidValue;
   }
 }

@@ -48,6 +48,7 @@ def test_null_arguments_rejected():
     assert L.cadv_create(None, 0, None, None, 0, 1) == cadv.CADV_ERR_INVALID_ARG
     assert L.cadv_load_trace(None, None, 0) == cadv.CADV_ERR_INVALID_ARG
     assert L.cadv_reuse_histogram(None, 128, 0, 0, None, 10, None) == cadv.CADV_ERR_INVALID_ARG
+    assert L.cadv_data_centric(None, None, 0, 128, 0, 0, 66, 32, None, None) == cadv.CADV_ERR_INVALID_ARG
     assert L.cadv_destroy(None) == cadv.CADV_ERR_INVALID_ARG
 
 

@@ -196,3 +196,22 @@ def test_exchange_collective_baseline(cadv, monkeypatch, scope):
     assert not any(err), err
     for h, s in out:
         assert (h == h_ref).all() and s == s_ref
+
+
+@pytest.mark.parametrize("name", ["srad", "rand_stores"])
+@pytest.mark.parametrize("G", [2, 3])
+@pytest.mark.parametrize("scope", [0, 1])
+def test_data_centric_shards(cadv, name, G, scope):
+    """Data-centric attribution (cadv_data_centric) on snapped shards: every
+    rank returns the oracle's global per-object rows."""
+    t = TRACES[name]()
+    cuts = snapped_cuts(t, G, seed=3 * G + scope)
+    if name == "srad":
+        objs = tg.objects("srad", rows=128, cols=128, iters=2)
+    else:
+        base = int(t.addr[(t.meta & 3) != 2].min())
+        objs = (np.array([base, base + 2048], np.uint64), np.array([1024, 1 << 20], np.uint64))
+    ref = orc.data_centric(t, objs, 128, scope, 0, 66, 32)
+    out, err = run_ranks(cadv, t, cuts, lambda c: c.data_centric(objs, 128, scope, 0, 66, 32))
+    assert not any(err), err
+    check_all_equal(out, ref)
