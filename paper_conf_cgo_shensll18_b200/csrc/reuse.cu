@@ -30,6 +30,7 @@
 //                    cross-tile queries get RD from prefix sums plus a global
 //                    inversion count on the compacted cross-tile set.
 #include <cuda_runtime.h>
+#include <stddef.h>
 #include <stdio.h>
 #include <stdlib.h>
 #include <string.h>
@@ -274,6 +275,9 @@ struct TileSmem {
   uint32_t misc[8];
   unsigned long long lmin, lmax;
 };
+// the warp path of k_rd_tile keeps 256 u32 per warp in pl + qx
+static_assert(offsetof(TileSmem, qx) == offsetof(TileSmem, pl) + sizeof(uint16_t) * TL_CAP, "pl, qx adjacent");
+static_assert(sizeof(uint16_t) * TL_CAP * 2 >= 16 * 256 * 4 && TL_CAP >= 16 * 16 * 4, "warp path scratch");
 // WIDE tiles (line range >= 2^52, practically never) keep lines and positions
 // in separate arrays.
 struct TileSmemWide {
@@ -327,6 +331,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     S.lmin = ~0ull;
     S.lmax = 0;
     S.misc[2] = m;
+    S.misc[3] = S.misc[4] = S.misc[5] = 0;  // warp path: longest segment, weight and query totals
   }
   __syncthreads();
   {
@@ -412,6 +417,179 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   const bool tail_cont = m > 0 && e < K && (!key || __ldg(key + e) == __ldg(key + e - 1));
   __syncthreads();
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) S.es[x] = 0;
+  // ---- warp path (MODE 0): the tile holds whole segments of <= 256 kept
+  //      records each (every CTA of the paper-shaped workloads at 128 B
+  //      lines): warp w resolves segments w, w + 16, ... alone with the same
+  //      two sorts as below over <= 256 keys (<= 5 merge levels instead of 9,
+  //      warp syncs only).  Segments cut by a tile boundary, longer segments
+  //      and the wider key modes take the block path.
+  if (MODE == 0 && !head_cont && !tail_cont && m) {
+    uint32_t ml = 0;
+#pragma unroll
+    for (int j = 0; j < IPT; ++j) {
+      const uint32_t x = tx * IPT + j;
+      if (x < m) ml = max(ml, x - S.sgs[x] + 1u);
+    }
+    ml = __reduce_max_sync(FULL, ml);
+    if (lane_id() == 0) atomicMax(&S.misc[3], ml);
+    __syncthreads();
+    if (S.misc[3] <= 256u) {
+      uint32_t nseg;
+      uint32_t so = block_exclusive_scan<TL_NT>(__popc(ssm), S.ws, &nseg);
+#pragma unroll
+      for (int j = 0; j < IPT; ++j)
+        if ((ssm >> j) & 1u) S.es[so++] = (uint16_t)(tx * IPT + j);
+      __syncthreads();
+      uint32_t stream = 0, wt = 0, qt = 0;
+      unsigned long long rdsum = 0;
+      const uint32_t warp = tx >> 5, lane = lane_id();
+      // warp-private scratch (arrays the block path would use): a line -> last
+      // position hash table of 512 slots (key[0] / key[1]), the inclusive
+      // weighted prefix by segment position (pl + qx), the "reused" position
+      // bitmap R and its word prefix counts (ffl)
+      uint32_t* const HK = reinterpret_cast<uint32_t*>(S.key) + warp * 1024;
+      uint32_t* const HP = HK + 512;
+      uint32_t* const WPI = reinterpret_cast<uint32_t*>(S.pl) + warp * 256;
+      uint32_t* const RW = reinterpret_cast<uint32_t*>(S.ffl) + warp * 16;  // [8] bitmap words
+      uint32_t* const CW8 = RW + 8;                                          // [8] set bits before each word
+      for (uint32_t sg = warp; sg < nseg; sg += TL_NT / 32) {
+        const uint32_t s0 = S.es[sg], n = (sg + 1 < nseg ? S.es[sg + 1] : m) - s0;
+        for (uint32_t k = lane; k < 512; k += 32) HK[k] = 0xffffffffu;
+        if (lane < 8) { RW[lane] = 0; CW8[lane] = 0; }
+        __syncwarp();
+        uint32_t wb = 0, qn = 0, rtot = 0;   // running weight, queries, reused positions (warp-uniform)
+        uint32_t qbits = 0, hbits = 0;       // this lane's positions 32 r + lane: query / has-dup flags
+        for (uint32_t r = 0; 32 * r < n; ++r) {
+          const uint32_t i = 32 * r + lane;
+          const bool valid = i < n;
+          const uint64_t v = valid ? __ldg(val + b + s0 + i) : 0ull;
+          const uint64_t lfull = v & LINE_MASK;
+          const uint32_t line = valid ? (uint32_t)(lfull - lmin) : 0xffffffffu;  // MODE 0: < 2^20
+          const bool st = (v >> VB_STORE) & 1u, hd = (v >> VB_DUP) & 1u;
+          const uint32_t w = valid ? (uint32_t)(v >> VB_W) + 1u : 0u;
+          // previous use of the line: an earlier lane of this round, else the table
+          const uint32_t peers = __match_any_sync(FULL, line);
+          const uint32_t lower = peers & lanemask_lt();
+          int32_t pp = -1;
+          if (valid) {
+            if (lower) {
+              pp = (int32_t)(32 * r + 31 - __clz(lower));
+            } else {
+              uint32_t h = (line * 0x9E3779B1u) >> 23;
+              while (true) {
+                const uint32_t k = HK[h];
+                if (k == line) { pp = (int32_t)HP[h]; break; }
+                if (k == 0xffffffffu) break;
+                h = (h + 1) & 511u;
+              }
+            }
+          }
+          const bool q = valid && !st && pp >= 0;  // a local query: RD = window - reused in window
+          const int32_t P = q ? pp : -1;
+          __syncwarp();
+          if (valid && (peers >> lane) == 1u) {  // the line's last lane in this round records it
+            uint32_t h = (line * 0x9E3779B1u) >> 23;
+            while (true) {  // lanes of other lines insert concurrently: claim slots with CAS
+              const uint32_t k = atomicCAS(&HK[h], 0xffffffffu, line);
+              if (k == 0xffffffffu || k == line) break;
+              h = (h + 1) & 511u;
+            }
+            HP[h] = i;
+          }
+          // weighted prefix (inclusive) by position
+          uint32_t xw = w;
+#pragma unroll
+          for (int o = 1; o < 32; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, xw, o);
+            if (lane >= (uint32_t)o) xw += y;
+          }
+          if (valid) WPI[i] = wb + xw;
+          // reused positions inside the window (P, i): earlier rounds (bitmap R) ...
+          uint32_t cnt = 0;
+          if (q && (uint32_t)P < 32 * r) {
+            const uint32_t pw = (uint32_t)P >> 5, pb = (uint32_t)P & 31u;
+            cnt = rtot - (CW8[pw] + __popc(RW[pw] & (0xffffffffu >> (31u - pb))));
+          }
+          // ... and this round: lanes s < lane with P(s) > P (bit-sliced compare)
+          const uint32_t qm = __ballot_sync(FULL, q);
+          const uint32_t pv = q ? (uint32_t)P : 0u;
+          uint32_t gt = 0, eq = FULL;
+#pragma unroll
+          for (int kb = 7; kb >= 0; --kb) {
+            const uint32_t bk = __ballot_sync(FULL, (pv >> kb) & 1u);
+            if ((pv >> kb) & 1u) eq &= bk;
+            else { gt |= eq & bk; eq &= ~bk; }
+          }
+          cnt += __popc(gt & qm & lanemask_lt());
+          __syncwarp();
+          // R4
+          if (valid) {
+            uint32_t bin, cntb = 1;
+            if (q) {
+              const uint32_t rd = (wb + xw - w) - WPI[P] - cnt;
+              bin = rd_bin(rd, log2bins, nbins);
+              rdsum += rd;
+            } else {
+              bin = nbins - 1;
+              if (st) cntb = w;
+            }
+            if (O.n) bin += obj_row(O, lfull) * nbins;
+            if (smem_hist) atomicAdd(&S.hist[bin], cntb);
+            else atomicAdd((unsigned long long*)&g_hist[bin], (unsigned long long)cntb);
+            if (st) stream += w - 1;  // all but the last of merged stores are one-shot elements
+          }
+          qbits |= (uint32_t)q << r;
+          hbits |= (uint32_t)hd << r;
+          // R += { P(s) } of this round's queries; word prefix counts
+          uint32_t nr = 0;
+#pragma unroll
+          for (int k = 0; k < 8; ++k) {
+            const uint32_t o = __reduce_or_sync(FULL, (q && ((uint32_t)P >> 5) == (uint32_t)k) ? 1u << (P & 31) : 0u);
+            if (lane == (uint32_t)k) nr = RW[k] | o;
+          }
+          __syncwarp();
+          if (lane < 8) RW[lane] = nr;
+          uint32_t pc = lane < 8 ? __popc(nr) : 0u, xc = pc;
+#pragma unroll
+          for (int o = 1; o < 8; o <<= 1) {
+            const uint32_t y = __shfl_up_sync(FULL, xc, o);
+            if (lane >= (uint32_t)o) xc += y;
+          }
+          if (lane < 8) CW8[lane] = xc - pc;
+          rtot = __shfl_sync(FULL, xc, 7);
+          wb += __shfl_sync(FULL, xw, 31);
+          qn += __popc(qm);
+          __syncwarp();
+        }
+        // streaming: positions whose element is never used again (not reused, no dup)
+        for (uint32_t r = 0; 32 * r < n; ++r) {
+          const uint32_t i = 32 * r + lane;
+          if (i < n && !((qbits >> r) & 1u) && !((hbits >> r) & 1u) && !((RW[i >> 5] >> (i & 31u)) & 1u)) stream += 1;
+        }
+        wt += wb;
+        qt += qn;
+        __syncwarp();
+      }
+      if (lane == 0) {
+        atomicAdd(&S.misc[4], wt);
+        atomicAdd(&S.misc[5], qt);
+      }
+      stream = __reduce_add_sync(FULL, stream);
+      if (lane == 0 && stream) atomicAdd((unsigned long long*)g_stream, (unsigned long long)stream);
+#pragma unroll
+      for (int o = 16; o; o >>= 1) rdsum += __shfl_xor_sync(FULL, rdsum, o);
+      if (lane == 0 && rdsum) atomicAdd((unsigned long long*)g_stream + 1, rdsum);
+      __syncthreads();
+      if (tx == 0) {
+        tile_w[tile] = S.misc[4];
+        tile_q[tile] = S.misc[5];
+      }
+      if (smem_hist)
+        for (uint32_t k = tx; k < hbins; k += TL_NT)
+          if (S.hist[k]) atomicAdd((unsigned long long*)&g_hist[k], (unsigned long long)S.hist[k]);
+      return;
+    }
+  }
   const uint32_t lastseg = m ? S.sgs[m - 1] : 0u;
   const uint32_t second = S.misc[2];
   auto partial = [&](uint32_t x) {

@@ -340,7 +340,10 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
         else md = true;
       }
     }
-    if (MD && md) finish_md<F>(A, C, whist, sites_smem, kind, u & PK_M, s, s);  // F_OBJ: s holds the row
+    // F_OBJ: the group's object from its first record's address (global; recently streamed, L2)
+    if (MD && md)
+      finish_md<F>(A, C, whist, sites_smem, kind, u & PK_M, s,
+                   (F & F_OBJ) ? row_of(A, C, __ldg(A.addr + c_lo + j) >> A.lbs_md) : 0u);
     if (BD) {
       const uint32_t cnt = (u >> PK_CNT) & PK_M;
       if (bd) {
@@ -764,8 +767,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
               Q.m[pos] = m2;
               Q.kt[pos] = ((((k < 4 ? mmx : mmy) >> (8 * (k & 3))) & 3u) << 16) | t[k];
               Q.cta[pos] = c[k];
-              // F_OBJ (no per-site counters): the slot carries the group's object row
-              Q.site[pos] = OBJ ? row_of(A, C, a[k] >> A.lbs_md) : (A.nsites ? R.site[ring_slot(j0 + k)] : 0u);
+              Q.site[pos] = A.nsites ? R.site[ring_slot(j0 + k)] : 0u;
             }
             qn += __popc(im);
           }
@@ -800,7 +802,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
               const uint32_t sl0 = ring_slot(j0 + lastk);
               qc[0] = ((R.meta[sl0] & 3u) << 16) | R.tid[sl0];
               qc[1] = R.cta[sl0];
-              qc[2] = OBJ ? row_of(A, C, R.addr[sl0] >> A.lbs_md) : (A.nsites ? R.site[sl0] : 0u);
+              qc[2] = A.nsites ? R.site[sl0] : 0u;
             }
           }
           cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
