@@ -23,7 +23,7 @@ import os
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libcadv.so")
+LIB_PATH = os.environ.get("CADV_LIB") or os.path.join(_HERE, "libcadv.so")  # CADV_LIB: A/B builds
 
 CADV_OK, CADV_ERR_INVALID_ARG, CADV_ERR_BAD_TRACE, CADV_ERR_NO_TRACE = 0, 1, 2, 3
 CADV_ERR_OOM, CADV_ERR_CUDA, CADV_ERR_NCCL, CADV_ERR_UNSUPPORTED = 4, 5, 6, 7

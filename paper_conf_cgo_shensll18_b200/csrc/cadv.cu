@@ -248,7 +248,9 @@ cadv_status create_ctx(cadv_ctx** out, int device, void* cuda_stream, const void
   c->nranks = nranks;
   c->num_sms = prop.multiProcessorCount;
   if (const char* e = getenv("CADV_SCAN_CTAS")) c->scan_ctas = atoi(e);
-  if (cudaEventCreate(&c->ev0) != cudaSuccess || cudaEventCreate(&c->ev1) != cudaSuccess) {
+  if (cudaEventCreate(&c->ev0) != cudaSuccess || cudaEventCreate(&c->ev1) != cudaSuccess ||
+      cudaMallocHost(&c->hstage, 512) != cudaSuccess) {
+    if (c->hstage) cudaFreeHost(c->hstage);
     delete c;
     return CADV_ERR_CUDA;
   }
@@ -261,6 +263,7 @@ cadv_status create_ctx(cadv_ctx** out, int device, void* cuda_stream, const void
       fprintf(stderr, "cadv_create: %s\n", err.c_str());
       cudaEventDestroy(c->ev0);
       cudaEventDestroy(c->ev1);
+      cudaFreeHost(c->hstage);
       delete c;
       return CADV_ERR_NCCL;
     }
@@ -309,6 +312,7 @@ CADV_API cadv_status cadv_destroy(cadv_ctx* c) {
   for (auto& b : c->buf)
     if (b.p) cudaFree(b.p);
   if (c->host_pinned) cudaFreeHost(c->host_pinned);
+  if (c->hstage) cudaFreeHost(c->hstage);
   if (c->ev0) cudaEventDestroy(c->ev0);
   if (c->ev1) cudaEventDestroy(c->ev1);
   for (auto e : c->prof_ev) cudaEventDestroy(e);
@@ -542,11 +546,14 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
   // one flag word for both site checks
   P.site_flag = d + (q.md ? o_mdf : o_bdf);
   if (flags && t.n) CK(launch_scan(c, flags, P), "scan launch");
-  // R0 results of the pass: CTA-id range, T_c / deferred-group capacity
+  // R0 results of the pass: CTA-id range, T_c / deferred-group capacity; the
+  // reuse compaction is queued behind them, so one synchronisation covers both
   {
-    Scalars hs;
-    CK(cudaMemcpyAsync(&hs, scalars(c), sizeof hs, cudaMemcpyDeviceToHost, c->stream), "D2H");
+    Scalars* hsp = (Scalars*)((uint8_t*)c->hstage + 64);
+    CK(cudaMemcpyAsync(hsp, scalars(c), sizeof(Scalars), cudaMemcpyDeviceToHost, c->stream), "D2H");
+    if (q.rd && (t.n || multi)) CK(rd_compact(c, rs), "reuse compaction");
     CK(cudaStreamSynchronize(c->stream), "scan");
+    const Scalars hs = *hsp;
     c->max_cta = (uint32_t)hs.max_cta;
     if (q.bd && t.n) {
       if (hs.max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
@@ -600,11 +607,10 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
       if (c->comm->allreduce_max_u32(c->tc_buf, c->max_cta + 1, c->stream))
         return fail(c, CADV_ERR_NCCL, c->comm->err);
     }
-    unsigned long long m = 0;
-    CK(cudaMemcpyAsync(&m, P.ndefer, 8, cudaMemcpyDeviceToHost, c->stream), "D2H");
-    CK(cudaStreamSynchronize(c->stream), "scan");
-    CK(launch_bd_resolve(c, defer, m, c->tc_buf, c->tc_gen, q.bd_ws, d + o_bdt, q.bd_sites ? d + o_bds : nullptr,
-                         q.bd_sites ? q.nsites : 0),
+    // the deferred-group count stays on the device (the scan's read-back
+    // already checked it against the capacity)
+    CK(launch_bd_resolve(c, defer, P.ndefer, c->defer_cap, c->tc_buf, c->tc_gen, q.bd_ws, d + o_bdt,
+                         q.bd_sites ? d + o_bds : nullptr, q.bd_sites ? q.nsites : 0),
        "bd resolve");
   }
   if (multi && c->comm->allreduce_sum_u64(d, total, c->stream)) return fail(c, CADV_ERR_NCCL, c->comm->err);

@@ -74,6 +74,9 @@ struct cadv_ctx {
   cadv::DevBuf buf[cadv::B_COUNT];
   void* host_pinned = nullptr;
   size_t host_pinned_bytes = 0;
+  // small pinned staging for the per-call scalars read back mid-call (one
+  // stream synchronisation for the scan scalars, kept count and CTA range)
+  void* hstage = nullptr;  // 512 B: [0] kept records, [1] kept CTA-id max, +64: Scalars
   // per-kernel profiling (cadv_set_profiling)
   bool profiling = false;
   std::vector<cudaEvent_t> prof_ev;   // 2 per launch
@@ -137,8 +140,9 @@ void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nwarps, ui
 cudaError_t launch_squeeze(cadv_ctx* c, const uint32_t* kin, const uint64_t* vin, uint32_t* kout, uint64_t* vout,
                            const uint64_t* cnt, const uint64_t* off, uint64_t nblocks, uint64_t chunk_cap);
 cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P);
-cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const uint32_t* tc, uint32_t tc_gen,
-                              uint32_t ws, uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites);
+cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, const unsigned long long* m, uint64_t cap,
+                              const uint32_t* tc, uint32_t tc_gen, uint32_t ws, uint64_t* bd_tot, uint64_t* bd_sites,
+                              uint32_t nsites);
 
 // ---- reuse distance around the scan (reuse.cu)
 struct RdState {
@@ -150,6 +154,10 @@ struct RdState {
   uint64_t* blkcnt = nullptr;  // [grid] kept per scan block, then [grid] offsets
   uint64_t grid = 0, chunk_cap = 0;
 };
+// R1 compaction of the scan's per-warp regions (exclusive scan of the counts
+// + squeeze), queued on the stream; the kept count and the kept CTA-id range
+// arrive in c->hstage (words 0, 1) once the stream reaches them.
+cudaError_t rd_compact(cadv_ctx* c, const RdState& st);
 // workspace for the run-compression output of the scan
 cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st);
 // CTA regroup, tiles, cross-tile phase after the scan wrote the kept records

@@ -1238,6 +1238,21 @@ cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const 
   return cudaSuccess;
 }
 
+cudaError_t rd_compact(cadv_ctx* c, const RdState& S) {
+  cudaError_t e;
+  uint64_t* h = (uint64_t*)c->hstage;
+  h[0] = h[1] = 0;
+  if (!S.grid) return cudaSuccess;
+  // pack the per-block regions: offsets = exclusive scan of the block counts
+  uint64_t* off = S.blkcnt + S.grid + 4;
+  if ((e = exclusive_scan_u64(c, S.blkcnt, off, S.grid + 1))) return e;
+  if ((e = cudaMemcpyAsync(&h[0], off + S.grid, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = launch_squeeze(c, (const uint32_t*)S.k1, (const uint64_t*)S.v1, (uint32_t*)S.k0, (uint64_t*)S.v0, S.blkcnt,
+                          off, S.grid, S.chunk_cap)))
+    return e;
+  return cudaMemcpyAsync(&h[1], &scalars(c)->max_cta, 8, cudaMemcpyDeviceToHost, c->stream);
+}
+
 cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbins, uint64_t* d_hist,
                       uint64_t* d_stats, const ObjTab* obj) {
   cudaError_t e;
@@ -1249,17 +1264,10 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   const uint32_t* key = nullptr;
   const uint64_t* val = nullptr;
   if (S.grid) {
+    // rd_compact ran and the caller synchronised the stream
     void *k0 = S.k0, *k1 = S.k1, *v0 = S.v0, *v1 = S.v1;
-    // pack the per-block regions: offsets = exclusive scan of the block counts
-    uint64_t* off = S.blkcnt + S.grid + 4;
-    if ((e = exclusive_scan_u64(c, S.blkcnt, off, S.grid + 1))) return e;
-    if ((e = cudaMemcpyAsync(&K, off + S.grid, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
-    if ((e = launch_squeeze(c, (const uint32_t*)k1, (const uint64_t*)v1, (uint32_t*)k0, (uint64_t*)v0, S.blkcnt, off,
-                            S.grid, S.chunk_cap)))
-      return e;
-    unsigned long long mxc = 0;  // CTA-id range of the kept records (and BB groups), from the scan / squeeze
-    if ((e = cudaMemcpyAsync(&mxc, &scalars(c)->max_cta, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
-    if ((e = cudaStreamSynchronize(c->stream))) return e;
+    K = ((const uint64_t*)c->hstage)[0];
+    const unsigned long long mxc = ((const unsigned long long*)c->hstage)[1];  // CTA-id range (scan / squeeze)
     if (mxc > c->max_cta) c->max_cta = (uint32_t)mxc;
     c->counts[0] = K;
     // ---- R1b regroup by CTA (stable)
@@ -1336,9 +1344,11 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
                        tile_q, En, sc, wide_list, O));
     if ((e = cudaGetLastError())) return e;
   }
-  unsigned long long nent;
-  if ((e = cudaMemcpyAsync(&nent, &sc->count[1], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
-  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  unsigned long long nent = cnt14[0];
+  if (cnt14[2] || cnt14[3]) {  // the wider-key tiles add entries too
+    if ((e = cudaMemcpyAsync(&nent, &sc->count[1], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+    if ((e = cudaStreamSynchronize(c->stream))) return e;
+  }
   c->counts[1] = nent;
   if (nent == 0) return cudaSuccess;
   // ---- cross-tile phase

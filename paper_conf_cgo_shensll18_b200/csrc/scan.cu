@@ -168,11 +168,16 @@ __device__ __forceinline__ void site_add(const ScanArgs& A, uint32_t* smem_tab, 
 // stream) into ring stage p % KS: one 1-D bulk copy per column, completion
 // counted on the stage's mbarrier.  Stateless: column pointers come from the
 // kernel parameters (constant bank), so no lane holds them in registers.
+// Called by the whole (converged) warp with warp-uniform operands: one
+// elected lane issues the copy (elect.sync inside the asm, so ptxas needs no
+// per-lane loop to move the operands to uniform registers).
 template <int F>
 __device__ __forceinline__ void bulk_cp(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
-  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(dst),
-               "l"(src), "r"(bytes), "r"(bar)
-               : "memory");
+  asm volatile(
+      "{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\n"
+      "@p cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n}" ::"r"(dst),
+      "l"(src), "r"(bytes), "r"(bar)
+      : "memory");
 }
 template <int F>
 __device__ __forceinline__ void issue_piece(const ScanArgs& A, uint32_t ring, uint32_t bar0, uint64_t c_lo,
@@ -191,7 +196,10 @@ __device__ __forceinline__ void issue_piece(const ScanArgs& A, uint32_t ring, ui
     if (NA) bytes += r16(cnt * 8);
     if (NG) bytes += r16(cnt * 2) + 2 * r16(cnt * 4);
   }
-  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(bar), "r"(bytes) : "memory");
+  asm volatile(
+      "{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\n@p mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n}" ::"r"(bar),
+      "r"(bytes)
+      : "memory");
   if (NA) bulk_cp<F>(ring + R_ADDR + stg * KR * 8, A.addr + q0, r16(cnt * 8), bar);
   bulk_cp<F>(ring + R_CTA + stg * KR * 4, A.cta + q0, r16(cnt * 4), bar);
   if (NG) {
@@ -469,8 +477,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     __syncwarp();
     const uint32_t ring_s = smem_u32(ring), bar_s = smem_u32(bar);
     uint32_t issued = npieces < (uint32_t)KS ? npieces : (uint32_t)KS, waited = 0;
-    if (lane == 0)
-      for (uint32_t p = 0; p < issued; ++p) issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, p);
+    for (uint32_t p = 0; p < issued; ++p) issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, p);
     const RingView R{(const uint64_t*)(ring + R_ADDR), (const uint32_t*)(ring + R_CTA),
                      (const uint16_t*)(ring + R_TID),  (const uint32_t*)(ring + R_WINST),
                      (const uint32_t*)(ring + R_SITE), ring + R_META};
@@ -502,10 +509,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       if (base >= clen && !(NG && cr_on && cr_own) && !(RD && open_rd)) break;
       // piece p + 1 goes into the stage of piece p - 1 (consumed)
       if (p >= 1 && issued < npieces) {
-        if (lane == 0) {
-          fence_proxy_async();
-          issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, issued);
-        }
+        fence_proxy_async();
+        issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, issued);
         ++issued;
       }
       mbar_wait(&bar[p % KS], (p / KS) & 1u);
@@ -888,9 +893,12 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
 }
 
 // Deferred BD groups: divergent iff active < clamp(T_c - w*W, 0, W).
-__global__ void __launch_bounds__(256) k_bd_resolve(const uint4* __restrict__ defer, uint64_t m,
+// m: number of deferred groups, read on the device (no host round trip)
+__global__ void __launch_bounds__(256) k_bd_resolve(const uint4* __restrict__ defer,
+                                                    const unsigned long long* __restrict__ pm, uint64_t cap,
                                                     const uint32_t* __restrict__ tc, uint32_t gen, uint32_t ws,
                                                     uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites) {
+  const uint64_t m = *pm < cap ? *pm : cap;
   __shared__ uint32_t s_div[NSITE_SMEM];
   const bool sm = nsites && nsites <= NSITE_SMEM;
   if (sm)
@@ -1023,12 +1031,13 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
   }
 }
 
-cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, uint64_t m, const uint32_t* tc, uint32_t tc_gen,
-                              uint32_t ws, uint64_t* bd_tot, uint64_t* bd_sites, uint32_t nsites) {
-  if (m == 0) return cudaSuccess;
-  const uint64_t want = (m + 255) / 256;
-  const int grid = (int)(want < (uint64_t)c->num_sms * 4 ? want : (uint64_t)c->num_sms * 4);
-  CADV_LAUNCH(c, k_bd_resolve<<<grid, 256, 0, c->stream>>>((const uint4*)defer, m, tc, tc_gen, ws, bd_tot, bd_sites, nsites));
+cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, const unsigned long long* m, uint64_t cap,
+                              const uint32_t* tc, uint32_t tc_gen, uint32_t ws, uint64_t* bd_tot, uint64_t* bd_sites,
+                              uint32_t nsites) {
+  const uint64_t want = (cap + 255) / 256;
+  const int grid = (int)(want < (uint64_t)c->num_sms * 4 ? (want ? want : 1) : (uint64_t)c->num_sms * 4);
+  CADV_LAUNCH(c, k_bd_resolve<<<grid, 256, 0, c->stream>>>((const uint4*)defer, m, cap, tc, tc_gen, ws, bd_tot,
+                                                           bd_sites, nsites));
   return cudaGetLastError();
 }
 
