@@ -237,7 +237,8 @@ CADV_API cadv_status cadv_destroy(cadv_ctx *ctx);
 CADV_API const char *cadv_last_error(const cadv_ctx *ctx);
 
 /* Device time (CUDA events on the context's stream) of the last successful
- * cadv_load_trace / analysis call, in milliseconds. */
+ * cadv_load_trace / analysis call, in milliseconds (0 for a load of device
+ * columns: they are only registered, no device work runs). */
 CADV_API float cadv_last_elapsed_ms(const cadv_ctx *ctx);
 
 /* Number of kernels the last call launched (for bench.py's gpu_launches). */

@@ -357,12 +357,14 @@ CADV_API cadv_status cadv_load_trace(cadv_ctx* c, const cadv_trace_desc* d, uint
       ((uintptr_t)d->winst & 3))
     return fail(c, CADV_ERR_INVALID_ARG, "trace columns must be naturally aligned");
   CK(cudaSetDevice(c->device), "cudaSetDevice");
-  cadv_status s = begin_call(c);
-  if (s != CADV_OK) return s;
+  cadv_status s = CADV_OK;
+  const bool copy = !d->on_device && d->n;
+  // device columns are only registered (no device work, no synchronisation)
+  if (copy && (s = begin_call(c)) != CADV_OK) return s;
   c->t = *d;
   c->t.on_device = 1;
   c->global_offset = global_offset;
-  if (!d->on_device && d->n) {
+  if (copy) {
     const void* src[6] = {d->addr, d->cta, d->tid, d->site, d->winst, d->meta};
     size_t es[6] = {8, 4, 2, 4, 4, 1};
     void* dst[6];
@@ -377,9 +379,17 @@ CADV_API cadv_status cadv_load_trace(cadv_ctx* c, const cadv_trace_desc* d, uint
     c->t.winst = (const uint32_t*)dst[4];
     c->t.meta = (const uint8_t*)dst[5];
   }
-  void* h;
-  s = end_call(c, nullptr, 0, &h);
-  if (s != CADV_OK) return s;
+  if (copy) {
+    void* h;
+    s = end_call(c, nullptr, 0, &h);
+    if (s != CADV_OK) return s;
+  } else {
+    c->launches = 0;
+    c->nprof = 0;
+    c->prof_ms.clear();
+    c->prof_name.clear();
+    c->elapsed_ms = 0.f;
+  }
   c->max_cta = 0;  // R0's CTA-id range comes out of each analysis' streaming pass
   if (c->comm) {
     s = load_trace_collective(c);

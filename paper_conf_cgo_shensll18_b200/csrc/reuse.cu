@@ -331,7 +331,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     S.lmin = ~0ull;
     S.lmax = 0;
     S.misc[2] = m;
-    S.misc[3] = S.misc[4] = S.misc[5] = 0;  // warp path: longest segment, weight and query totals
+    S.misc[3] = S.misc[4] = S.misc[5] = S.misc[6] = 0;  // warp path: longest segment, weight / query totals, queue
   }
   __syncthreads();
   {
@@ -368,26 +368,8 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   }
   if (smem_hist)
     for (uint32_t k = tx; k < hbins; k += TL_NT) S.hist[k] = 0;
-  // ---- load (striped)
-  uint16_t* PSW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[0] : nullptr;
   uint32_t* const K32a = reinterpret_cast<uint32_t*>(S.key[0]);
   uint32_t* const K32b = reinterpret_cast<uint32_t*>(S.key[1]);
-  for (uint32_t x = tx; x < TL_CAP; x += TL_NT) {
-    if (x < m) {
-      uint64_t v = __ldg(val + b + x);
-      uint64_t l = v & LINE_MASK;
-      if (MODE == 0) K32a[swz<uint32_t>(x)] = (uint32_t)(((l - lmin) << 12) | x);
-      else S.key[0][WIDE ? x : swz<uint64_t>(x)] = WIDE ? l : (((l - lmin) << 12) | x);
-      uint32_t w = (uint32_t)(v >> VB_W) + 1u;
-      S.sdw[x] = (uint8_t)(((v >> VB_STORE) & 1u) | (((v >> VB_DUP) & 1u) << 1) | (w << 2));
-    } else {
-      if (MODE == 0) K32a[swz<uint32_t>(x)] = 0xffffffffu;
-      else S.key[0][WIDE ? x : swz<uint64_t>(x)] = ~0ull;
-      S.sdw[x] = 0;
-    }
-    if (WIDE) PSW[x] = (uint16_t)x;
-    S.fnx[x] = 0;
-  }
   // ---- segment starts (blocked: thread owns 8 consecutive positions)
   constexpr int IPT = TL_CAP / TL_NT;
   uint32_t ssm = 0, ss_local = 0;
@@ -452,7 +434,9 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       uint32_t* const WPI = reinterpret_cast<uint32_t*>(S.pl) + warp * 256;
       uint32_t* const RW = reinterpret_cast<uint32_t*>(S.ffl) + warp * 16;  // [8] bitmap words
       uint32_t* const CW8 = RW + 8;                                          // [8] set bits before each word
-      for (uint32_t sg = warp; sg < nseg; sg += TL_NT / 32) {
+      // segments longest first would be ideal; a shared counter hands them out in order
+      for (uint32_t sg = __shfl_sync(FULL, lane == 0 ? atomicAdd(&S.misc[6], 1u) : 0u, 0); sg < nseg;
+           sg = __shfl_sync(FULL, lane == 0 ? atomicAdd(&S.misc[6], 1u) : 0u, 0)) {
         const uint32_t s0 = S.es[sg], n = (sg + 1 < nseg ? S.es[sg + 1] : m) - s0;
         for (uint32_t k = lane; k < 512; k += 32) HK[k] = 0xffffffffu;
         if (lane < 8) { RW[lane] = 0; CW8[lane] = 0; }
@@ -590,6 +574,25 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       return;
     }
   }
+  // ---- block path: load (striped)
+  uint16_t* PSW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[0] : nullptr;
+  for (uint32_t x = tx; x < TL_CAP; x += TL_NT) {
+    if (x < m) {
+      uint64_t v = __ldg(val + b + x);
+      uint64_t l = v & LINE_MASK;
+      if (MODE == 0) K32a[swz<uint32_t>(x)] = (uint32_t)(((l - lmin) << 12) | x);
+      else S.key[0][WIDE ? x : swz<uint64_t>(x)] = WIDE ? l : (((l - lmin) << 12) | x);
+      uint32_t w = (uint32_t)(v >> VB_W) + 1u;
+      S.sdw[x] = (uint8_t)(((v >> VB_STORE) & 1u) | (((v >> VB_DUP) & 1u) << 1) | (w << 2));
+    } else {
+      if (MODE == 0) K32a[swz<uint32_t>(x)] = 0xffffffffu;
+      else S.key[0][WIDE ? x : swz<uint64_t>(x)] = ~0ull;
+      S.sdw[x] = 0;
+    }
+    if (WIDE) PSW[x] = (uint16_t)x;
+    S.fnx[x] = 0;
+  }
+  __syncthreads();
   const uint32_t lastseg = m ? S.sgs[m - 1] : 0u;
   const uint32_t second = S.misc[2];
   auto partial = [&](uint32_t x) {
