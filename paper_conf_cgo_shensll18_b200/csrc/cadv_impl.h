@@ -39,7 +39,7 @@ enum BufId {
   B_RD_KEY, B_RD_VAL, B_RD_TILESTAT, B_RD_TILEW, B_RD_TILEQ, B_RD_ENT, B_RD_ENT_KEY0, B_RD_ENT_KEY1,
   B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP, B_DEFER, B_OUT2,
   B_ALIGN0, B_ALIGN1, B_ALIGN2, B_ALIGN3, B_ALIGN4, B_ALIGN5,
-  B_XCH_K0, B_XCH_K1, B_XCH_V0, B_XCH_V1, B_XCH_CNT, B_COMM, B_OBJ,
+  B_XCH_K0, B_XCH_K1, B_XCH_V0, B_XCH_V1, B_XCH_CNT, B_COMM, B_OBJ, B_RD_ENT_ALL,
   B_COUNT
 };
 

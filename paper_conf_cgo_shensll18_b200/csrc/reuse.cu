@@ -285,6 +285,15 @@ struct TileSmemWide {
   uint16_t ps[2][TL_CAP];
 };
 
+// Where a rank's tiles sit in the global kept sequence (kernel scope over
+// ranks; zeros / K for one GPU and for CTA scope): entry positions, tile ids
+// and the continuation of the one segment across shard edges are global.
+struct TilePos {
+  uint64_t pos_base;   // global kept position of this rank's first kept record
+  uint32_t tile_base;  // global index of this rank's first tile
+  uint64_t k_glob;     // kept records of all ranks
+};
+
 struct EntryCols {
   uint32_t* seg;
   uint64_t* line;
@@ -315,7 +324,8 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     k_rd_tile(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val, uint64_t K,
               const uint32_t* __restrict__ bounds, uint32_t ntiles, int log2bins, uint32_t nbins,
               uint64_t* __restrict__ g_hist, uint64_t* __restrict__ g_stream, uint32_t* __restrict__ tile_w,
-              uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc, uint32_t* wide_list, ObjTab O) {
+              uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc, uint32_t* wide_list, ObjTab O,
+              TilePos TP) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
   const uint32_t tx = threadIdx.x;
@@ -377,7 +387,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   for (int j = 0; j < IPT; ++j) {
     uint32_t x = tx * IPT + j;
     uint64_t gx = b + x;
-    bool sflag = x < m && (gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1)));
+    bool sflag = x < m && (TP.pos_base + gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1)));
     if (sflag) { ssm |= 1u << j; ss_local = x; }
   }
   uint32_t* tmax = reinterpret_cast<uint32_t*>(S.es);
@@ -395,8 +405,9 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       S.sgs[x] = (uint16_t)cur;
     }
   }
-  const bool head_cont = m > 0 && b > 0 && (!key || __ldg(key + b) == __ldg(key + b - 1));
-  const bool tail_cont = m > 0 && e < K && (!key || __ldg(key + e) == __ldg(key + e - 1));
+  // (kernel scope over ranks: the one segment continues across the shards' kept records)
+  const bool head_cont = m > 0 && TP.pos_base + b > 0 && (!key || __ldg(key + b) == __ldg(key + b - 1));
+  const bool tail_cont = m > 0 && TP.pos_base + e < TP.k_glob && (!key || __ldg(key + e) == __ldg(key + e - 1));
   __syncthreads();
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) S.es[x] = 0;
   // ---- warp path (MODE 0): the tile holds whole segments of <= 256 kept
@@ -565,8 +576,8 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       if (lane == 0 && rdsum) atomicAdd((unsigned long long*)g_stream + 1, rdsum);
       __syncthreads();
       if (tx == 0) {
-        tile_w[tile] = S.misc[4];
-        tile_q[tile] = S.misc[5];
+        tile_w[TP.tile_base + tile] = S.misc[4];
+        tile_q[TP.tile_base + tile] = S.misc[5];
       }
       if (smem_hist)
         for (uint32_t k = tx; k < hbins; k += TL_NT)
@@ -660,7 +671,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       const uint32_t slot = ebase + run;
       E.seg[slot] = key ? __ldg(key + b + x) : 0u;
       E.line[slot] = WIDE ? LN(s_) : LN(s_) + lmin;
-      E.tile[slot] = tile;
+      E.tile[slot] = TP.tile_base + tile;
       S.es[x] = (uint16_t)(run + 1);
       run++;
     }
@@ -762,7 +773,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       const uint32_t sdw = S.sdw[x];
       if (f & 1u) {
         const bool head_piece = S.sgs[x] == 0 && head_cont;
-        E.f[slot] = (uint32_t)(b + x);
+        E.f[slot] = (uint32_t)(TP.pos_base + b + x);
         E.fa[slot] = (uint32_t)S.qx[x] - (uint32_t)S.qx[S.sgs[x]];
         E.fw[slot] = WP[x];
         E.ff[slot] = (uint8_t)(((sdw & 1u) ? 0u : 1u) | (((sdw >> 1) & 1u) ? 0u : 2u) | (S.fnx[x] ? 4u : 0u) |
@@ -776,7 +787,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
         while (a0 < a1) { uint32_t md = (a0 + a1) >> 1; if (QS[swz<uint32_t>(md)] < lo_key) a0 = md + 1; else a1 = md; }
         uint32_t c0 = a0, c1 = Q;
         while (c0 < c1) { uint32_t md = (c0 + c1) >> 1; if (QS[swz<uint32_t>(md)] < hi_key) c0 = md + 1; else c1 = md; }
-        E.l[slot] = (uint32_t)(b + x);
+        E.l[slot] = (uint32_t)(TP.pos_base + b + x);
         E.lw[slot] = WP[x];
         E.ld[slot] = c0 - a0;
         E.lf[slot] = (uint8_t)((sdw & 1u) | (((sdw >> 1) & 1u) ? 0u : 2u) | ((sdw >> 2) << 2));
@@ -790,8 +801,8 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   for (int o = 16; o; o >>= 1) rdsum += __shfl_xor_sync(FULL, rdsum, o);
   if (lane_id() == 0 && rdsum) atomicAdd((unsigned long long*)g_stream + 1, rdsum);
   if (tx == 0) {
-    tile_w[tile] = WT;
-    tile_q[tile] = Q;
+    tile_w[TP.tile_base + tile] = WT;
+    tile_q[TP.tile_base + tile] = Q;
   }
   __syncthreads();
   if (smem_hist)
@@ -837,6 +848,7 @@ struct CrossOut {
   uint32_t* xpos;   // query global kept position
   uint32_t* xq;     // its previous use (global kept position)
   int64_t* part;    // RD before subtracting the cross-tile dominance count
+  uint64_t* xline;  // its line (data-centric rows)
 };
 
 __global__ void k_link(const uint32_t* __restrict__ order, uint64_t E, EntryCols En,
@@ -872,6 +884,7 @@ __global__ void k_link(const uint32_t* __restrict__ order, uint64_t E, EntryCols
         X.xpos[slot] = En.f[e];
         X.xq[slot] = En.l[p];
         X.part[slot] = part;
+        X.xline[slot] = En.line[e];
       } else {
         const uint32_t row = O.n ? obj_row(O, En.line[e]) : 0u;
         atomicAdd((unsigned long long*)&g_hist[(uint64_t)row * nbins + nbins - 1], 1ull);
@@ -961,13 +974,11 @@ __global__ void k_iota_gather(const uint32_t* __restrict__ order, const uint32_t
 }
 
 constexpr uint32_t XF_SMEM_BINS = 4096;
-// O.n > 0 (data-centric attribution): the query's row comes from its line,
-// val[xpos[i]] (the CTA-major kept records)
+// O.n > 0 (data-centric attribution): the query's row comes from its line
 __global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__ part,
                                                      const uint32_t* __restrict__ cnt, uint64_t M, int log2bins,
                                                      uint32_t nbins, uint64_t* g_hist, uint64_t* g_stats,
-                                                     Scalars* sc, ObjTab O, const uint32_t* __restrict__ xpos,
-                                                     const uint64_t* __restrict__ val) {
+                                                     Scalars* sc, ObjTab O, const uint64_t* __restrict__ xline) {
   unsigned long long rdsum = 0;
   __shared__ uint32_t h[XF_SMEM_BINS];
   const uint32_t hbins = (O.n + 1) * nbins;
@@ -982,7 +993,7 @@ __global__ void __launch_bounds__(256) k_cross_final(const int64_t* __restrict__
       rd = 0;
     }
     uint32_t b = rd_bin((uint64_t)rd, log2bins, nbins);
-    if (O.n) b += obj_row(O, __ldg(val + xpos[i]) & LINE_MASK) * nbins;
+    if (O.n) b += obj_row(O, __ldg(xline + i)) * nbins;
     rdsum += (unsigned long long)rd;
     if (sm) {
       // warp-aggregated: one shared-memory atomic per distinct bin in the warp
@@ -1241,6 +1252,63 @@ cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const 
   return cudaSuccess;
 }
 
+// Spread kernel scope: every rank's cross-tile entries gathered on rank 0
+// (column by column, in rank order); *En / *nent become the gathered set
+// there and nent = 0 elsewhere.  Collective.
+cudaError_t gather_entries(cadv_ctx* c, EntryCols* En, unsigned long long* nent) {
+  cudaError_t e;
+  const int G = c->nranks, me = c->rank;
+  void* cb;
+  if ((e = ensure(c, B_COMM, (size_t)(2 + 2 * G) * 8 + 64, &cb))) return e;
+  uint64_t* d = (uint64_t*)cb;
+  const uint64_t mine = *nent;
+  if ((e = cudaMemcpyAsync(d, &mine, 8, cudaMemcpyHostToDevice, c->stream))) return e;
+  if (c->comm->allgather(d, d + 1, 8, c->stream)) return cudaErrorUnknown;
+  std::vector<uint64_t> cnt(G);
+  if ((e = cudaMemcpyAsync(cnt.data(), d + 1, 8 * G, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  std::vector<uint64_t> off(G + 1, 0);
+  for (int r = 0; r < G; ++r) off[r + 1] = off[r] + cnt[r];
+  const uint64_t N = off[G];
+  if (N == 0) { *nent = 0; return cudaSuccess; }
+  EntryCols A{};
+  if (me == 0) {
+    void* ent;
+    if ((e = ensure(c, B_RD_ENT_ALL, N * (4 + 8 + 4 + 4 + 4 + 4 + 1 + 4 + 4 + 4 + 1) + 16 * 16, &ent))) return e;
+    uint8_t* p = (uint8_t*)ent;
+    auto take = [&](size_t bytes) { uint8_t* q = p; p += (bytes + 15) & ~size_t(15); return q; };
+    A.line = (uint64_t*)take(N * 8);
+    A.seg = (uint32_t*)take(N * 4);
+    A.tile = (uint32_t*)take(N * 4);
+    A.f = (uint32_t*)take(N * 4);
+    A.fa = (uint32_t*)take(N * 4);
+    A.fw = (uint32_t*)take(N * 4);
+    A.l = (uint32_t*)take(N * 4);
+    A.lw = (uint32_t*)take(N * 4);
+    A.ld = (uint32_t*)take(N * 4);
+    A.ff = (uint8_t*)take(N);
+    A.lf = (uint8_t*)take(N);
+  }
+  auto col = [&](const void* src, void* dst, size_t es) -> int {
+    std::vector<uint64_t> soff(G, 0), scnt(G, 0), roff(G, 0), rcnt(G, 0);
+    scnt[0] = mine * es;
+    if (me == 0)
+      for (int r = 0; r < G; ++r) { roff[r] = off[r] * es; rcnt[r] = cnt[r] * es; }
+    return c->comm->alltoallv(src, soff.data(), scnt.data(), dst, roff.data(), rcnt.data(), c->stream);
+  };
+  if (col(En->line, A.line, 8) || col(En->seg, A.seg, 4) || col(En->tile, A.tile, 4) || col(En->f, A.f, 4) ||
+      col(En->fa, A.fa, 4) || col(En->fw, A.fw, 4) || col(En->l, A.l, 4) || col(En->lw, A.lw, 4) ||
+      col(En->ld, A.ld, 4) || col(En->ff, A.ff, 1) || col(En->lf, A.lf, 1))
+    return cudaErrorUnknown;
+  if (me == 0) {
+    *En = A;
+    *nent = N;
+  } else {
+    *nent = 0;
+  }
+  return cudaSuccess;
+}
+
 cudaError_t rd_compact(cadv_ctx* c, const RdState& S) {
   cudaError_t e;
   uint64_t* h = (uint64_t*)c->hstage;
@@ -1286,17 +1354,54 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
       val = res ? (const uint64_t*)v1 : (const uint64_t*)v0;
     }
   }
-  if (c->comm && (e = rd_exchange(c, cta_scope, &key, &val, &K))) return e;
-  if (K == 0) return cudaSuccess;
+  // Kernel scope over ranks ("spread"): the kept records stay on their rank
+  // and are tiled there as consecutive parts of the global kept sequence;
+  // only the cross-tile entries (first / last use of each line per tile
+  // piece) and the per-tile weight / query counts travel, to rank 0, which
+  // runs the cross-tile phase over all of them.  CTA scope
+  // redistributes the kept records by CTA range instead (rd_exchange).
+  const bool spread = c->comm != nullptr && !cta_scope;
+  if (c->comm && !spread && (e = rd_exchange(c, cta_scope, &key, &val, &K))) return e;
+  const uint64_t ntiles_loc = (K + TL_NOM - 1) / TL_NOM;
+  uint64_t ntiles = ntiles_loc;  // tiles of all ranks (global tile ids)
+  TilePos TP{0, 0, K};
+  std::vector<uint64_t> kk;       // spread: (K, ntiles) of every rank
+  if (spread) {
+    const int G = c->nranks;
+    void* cb;
+    if ((e = ensure(c, B_COMM, (size_t)(2 + 2 * G) * 8 + 64, &cb))) return e;
+    uint64_t* d = (uint64_t*)cb;
+    const uint64_t mine[2] = {K, ntiles_loc};
+    if ((e = cudaMemcpyAsync(d, mine, 16, cudaMemcpyHostToDevice, c->stream))) return e;
+    if (c->comm->allgather(d, d + 2, 16, c->stream)) return cudaErrorUnknown;
+    kk.resize(2 * G);
+    if ((e = cudaMemcpyAsync(kk.data(), d + 2, 16 * G, cudaMemcpyDeviceToHost, c->stream))) return e;
+    if ((e = cudaStreamSynchronize(c->stream))) return e;
+    uint64_t kg = 0, tg = 0;
+    for (int r = 0; r < G; ++r) {
+      if (r == c->rank) { TP.pos_base = kg; TP.tile_base = (uint32_t)tg; }
+      kg += kk[2 * r];
+      tg += kk[2 * r + 1];
+    }
+    if (kg >= 0xffffffffull) return cudaErrorNotSupported;  // global kept positions are u32
+    TP.k_glob = kg;
+    ntiles = tg;
+    if (kg == 0) return cudaSuccess;  // every rank sees it
+  } else if (K == 0) {
+    return cudaSuccess;
+  }
   // ---- tiles
-  uint64_t ntiles = (K + TL_NOM - 1) / TL_NOM;
-  c->counts[3] = ntiles;
+  c->counts[3] = ntiles_loc;
   void *bnd, *tw, *tq;
-  if ((e = ensure(c, B_RD_XTMP, (3 * ntiles + 8) * 4 + 64, &bnd))) return e;  // bounds + MODE 2 / MODE 1 lists
+  if ((e = ensure(c, B_RD_XTMP, (3 * ntiles_loc + 8) * 4 + 64, &bnd))) return e;  // bounds + MODE 2 / MODE 1 lists
   if ((e = ensure(c, B_RD_TILEW, (ntiles + 2) * 8 * 2, &tw))) return e;
   if ((e = ensure(c, B_RD_TILEQ, (ntiles + 2) * 8 * 2, &tq))) return e;
-  CADV_LAUNCH(c, k_tile_bounds<<<(unsigned)((ntiles + 1 + 7) / 8), 256, 0, c->stream>>>(key, K, (uint32_t*)bnd,
-                                                                                       ntiles));
+  if (spread && ((e = cudaMemsetAsync(tw, 0, (ntiles + 2) * 4, c->stream)) ||
+                 (e = cudaMemsetAsync(tq, 0, (ntiles + 2) * 4, c->stream))))
+    return e;
+  if (ntiles_loc)
+    CADV_LAUNCH(c, k_tile_bounds<<<(unsigned)((ntiles_loc + 1 + 7) / 8), 256, 0, c->stream>>>(key, K, (uint32_t*)bnd,
+                                                                                             ntiles_loc));
   // entries: at most one per kept record
   void* ent;
   size_t ent_bytes = K * (4 + 8 + 4 + 4 + 4 + 4 + 1 + 4 + 4 + 4 + 1) + 16 * 16;
@@ -1327,24 +1432,26 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   }
   uint32_t* tile_w = (uint32_t*)tw;
   uint32_t* tile_q = (uint32_t*)tq;
-  uint32_t* wide_list = (uint32_t*)bnd + (ntiles + 2);
-  CADV_LAUNCH(c, k_rd_tile<0><<<(unsigned)ntiles, TL_NT, sizeof(TileSmem), c->stream>>>(
-                     key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
-                     tile_q, En, sc, wide_list, O));
-  if ((e = cudaGetLastError())) return e;
+  uint32_t* wide_list = (uint32_t*)bnd + (ntiles_loc + 2);
+  if (ntiles_loc) {
+    CADV_LAUNCH(c, k_rd_tile<0><<<(unsigned)ntiles_loc, TL_NT, sizeof(TileSmem), c->stream>>>(
+                       key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
+                       tile_w, tile_q, En, sc, wide_list, O, TP));
+    if ((e = cudaGetLastError())) return e;
+  }
   unsigned long long cnt14[4];  // count[1..4]: entries, cross queries, MODE 2 tiles, MODE 1 tiles
   if ((e = cudaMemcpyAsync(cnt14, &sc->count[1], 32, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
   if (cnt14[3]) {
     CADV_LAUNCH(c, k_rd_tile<1><<<(unsigned)cnt14[3], TL_NT, sizeof(TileSmem), c->stream>>>(
-                       key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
-                       tile_q, En, sc, wide_list, O));
+                       key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
+                       tile_w, tile_q, En, sc, wide_list, O, TP));
     if ((e = cudaGetLastError())) return e;
   }
   if (cnt14[2]) {
     CADV_LAUNCH(c, k_rd_tile<2><<<(unsigned)cnt14[2], TL_NT, sizeof(TileSmemWide), c->stream>>>(
-                       key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles, log2bins, nbins, d_hist, d_stats, tile_w,
-                       tile_q, En, sc, wide_list, O));
+                       key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
+                       tile_w, tile_q, En, sc, wide_list, O, TP));
     if ((e = cudaGetLastError())) return e;
   }
   unsigned long long nent = cnt14[0];
@@ -1353,21 +1460,27 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     if ((e = cudaStreamSynchronize(c->stream))) return e;
   }
   c->counts[1] = nent;
-  if (nent == 0) return cudaSuccess;
-  // ---- cross-tile phase
-  // tile prefix sums of weights and local query counts (u64)
-  unsigned long long* twb = (unsigned long long*)((uint8_t*)tw + (ntiles + 2) * 8);
-  unsigned long long* tqb = (unsigned long long*)((uint8_t*)tq + (ntiles + 2) * 8);
+  // tile weight / local-query counts (u64); spread: summed over ranks (each rank filled its own tiles)
   void* wide;
   if ((e = ensure(c, B_RD_XQ2, (ntiles + 2) * 16 + 64, &wide))) return e;
-  {
-    unsigned long long* w64 = (unsigned long long*)wide;
-    unsigned long long* q64 = w64 + (ntiles + 2);
+  unsigned long long* w64 = (unsigned long long*)wide;
+  unsigned long long* q64 = w64 + (ntiles + 2);
+  if (spread) {
     CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_w, w64, ntiles, ntiles + 1));
     CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_q, q64, ntiles, ntiles + 1));
-    if ((e = exclusive_scan_u64(c, (const uint64_t*)w64, (uint64_t*)twb, ntiles + 1))) return e;
-    if ((e = exclusive_scan_u64(c, (const uint64_t*)q64, (uint64_t*)tqb, ntiles + 1))) return e;
+    if (c->comm->allreduce_sum_u64((uint64_t*)w64, 2 * (ntiles + 2), c->stream)) return cudaErrorUnknown;
+    if ((e = gather_entries(c, &En, &nent))) return e;  // rank 0: everyone's entries; others: nent = 0
+  } else if (nent) {
+    CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_w, w64, ntiles, ntiles + 1));
+    CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_q, q64, ntiles, ntiles + 1));
   }
+  if (nent == 0) return cudaSuccess;
+  // ---- cross-tile phase
+  // tile prefix sums of weights and local query counts
+  unsigned long long* twb = (unsigned long long*)((uint8_t*)tw + (ntiles + 2) * 8);
+  unsigned long long* tqb = (unsigned long long*)((uint8_t*)tq + (ntiles + 2) * 8);
+  if ((e = exclusive_scan_u64(c, (const uint64_t*)w64, (uint64_t*)twb, ntiles + 1))) return e;
+  if ((e = exclusive_scan_u64(c, (const uint64_t*)q64, (uint64_t*)tqb, ntiles + 1))) return e;
   // sort entries by (seg, line, tile)
   void *ek0, *ek1, *ei0, *ei1;
   if ((e = ensure(c, B_RD_ENT_KEY0, nent * 8, &ek0)) || (e = ensure(c, B_RD_ENT_KEY1, nent * 8, &ek1)) ||
@@ -1416,11 +1529,12 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   }
   // link
   void *xq, *xq2;
-  if ((e = ensure(c, B_RD_XQ, nent * (4 + 4 + 8) + 64, &xq))) return e;
+  if ((e = ensure(c, B_RD_XQ, nent * (4 + 4 + 8 + 8) + 64, &xq))) return e;
   CrossOut X;
   X.xpos = (uint32_t*)xq;
   X.xq = X.xpos + nent;
   X.part = (int64_t*)(((uintptr_t)(X.xq + nent) + 15) & ~(uintptr_t)15);
+  X.xline = (uint64_t*)(X.part + nent);
   CADV_LAUNCH(c, k_link<<<grid_ls, 256, 0, c->stream>>>(order, nent, En, twb, tqb, nbins, d_hist, d_stats, X, sc, O));
   unsigned long long M;
   if ((e = cudaMemcpyAsync(&M, &sc->count[2], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
@@ -1467,7 +1581,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     std::swap(ia, ib);
   }
   CADV_LAUNCH(c, k_cross_final<<<grid_ls, 256, 0, c->stream>>>(X.part, cnt, M, log2bins, nbins, d_hist, d_stats, sc, O,
-                                                                      X.xpos, val));
+                                                                      X.xline));
   return cudaGetLastError();
 }
 

@@ -215,3 +215,21 @@ def test_data_centric_shards(cadv, name, G, scope):
     out, err = run_ranks(cadv, t, cuts, lambda c: c.data_centric(objs, 128, scope, 0, 66, 32))
     assert not any(err), err
     check_all_equal(out, ref)
+
+
+@pytest.mark.parametrize("G", [2, 3, 4])
+def test_kernel_scope_spread_cyclic(cadv, G):
+    """Kernel scope over ranks keeps every kept record on its rank: K lines
+    read cyclically R times (27,000 records, several tiles per rank) split at
+    random positions; the cross-tile entries travel to rank 0.  Closed form:
+    K at ∞ and K (R - 1) at distance K - 1, on every rank."""
+    K, R = 9000, 3
+    n = K * R
+    addr = 0x7F0000000000 + 128 * (np.arange(n) % K)
+    t = tg.from_arrays(addr, np.zeros(n), np.zeros(n), np.zeros(n), np.arange(n), np.full(n, 2 << 2), nsites=1)
+    cuts = random_cuts(n, G, seed=40 + G, empty=(G == 4))
+    out, err = run_ranks(cadv, t, cuts, lambda c: c.reuse_histogram(128, 1, 0, K + 3))
+    assert not any(err), err
+    for h, s in out:
+        assert h[-1] == K and h[K - 1] == K * (R - 1) and h.sum() == n
+        assert s["streaming"] == 0 and s["finite_sum"] == K * (R - 1) * (K - 1)
