@@ -40,26 +40,29 @@ namespace {
 constexpr int LPR = 8;                 // consecutive records per lane in one warp step
 constexpr int KR = 32 * LPR;           // records per piece = one warp step
 constexpr int KS = 2;                  // ring stages per warp (piece p and piece p + 1 in flight)
-constexpr int RING = KR * KS;          // ring slots: record j lives in stage (j / KR) % KS
 constexpr int NWARP = 12;              // warps per CTA (one CTA per SM; 3 per SM sub-partition)
 constexpr int NTHR = NWARP * 32;
 constexpr int NSITE_SMEM = 512;        // per-site counters kept in shared memory up to this many sites
-constexpr int QCAP = 160;              // per-warp queue of complete runs awaiting finalization
+constexpr int QCAP = 288;              // per-warp queue of complete runs awaiting finalization (31 + 1 + KR)
 constexpr int OBJ_SMEM = 64;           // F_OBJ: object rows (objects + 1) kept in shared memory up to this many
 
-__device__ __forceinline__ uint32_t ring_slot(uint32_t j) {  // chunk-relative record -> ring slot
-  const uint32_t p = j / KR;
-  return (p - (p / KS) * KS) * KR + (j & (KR - 1));
-}
+// per-warp ring, stage-major: stage s occupies [s * STG_BYTES, (s + 1) * STG_BYTES)
+// and holds the KR records of one piece column by column (every column region
+// a multiple of 128 B), so one stage base + constant offsets address a piece
+constexpr uint32_t S_ADDR = 0;
+constexpr uint32_t S_CTA = S_ADDR + KR * 8;
+constexpr uint32_t S_TID = S_CTA + KR * 4;
+constexpr uint32_t S_WINST = S_TID + KR * 2;
+constexpr uint32_t S_SITE = S_WINST + KR * 4;
+constexpr uint32_t S_META = S_SITE + KR * 4;
+constexpr uint32_t STG_BYTES = S_META + KR;
+constexpr uint32_t R_BYTES = KS * STG_BYTES;
 
-// per-warp ring (bytes); every column region is a multiple of 128 B
-constexpr uint32_t R_ADDR = 0;
-constexpr uint32_t R_CTA = R_ADDR + RING * 8;
-constexpr uint32_t R_TID = R_CTA + RING * 4;
-constexpr uint32_t R_WINST = R_TID + RING * 2;
-constexpr uint32_t R_SITE = R_WINST + RING * 4;
-constexpr uint32_t R_META = R_SITE + RING * 4;
-constexpr uint32_t R_BYTES = R_META + RING;
+// chunk-relative record j -> byte offset of its stage in the ring
+__device__ __forceinline__ uint32_t stage_off(uint32_t j) {
+  const uint32_t p = j / KR;
+  return (p - (p / KS) * KS) * STG_BYTES;
+}
 
 constexpr uint64_t LINE_MASK = (1ull << 58) - 1;
 constexpr int VB_STORE = 58, VB_DUP = 59, VB_W = 60;
@@ -166,11 +169,44 @@ __device__ __forceinline__ void site_add(const ScanArgs& A, uint32_t* smem_tab, 
 
 // Per-warp TMA issue of piece p (records [c_lo + p KR, ...) of the warp's
 // stream) into ring stage p % KS: one 1-D bulk copy per column, completion
-// counted on the stage's mbarrier.  Stateless: column pointers come from the
-// kernel parameters (constant bank), so no lane holds them in registers.
-// Called by the whole (converged) warp with warp-uniform operands: one
-// elected lane issues the copy (elect.sync inside the asm, so ptxas needs no
-// per-lane loop to move the operands to uniform registers).
+// counted on the stage's mbarrier.  Called by the whole (converged) warp with
+// warp-uniform operands: one elected lane (elect.sync inside the asm, so
+// ptxas needs no per-lane loop to move the operands to uniform registers)
+// issues the expect-tx and every copy of a full piece from ONE asm block
+// (one election, destinations = stage base + constant column offsets).
+#define CADV_CP(DOFF, SRC, BYTES) \
+  "@p cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0+" #DOFF "], [" SRC "], " #BYTES ", [%1];\n"
+template <int F>
+__device__ __forceinline__ void issue_full(const ScanArgs& A, uint32_t dst, uint32_t bar, uint64_t q0) {
+  constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
+  static_assert(KR == 256 && S_CTA == 2048 && S_TID == 3072 && S_WINST == 3584 && S_SITE == 4608 && S_META == 5632,
+                "column offsets / byte counts below are for 256-record pieces");
+  if (NA && NG) {
+    asm volatile(
+        "{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\n"
+        "@p mbarrier.arrive.expect_tx.shared::cta.b64 _, [%1], 5888;\n"
+        CADV_CP(0, "%2", 2048) CADV_CP(2048, "%3", 1024) CADV_CP(3072, "%4", 512) CADV_CP(3584, "%5", 1024)
+        CADV_CP(4608, "%6", 1024) CADV_CP(5632, "%7", 256) "}" ::"r"(dst), "r"(bar), "l"(A.addr + q0),
+        "l"(A.cta + q0), "l"(A.tid + q0), "l"(A.winst + q0), "l"(A.site + q0), "l"(A.meta + q0)
+        : "memory");
+  } else if (NA) {
+    asm volatile(
+        "{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\n"
+        "@p mbarrier.arrive.expect_tx.shared::cta.b64 _, [%1], 3328;\n"
+        CADV_CP(0, "%2", 2048) CADV_CP(2048, "%3", 1024) CADV_CP(5632, "%4", 256) "}" ::"r"(dst), "r"(bar),
+        "l"(A.addr + q0), "l"(A.cta + q0), "l"(A.meta + q0)
+        : "memory");
+  } else {
+    asm volatile(
+        "{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\n"
+        "@p mbarrier.arrive.expect_tx.shared::cta.b64 _, [%1], 3840;\n"
+        CADV_CP(2048, "%2", 1024) CADV_CP(3072, "%3", 512) CADV_CP(3584, "%4", 1024) CADV_CP(4608, "%5", 1024)
+        CADV_CP(5632, "%6", 256) "}" ::"r"(dst), "r"(bar), "l"(A.cta + q0), "l"(A.tid + q0), "l"(A.winst + q0),
+        "l"(A.site + q0), "l"(A.meta + q0)
+        : "memory");
+  }
+}
+#undef CADV_CP
 template <int F>
 __device__ __forceinline__ void bulk_cp(uint32_t dst, const void* src, uint32_t bytes, uint32_t bar) {
   asm volatile(
@@ -179,35 +215,34 @@ __device__ __forceinline__ void bulk_cp(uint32_t dst, const void* src, uint32_t 
       "l"(src), "r"(bytes), "r"(bar)
       : "memory");
 }
+// the partial last piece of a stream: sizes rounded up to 16 bytes (sources stay in the padded columns)
 template <int F>
-__device__ __forceinline__ void issue_piece(const ScanArgs& A, uint32_t ring, uint32_t bar0, uint64_t c_lo,
-                                            uint64_t s_end, uint32_t p) {
+__device__ __noinline__ void issue_partial(const ScanArgs& A, uint32_t dst, uint32_t bar, uint64_t q0, uint32_t cnt) {
   constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
-  constexpr uint32_t FULL_BYTES = KR * (4 + 1 + (NA ? 8 : 0) + (NG ? 2 + 4 + 4 : 0));
-  const uint32_t stg = p % KS, bar = bar0 + stg * 8;
-  const uint64_t q0 = c_lo + (uint64_t)p * KR;
-  const bool full = q0 + KR <= s_end;
-  const uint32_t cnt = full ? (uint32_t)KR : (uint32_t)(s_end - q0);
-  // partial last piece: sizes rounded up to 16 bytes (sources stay in the padded columns)
   auto r16 = [](uint32_t b_) { return (b_ + 15u) & ~15u; };
-  uint32_t bytes = FULL_BYTES;
-  if (!full) {
-    bytes = r16(cnt * 4) + r16(cnt);
-    if (NA) bytes += r16(cnt * 8);
-    if (NG) bytes += r16(cnt * 2) + 2 * r16(cnt * 4);
-  }
+  uint32_t bytes = r16(cnt * 4) + r16(cnt);
+  if (NA) bytes += r16(cnt * 8);
+  if (NG) bytes += r16(cnt * 2) + 2 * r16(cnt * 4);
   asm volatile(
       "{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\n@p mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;\n}" ::"r"(bar),
       "r"(bytes)
       : "memory");
-  if (NA) bulk_cp<F>(ring + R_ADDR + stg * KR * 8, A.addr + q0, r16(cnt * 8), bar);
-  bulk_cp<F>(ring + R_CTA + stg * KR * 4, A.cta + q0, r16(cnt * 4), bar);
+  if (NA) bulk_cp<F>(dst + S_ADDR, A.addr + q0, r16(cnt * 8), bar);
+  bulk_cp<F>(dst + S_CTA, A.cta + q0, r16(cnt * 4), bar);
   if (NG) {
-    bulk_cp<F>(ring + R_TID + stg * KR * 2, A.tid + q0, r16(cnt * 2), bar);
-    bulk_cp<F>(ring + R_WINST + stg * KR * 4, A.winst + q0, r16(cnt * 4), bar);
-    bulk_cp<F>(ring + R_SITE + stg * KR * 4, A.site + q0, r16(cnt * 4), bar);
+    bulk_cp<F>(dst + S_TID, A.tid + q0, r16(cnt * 2), bar);
+    bulk_cp<F>(dst + S_WINST, A.winst + q0, r16(cnt * 4), bar);
+    bulk_cp<F>(dst + S_SITE, A.site + q0, r16(cnt * 4), bar);
   }
-  bulk_cp<F>(ring + R_META + stg * KR, A.meta + q0, r16(cnt), bar);
+  bulk_cp<F>(dst + S_META, A.meta + q0, r16(cnt), bar);
+}
+template <int F>
+__device__ __forceinline__ void issue_piece(const ScanArgs& A, uint32_t ring, uint32_t bar0, uint64_t c_lo,
+                                            uint64_t s_end, uint32_t p) {
+  const uint32_t stg = p % KS, bar = bar0 + stg * 8, dst = ring + stg * STG_BYTES;
+  const uint64_t q0 = c_lo + (uint64_t)p * KR;
+  if (q0 + KR <= s_end) issue_full<F>(A, dst, bar, q0);
+  else issue_partial<F>(A, dst, bar, q0, (uint32_t)(s_end - q0));
 }
 
 // run identity: (cta, warp32, winst, family)
@@ -258,14 +293,6 @@ __device__ __forceinline__ void finish_bd(const ScanArgs& A, const Counters& C, 
   }
 }
 
-struct RingView {
-  const uint64_t* addr;
-  const uint32_t* cta;
-  const uint16_t* tid;
-  const uint32_t* winst;
-  const uint32_t* site;
-  const uint8_t* meta;
-};
 
 // Exact resolution of one run [j0, j0 + nrec) read back from the ring: every
 // sub-warp group's distinct lines (MD) / lanes (BD) by pairwise comparison.
@@ -314,10 +341,12 @@ constexpr uint32_t PK_CNT = 10, PK_VIOL = 20, PK_M = 1023;
 // Finalizes the queued complete runs (one per lane, the warp converged).  A
 // run is one warp32 instruction of one CTA: with W = 32 it is the group, and
 // when its lines never decrease (viol = 0) deg = the number of line changes.
-// Entries are self-contained (run start j, aggregate u, lane bits m, kind |
-// tid, CTA and site of the first record), so flushes are batched across steps.
+// Entries are self-contained (run start j, aggregate u, lane bits m), so
+// flushes are batched across steps; the kind, tid, CTA and site of a run's
+// first record are read back from global memory (streamed moments ago, an L2
+// hit), which keeps the queue at 3 words per run and the carried run stateless.
 struct RunQueue {
-  uint32_t *j, *u, *m, *kt, *cta, *site;
+  uint32_t *j, *u, *m;
 };
 
 template <int F>
@@ -334,11 +363,11 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
       j = Q.j[q];
       u = Q.u[q];
       m = Q.m[q];
-      const uint32_t kt = Q.kt[q];
-      kind = kt >> 16;
-      t = kt & 0xffffu;
-      cta = Q.cta[q];
-      s = Q.site[q];
+      const uint64_t g = c_lo + j;
+      kind = __ldg(A.meta + g) & 3u;
+      t = __ldg(A.tid + g);
+      cta = __ldg(A.cta + g);
+      s = A.nsites ? __ldg(A.site + g) : 0u;
     const bool bb = kind == 2u;
       if (bb ? BD : MD) {
         const uint32_t cnt = (u >> PK_CNT) & PK_M;
@@ -393,16 +422,26 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
 }
 
 // Segmented suffix scans: lane l gets the sum (OR) of lanes l .. h, h the
-// first lane >= l whose head flag is set (h = 31 if none).
+// first lane >= l whose head flag is set (h = 31 if none).  The head flag
+// rides in bit 31 of the sum (v < 2^30: adding a lane's packed value to one
+// without the flag copies that lane's flag); lane 31 always stops a segment,
+// so no lane ever reads past it.
 __device__ __forceinline__ void seg_scan2(uint32_t& v, uint32_t& m, uint32_t head) {
-  const uint32_t lane = lane_id();
-  uint32_t h = head;
+  uint32_t x = v | ((head || lane_id() == 31u) ? 0x80000000u : 0u);
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
-    const uint32_t vo = __shfl_down_sync(FULL, v, d), mo = __shfl_down_sync(FULL, m, d),
-                   ho = __shfl_down_sync(FULL, h, d);
-    if (lane + d < 32 && !h) { v += vo; m |= mo; h = ho; }
+    const uint32_t xo = __shfl_down_sync(FULL, x, d), mo = __shfl_down_sync(FULL, m, d);
+    if (!(x >> 31)) { x += xo; m |= mo; }
   }
+  v = x & 0x7fffffffu;
+}
+
+// r[k] for a lane-varying k < 8 (a 3-level select tree instead of local memory)
+__device__ __forceinline__ uint32_t sel8(const uint32_t (&r)[8], uint32_t k) {
+  const bool b0 = k & 1u, b1 = k & 2u, b2 = k & 4u;
+  const uint32_t x01 = b0 ? r[1] : r[0], x23 = b0 ? r[3] : r[2];
+  const uint32_t x45 = b0 ? r[5] : r[4], x67 = b0 ? r[7] : r[6];
+  return b2 ? (b1 ? x67 : x45) : (b1 ? x23 : x01);
 }
 
 template <int F>
@@ -420,7 +459,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   const bool sites_smem = A.nsites && A.nsites <= NSITE_SMEM;
   // F_OBJ tables after the run queues (scan_smem)
   uint8_t* objm = smem + NWARP * R_BYTES + ((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + NWARP * 68 * 4 +
-                  NWARP * (QCAP * 24 + 16);
+                  NWARP * (QCAP * 12);
   const bool obj_sm = OBJ && A.nobj < OBJ_SMEM;
   uint64_t* s_olo = (uint64_t*)objm;
   uint64_t* s_ohi = s_olo + OBJ_SMEM;
@@ -441,9 +480,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   if (sites_smem)
     for (uint32_t k = tx; k < (uint32_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM; k += NTHR) sites[k] = 0;
   uint32_t* whist = wh_all + warp * 68;  // warp-private MD histogram [2][33]
-  uint32_t* qbase = wh_all + NWARP * 68 + warp * (QCAP * 6 + 4);
-  const RunQueue Q{qbase, qbase + QCAP, qbase + 2 * QCAP, qbase + 3 * QCAP, qbase + 4 * QCAP, qbase + 5 * QCAP};
-  uint32_t* qc = qbase + 6 * QCAP;  // the carried run's first record: kind << 16 | tid, cta, site
+  uint32_t* qbase = wh_all + NWARP * 68 + warp * (QCAP * 3);
+  const RunQueue Q{qbase, qbase + QCAP, qbase + 2 * QCAP};
   for (uint32_t k = lane; k < 68; k += 32) whist[k] = 0;
   __syncthreads();
 
@@ -478,9 +516,6 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     const uint32_t ring_s = smem_u32(ring), bar_s = smem_u32(bar);
     uint32_t issued = npieces < (uint32_t)KS ? npieces : (uint32_t)KS, waited = 0;
     for (uint32_t p = 0; p < issued; ++p) issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, p);
-    const RingView R{(const uint64_t*)(ring + R_ADDR), (const uint32_t*)(ring + R_CTA),
-                     (const uint16_t*)(ring + R_TID),  (const uint32_t*)(ring + R_WINST),
-                     (const uint32_t*)(ring + R_SITE), ring + R_META};
     // the record before the step (warp-uniform); meta 3 = "no record"
     // p_kb: kind bits of that record (bit 0 memory, 1 store, 2 BB; 0 = invalid / none)
     uint32_t p_cta = 0xffffffffu, p_t = 0, p_kb = 0, p_winst = 0;
@@ -517,21 +552,29 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       waited = p + 1;
       // ---- this lane's LPR consecutive records (vector shared-memory loads)
       const uint32_t j0 = base + lane * LPR;
-      const uint32_t sl = ring_slot(j0);
+      // this step's stage in the ring; the lane's records start at slot lane * LPR
+      const uint8_t* stg = ring + stage_off(base);
+      const uint32_t sl = lane * LPR;
+      const uint64_t* r_addr = (const uint64_t*)(stg + S_ADDR);
+      const uint32_t* r_cta = (const uint32_t*)(stg + S_CTA);
+      const uint16_t* r_tid = (const uint16_t*)(stg + S_TID);
+      const uint32_t* r_winst = (const uint32_t*)(stg + S_WINST);
+      const uint32_t* r_site = (const uint32_t*)(stg + S_SITE);
+      const uint8_t* r_meta = stg + S_META;
       uint32_t c[LPR], t[LPR], w[LPR], mmx, mmy, tor = 0;
       uint64_t a[LPR];
       {
-        const uint4 c0 = *(const uint4*)(R.cta + sl), c1 = *(const uint4*)(R.cta + sl + 4);
+        const uint4 c0 = *(const uint4*)(r_cta + sl), c1 = *(const uint4*)(r_cta + sl + 4);
         c[0] = c0.x; c[1] = c0.y; c[2] = c0.z; c[3] = c0.w; c[4] = c1.x; c[5] = c1.y; c[6] = c1.z; c[7] = c1.w;
-        const uint2 mm = *(const uint2*)(R.meta + sl);
+        const uint2 mm = *(const uint2*)(r_meta + sl);
         mmx = mm.x;
         mmy = mm.y;
         if (NG) {
-          const uint4 t4 = *(const uint4*)(R.tid + sl);
+          const uint4 t4 = *(const uint4*)(r_tid + sl);
           tor = t4.x | t4.y | t4.z | t4.w;
           t[0] = t4.x & 0xffffu; t[1] = t4.x >> 16; t[2] = t4.y & 0xffffu; t[3] = t4.y >> 16;
           t[4] = t4.z & 0xffffu; t[5] = t4.z >> 16; t[6] = t4.w & 0xffffu; t[7] = t4.w >> 16;
-          const uint4 w0 = *(const uint4*)(R.winst + sl), w1 = *(const uint4*)(R.winst + sl + 4);
+          const uint4 w0 = *(const uint4*)(r_winst + sl), w1 = *(const uint4*)(r_winst + sl + 4);
           w[0] = w0.x; w[1] = w0.y; w[2] = w0.z; w[3] = w0.w; w[4] = w1.x; w[5] = w1.y; w[6] = w1.z; w[7] = w1.w;
         } else {
 #pragma unroll
@@ -540,7 +583,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         if (NA) {
 #pragma unroll
           for (int q = 0; q < LPR / 2; ++q) {
-            const uint4 v = *(const uint4*)(R.addr + sl + 2 * q);
+            const uint4 v = *(const uint4*)(r_addr + sl + 2 * q);
             a[2 * q] = ((uint64_t)v.y << 32) | v.x;
             a[2 * q + 1] = ((uint64_t)v.w << 32) | v.z;
           }
@@ -556,28 +599,32 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       const uint32_t glo = gather8(mmx, mmy), ghi = gather8(mmx >> 1, mmy >> 1);
       uint32_t okm = inbm;
       {
-        // validation: SWAR checks over the lane's records, exact per record only if one fails
-        uint32_t badm = 0;
+        // validation trigger: SWAR over the lane's records, 4 per meta word (byte
+        // permutes gather the low address byte / the address's top byte of 4
+        // records); a superset of the bad records (it may also fire on records
+        // past the chunk) - the exact per-record check below decides
+        uint32_t trig = 0;
 #pragma unroll
         for (int h = 0; h < 2; ++h) {
-          const uint32_t v = h ? mmy : mmx;
-          const uint32_t lo = v & 0x01010101u, hi = (v >> 1) & 0x01010101u;
-          const uint32_t b = (lo & hi) | (((v >> 5) | (v >> 6) | (v >> 7)) & 0x01010101u) |  // kind 3, reserved bits
-                             ((v >> 4) & ((v >> 3) | (v >> 2)) & ~hi & 0x01010101u);        // memory size > 16 B
-          badm |= gather4(b) << (4 * h);
-        }
-        uint32_t abad = 0;  // memory records: address bits below the access size, or >= 2^58 (lane-level)
-        if (NA) {
-          const uint32_t memk = ~ghi & ownm;
-#pragma unroll
-          for (int k = 0; k < LPR; ++k) {
-            const uint32_t msk = (1u << ((((k < 4 ? mmx : mmy) >> (8 * (k & 3))) >> 2) & 7u)) - 1u;
-            const uint32_t v = ((uint32_t)a[k] & msk) | ((uint32_t)(a[k] >> 32) & 0xfc000000u);
-            abad |= (memk >> k) & 1u ? v : 0u;
+          const uint32_t v = h ? mmy : mmx, v1 = v >> 1;
+          const uint32_t K = (~v1 & 0x01010101u) * 0xffu;  // memory records (kind bit 1 clear)
+          const uint32_t S = (v >> 2) & 0x07070707u;        // log2(bytes)
+          // (1 << log2(bytes)) - 1 per memory record (bit 4 set iff more than 16 bytes)
+          const uint32_t M = __byte_perm(0x07030100u, 0x7f3f1f0fu, __byte_perm(S | (S >> 4), 0u, 0x0020u)) & K;
+          trig |= (v & 0xe0e0e0e0u) | (v & v1 & 0x01010101u);  // reserved bits, kind 3
+          if (NA) {
+            const int i = 4 * h;
+            const uint32_t L = __byte_perm(__byte_perm((uint32_t)a[i], (uint32_t)a[i + 1], 0x0040u),
+                                           __byte_perm((uint32_t)a[i + 2], (uint32_t)a[i + 3], 0x0040u), 0x5410u);
+            const uint32_t H = __byte_perm(__byte_perm((uint32_t)(a[i] >> 32), (uint32_t)(a[i + 1] >> 32), 0x0073u),
+                                           __byte_perm((uint32_t)(a[i + 2] >> 32), (uint32_t)(a[i + 3] >> 32), 0x0073u),
+                                           0x5410u);
+            trig |= ((L | 0x10101010u) & M) | (H & K & 0xfcfcfcfcu);  // misaligned / > 16 B, address >= 2^58
+          } else {
+            trig |= M & 0x10101010u;
           }
         }
-        badm &= ownm;
-        if (__any_sync(FULL, (badm | abad) != 0 || (NG && (tor & 0xfc00fc00u)))) {
+        if (__any_sync(FULL, trig != 0 || (NG && (tor & 0xfc00fc00u)))) {
 #pragma unroll
           for (int k = 0; k < LPR; ++k) {
             if (!((ownm >> k) & 1u)) continue;
@@ -740,9 +787,6 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
                 Q.j[qn] = cr_j;
                 Q.u[qn] = cr_v;
                 Q.m[qn] = cr_mask;
-                Q.kt[qn] = qc[0];
-                Q.cta[qn] = qc[1];
-                Q.site[qn] = qc[2];
               }
               ++qn;
             }
@@ -755,34 +799,24 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         const uint32_t starts = rsm & inbm;
         const bool tail_open = !above && ((starts >> lastk) & 1u);  // continues past the step end
         const uint32_t todo = starts & ownm & ~(tail_open ? 1u << lastk : 0u);
-#pragma unroll
-        for (int k = 0; k < LPR; ++k) {
-          const bool it = (todo >> k) & 1u;
-          const uint32_t im = __ballot_sync(FULL, it);
-          if (im) {
-            if (it) {
-              const uint32_t nxt = rsm & (0xfeu << k) & 0xffu;
-              const uint32_t seg = (nxt ? (nxt & (0u - nxt)) - 1u : 0xffu) & (0xffu << k);
-              uint32_t u2 = __popc(nlm & seg) | (__popc(seg) << PK_CNT) | (__popc(vim & seg) << PK_VIOL);
-              uint32_t m2 = rm[k];
-              if ((uint32_t)k == lastk) { u2 += S_next; m2 |= M_next; }  // closed by a later lane's head
-              const uint32_t pos = qn + __popc(im & lanemask_lt());
-              Q.j[pos] = j0 + k;
-              Q.u[pos] = u2;
-              Q.m[pos] = m2;
-              Q.kt[pos] = ((((k < 4 ? mmx : mmy) >> (8 * (k & 3))) & 3u) << 16) | t[k];
-              Q.cta[pos] = c[k];
-              Q.site[pos] = A.nsites ? R.site[ring_slot(j0 + k)] : 0u;
-            }
-            qn += __popc(im);
+        // rounds over the lanes' run starts (one per lane per round; usually one round)
+        for (uint32_t td = todo;;) {
+          const uint32_t bm = __ballot_sync(FULL, td != 0);
+          if (!bm) break;
+          if (td) {
+            const uint32_t k = __ffs(td) - 1;
+            td &= td - 1;
+            const uint32_t nxt = rsm & (0xfeu << k) & 0xffu;
+            const uint32_t seg = (nxt ? (nxt & (0u - nxt)) - 1u : 0xffu) & (0xffu << k);
+            uint32_t u2 = __popc(nlm & seg) | (__popc(seg) << PK_CNT) | (__popc(vim & seg) << PK_VIOL);
+            uint32_t m2 = sel8(rm, k);
+            if (k == lastk) { u2 += S_next; m2 |= M_next; }  // closed by a later lane's head
+            const uint32_t pos = qn + __popc(bm & lanemask_lt());
+            Q.j[pos] = j0 + k;
+            Q.u[pos] = u2;
+            Q.m[pos] = m2;
           }
-          // flushes are batched (>= 32 runs), always leaving room for half a step
-          if (k == LPR / 2 - 1 && qn > QCAP - 32 * LPR / 2 - 1) {
-            __syncwarp();
-            flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
-            qn = 0;
-            __syncwarp();
-          }
+          qn += __popc(bm);
         }
         if (qn >= 32) {
           __syncwarp();
@@ -796,19 +830,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           if (tail_open) {
             const uint32_t msk = 0xffu << lastk;
             tu = __popc(nlm & msk) | ((LPR - lastk) << PK_CNT) | (__popc(vim & msk) << PK_VIOL);
-            {  // rm[lastk] by a 3-level select on the bits of lastk
-              const bool b0 = lastk & 1u, b1 = lastk & 2u, b2 = lastk & 4u;
-              const uint32_t x01 = b0 ? rm[1] : rm[0], x23 = b0 ? rm[3] : rm[2];
-              const uint32_t x45 = b0 ? rm[5] : rm[4], x67 = b0 ? rm[7] : rm[6];
-              tmk = b2 ? (b1 ? x67 : x45) : (b1 ? x23 : x01);
-            }
+            tmk = sel8(rm, lastk);
             if (lane < 31) { tu += S_next; tmk |= M_next; }
-            {  // the carried run's first record (its piece is recycled before the run closes)
-              const uint32_t sl0 = ring_slot(j0 + lastk);
-              qc[0] = ((R.meta[sl0] & 3u) << 16) | R.tid[sl0];
-              qc[1] = R.cta[sl0];
-              qc[2] = A.nsites ? R.site[sl0] : 0u;
-            }
           }
           cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
           cr_v = __shfl_sync(FULL, tu, hl);
@@ -833,9 +856,6 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         Q.j[qn] = cr_j;
         Q.u[qn] = cr_v;
         Q.m[qn] = cr_mask;
-        Q.kt[qn] = qc[0];
-        Q.cta[qn] = qc[1];
-        Q.site[qn] = qc[2];
       }
       ++qn;
     }
@@ -954,7 +974,7 @@ template <int F>
 size_t scan_smem() {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0, OBJ = (F & F_OBJ) != 0;
   return (size_t)NWARP * R_BYTES + (size_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + (size_t)NWARP * 68 * 4 +
-         (size_t)NWARP * (QCAP * 24 + 16) + (OBJ ? (size_t)OBJ_SMEM * (16 + 4 + (MD ? 66 * 4 : 0)) : 0);
+         (size_t)NWARP * (QCAP * 12) + (OBJ ? (size_t)OBJ_SMEM * (16 + 4 + (MD ? 66 * 4 : 0)) : 0);
 }
 
 int g_scan_ready[16] = {0};
