@@ -40,10 +40,10 @@ namespace {
 constexpr int LPR = 8;                 // consecutive records per lane in one warp step
 constexpr int KR = 32 * LPR;           // records per piece = one warp step
 constexpr int KS = 2;                  // ring stages per warp (piece p and piece p + 1 in flight)
-constexpr int NWARP = 12;              // warps per CTA (one CTA per SM; 3 per SM sub-partition)
+constexpr int NWARP = 16;              // warps per CTA (one CTA per SM; 4 per SM sub-partition)
 constexpr int NTHR = NWARP * 32;
 constexpr int NSITE_SMEM = 512;        // per-site counters kept in shared memory up to this many sites
-constexpr int QCAP = 288;              // per-warp queue of complete runs awaiting finalization (31 + 1 + KR)
+constexpr int QCAP = 64;               // per-warp queue of complete runs awaiting finalization (31 + 1 + 32)
 constexpr int OBJ_SMEM = 64;           // F_OBJ: object rows (objects + 1) kept in shared memory up to this many
 
 // per-warp ring, stage-major: stage s occupies [s * STG_BYTES, (s + 1) * STG_BYTES)
@@ -803,6 +803,12 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         for (uint32_t td = todo;;) {
           const uint32_t bm = __ballot_sync(FULL, td != 0);
           if (!bm) break;
+          if (qn >= 32) {  // room for one more round (QCAP >= 31 + 1 + 32)
+            __syncwarp();
+            flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
+            qn = 0;
+            __syncwarp();
+          }
           if (td) {
             const uint32_t k = __ffs(td) - 1;
             td &= td - 1;
