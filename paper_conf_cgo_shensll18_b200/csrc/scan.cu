@@ -43,7 +43,10 @@ constexpr int KS = 2;                  // ring stages per warp (piece p and piec
 constexpr int NWARP = 16;              // warps per CTA (one CTA per SM; 4 per SM sub-partition)
 constexpr int NTHR = NWARP * 32;
 constexpr int NSITE_SMEM = 512;        // per-site counters kept in shared memory up to this many sites
-constexpr int QCAP = 64;               // per-warp queue of complete runs awaiting finalization (31 + 1 + 32)
+// per-warp queue of complete runs awaiting finalization: a round of enqueues
+// (<= 32) starts with at most QCAP - 32 entries queued
+template <int F>
+constexpr int qcap() { return (F & F_OBJ) ? 40 : 64; }
 constexpr int OBJ_SMEM = 64;           // F_OBJ: object rows (objects + 1) kept in shared memory up to this many
 
 // per-warp ring, stage-major: stage s occupies [s * STG_BYTES, (s + 1) * STG_BYTES)
@@ -341,17 +344,25 @@ constexpr uint32_t PK_CNT = 10, PK_VIOL = 20, PK_M = 1023;
 // Finalizes the queued complete runs (one per lane, the warp converged).  A
 // run is one warp32 instruction of one CTA: with W = 32 it is the group, and
 // when its lines never decrease (viol = 0) deg = the number of line changes.
-// Entries are self-contained (run start j, aggregate u, lane bits m), so
-// flushes are batched across steps; the kind, tid, CTA and site of a run's
-// first record are read back from global memory (streamed moments ago, an L2
-// hit), which keeps the queue at 3 words per run and the carried run stateless.
-struct RunQueue {
-  uint32_t *j, *u, *m;
+// Entries are self-contained (run start j, aggregate u, lane bits m, kind |
+// tid, CTA and site of the first record, copied from the ring when queued),
+// so flushes are batched across steps.
+template <int F>
+struct RunQueue {  // six columns of QCAP words from one base (one live register)
+  uint32_t* b;
+  static constexpr uint32_t C = qcap<F>();
+  __device__ __forceinline__ uint32_t& j(uint32_t i) const { return b[i]; }
+  __device__ __forceinline__ uint32_t& u(uint32_t i) const { return b[C + i]; }
+  __device__ __forceinline__ uint32_t& m(uint32_t i) const { return b[2 * C + i]; }
+  __device__ __forceinline__ uint32_t& kt(uint32_t i) const { return b[3 * C + i]; }
+  __device__ __forceinline__ uint32_t& cta(uint32_t i) const { return b[4 * C + i]; }
+  __device__ __forceinline__ uint32_t& site(uint32_t i) const { return b[5 * C + i]; }
+  __device__ __forceinline__ uint32_t* carry() const { return b + 6 * C; }  // the carried run's first record
 };
 
 template <int F>
 __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
-                                        const RunQueue Q, uint32_t qn, uint64_t c_lo) {
+                                        const RunQueue<F> Q, uint32_t qn, uint64_t c_lo) {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   const uint32_t lane = lane_id();
   uint32_t exec = 0, thr = 0, mxc = 0;
@@ -360,14 +371,14 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
     bool md = false, bd = false;
     uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0;
     if (q < qn) {
-      j = Q.j[q];
-      u = Q.u[q];
-      m = Q.m[q];
-      const uint64_t g = c_lo + j;
-      kind = __ldg(A.meta + g) & 3u;
-      t = __ldg(A.tid + g);
-      cta = __ldg(A.cta + g);
-      s = A.nsites ? __ldg(A.site + g) : 0u;
+      j = Q.j(q);
+      u = Q.u(q);
+      m = Q.m(q);
+      const uint32_t kt = Q.kt(q);
+      kind = kt >> 16;
+      t = kt & 0xffffu;
+      cta = Q.cta(q);
+      s = Q.site(q);
     const bool bb = kind == 2u;
       if (bb ? BD : MD) {
         const uint32_t cnt = (u >> PK_CNT) & PK_M;
@@ -459,7 +470,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   const bool sites_smem = A.nsites && A.nsites <= NSITE_SMEM;
   // F_OBJ tables after the run queues (scan_smem)
   uint8_t* objm = smem + NWARP * R_BYTES + ((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + NWARP * 68 * 4 +
-                  NWARP * (QCAP * 12);
+                  NWARP * (qcap<F>() * 24 + 16);
   const bool obj_sm = OBJ && A.nobj < OBJ_SMEM;
   uint64_t* s_olo = (uint64_t*)objm;
   uint64_t* s_ohi = s_olo + OBJ_SMEM;
@@ -480,8 +491,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   if (sites_smem)
     for (uint32_t k = tx; k < (uint32_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM; k += NTHR) sites[k] = 0;
   uint32_t* whist = wh_all + warp * 68;  // warp-private MD histogram [2][33]
-  uint32_t* qbase = wh_all + NWARP * 68 + warp * (QCAP * 3);
-  const RunQueue Q{qbase, qbase + QCAP, qbase + 2 * QCAP};
+  constexpr uint32_t QCAP = qcap<F>();
+  const RunQueue<F> Q{wh_all + NWARP * 68 + warp * (QCAP * 6 + 4)};
   for (uint32_t k = lane; k < 68; k += 32) whist[k] = 0;
   __syncthreads();
 
@@ -784,9 +795,12 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           if (heads) {
             if (cr_own) {
               if (lane == 0) {
-                Q.j[qn] = cr_j;
-                Q.u[qn] = cr_v;
-                Q.m[qn] = cr_mask;
+                Q.j(qn) = cr_j;
+                Q.u(qn) = cr_v;
+                Q.m(qn) = cr_mask;
+                Q.kt(qn) = Q.carry()[0];
+                Q.cta(qn) = Q.carry()[1];
+                Q.site(qn) = Q.carry()[2];
               }
               ++qn;
             }
@@ -803,7 +817,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         for (uint32_t td = todo;;) {
           const uint32_t bm = __ballot_sync(FULL, td != 0);
           if (!bm) break;
-          if (qn >= 32) {  // room for one more round (QCAP >= 31 + 1 + 32)
+          if (qn > QCAP - 32) {  // room for one more round
             __syncwarp();
             flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
             qn = 0;
@@ -818,9 +832,12 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             uint32_t m2 = sel8(rm, k);
             if (k == lastk) { u2 += S_next; m2 |= M_next; }  // closed by a later lane's head
             const uint32_t pos = qn + __popc(bm & lanemask_lt());
-            Q.j[pos] = j0 + k;
-            Q.u[pos] = u2;
-            Q.m[pos] = m2;
+            Q.j(pos) = j0 + k;
+            Q.u(pos) = u2;
+            Q.m(pos) = m2;
+            Q.kt(pos) = ((r_meta[sl + k] & 3u) << 16) | r_tid[sl + k];
+            Q.cta(pos) = r_cta[sl + k];
+            Q.site(pos) = A.nsites ? r_site[sl + k] : 0u;
           }
           qn += __popc(bm);
         }
@@ -838,6 +855,11 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             tu = __popc(nlm & msk) | ((LPR - lastk) << PK_CNT) | (__popc(vim & msk) << PK_VIOL);
             tmk = sel8(rm, lastk);
             if (lane < 31) { tu += S_next; tmk |= M_next; }
+            // the carried run's first record (its stage is recycled before the run closes)
+            const uint32_t sl0 = sl + lastk;
+            Q.carry()[0] = ((r_meta[sl0] & 3u) << 16) | r_tid[sl0];
+            Q.carry()[1] = r_cta[sl0];
+            Q.carry()[2] = A.nsites ? r_site[sl0] : 0u;
           }
           cr_on = __shfl_sync(FULL, (uint32_t)tail_open, hl) != 0;
           cr_v = __shfl_sync(FULL, tu, hl);
@@ -859,9 +881,12 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     // a run open at the end of the stream ends with the trace; then the rest of the queue
     if (NG && cr_on && cr_own) {
       if (lane == 0) {
-        Q.j[qn] = cr_j;
-        Q.u[qn] = cr_v;
-        Q.m[qn] = cr_mask;
+        Q.j(qn) = cr_j;
+        Q.u(qn) = cr_v;
+        Q.m(qn) = cr_mask;
+        Q.kt(qn) = Q.carry()[0];
+        Q.cta(qn) = Q.carry()[1];
+        Q.site(qn) = Q.carry()[2];
       }
       ++qn;
     }
@@ -980,7 +1005,7 @@ template <int F>
 size_t scan_smem() {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0, OBJ = (F & F_OBJ) != 0;
   return (size_t)NWARP * R_BYTES + (size_t)((MD ? 2 : 0) + (BD ? 3 : 0)) * NSITE_SMEM * 4 + (size_t)NWARP * 68 * 4 +
-         (size_t)NWARP * (QCAP * 12) + (OBJ ? (size_t)OBJ_SMEM * (16 + 4 + (MD ? 66 * 4 : 0)) : 0);
+         (size_t)NWARP * (qcap<F>() * 24 + 16) + (OBJ ? (size_t)OBJ_SMEM * (16 + 4 + (MD ? 66 * 4 : 0)) : 0);
 }
 
 int g_scan_ready[16] = {0};
