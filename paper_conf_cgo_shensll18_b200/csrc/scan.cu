@@ -248,6 +248,19 @@ __device__ __forceinline__ void issue_piece(const ScanArgs& A, uint32_t ring, ui
   else issue_partial<F>(A, dst, bar, q0, (uint32_t)(s_end - q0));
 }
 
+// shared-memory re-reads of ring values (asm: not folded into the registers
+// that held them, which are dead by then)
+__device__ __forceinline__ uint64_t lds_u64(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(smem_u32(p)));
+  return v;
+}
+__device__ __forceinline__ uint32_t lds_u32(const uint32_t* p) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)));
+  return v;
+}
+
 // run identity: (cta, warp32, winst, family)
 __device__ __forceinline__ uint32_t run_hi(uint32_t tid, uint32_t meta) {
   return (tid >> 5) | (((meta & 3u) == 2u) ? 64u : 0u);
@@ -659,23 +672,45 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       uint64_t pa = NA ? __shfl_up_sync(FULL, a[LPR - 1], 1) : 0ull;
       if (lane == 0) { pc = p_cta; pkb = p_kb; pt = p_t; pwi = p_winst; pa = p_addr; }
 
+      // ---- every comparison with the predecessor first, so that the record
+      //      registers die here (kept-record writes below re-read the ring)
+      // RD  eqm: same (scope, line) as the predecessor (32-bit halves, line bits only, lbs <= 12)
+      // NG  rsm: run starts ((cta, winst, warp32) differ); nlm: MD line changes; vim: line decreases
+      uint32_t eqm = 0, rsm = 0, nlm = 0, vim = 0;
+      uint64_t tl5 = 0;  // NG: the records' lanes, 5 bits each
+      {
+        const uint32_t mlr = ~((1u << A.lbs_rd) - 1u), msc = A.cta_scope ? 0xffffffffu : 0u;
+        const uint32_t mlm = ~((1u << A.lbs_md) - 1u);
+#pragma unroll
+        for (int k = 0; k < LPR; ++k) {
+          const uint64_t qa = k == 0 ? pa : a[k - 1];
+          const uint32_t qc = k == 0 ? pc : c[k - 1];
+          const uint32_t dlo = (uint32_t)a[k] ^ (uint32_t)qa, dhi = (uint32_t)(a[k] >> 32) ^ (uint32_t)(qa >> 32);
+          if (RD) eqm |= (uint32_t)(((dlo & mlr) | dhi | ((c[k] ^ qc) & msc)) == 0u) << k;
+          if (NG) {
+            const uint32_t qw = k == 0 ? pwi : w[k - 1], qt = k == 0 ? pt : t[k - 1];
+            rsm |= (uint32_t)(((c[k] ^ qc) | (w[k] ^ qw) | ((t[k] ^ qt) & ~31u)) != 0u) << k;
+            if (MD) {
+              nlm |= (uint32_t)(((dlo & mlm) | dhi) != 0u) << k;
+              vim |= (uint32_t)(a[k] < qa) << k;  // only where the line changes (masked below)
+            }
+            tl5 |= (uint64_t)(t[k] & 31u) << (5 * k);
+          }
+        }
+      }
+      // ---- carry the step's last record to the next step
+      p_cta = __shfl_sync(FULL, c[LPR - 1], 31);
+      p_kb = __shfl_sync(FULL, ((memm >> 7) & 1u) | ((stm >> 6) & 2u) | ((bbm >> 5) & 4u), 31);
+      if (NG) p_t = __shfl_sync(FULL, t[LPR - 1], 31);
+      if (NG) p_winst = __shfl_sync(FULL, w[LPR - 1], 31);
+      if (NA) p_addr = __shfl_sync(FULL, a[LPR - 1], 31);
+
       // ================= R1: run compression of the chunk's records
       // dup  : a load repeating its predecessor's (scope, line): RD 0, never kept;
       // chain: consecutive stores to one (scope, line); every 16th one is kept
       //        with the weight of the chain piece it heads.  Chains are cut at
       //        step starts and at the chunk end (both only split a piece).
       if (RD) {
-        // same (scope, line) as the predecessor: 32-bit halves, line bits only (lbs <= 12)
-        uint32_t eqm = 0;
-        const uint32_t mlo = ~((1u << A.lbs_rd) - 1u), msc = A.cta_scope ? 0xffffffffu : 0u;
-#pragma unroll
-        for (int k = 0; k < LPR; ++k) {
-          const uint64_t q = k == 0 ? pa : a[k - 1];
-          const uint32_t qs = k == 0 ? pc : c[k - 1];
-          const uint32_t x = (((uint32_t)a[k] ^ (uint32_t)q) & mlo) | ((uint32_t)(a[k] >> 32) ^ (uint32_t)(q >> 32)) |
-                             ((c[k] ^ qs) & msc);
-          eqm |= (uint32_t)(x == 0u) << k;
-        }
         const uint32_t pm = ((memm << 1) | (pkb & 1u)) & 0xffu, ps = ((stm << 1) | ((pkb >> 1) & 1u)) & 0xffu;
         const uint32_t dupm = eqm & memm & ~stm & pm;
         const uint32_t contm = eqm & stm & ps & (lane == 0 ? 0xfeu : 0xffu);
@@ -717,9 +752,9 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           bool hd = nd;
           if (wgt > 16u) { wgt = 16u; hd = false; }      // the chain goes on with another kept store
           else last_open = nb == (uint32_t)KR;           // decided by the next step's first record
-          wbv[pos] = (a[k] >> A.lbs_rd) | ((uint64_t)((stm >> k) & 1u) << VB_STORE) | ((uint64_t)hd << VB_DUP) |
+          wbv[pos] = (lds_u64(r_addr + sl + k) >> A.lbs_rd) | ((uint64_t)((stm >> k) & 1u) << VB_STORE) | ((uint64_t)hd << VB_DUP) |
                      ((uint64_t)(wgt - 1u) << VB_W);
-          if (wbk) wbk[pos] = A.cta_scope ? c[k] : 0u;
+          if (wbk) wbk[pos] = A.cta_scope ? lds_u32(r_cta + sl + k) : 0u;
           ++pos;
         }
         open_rd = __ballot_sync(FULL, last_open) != 0;
@@ -730,7 +765,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
 #pragma unroll
             for (int k = 0; k < LPR; ++k) {
               if (!((dm >> k) & 1u)) continue;
-              const uint64_t ln = a[k] >> A.lbs_rd;
+              const uint64_t ln = lds_u64(r_addr + sl + k) >> A.lbs_rd;
               if (ln != dc_line) {
                 dc_flush();
                 dc_line = ln;
@@ -747,21 +782,6 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
 
       // ================= M1-M3 / B1-B3: runs = warp-level groups
       if (NG) {
-        uint32_t rsm = 0, nlm = 0, vim = 0, bits[LPR];
-        const uint32_t mlo = ~((1u << A.lbs_md) - 1u);
-#pragma unroll
-        for (int k = 0; k < LPR; ++k) {
-          const uint32_t qc = k == 0 ? pc : c[k - 1], qw = k == 0 ? pwi : w[k - 1], qt = k == 0 ? pt : t[k - 1];
-          const uint32_t x = (c[k] ^ qc) | (w[k] ^ qw) | ((t[k] ^ qt) & ~31u);  // (cta, winst, warp32) differ
-          rsm |= (uint32_t)(x != 0u) << k;
-          if (MD) {
-            const uint64_t qa = k == 0 ? pa : a[k - 1];
-            const uint32_t y = (((uint32_t)a[k] ^ (uint32_t)qa) & mlo) | ((uint32_t)(a[k] >> 32) ^ (uint32_t)(qa >> 32));
-            nlm |= (uint32_t)(y != 0u) << k;
-            vim |= (uint32_t)(a[k] < qa) << k;  // only where the line changes (masked below)
-          }
-          bits[k] = 1u << (t[k] & 31u);
-        }
         vim &= nlm;
         rsm |= (bbm ^ ((bbm << 1) | ((pkb >> 2) & 1u))) & 0xffu;  // BB and memory records never share a run
         rsm |= ~inbm & 0xffu;  // every record past the stream is a run of its own (never finalized)
@@ -772,7 +792,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         uint32_t m = 0;
 #pragma unroll
         for (int k = LPR - 1; k >= 0; --k) {
-          m |= bits[k];
+          m |= 1u << (tl5 >> (5 * k) & 31u);
           rm[k] = m;
           if ((rsm >> k) & 1u) m = 0;
         }
@@ -870,12 +890,6 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         }
         __syncwarp();
       }
-      // ---- carry the step's last record; recycle piece p - 1 for piece p + 2
-      p_cta = __shfl_sync(FULL, c[LPR - 1], 31);
-      p_kb = __shfl_sync(FULL, ((memm >> 7) & 1u) | ((stm >> 6) & 2u) | ((bbm >> 5) & 4u), 31);
-      if (NG) p_t = __shfl_sync(FULL, t[LPR - 1], 31);
-      if (NG) p_winst = __shfl_sync(FULL, w[LPR - 1], 31);
-      if (NA) p_addr = __shfl_sync(FULL, a[LPR - 1], 31);
       __syncwarp();
     }
     // a run open at the end of the stream ends with the trace; then the rest of the queue
