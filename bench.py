@@ -312,14 +312,19 @@ def main():
     # ---- warm-up (allocates the library workspace)
     for _ in range(max(args.warmup, 0)):
         step(dev)
-    # ---- timed region
-    ctx.set_profiling(True)
+    # ---- timed region (CUDA events around the streaming pass only: the
+    # dominant kernel's live duration without two event records per launch)
+    ctx.set_profiling(2)
     clocks = Clocks(local)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
     if not args.profile_run:
         clocks.start()
+    else:
+        # ncu --profile-from-start off: capture the timed steps only (not the
+        # warm-up, whose first call also sizes the workspace)
+        torch.cuda.profiler.start()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     e0.record(stream)
     launches, kt, stats = 0, [], None
@@ -332,6 +337,8 @@ def main():
     if world > 1:
         dist.barrier()
     ck = clocks.stop() if not args.profile_run else {}
+    if args.profile_run:
+        torch.cuda.profiler.stop()
     ctx.set_profiling(False)
     ms = e0.elapsed_time(e1)
     ms_max = ms
@@ -367,7 +374,23 @@ def main():
                     "traffic_source": "profiles/ncu_full_latest.csv (dram read+write bytes per launch, ncu --set full)",
                     "avg_launch_ms": round(avg_ms, 4), "algorithmic_bytes_per_launch": per,
                     "share_of_step": round(tot_ms / (ms * 1.0), 4)}
-    kernels = {k: {"launches": v[1], "total_ms": round(v[0], 3)} for k, v in sorted(agg.items(), key=lambda kv: -kv[1][0])}
+    # ---- per-kernel breakdown of the step: a separate, untimed pass with
+    # events around every launch
+    kernels = {}
+    if not args.profile_run:
+        ctx.set_profiling(1)
+        nb = max(1, min(args.steps, 3))
+        kall = {}
+        for _ in range(nb):
+            _, k, _ = step(dev)
+            for name, t_ms in k:
+                a = kall.setdefault(name, [0.0, 0])
+                a[0] += t_ms
+                a[1] += 1
+        torch.cuda.synchronize()
+        ctx.set_profiling(False)
+        kernels = {k: {"launches_per_step": v[1] / nb, "ms_per_step": round(v[0] / nb, 4)}
+                   for k, v in sorted(kall.items(), key=lambda kv: -kv[1][0])}
 
     # ---- data-centric attribution: the same trace, per-object
     # RD + MD rows over the workload's allocation table (one fused pass)
@@ -382,7 +405,7 @@ def main():
                 return ctx.last_launches(), ctx.last_kernel_times(), ctx.last_count(0)
             for _ in range(2):
                 dstep()
-            ctx.set_profiling(True)
+            ctx.set_profiling(2)
             torch.cuda.synchronize()
             g0, g1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             g0.record(stream)

@@ -244,9 +244,11 @@ CADV_API float cadv_last_elapsed_ms(const cadv_ctx *ctx);
 /* Number of kernels the last call launched (for bench.py's gpu_launches). */
 CADV_API uint32_t cadv_last_launches(const cadv_ctx *ctx);
 
-/* Per-kernel timing of the calls that follow (enable != 0): CUDA events are
- * recorded on the context's stream around every kernel launch.  Off by
- * default (it adds two event records per launch). */
+/* Per-kernel timing of the calls that follow: CUDA events are recorded on
+ * the context's stream around every kernel launch (enable = 1) or around the
+ * launches of the fused streaming pass k_scan<F> only (enable = 2, what a
+ * timed loop needs for the dominant kernel's roofline without the host cost
+ * of 2 event records per launch).  0 (default) turns it off. */
 CADV_API cadv_status cadv_set_profiling(cadv_ctx *ctx, int enable);
 
 /* Kernel names and device times (ms) of the last call's launches, in launch

@@ -162,9 +162,10 @@ class Context:
     def last_launches(self) -> int:
         return int(lib().cadv_last_launches(self._h))
 
-    def set_profiling(self, enable: bool):
-        """cadv_set_profiling: CUDA events around every kernel launch."""
-        self._check(lib().cadv_set_profiling(self._h, 1 if enable else 0))
+    def set_profiling(self, enable):
+        """cadv_set_profiling: CUDA events around every kernel launch (True / 1)
+        or around the streaming-pass (k_scan<F>) launches only (2)."""
+        self._check(lib().cadv_set_profiling(self._h, int(enable)))
 
     def last_kernel_times(self):
         """cadv_last_kernel_times: [(kernel name, device ms)] of the last call."""

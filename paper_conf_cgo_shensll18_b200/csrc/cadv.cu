@@ -53,11 +53,16 @@ cudaError_t ensure_host(cadv_ctx* c, size_t bytes, void** out) {
 Scalars* scalars(cadv_ctx* c) { return (Scalars*)c->buf[B_SCALARS].p; }
 
 void prof_begin(cadv_ctx* c, const char* src) {
+  c->prof_skip = false;
   if (!c->profiling) return;
+  if (c->profiling == 2 && strncmp(src, "k_scan<", 7) != 0) {
+    c->prof_skip = true;
+    return;
+  }
   uint32_t k = c->nprof;
   while (c->prof_ev.size() < 2ull * (k + 1)) {
     cudaEvent_t e;
-    if (cudaEventCreate(&e) != cudaSuccess) { c->profiling = false; return; }
+    if (cudaEventCreate(&e) != cudaSuccess) { c->profiling = 0; return; }
     c->prof_ev.push_back(e);
   }
   if (c->prof_src.size() <= k) c->prof_src.resize(k + 1);
@@ -66,7 +71,7 @@ void prof_begin(cadv_ctx* c, const char* src) {
 }
 
 void prof_end(cadv_ctx* c) {
-  if (!c->profiling || c->prof_ev.size() < 2ull * (c->nprof + 1)) return;
+  if (!c->profiling || c->prof_skip || c->prof_ev.size() < 2ull * (c->nprof + 1)) return;
   cudaEventRecord(c->prof_ev[2 * c->nprof + 1], c->stream);
   c->nprof++;
 }
@@ -332,7 +337,8 @@ CADV_API uint64_t cadv_last_count(const cadv_ctx* c, int which) {
 
 CADV_API cadv_status cadv_set_profiling(cadv_ctx* c, int enable) {
   if (!c) return CADV_ERR_INVALID_ARG;
-  c->profiling = enable != 0;
+  if (enable < 0 || enable > 2) return CADV_ERR_INVALID_ARG;
+  c->profiling = enable;
   return CADV_OK;
 }
 

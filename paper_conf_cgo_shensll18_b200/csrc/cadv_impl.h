@@ -78,7 +78,8 @@ struct cadv_ctx {
   // stream synchronisation for the scan scalars, kept count and CTA range)
   void* hstage = nullptr;  // 512 B: [0] kept records, [1] kept CTA-id max, +64: Scalars
   // per-kernel profiling (cadv_set_profiling)
-  bool profiling = false;
+  int profiling = 0;                  // 1: every launch, 2: k_scan<F> launches only
+  bool prof_skip = false;             // the current launch is not profiled (mode 2)
   std::vector<cudaEvent_t> prof_ev;   // 2 per launch
   std::vector<const char*> prof_src;  // stringified launch expression
   std::vector<std::string> prof_name;
