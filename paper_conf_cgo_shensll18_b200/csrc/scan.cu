@@ -13,22 +13,24 @@
 //         k_bd_resolve classifies once T_c (1 + max tid of the CTA's BB
 //         records, reduced with fire-and-forget RED.MAX) is complete.
 //
-// Data movement (B200): one persistent CTA per SM, 20 independent warps.
-// Every warp owns a contiguous chunk of the trace and streams it through a
-// private ring of 3 x 128-record pieces in shared memory, filled by 1-D TMA
-// bulk copies (cp.async.bulk + a per-warp mbarrier per piece).  There is no
-// block-level barrier in the loop.  A warp walks its chunk in batches of 32
-// records that start at a run start (run = records of one (cta, warp32,
-// winst, family)); every run that is complete inside the batch is resolved
-// at once:
-//   fast path  (lanes ascend inside the run and, for MD, lines do not
-//              decrease inside a sub-warp group): group boundaries and
-//              "first use of a line" flags come from one __shfl_up_sync per
-//              field plus ballots and popcounts;
-//   otherwise  __match_any_sync on (group, line) and (group, lane).
-// The batch then advances to the first run that is not complete.  Runs are
-// owned by the chunk that contains their first record; reuse-distance run
-// compression consumes exactly the chunk's records.
+// Data movement (B200): one persistent CTA per SM, 16 independent warps
+// (128 registers).  Every warp owns a contiguous chunk of the trace and
+// streams it through a private stage-major ring of 2 x 256-record pieces in
+// shared memory, filled by 1-D TMA bulk copies (cp.async.bulk, one elected
+// lane, one mbarrier per stage).  There is no block-level barrier in the
+// loop.  A step = one piece: every lane takes 8 consecutive records, builds
+// 8-bit masks from the comparisons with each record's predecessor (RD line /
+// scope equality, run starts, MD line changes and decreases), and the warp
+// combines lanes with ballots, shuffles and one segmented suffix scan:
+//   R1   duplicate loads are counted and dropped, store chains merged; the
+//        kept records are written to the warp's region of the kept buffer;
+//   M/B  runs (records of one (cta, warp32, winst, family)) complete in the
+//        step are queued in shared memory and finalized 32 at a time
+//        (flush_runs); the run open at the step end is carried.  Runs whose
+//        lines decrease (MD), analysis warp sizes below 32 and malformed
+//        runs take an exact pairwise walk over global memory.
+// Runs are owned by the chunk that contains their first record; reuse-
+// distance run compression consumes exactly the chunk's records.
 #include <cuda_runtime.h>
 
 #include "cadv_impl.h"
@@ -1003,12 +1005,28 @@ __global__ void __launch_bounds__(256) k_squeeze(const uint32_t* __restrict__ ki
   const uint64_t b = blockIdx.x, m = cnt[b], o = off[b];
   const uint64_t src = b * chunk;
   uint32_t mx = 0;
-  for (uint64_t k = threadIdx.x; k < m; k += blockDim.x) {
-    vout[o + k] = vin[src + k];
-    if (kin) {
-      const uint32_t key = kin[src + k];
-      kout[o + k] = key;
-      mx = max(mx, key);
+  // 4 elements per thread per round: all loads issued before the stores
+  for (uint64_t k0 = threadIdx.x; k0 < m; k0 += 4ull * blockDim.x) {
+    uint64_t v[4];
+    uint32_t key[4];
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint64_t k = k0 + (uint64_t)u * blockDim.x;
+      if (k < m) {
+        v[u] = vin[src + k];
+        key[u] = kin ? kin[src + k] : 0u;
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const uint64_t k = k0 + (uint64_t)u * blockDim.x;
+      if (k < m) {
+        vout[o + k] = v[u];
+        if (kin) {
+          kout[o + k] = key[u];
+          mx = max(mx, key[u]);
+        }
+      }
     }
   }
   mx = __reduce_max_sync(FULL, mx);
