@@ -535,16 +535,12 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
           }
           qbits |= (uint32_t)q << r;
           hbits |= (uint32_t)hd << r;
-          // R += { P(s) } of this round's queries; word prefix counts
-          uint32_t nr = 0;
-#pragma unroll
-          for (int k = 0; k < 8; ++k) {
-            const uint32_t o = __reduce_or_sync(FULL, (q && ((uint32_t)P >> 5) == (uint32_t)k) ? 1u << (P & 31) : 0u);
-            if (lane == (uint32_t)k) nr = RW[k] | o;
-          }
+          // R += { P(s) } of this round's queries (shared-memory atomics; every
+          // lane finished reading R above); word prefix counts
+          if (q) atomicOr(&RW[(uint32_t)P >> 5], 1u << (P & 31));
           __syncwarp();
-          if (lane < 8) RW[lane] = nr;
-          uint32_t pc = lane < 8 ? __popc(nr) : 0u, xc = pc;
+          const uint32_t nr = lane < 8 ? RW[lane] : 0u;
+          uint32_t pc = __popc(nr), xc = pc;
 #pragma unroll
           for (int o = 1; o < 8; o <<= 1) {
             const uint32_t y = __shfl_up_sync(FULL, xc, o);
