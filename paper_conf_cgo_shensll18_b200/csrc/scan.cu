@@ -108,6 +108,7 @@ struct ScanArgs {
   const uint64_t* obj_lo;
   const uint64_t* obj_hi;
   uint32_t nobj, rd_nbins;
+  uint32_t one;          // = 1 (opaque to the compiler: see add_if)
 };
 
 __device__ __forceinline__ void report(Scalars* sc, uint64_t i, uint32_t code) {
@@ -261,6 +262,16 @@ __device__ __forceinline__ uint32_t lds_u32(const uint32_t* p) {
   uint32_t v;
   asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(smem_u32(p)));
   return v;
+}
+
+// Mask building off the integer ALU pipe (the scan's bottleneck): m += bit
+// when the condition holds, as a predicated IMAD by an opaque 1 (FMA pipe)
+// instead of SEL + IADD3 on the ALU pipe.
+__device__ __forceinline__ void add_if_nz(uint32_t& m, uint32_t x, uint32_t one, uint32_t bit) {
+  asm("{\n.reg .pred q;\nsetp.ne.u32 q, %1, 0;\n@q mad.lo.u32 %0, %2, %3, %0;\n}" : "+r"(m) : "r"(x), "r"(one), "r"(bit));
+}
+__device__ __forceinline__ void add_if_lt(uint32_t& m, uint64_t a, uint64_t b, uint32_t one, uint32_t bit) {
+  asm("{\n.reg .pred q;\nsetp.lt.u64 q, %1, %2;\n@q mad.lo.u32 %0, %3, %4, %0;\n}" : "+r"(m) : "l"(a), "l"(b), "r"(one), "r"(bit));
 }
 
 // run identity: (cta, warp32, winst, family)
@@ -681,6 +692,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       uint32_t eqm = 0, rsm = 0, nlm = 0, vim = 0;
       uint64_t tl5 = 0;  // NG: the records' lanes, 5 bits each
       {
+        const uint32_t one = A.one;
         const uint32_t mlr = ~((1u << A.lbs_rd) - 1u), msc = A.cta_scope ? 0xffffffffu : 0u;
         const uint32_t mlm = ~((1u << A.lbs_md) - 1u);
 #pragma unroll
@@ -688,17 +700,18 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           const uint64_t qa = k == 0 ? pa : a[k - 1];
           const uint32_t qc = k == 0 ? pc : c[k - 1];
           const uint32_t dlo = (uint32_t)a[k] ^ (uint32_t)qa, dhi = (uint32_t)(a[k] >> 32) ^ (uint32_t)(qa >> 32);
-          if (RD) eqm |= (uint32_t)(((dlo & mlr) | dhi | ((c[k] ^ qc) & msc)) == 0u) << k;
+          if (RD) add_if_nz(eqm, (dlo & mlr) | dhi | ((c[k] ^ qc) & msc), one, 1u << k);  // (inverted below)
           if (NG) {
             const uint32_t qw = k == 0 ? pwi : w[k - 1], qt = k == 0 ? pt : t[k - 1];
-            rsm |= (uint32_t)(((c[k] ^ qc) | (w[k] ^ qw) | ((t[k] ^ qt) & ~31u)) != 0u) << k;
+            add_if_nz(rsm, (c[k] ^ qc) | (w[k] ^ qw) | ((t[k] ^ qt) & ~31u), one, 1u << k);
             if (MD) {
-              nlm |= (uint32_t)(((dlo & mlm) | dhi) != 0u) << k;
-              vim |= (uint32_t)(a[k] < qa) << k;  // only where the line changes (masked below)
+              add_if_nz(nlm, (dlo & mlm) | dhi, one, 1u << k);
+              add_if_lt(vim, a[k], qa, one, 1u << k);  // only where the line changes (masked below)
             }
             tl5 |= (uint64_t)(t[k] & 31u) << (5 * k);
           }
         }
+        eqm = ~eqm & 0xffu;
       }
       // ---- carry the step's last record to the next step
       p_cta = __shfl_sync(FULL, c[LPR - 1], 31);
@@ -1098,6 +1111,7 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
   A.ndefer = P.ndefer;
   A.nsites = P.nsites; A.site_flag = P.site_flag; A.sc = scalars(c);
   A.obj_lo = P.obj_lo; A.obj_hi = P.obj_hi; A.nobj = P.nobj; A.rd_nbins = P.rd_nbins;
+  A.one = 1;
   switch (flags) {
     case 1: return launch_scan_t<1>(c, A, grid);
     case 2: return launch_scan_t<2>(c, A, grid);
