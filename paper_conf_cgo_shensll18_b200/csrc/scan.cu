@@ -463,12 +463,16 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
 // rides in bit 31 of the sum (v < 2^30: adding a lane's packed value to one
 // without the flag copies that lane's flag); lane 31 always stops a segment,
 // so no lane ever reads past it.
-__device__ __forceinline__ void seg_scan2(uint32_t& v, uint32_t& m, uint32_t head) {
+// The lane-bit masks of one valid run are disjoint, so they are ADDED
+// (predicated IMADs by an opaque 1, off the ALU pipe); a repeated lane makes
+// a carry, so popc(mask) < count still exposes it (flush_runs).
+__device__ __forceinline__ void seg_scan2(uint32_t& v, uint32_t& m, uint32_t head, uint32_t one) {
   uint32_t x = v | ((head || lane_id() == 31u) ? 0x80000000u : 0u);
 #pragma unroll
   for (int d = 1; d < 32; d <<= 1) {
     const uint32_t xo = __shfl_down_sync(FULL, x, d), mo = __shfl_down_sync(FULL, m, d);
-    if (!(x >> 31)) { x += xo; m |= mo; }
+    asm("{\n.reg .pred q;\nsetp.lt.s32 q, %2, 0;\n@!q mad.lo.u32 %0, %4, %3, %0;\n@!q mad.lo.u32 %1, %4, %5, %1;\n}"
+        : "+r"(x), "+r"(m) : "r"(x), "r"(xo), "r"(one), "r"(mo));
   }
   v = x & 0x7fffffffu;
 }
@@ -807,7 +811,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         uint32_t m = 0;
 #pragma unroll
         for (int k = LPR - 1; k >= 0; --k) {
-          m |= 1u << (tl5 >> (5 * k) & 31u);
+          m = A.one * (1u << (tl5 >> (5 * k) & 31u)) + m;  // disjoint lanes: + == | (IMAD, FMA pipe)
           rm[k] = m;
           if ((rsm >> k) & 1u) m = 0;
         }
@@ -816,7 +820,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         const uint32_t pre = (1u << fr) - 1u;
         uint32_t u = __popc(nlm & pre) | (fr << PK_CNT) | (__popc(vim & pre) << PK_VIOL);
         const uint32_t head = rsm != 0;
-        seg_scan2(u, m, head);
+        seg_scan2(u, m, head, A.one);
         const uint32_t S_next = __shfl_down_sync(FULL, u, 1), M_next = __shfl_down_sync(FULL, m, 1);
         const uint32_t heads = __ballot_sync(FULL, head);
         // ---- the run carried in from the previous step ends at the first head
