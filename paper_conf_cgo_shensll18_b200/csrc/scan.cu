@@ -634,8 +634,11 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         }
       }
       // owned / in-stream records of the lane (all of them except near the chunk end)
-      const uint32_t ownm = j0 >= clen ? 0u : (clen - j0 >= LPR ? 0xffu : (1u << (clen - j0)) - 1u);
-      const uint32_t inbm = j0 >= slen ? 0u : (slen - j0 >= LPR ? 0xffu : (1u << (slen - j0)) - 1u);
+      uint32_t ownm = 0xffu, inbm = 0xffu;
+      if (base + KR > clen) {  // (warp-uniform: only the chunk's last steps)
+        ownm = j0 >= clen ? 0u : (clen - j0 >= LPR ? 0xffu : (1u << (clen - j0)) - 1u);
+        inbm = j0 >= slen ? 0u : (slen - j0 >= LPR ? 0xffu : (1u << (slen - j0)) - 1u);
+      }
       // kind masks (bit k = record k) from the meta bytes
       const uint32_t glo = gather8(mmx, mmy), ghi = gather8(mmx >> 1, mmy >> 1);
       uint32_t okm = inbm;
@@ -755,7 +758,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
 #pragma unroll
         for (int o = 1; o < 32; o <<= 1) {
           const uint32_t y = __shfl_up_sync(FULL, x, o);
-          if (lane >= (uint32_t)o) x += y;
+          if (lane >= (uint32_t)o) x = A.one * y + x;  // (IMAD: off the ALU pipe)
         }
         const uint32_t tot = __shfl_sync(FULL, x, 31);
         uint32_t pos = kept + x - nk;

@@ -252,6 +252,43 @@ def test_long_run_detected(ctx, cadv):
     assert e.value.status == cadv.CADV_ERR_BAD_TRACE
 
 
+@pytest.mark.parametrize("bb", [False, True])
+@pytest.mark.parametrize("lead,size,dup", [(0, 32, (3, 4)), (5, 20, (0, 19)), (13, 32, (30, 31)), (250, 12, (2, 9))])
+def test_repeated_lane_detected(ctx, cadv, bb, lead, size, dup):
+    """A warp-level group of <= 32 records with one lane twice (the run's lane
+    masks are accumulated by addition in the scan: the carry must still fail
+    the popcount check), at various offsets inside a 256-record step; the
+    same trace without the repeat is valid and matches the oracle."""
+    def build(repeat):
+        recs = []  # (addr, tid, winst)
+        for g in range(lead):      # filler groups of 1 record (warp 1), before the tested group
+            recs.append((0x7F0000000000 + 128 * g, 32, g))
+        lanes = list(range(size))
+        if repeat:
+            lanes[dup[1]] = lanes[dup[0]]
+        for q, l in enumerate(lanes):
+            recs.append((0x7F0000100000 + 4 * q, l, 0))
+        for g in range(40):        # trailing groups
+            recs.append((0x7F0000200000 + 128 * g, 32, lead + g))
+        a = np.array(recs, dtype=np.uint64)
+        meta = np.full(len(a), (2 if bb else 0) | (2 << 2))
+        return tg.from_arrays(a[:, 0], np.zeros(len(a)), a[:, 1], np.zeros(len(a)), a[:, 2], meta, nsites=1)
+    ok = build(False)
+    ctx.load_trace(cadv.to_device(ok))
+    if bb:
+        psb, tot = ctx.branch_divergence(32, 1)
+        psb_ref, tot_ref = orc.branch_div(ok, 32)
+        assert (tot == tot_ref).all() and (psb == psb_ref).all()
+    else:
+        hm, psm = ctx.mem_divergence(128, 32, 1)
+        hm_ref, psm_ref = orc.mem_div(ok, 128, 32)
+        assert (hm == hm_ref).all() and (psm == psm_ref).all()
+    ctx.load_trace(cadv.to_device(build(True)))
+    with pytest.raises(cadv.CadvError) as e:
+        ctx.branch_divergence(32, 1) if bb else ctx.mem_divergence(128, 32, 1)
+    assert e.value.status == cadv.CADV_ERR_BAD_TRACE
+
+
 def test_invalid_args(ctx, cadv):
     t = tg.generate("vecadd")
     load(ctx, cadv, t)
