@@ -29,6 +29,7 @@ struct Scalars {
   unsigned long long tc_overflow;  // scan: a CTA id >= the T_c capacity was seen
   unsigned long long ndefer;     // branch divergence: deferred partial groups
   unsigned long long rd_line_min, rd_line_max;  // reuse cross-tile phase: entry line range
+  unsigned long long rg_overflow;  // regroup: a scan region holds more than RG_MAX distinct CTAs
 };
 
 enum BufId {
@@ -40,6 +41,7 @@ enum BufId {
   B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP, B_DEFER, B_OUT2,
   B_ALIGN0, B_ALIGN1, B_ALIGN2, B_ALIGN3, B_ALIGN4, B_ALIGN5,
   B_XCH_K0, B_XCH_K1, B_XCH_V0, B_XCH_V1, B_XCH_CNT, B_COMM, B_OBJ, B_RD_ENT_ALL,
+  B_RG_PK, B_RG_PN, B_RG_NP, B_RG_SORT,
   B_COUNT
 };
 
@@ -146,6 +148,21 @@ cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, const unsigned lon
                               uint32_t nsites);
 
 // ---- reuse distance around the scan (reuse.cu)
+// R1 regroup by CTA through per-region CTA tables (regroup.cu; CTA scope on
+// one rank): a region = one scan warp's kept records
+constexpr uint32_t RG_MAX = 768;  // distinct CTAs per region (more: squeeze + radix sort)
+struct RgState {
+  uint32_t* pk = nullptr;    // [region][RG_MAX] CTA ids
+  uint32_t* pn = nullptr;    // [region][RG_MAX] record counts, later output offsets
+  uint32_t* np = nullptr;    // [region + 1] pairs per region
+  uint32_t* poff = nullptr;  // [region + 1] exclusive scan of np (poff[nregions] = total)
+  uint64_t nregions = 0;
+};
+cudaError_t rg_count(cadv_ctx* c, const uint32_t* key, const uint64_t* cnt, uint64_t nregions, uint64_t chunk,
+                     RgState* st);
+cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, const uint32_t* key,
+                      const uint64_t* val, const uint64_t* cnt, uint64_t chunk, uint32_t* kout, uint64_t* vout);
+
 struct RdState {
   int cta_scope = 1;
   uint32_t* k0 = nullptr;   // final kept records (after the squeeze) / radix sort ping
@@ -154,6 +171,8 @@ struct RdState {
   uint64_t* v1 = nullptr;
   uint64_t* blkcnt = nullptr;  // [grid] kept per scan block, then [grid] offsets
   uint64_t grid = 0, chunk_cap = 0;
+  bool rg = false;  // regroup through region tables (regroup.cu) instead of squeeze + radix sort
+  RgState rgs;
 };
 // R1 compaction of the scan's per-warp regions (exclusive scan of the counts
 // + squeeze), queued on the stream; the kept count and the kept CTA-id range

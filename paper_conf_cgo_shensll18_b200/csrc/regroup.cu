@@ -1,0 +1,241 @@
+// regroup.cu — R1 regroup by CTA (CTA scope, one rank) without a global sort
+// of the kept records.
+//
+// The scan leaves the kept records in per-warp regions, each in trace order
+// (region w = records [w * chunk, w * chunk + cnt[w]) of the gapped buffer).
+// CTA-major order with trace order inside a CTA (DESIGN.md reading
+// R2) puts record i of CTA c of region w at
+//     base(c) + sum_{w' < w} n(c, w') + rank of i among c's records in w,
+// n(c, w) the number of c's kept records in region w.  A region only sees
+// the CTAs resident while it was traced (a few hundred), so:
+//   1. k_rg_count   one warp per region: a shared-memory table CTA -> n(c, w)
+//                   (open addressing, RG_SLOTS slots); emits the region's
+//                   (c, n) pairs into its slice of the pair buffer; a region
+//                   with more than RG_MAX distinct CTAs sets the overflow flag
+//                   and the host takes the squeeze + radix-sort path instead;
+//   2. pairs packed in region order, stably radix-sorted by CTA (a few
+//      hundred thousand pairs instead of the tens of millions of records),
+//      exclusive scan of n in that order = the output offset of every (c, w);
+//   3. k_rg_scatter one warp per region: rebuilds the table CTA -> offset,
+//                   walks its records in order, rank = offset + earlier peers
+//                   (__match_any_sync) and writes key and value once.
+// Data movement: keys read twice, values once, both written once: 28 B per
+// kept record instead of 80 B for squeeze + two radix passes.
+#include <cuda_runtime.h>
+
+#include "cadv_impl.h"
+#include "common.cuh"
+
+namespace cadv {
+namespace {
+
+constexpr uint32_t RG_SLOTS = 1024;  // table slots per region (power of two)
+constexpr uint32_t RG_EMPTY = 0xffffffffu;
+
+__device__ __forceinline__ uint32_t rg_hash(uint32_t c) { return (c * 0x9E3779B1u) >> (32 - 10); }
+
+// Slot of CTA c in the region table (inserted if absent); RG_EMPTY if full.
+__device__ __forceinline__ uint32_t rg_slot(uint32_t* tk, uint32_t c) {
+  uint32_t h = rg_hash(c);
+  for (uint32_t probe = 0; probe < RG_SLOTS; ++probe) {
+    const uint32_t k = tk[h];
+    if (k == c) return h;
+    if (k == RG_EMPTY) {
+      const uint32_t old = atomicCAS(&tk[h], RG_EMPTY, c);
+      if (old == RG_EMPTY || old == c) return h;
+    }
+    h = (h + 1) & (RG_SLOTS - 1);
+  }
+  return RG_EMPTY;
+}
+
+// 1. per-region CTA counts -> pairs (cta, n) at pk/pn + w * RG_MAX, np[w];
+//    the kept CTA-id range (radix bits) and the overflow flag in sc.  Counts
+//    do not depend on order: RG_NT threads per region, warp-aggregated
+//    shared-memory atomics.
+constexpr int RG_NT = 256;
+__global__ void __launch_bounds__(RG_NT) k_rg_count(const uint32_t* __restrict__ key, const uint64_t* __restrict__ cnt,
+                                                    uint64_t chunk, uint32_t* __restrict__ pk,
+                                                    uint32_t* __restrict__ pn, uint32_t* __restrict__ np,
+                                                    Scalars* sc) {
+  __shared__ uint32_t tk[RG_SLOTS], tn[RG_SLOTS];
+  __shared__ uint32_t s_full, s_base;
+  const uint32_t lane = lane_id(), tx = threadIdx.x, w = blockIdx.x;
+  for (uint32_t k = tx; k < RG_SLOTS; k += RG_NT) { tk[k] = RG_EMPTY; tn[k] = 0; }
+  if (tx == 0) { s_full = 0; s_base = 0; }
+  __syncthreads();
+  const uint64_t m = cnt[w];
+  const uint32_t* kr = key + (uint64_t)w * chunk;
+  uint32_t mx = 0, full = 0;
+  for (uint64_t r0 = 0; r0 < m; r0 += RG_NT) {  // (uniform trip count: every lane reaches the match)
+    const uint64_t r = r0 + tx;
+    const bool ok = r < m;
+    const uint32_t c = ok ? __ldg(kr + r) : RG_EMPTY;
+    const uint32_t peers = __match_any_sync(FULL, c);
+    if (ok && (uint32_t)(__ffs(peers) - 1) == lane) {  // one lane per CTA of the warp's 32 records
+      const uint32_t s = rg_slot(tk, c);
+      if (s != RG_EMPTY) atomicAdd(&tn[s], (uint32_t)__popc(peers));
+      else full = 1;
+      mx = max(mx, c);
+    }
+  }
+  if (full) s_full = 1;
+  __syncthreads();
+  // compact the table into the region's pair slice (order within a region is free)
+  const uint32_t k = tx;
+  for (uint32_t k0 = 0; k0 < RG_SLOTS; k0 += RG_NT) {
+    const uint32_t kk = k0 + k, c = tk[kk];
+    const bool used = c != RG_EMPTY;
+    const uint32_t b = __ballot_sync(FULL, used);
+    uint32_t wb = 0;
+    if (lane == 0 && b) wb = atomicAdd(&s_base, (uint32_t)__popc(b));
+    wb = __shfl_sync(FULL, wb, 0);
+    if (used) {
+      const uint32_t j = wb + __popc(b & lanemask_lt());
+      if (j < RG_MAX) {
+        pk[(uint64_t)w * RG_MAX + j] = c;
+        pn[(uint64_t)w * RG_MAX + j] = tn[kk];
+      }
+    }
+  }
+  mx = __reduce_max_sync(FULL, mx);
+  if (lane == 0 && mx) atomicMax(&sc->max_cta, (unsigned long long)mx);
+  __syncthreads();
+  if (tx == 0) {
+    const uint32_t base = s_base;
+    np[w] = base < RG_MAX ? base : RG_MAX;
+    if (s_full || base > RG_MAX) sc->rg_overflow = 1;
+  }
+}
+
+// 2a. pack the pair slices in region order: (cta, w << 10 | j), n
+__global__ void k_rg_pack(const uint32_t* __restrict__ pk, const uint32_t* __restrict__ pn,
+                          const uint32_t* __restrict__ np, const uint32_t* __restrict__ poff,
+                          uint32_t* __restrict__ ok_, uint32_t* __restrict__ ov, uint32_t* __restrict__ on) {
+  const uint32_t w = blockIdx.x, n = np[w], o = poff[w];
+  for (uint32_t j = threadIdx.x; j < n; j += blockDim.x) {
+    ok_[o + j] = pk[(uint64_t)w * RG_MAX + j];
+    ov[o + j] = (w << 10) | j;
+    on[o + j] = pn[(uint64_t)w * RG_MAX + j];
+  }
+}
+
+// 2b. counts in CTA-sorted order (gathered through the sorted pair ids)
+__global__ void k_rg_gather_n(const uint32_t* __restrict__ sv, const uint32_t* __restrict__ pn, uint64_t P,
+                              uint32_t* __restrict__ sn) {
+  for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < P; s += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t v = sv[s];
+    sn[s] = pn[(uint64_t)(v >> 10) * RG_MAX + (v & 1023u)];
+  }
+}
+
+// 2c. offsets back into the region slices: po[w][j] = offset of (c, w)
+__global__ void k_rg_offsets(const uint32_t* __restrict__ sv, const uint32_t* __restrict__ so, uint64_t P,
+                             uint32_t* __restrict__ po) {
+  for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < P; s += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t v = sv[s];
+    po[(uint64_t)(v >> 10) * RG_MAX + (v & 1023u)] = so[s];
+  }
+}
+
+// 3. scatter: one warp per region, records in order
+__global__ void __launch_bounds__(32) k_rg_scatter(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val,
+                                                   const uint64_t* __restrict__ cnt, uint64_t chunk,
+                                                   const uint32_t* __restrict__ pk, const uint32_t* __restrict__ po,
+                                                   const uint32_t* __restrict__ np, uint32_t* __restrict__ kout,
+                                                   uint64_t* __restrict__ vout) {
+  __shared__ uint32_t tk[RG_SLOTS], to[RG_SLOTS];
+  const uint32_t lane = lane_id(), w = blockIdx.x;
+  for (uint32_t k = lane; k < RG_SLOTS; k += 32) tk[k] = RG_EMPTY;
+  __syncwarp();
+  const uint32_t n = np[w];
+  for (uint32_t j = lane; j < n; j += 32) {
+    const uint32_t c = pk[(uint64_t)w * RG_MAX + j];
+    const uint32_t s = rg_slot(tk, c);  // (n <= RG_MAX < RG_SLOTS: always found a slot)
+    to[s] = po[(uint64_t)w * RG_MAX + j];
+  }
+  __syncwarp();
+  const uint64_t m = cnt[w];
+  const uint32_t* kr = key + (uint64_t)w * chunk;
+  const uint64_t* vr = val + (uint64_t)w * chunk;
+  // batches of RG_B rounds: all loads of a batch are issued before its rounds
+  constexpr int RG_B = 8;
+  for (uint64_t r0 = 0; r0 < m; r0 += 32 * RG_B) {
+    uint32_t cb[RG_B];
+    uint64_t vb[RG_B];
+#pragma unroll
+    for (int b = 0; b < RG_B; ++b) {
+      const uint64_t r = r0 + 32 * b + lane;
+      cb[b] = r < m ? __ldg(kr + r) : RG_EMPTY;
+      vb[b] = r < m ? __ldg(vr + r) : 0ull;
+    }
+#pragma unroll
+    for (int b = 0; b < RG_B; ++b) {
+      const bool ok = r0 + 32 * b + lane < m;
+      const uint32_t c = cb[b];
+      const uint32_t peers = __match_any_sync(FULL, c);
+      uint32_t s = 0, dst = 0;
+      if (ok) {
+        s = rg_slot(tk, c);  // present: every CTA of the region is in the table
+        dst = to[s] + __popc(peers & lanemask_lt());
+        kout[dst] = c;
+        vout[dst] = vb[b];
+      }
+      __syncwarp();
+      if (ok && (peers >> lane) == 1u) to[s] = dst + 1;  // the CTA's last record of the round
+      __syncwarp();
+    }
+  }
+}
+
+}  // namespace
+
+// Phase 1 (queued before the scan's synchronisation): per-region CTA counts.
+cudaError_t rg_count(cadv_ctx* c, const uint32_t* key, const uint64_t* cnt, uint64_t nregions, uint64_t chunk,
+                     RgState* st) {
+  void *pk, *pn, *np;
+  cudaError_t e;
+  if ((e = ensure(c, B_RG_PK, nregions * RG_MAX * 4 + 64, &pk)) ||
+      (e = ensure(c, B_RG_PN, nregions * RG_MAX * 4 + 64, &pn)) ||
+      (e = ensure(c, B_RG_NP, (nregions + 2) * 4 * 2 + 64, &np)))
+    return e;
+  st->pk = (uint32_t*)pk;
+  st->pn = (uint32_t*)pn;
+  st->np = (uint32_t*)np;
+  st->poff = st->np + nregions + 2;
+  st->nregions = nregions;
+  if ((e = cudaMemsetAsync(st->np + nregions, 0, 8, c->stream))) return e;
+  CADV_LAUNCH(c, k_rg_count<<<(unsigned)nregions, RG_NT, 0, c->stream>>>(key, cnt, chunk, st->pk, st->pn, st->np,
+                                                                       scalars(c)));
+  // region offsets of the packed pairs; the total arrives with the scan's read-back
+  return exclusive_scan_u32(c, st->np, st->poff, nregions + 1, nullptr);
+}
+
+// Phases 2-3 (after the synchronisation; P = total pairs, no overflow).
+cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, const uint32_t* key,
+                      const uint64_t* val, const uint64_t* cnt, uint64_t chunk, uint32_t* kout, uint64_t* vout) {
+  void *b;
+  cudaError_t e;
+  // packed pairs (ping-pong for the sort) + counts + offsets
+  if ((e = ensure(c, B_RG_SORT, (P + 16) * 4 * 6 + 64, &b))) return e;
+  uint32_t* k0 = (uint32_t*)b;
+  uint32_t* k1 = k0 + (P + 16);
+  uint32_t* v0 = k1 + (P + 16);
+  uint32_t* v1 = v0 + (P + 16);
+  uint32_t* n0 = v1 + (P + 16);
+  uint32_t* n1 = n0 + (P + 16);
+  CADV_LAUNCH(c, k_rg_pack<<<(unsigned)st.nregions, 128, 0, c->stream>>>(st.pk, st.pn, st.np, st.poff, k0, v0, n0));
+  int res = 0;
+  if ((e = radix_sort_pairs<uint32_t, uint32_t>(c, k0, v0, k1, v1, P, 0, bits, &res))) return e;
+  const uint32_t* sv = res ? v1 : v0;
+  const int grid = c->num_sms * 4;
+  CADV_LAUNCH(c, k_rg_gather_n<<<grid, 256, 0, c->stream>>>(sv, st.pn, P, n1));
+  if ((e = exclusive_scan_u32(c, n1, n0, P, nullptr))) return e;
+  // the offsets overwrite the pair counts (pn is no longer needed)
+  CADV_LAUNCH(c, k_rg_offsets<<<grid, 256, 0, c->stream>>>(sv, n0, P, st.pn));
+  CADV_LAUNCH(c, k_rg_scatter<<<(unsigned)st.nregions, 32, 0, c->stream>>>(key, val, cnt, chunk, st.pk, st.pn, st.np,
+                                                                           kout, vout));
+  return cudaGetLastError();
+}
+
+}  // namespace cadv

@@ -1102,6 +1102,7 @@ cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st) {
   st->v0 = (uint64_t*)v0;
   st->v1 = (uint64_t*)v1;
   st->blkcnt = (uint64_t*)bc;
+  st->rg = st->cta_scope && c->comm == nullptr && getenv("CADV_REGROUP_RADIX") == nullptr;
   return cudaSuccess;
 }
 
@@ -1314,6 +1315,16 @@ cudaError_t rd_compact(cadv_ctx* c, const RdState& S) {
   uint64_t* off = S.blkcnt + S.grid + 4;
   if ((e = exclusive_scan_u64(c, S.blkcnt, off, S.grid + 1))) return e;
   if ((e = cudaMemcpyAsync(&h[0], off + S.grid, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if (S.rg) {
+    // regroup tables (regroup.cu): pair total, overflow flag and CTA-id range
+    // arrive with the same read-back; the squeeze only runs on overflow
+    RgState& G = const_cast<RdState&>(S).rgs;
+    if ((e = rg_count(c, S.k1, S.blkcnt, S.grid, S.chunk_cap, &G))) return e;
+    h[2] = h[3] = 0;
+    if ((e = cudaMemcpyAsync(&h[2], G.poff + S.grid, 4, cudaMemcpyDeviceToHost, c->stream))) return e;
+    if ((e = cudaMemcpyAsync(&h[3], &scalars(c)->rg_overflow, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+    return cudaMemcpyAsync(&h[1], &scalars(c)->max_cta, 8, cudaMemcpyDeviceToHost, c->stream);
+  }
   if ((e = launch_squeeze(c, (const uint32_t*)S.k1, (const uint64_t*)S.v1, (uint32_t*)S.k0, (uint64_t*)S.v0, S.blkcnt,
                           off, S.grid, S.chunk_cap)))
     return e;
@@ -1339,7 +1350,28 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     c->counts[0] = K;
     // ---- R1b regroup by CTA (stable)
     val = (const uint64_t*)v0;
-    if (cta_scope && K) {
+    if (S.rg && K) {
+      const uint64_t* hs = (const uint64_t*)c->hstage;
+      int bits = bits_for(c->max_cta);
+      if (bits == 0) bits = 1;
+      if (hs[3] == 0) {  // every region's CTAs fit its table
+        if ((e = rg_finish(c, S.rgs, hs[2], bits, (const uint32_t*)k1, (const uint64_t*)v1, S.blkcnt, S.chunk_cap,
+                           (uint32_t*)k0, (uint64_t*)v0)))
+          return e;
+        key = (const uint32_t*)k0;
+        val = (const uint64_t*)v0;
+      } else {  // overflow: pack, then the radix sort
+        if ((e = launch_squeeze(c, (const uint32_t*)k1, (const uint64_t*)v1, (uint32_t*)k0, (uint64_t*)v0, S.blkcnt,
+                                S.blkcnt + S.grid + 4, S.grid, S.chunk_cap)))
+          return e;
+        int res;
+        if ((e = radix_sort_pairs<uint32_t, uint64_t>(c, (uint32_t*)k0, (uint64_t*)v0, (uint32_t*)k1, (uint64_t*)v1,
+                                                      K, 0, bits, &res)))
+          return e;
+        key = res ? (const uint32_t*)k1 : (const uint32_t*)k0;
+        val = res ? (const uint64_t*)v1 : (const uint64_t*)v0;
+      }
+    } else if (cta_scope && K) {
       int res;
       int bits = bits_for(c->max_cta);
       if (bits == 0) bits = 1;

@@ -183,7 +183,8 @@ __device__ __forceinline__ void site_add(const ScanArgs& A, uint32_t* smem_tab, 
 #define CADV_CP(DOFF, SRC, BYTES) \
   "@p cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0+" #DOFF "], [" SRC "], " #BYTES ", [%1];\n"
 template <int F>
-__device__ __forceinline__ void issue_full(const ScanArgs& A, uint32_t dst, uint32_t bar, uint64_t q0) {
+__device__ __forceinline__ void issue_full(const ScanArgs& A, uint32_t dst, uint32_t bar, uint32_t q0) {
+  // (q0 < n < 2^32: 32-bit element offsets, so the addresses are IMAD.WIDEs on the FMA pipe)
   constexpr bool NA = (F & (F_RD | F_MD)) != 0, NG = (F & (F_MD | F_BD)) != 0;
   static_assert(KR == 256 && S_CTA == 2048 && S_TID == 3072 && S_WINST == 3584 && S_SITE == 4608 && S_META == 5632,
                 "column offsets / byte counts below are for 256-record pieces");
@@ -192,7 +193,8 @@ __device__ __forceinline__ void issue_full(const ScanArgs& A, uint32_t dst, uint
         "{\n.reg .pred p;\nelect.sync _|p, 0xffffffff;\n"
         "@p mbarrier.arrive.expect_tx.shared::cta.b64 _, [%1], 5888;\n"
         CADV_CP(0, "%2", 2048) CADV_CP(2048, "%3", 1024) CADV_CP(3072, "%4", 512) CADV_CP(3584, "%5", 1024)
-        CADV_CP(4608, "%6", 1024) CADV_CP(5632, "%7", 256) "}" ::"r"(dst), "r"(bar), "l"(A.addr + q0),
+        CADV_CP(4608, "%6", 1024) CADV_CP(5632, "%7", 256) "}" ::"r"(dst), "r"(bar),
+        "l"(A.addr + q0),
         "l"(A.cta + q0), "l"(A.tid + q0), "l"(A.winst + q0), "l"(A.site + q0), "l"(A.meta + q0)
         : "memory");
   } else if (NA) {
@@ -246,8 +248,8 @@ template <int F>
 __device__ __forceinline__ void issue_piece(const ScanArgs& A, uint32_t ring, uint32_t bar0, uint64_t c_lo,
                                             uint64_t s_end, uint32_t p) {
   const uint32_t stg = p % KS, bar = bar0 + stg * 8, dst = ring + stg * STG_BYTES;
-  const uint64_t q0 = c_lo + (uint64_t)p * KR;
-  if (q0 + KR <= s_end) issue_full<F>(A, dst, bar, q0);
+  const uint32_t q0 = (uint32_t)c_lo + p * KR;  // < n < 2^32 (cadv_load_trace)
+  if ((uint64_t)q0 + KR <= s_end) issue_full<F>(A, dst, bar, q0);
   else issue_partial<F>(A, dst, bar, q0, (uint32_t)(s_end - q0));
 }
 

@@ -478,3 +478,16 @@ def test_eq1_from_gpu_outputs(ctx, cadv):
     assert rd == M.mean_reuse_distance(s_ref) and md == M.md_degree(orc.mem_div(t, 128)[0])
     assert M.opt_num_warps(16384, rd, 128, md, 4) == M.opt_num_warps(16384, M.mean_reuse_distance(s_ref), 128,
                                                                        orc.md_degree(orc.mem_div(t, 128)[0]), 4)
+
+
+@pytest.mark.parametrize("ctas", [40, 1500])
+def test_regroup_tables_and_overflow(ctx, ctx_long, cadv, ctas):
+    """CTA regroup through per-region CTA tables (regroup.cu): with 1 scan CTA
+    (16 regions) 1500 CTAs overflow a region's table (> RG_MAX = 768
+    distinct CTAs) and the squeeze + radix-sort path takes over; 40 CTAs fit.
+    Both contexts, both line sizes, CTA scope, against the oracle."""
+    t = tg.generate("rand", seed=31, ctas=ctas, threads=64, instrs=12, lines=50, pstore=0.2, pbb=0.2)
+    for c in (ctx, ctx_long):
+        load(c, cadv, t)
+        check_reuse(c, t, 128, 0)
+        check_reuse(c, t, 32, 0, 1, 20)
