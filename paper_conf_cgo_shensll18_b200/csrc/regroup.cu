@@ -67,16 +67,26 @@ __global__ void __launch_bounds__(RG_NT) k_rg_count(const uint32_t* __restrict__
   const uint64_t m = cnt[w];
   const uint32_t* kr = key + (uint64_t)w * chunk;
   uint32_t mx = 0, full = 0;
-  for (uint64_t r0 = 0; r0 < m; r0 += RG_NT) {  // (uniform trip count: every lane reaches the match)
-    const uint64_t r = r0 + tx;
-    const bool ok = r < m;
-    const uint32_t c = ok ? __ldg(kr + r) : RG_EMPTY;
-    const uint32_t peers = __match_any_sync(FULL, c);
-    if (ok && (uint32_t)(__ffs(peers) - 1) == lane) {  // one lane per CTA of the warp's 32 records
-      const uint32_t s = rg_slot(tk, c);
-      if (s != RG_EMPTY) atomicAdd(&tn[s], (uint32_t)__popc(peers));
-      else full = 1;
-      mx = max(mx, c);
+  constexpr int RB = 4;  // rounds whose loads are issued together
+  for (uint64_t r0 = 0; r0 < m; r0 += RG_NT * RB) {  // (uniform trip count: every lane reaches the match)
+    uint32_t cb[RB];
+#pragma unroll
+    for (int b = 0; b < RB; ++b) {
+      const uint64_t r = r0 + (uint64_t)b * RG_NT + tx;
+      cb[b] = r < m ? __ldg(kr + r) : RG_EMPTY;
+    }
+#pragma unroll
+    for (int b = 0; b < RB; ++b) {
+      const bool ok = r0 + (uint64_t)b * RG_NT + tx < m;
+      const uint32_t c = cb[b];
+      if (ok && c == RG_EMPTY) full = 1;  // (the table's empty marker: such a trace takes the radix path)
+      const uint32_t peers = __match_any_sync(FULL, c);
+      if (ok && c != RG_EMPTY && (uint32_t)(__ffs(peers) - 1) == lane) {  // one lane per CTA of the warp's 32 records
+        const uint32_t s = rg_slot(tk, c);
+        if (s != RG_EMPTY) atomicAdd(&tn[s], (uint32_t)__popc(peers));
+        else full = 1;
+        mx = max(mx, c);
+      }
     }
   }
   if (full) s_full = 1;
@@ -138,45 +148,76 @@ __global__ void k_rg_offsets(const uint32_t* __restrict__ sv, const uint32_t* __
   }
 }
 
-// 3. scatter: one warp per region, records in order
-__global__ void __launch_bounds__(32) k_rg_scatter(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val,
-                                                   const uint64_t* __restrict__ cnt, uint64_t chunk,
-                                                   const uint32_t* __restrict__ pk, const uint32_t* __restrict__ po,
-                                                   const uint32_t* __restrict__ np, uint32_t* __restrict__ kout,
-                                                   uint64_t* __restrict__ vout) {
-  __shared__ uint32_t tk[RG_SLOTS], to[RG_SLOTS];
-  const uint32_t lane = lane_id(), w = blockIdx.x;
-  for (uint32_t k = lane; k < RG_SLOTS; k += 32) tk[k] = RG_EMPTY;
-  __syncwarp();
+// 3. scatter: RG_NT threads per region; warp q takes the q-th contiguous
+//    slice of the region (whole 32-record rounds).  The warps first count
+//    their slices' CTAs, a prefix over the warps turns the region offsets of
+//    the CTAs into per-slice starts, then every warp writes its slice in
+//    order (rank among a round's peers by __match_any_sync; the peer group's
+//    leader probes the table once).
+constexpr int RG_W = RG_NT / 32;
+__global__ void __launch_bounds__(RG_NT) k_rg_scatter(const uint32_t* __restrict__ key,
+                                                      const uint64_t* __restrict__ val,
+                                                      const uint64_t* __restrict__ cnt, uint64_t chunk,
+                                                      const uint32_t* __restrict__ pk, const uint32_t* __restrict__ po,
+                                                      const uint32_t* __restrict__ np, uint32_t* __restrict__ kout,
+                                                      uint64_t* __restrict__ vout) {
+  __shared__ uint32_t tk[RG_SLOTS];
+  __shared__ uint32_t st[RG_W][RG_SLOTS];  // per slice: CTA counts, then starts
+  const uint32_t lane = lane_id(), tx = threadIdx.x, q = tx >> 5, w = blockIdx.x;
+  for (uint32_t k = tx; k < RG_SLOTS; k += RG_NT) tk[k] = RG_EMPTY;
+  for (uint32_t k = tx; k < RG_W * RG_SLOTS; k += RG_NT) (&st[0][0])[k] = 0;
+  __syncthreads();
   const uint32_t n = np[w];
-  for (uint32_t j = lane; j < n; j += 32) {
-    const uint32_t c = pk[(uint64_t)w * RG_MAX + j];
-    const uint32_t s = rg_slot(tk, c);  // (n <= RG_MAX < RG_SLOTS: always found a slot)
-    to[s] = po[(uint64_t)w * RG_MAX + j];
-  }
-  __syncwarp();
+  for (uint32_t j = tx; j < n; j += RG_NT) rg_slot(tk, pk[(uint64_t)w * RG_MAX + j]);
+  __syncthreads();
   const uint64_t m = cnt[w];
   const uint32_t* kr = key + (uint64_t)w * chunk;
   const uint64_t* vr = val + (uint64_t)w * chunk;
-  // batches of RG_B rounds: all loads of a batch are issued before its rounds
-  constexpr int RG_B = 8;
-  for (uint64_t r0 = 0; r0 < m; r0 += 32 * RG_B) {
+  const uint64_t rounds = (m + 31) / 32, per = (rounds + RG_W - 1) / RG_W;
+  const uint64_t lo = min(m, q * per * 32), hi = min(m, (q + 1) * per * 32);
+  // (a) count the slice's CTAs
+  for (uint64_t r = lo; r < hi; r += 32) {
+    const bool ok = r + lane < hi;
+    const uint32_t c = ok ? __ldg(kr + r + lane) : RG_EMPTY;
+    const uint32_t peers = __match_any_sync(FULL, c);
+    if (ok && (uint32_t)(__ffs(peers) - 1) == lane) st[q][rg_slot(tk, c)] += __popc(peers);
+  }
+  __syncthreads();
+  // (b) slice starts = the CTA's region offset + its records in earlier slices
+  for (uint32_t j = tx; j < n; j += RG_NT) {
+    const uint32_t s = rg_slot(tk, pk[(uint64_t)w * RG_MAX + j]);
+    uint32_t run = po[(uint64_t)w * RG_MAX + j];
+#pragma unroll
+    for (int x = 0; x < RG_W; ++x) {
+      const uint32_t t = st[x][s];
+      st[x][s] = run;
+      run += t;
+    }
+  }
+  __syncthreads();
+  // (c) write the slice in order
+  uint32_t* const to = st[q];
+  constexpr int RG_B = 4;  // rounds whose loads are issued together
+  for (uint64_t r0 = lo; r0 < hi; r0 += 32 * RG_B) {
     uint32_t cb[RG_B];
     uint64_t vb[RG_B];
 #pragma unroll
     for (int b = 0; b < RG_B; ++b) {
       const uint64_t r = r0 + 32 * b + lane;
-      cb[b] = r < m ? __ldg(kr + r) : RG_EMPTY;
-      vb[b] = r < m ? __ldg(vr + r) : 0ull;
+      cb[b] = r < hi ? __ldg(kr + r) : RG_EMPTY;
+      vb[b] = r < hi ? __ldg(vr + r) : 0ull;
     }
 #pragma unroll
     for (int b = 0; b < RG_B; ++b) {
-      const bool ok = r0 + 32 * b + lane < m;
+      const bool ok = r0 + 32 * b + lane < hi;
       const uint32_t c = cb[b];
       const uint32_t peers = __match_any_sync(FULL, c);
-      uint32_t s = 0, dst = 0;
+      const uint32_t lead = __ffs(peers) - 1;
+      uint32_t s = 0;
+      if (ok && lead == lane) s = rg_slot(tk, c);  // present: every CTA of the region is in the table
+      s = __shfl_sync(FULL, s, lead);
+      uint32_t dst = 0;
       if (ok) {
-        s = rg_slot(tk, c);  // present: every CTA of the region is in the table
         dst = to[s] + __popc(peers & lanemask_lt());
         kout[dst] = c;
         vout[dst] = vb[b];
@@ -233,7 +274,7 @@ cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, cons
   if ((e = exclusive_scan_u32(c, n1, n0, P, nullptr))) return e;
   // the offsets overwrite the pair counts (pn is no longer needed)
   CADV_LAUNCH(c, k_rg_offsets<<<grid, 256, 0, c->stream>>>(sv, n0, P, st.pn));
-  CADV_LAUNCH(c, k_rg_scatter<<<(unsigned)st.nregions, 32, 0, c->stream>>>(key, val, cnt, chunk, st.pk, st.pn, st.np,
+  CADV_LAUNCH(c, k_rg_scatter<<<(unsigned)st.nregions, RG_NT, 0, c->stream>>>(key, val, cnt, chunk, st.pk, st.pn, st.np,
                                                                            kout, vout));
   return cudaGetLastError();
 }

@@ -491,3 +491,16 @@ def test_regroup_tables_and_overflow(ctx, ctx_long, cadv, ctas):
         load(c, cadv, t)
         check_reuse(c, t, 128, 0)
         check_reuse(c, t, 32, 0, 1, 20)
+
+
+def test_cta_id_all_ones(ctx, cadv):
+    """CTA id 0xffffffff (the regroup tables' empty marker) in a reuse trace:
+    such a trace takes the radix-sort regroup and still matches the oracle."""
+    rng = np.random.default_rng(5)
+    n = 5000
+    cta = rng.choice(np.array([0, 7, 0xFFFFFFFF, 12345], dtype=np.uint64), n)
+    addr = 0x7F0000000000 + 128 * rng.integers(0, 300, n).astype(np.uint64)
+    t = _mk(addr, cta, tid=rng.integers(0, 64, n), meta=np.full(n, 2 << 2))
+    load(ctx, cadv, t)
+    check_reuse(ctx, t, 128, 0)
+    check_reuse(ctx, t, 128, 1)
