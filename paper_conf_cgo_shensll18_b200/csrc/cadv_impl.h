@@ -41,7 +41,7 @@ enum BufId {
   B_RD_ENT_IDX0, B_RD_ENT_IDX1, B_RD_XQ, B_RD_XQ2, B_RD_XTMP, B_DEFER, B_OUT2,
   B_ALIGN0, B_ALIGN1, B_ALIGN2, B_ALIGN3, B_ALIGN4, B_ALIGN5,
   B_XCH_K0, B_XCH_K1, B_XCH_V0, B_XCH_V1, B_XCH_CNT, B_COMM, B_OBJ, B_RD_ENT_ALL,
-  B_RG_PK, B_RG_PN, B_RG_NP, B_RG_SORT,
+  B_RG_PK, B_RG_PN, B_RG_NP, B_RG_SORT, B_RG_SEG,
   B_COUNT
 };
 
@@ -160,8 +160,11 @@ struct RgState {
 };
 cudaError_t rg_count(cadv_ctx* c, const uint32_t* key, const uint64_t* cnt, uint64_t nregions, uint64_t chunk,
                      RgState* st);
+// seg (nullable, >= P entries): the output's CTA segments (start, length), unordered;
+// seg_cm[0] = their number, seg_cm[1] = the longest (device)
 cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, const uint32_t* key,
-                      const uint64_t* val, const uint64_t* cnt, uint64_t chunk, uint32_t* kout, uint64_t* vout);
+                      const uint64_t* val, const uint64_t* cnt, uint64_t chunk, uint32_t* kout, uint64_t* vout,
+                      uint2* seg, unsigned int* seg_cm);
 
 struct RdState {
   int cta_scope = 1;

@@ -229,6 +229,24 @@ __global__ void __launch_bounds__(RG_NT) k_rg_scatter(const uint32_t* __restrict
   }
 }
 
+// 4. the CTA segments of the output: for every CTA's first sorted pair,
+//    (start, length) appended to seg (unordered: segments are independent);
+//    cnt_max[0] = number of segments, cnt_max[1] = longest segment
+__global__ void k_rg_segments(const uint32_t* __restrict__ sk, const uint32_t* __restrict__ sn,
+                              const uint32_t* __restrict__ so, uint64_t P, uint2* __restrict__ seg,
+                              unsigned int* __restrict__ cnt_max) {
+  for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < P; s += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t c = sk[s];
+    if (s > 0 && sk[s - 1] == c) continue;
+    uint32_t len = 0;
+    for (uint64_t x = s; x < P && sk[x] == c; ++x) len += sn[x];
+    if (len == 0) continue;
+    const uint32_t k = atomicAdd(&cnt_max[0], 1u);
+    seg[k] = make_uint2(so[s], len);
+    atomicMax(&cnt_max[1], len);
+  }
+}
+
 }  // namespace
 
 // Phase 1 (queued before the scan's synchronisation): per-region CTA counts.
@@ -254,7 +272,8 @@ cudaError_t rg_count(cadv_ctx* c, const uint32_t* key, const uint64_t* cnt, uint
 
 // Phases 2-3 (after the synchronisation; P = total pairs, no overflow).
 cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, const uint32_t* key,
-                      const uint64_t* val, const uint64_t* cnt, uint64_t chunk, uint32_t* kout, uint64_t* vout) {
+                      const uint64_t* val, const uint64_t* cnt, uint64_t chunk, uint32_t* kout, uint64_t* vout,
+                      uint2* seg, unsigned int* seg_cm) {
   void *b;
   cudaError_t e;
   // packed pairs (ping-pong for the sort) + counts + offsets
@@ -276,6 +295,10 @@ cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, cons
   CADV_LAUNCH(c, k_rg_offsets<<<grid, 256, 0, c->stream>>>(sv, n0, P, st.pn));
   CADV_LAUNCH(c, k_rg_scatter<<<(unsigned)st.nregions, RG_NT, 0, c->stream>>>(key, val, cnt, chunk, st.pk, st.pn, st.np,
                                                                            kout, vout));
+  if (seg) {  // the CTA segments of the output (count and longest in seg_cm)
+    if ((e = cudaMemsetAsync(seg_cm, 0, 16, c->stream))) return e;
+    CADV_LAUNCH(c, k_rg_segments<<<grid, 256, 0, c->stream>>>(res ? k1 : k0, n1, n0, P, seg, seg_cm));
+  }
   return cudaGetLastError();
 }
 

@@ -319,6 +319,168 @@ struct EntryCols {
 //   1  R < 2^52: packed u64 keys;  2: lines and positions in separate arrays.
 // The MODE 0 launch covers all tiles and lists the others (sc->count[4] /
 // tile_list + ntiles, sc->count[3] / wide_list) for the MODE 1 / 2 launches.
+// ------------------------------------------------------------------ R2-R4 segment kernel
+// CTA scope on one rank with every CTA segment <= 256 kept records (every
+// segment of the paper-shaped workloads at 128 B lines): the regroup knows
+// the segments, so no tiles are needed.  Persistent warps take whole
+// segments from a global counter and resolve each exactly like the tile
+// kernel's warp path (rounds of 32 records: previous use from
+// __match_any_sync or a per-warp line -> last-position hash table, weighted
+// prefix, reused-position bitmap + bit-sliced compare), but with 64-bit line
+// keys (no tile line range) and no block barrier until the final flush.
+constexpr int SG_NT = 256, SG_W = SG_NT / 32;
+struct SegSmem {
+  unsigned long long hk[SG_W][512];  // line -> (slot) ; ~0 = empty
+  uint16_t hp[SG_W][512];            // slot -> last position
+  uint32_t wpi[SG_W][256];           // inclusive weighted prefix by position
+  uint32_t rw[SG_W][16];             // reused-position bitmap [8] + word prefix counts [8]
+  uint32_t hist[TL_SMEM_BINS];
+};
+
+__global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ val, const uint2* __restrict__ seg,
+                                                  const unsigned int* __restrict__ seg_cm, unsigned int* next,
+                                                  int log2bins, uint32_t nbins, uint64_t* __restrict__ g_hist,
+                                                  uint64_t* __restrict__ g_stream, ObjTab O) {
+  extern __shared__ __align__(16) uint8_t sg_smem[];
+  SegSmem& S = *reinterpret_cast<SegSmem*>(sg_smem);
+  const uint32_t tx = threadIdx.x, warp = tx >> 5, lane = lane_id();
+  const uint32_t hbins = (O.n + 1) * nbins;
+  const bool smem_hist = hbins <= TL_SMEM_BINS;
+  if (smem_hist)
+    for (uint32_t k = tx; k < hbins; k += SG_NT) S.hist[k] = 0;
+  __syncthreads();
+  const uint32_t nseg = seg_cm[0];
+  unsigned long long* const HK = S.hk[warp];
+  uint16_t* const HP = S.hp[warp];
+  uint32_t* const WPI = S.wpi[warp];
+  uint32_t* const RW = S.rw[warp];
+  uint32_t* const CW8 = RW + 8;
+  uint32_t stream = 0;
+  unsigned long long rdsum = 0;
+  for (uint32_t sg = __shfl_sync(FULL, lane == 0 ? atomicAdd(next, 1u) : 0u, 0); sg < nseg;
+       sg = __shfl_sync(FULL, lane == 0 ? atomicAdd(next, 1u) : 0u, 0)) {
+    const uint2 sd = seg[sg];
+    const uint64_t* const vs = val + sd.x;
+    const uint32_t n = sd.y;  // <= 256 (the host checked the longest)
+    for (uint32_t k = lane; k < 512; k += 32) HK[k] = ~0ull;
+    if (lane < 8) { RW[lane] = 0; CW8[lane] = 0; }
+    __syncwarp();
+    uint32_t wb = 0, rtot = 0;          // running weight, reused positions (warp-uniform)
+    uint32_t qbits = 0, hbits = 0;      // this lane's positions 32 r + lane: query / has-dup flags
+    for (uint32_t r = 0; 32 * r < n; ++r) {
+      const uint32_t i = 32 * r + lane;
+      const bool valid = i < n;
+      const uint64_t v = valid ? __ldg(vs + i) : 0ull;
+      const unsigned long long line = valid ? (v & LINE_MASK) : ~0ull;
+      const bool st = (v >> VB_STORE) & 1u, hd = (v >> VB_DUP) & 1u;
+      const uint32_t w = valid ? (uint32_t)(v >> VB_W) + 1u : 0u;
+      // previous use of the line: an earlier lane of this round, else the table
+      const uint32_t peers = __match_any_sync(FULL, line);
+      const uint32_t lower = peers & lanemask_lt();
+      const uint32_t h0 = (uint32_t)((line * 0x9E3779B97F4A7C15ull) >> 55);
+      int32_t pp = -1;
+      if (valid) {
+        if (lower) {
+          pp = (int32_t)(32 * r + 31 - __clz(lower));
+        } else {
+          uint32_t h = h0;
+          while (true) {
+            const unsigned long long k = HK[h];
+            if (k == line) { pp = (int32_t)HP[h]; break; }
+            if (k == ~0ull) break;
+            h = (h + 1) & 511u;
+          }
+        }
+      }
+      const bool q = valid && !st && pp >= 0;  // a local query: RD = window - reused in window
+      const int32_t P = q ? pp : -1;
+      __syncwarp();
+      if (valid && (peers >> lane) == 1u) {  // the line's last lane in this round records it
+        uint32_t h = h0;
+        while (true) {  // lanes of other lines insert concurrently: claim slots with CAS
+          const unsigned long long k = atomicCAS(&HK[h], ~0ull, line);
+          if (k == ~0ull || k == line) break;
+          h = (h + 1) & 511u;
+        }
+        HP[h] = (uint16_t)i;
+      }
+      // weighted prefix (inclusive) by position
+      uint32_t xw = w;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, xw, o);
+        if (lane >= (uint32_t)o) xw += y;
+      }
+      if (valid) WPI[i] = wb + xw;
+      // reused positions inside the window (P, i): earlier rounds (bitmap R) ...
+      uint32_t cnt = 0;
+      if (q && (uint32_t)P < 32 * r) {
+        const uint32_t pw = (uint32_t)P >> 5, pb = (uint32_t)P & 31u;
+        cnt = rtot - (CW8[pw] + __popc(RW[pw] & (0xffffffffu >> (31u - pb))));
+      }
+      // ... and this round: lanes s < lane with P(s) > P (bit-sliced compare)
+      const uint32_t qm = __ballot_sync(FULL, q);
+      const uint32_t pv = q ? (uint32_t)P : 0u;
+      uint32_t gt = 0, eq = FULL;
+#pragma unroll
+      for (int kb = 7; kb >= 0; --kb) {
+        const uint32_t bk = __ballot_sync(FULL, (pv >> kb) & 1u);
+        if ((pv >> kb) & 1u) eq &= bk;
+        else { gt |= eq & bk; eq &= ~bk; }
+      }
+      cnt += __popc(gt & qm & lanemask_lt());
+      __syncwarp();
+      // R4
+      if (valid) {
+        uint32_t bin, cntb = 1;
+        if (q) {
+          const uint32_t rd = (wb + xw - w) - WPI[P] - cnt;
+          bin = rd_bin(rd, log2bins, nbins);
+          rdsum += rd;
+        } else {
+          bin = nbins - 1;
+          if (st) cntb = w;
+        }
+        if (O.n) bin += obj_row(O, line) * nbins;
+        if (smem_hist) atomicAdd(&S.hist[bin], cntb);
+        else atomicAdd((unsigned long long*)&g_hist[bin], (unsigned long long)cntb);
+        if (st) stream += w - 1;  // all but the last of merged stores are one-shot elements
+      }
+      qbits |= (uint32_t)q << r;
+      hbits |= (uint32_t)hd << r;
+      // R += { P(s) } of this round's queries; word prefix counts
+      if (q) atomicOr(&RW[(uint32_t)P >> 5], 1u << (P & 31));
+      __syncwarp();
+      const uint32_t nr = lane < 8 ? RW[lane] : 0u;
+      uint32_t pc = __popc(nr), xc = pc;
+#pragma unroll
+      for (int o = 1; o < 8; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, xc, o);
+        if (lane >= (uint32_t)o) xc += y;
+      }
+      if (lane < 8) CW8[lane] = xc - pc;
+      rtot = __shfl_sync(FULL, xc, 7);
+      wb += __shfl_sync(FULL, xw, 31);
+      __syncwarp();
+    }
+    // streaming: positions whose element is never used again (not reused, no dup)
+    for (uint32_t r = 0; 32 * r < n; ++r) {
+      const uint32_t i = 32 * r + lane;
+      if (i < n && !((qbits >> r) & 1u) && !((hbits >> r) & 1u) && !((RW[i >> 5] >> (i & 31u)) & 1u)) stream += 1;
+    }
+    __syncwarp();
+  }
+  stream = __reduce_add_sync(FULL, stream);
+  if (lane == 0 && stream) atomicAdd((unsigned long long*)g_stream, (unsigned long long)stream);
+#pragma unroll
+  for (int o = 16; o; o >>= 1) rdsum += __shfl_xor_sync(FULL, rdsum, o);
+  if (lane == 0 && rdsum) atomicAdd((unsigned long long*)g_stream + 1, rdsum);
+  __syncthreads();
+  if (smem_hist)
+    for (uint32_t k = tx; k < hbins; k += SG_NT)
+      if (S.hist[k]) atomicAdd((unsigned long long*)&g_hist[k], (unsigned long long)S.hist[k]);
+}
+
 template <int MODE>
 __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     k_rd_tile(const uint32_t* __restrict__ key, const uint64_t* __restrict__ val, uint64_t K,
@@ -1355,11 +1517,36 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
       int bits = bits_for(c->max_cta);
       if (bits == 0) bits = 1;
       if (hs[3] == 0) {  // every region's CTAs fit its table
-        if ((e = rg_finish(c, S.rgs, hs[2], bits, (const uint32_t*)k1, (const uint64_t*)v1, S.blkcnt, S.chunk_cap,
-                           (uint32_t*)k0, (uint64_t*)v0)))
+        const uint64_t P = hs[2];
+        void* sb;
+        if ((e = ensure(c, B_RG_SEG, (P + 16) * 8 + 64, &sb))) return e;
+        uint2* seg = (uint2*)sb;
+        unsigned int* seg_cm = (unsigned int*)((uint8_t*)sb + (P + 16) * 8);  // count, longest, next
+        if ((e = rg_finish(c, S.rgs, P, bits, (const uint32_t*)k1, (const uint64_t*)v1, S.blkcnt, S.chunk_cap,
+                           (uint32_t*)k0, (uint64_t*)v0, seg, seg_cm)))
           return e;
         key = (const uint32_t*)k0;
         val = (const uint64_t*)v0;
+        // every CTA segment <= 256 kept records: the segment kernel, no tiles
+        unsigned int* hcm = (unsigned int*)((uint8_t*)c->hstage + 40);
+        if ((e = cudaMemcpyAsync(hcm, seg_cm, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+        if ((e = cudaStreamSynchronize(c->stream))) return e;
+        if (hcm[1] <= 256u && getenv("CADV_RD_TILES") == nullptr) {
+          static bool seg_smem_set = false;
+          if (!seg_smem_set) {
+            if ((e = cudaFuncSetAttribute(k_rd_seg, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SegSmem))))
+              return e;
+            seg_smem_set = true;
+          }
+          if (hcm[0]) {
+            const unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * 4, (hcm[0] + SG_W - 1) / SG_W);
+            CADV_LAUNCH(c, k_rd_seg<<<grid, SG_NT, sizeof(SegSmem), c->stream>>>(val, seg, seg_cm, seg_cm + 2, log2bins,
+                                                                                nbins, d_hist, d_stats, O));
+          }
+          c->counts[1] = 0;
+          c->counts[3] = 0;
+          return cudaGetLastError();
+        }
       } else {  // overflow: pack, then the radix sort
         if ((e = launch_squeeze(c, (const uint32_t*)k1, (const uint64_t*)v1, (uint32_t*)k0, (uint64_t*)v0, S.blkcnt,
                                 S.blkcnt + S.grid + 4, S.grid, S.chunk_cap)))
