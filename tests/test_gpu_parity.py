@@ -504,3 +504,25 @@ def test_cta_id_all_ones(ctx, cadv):
     load(ctx, cadv, t)
     check_reuse(ctx, t, 128, 0)
     check_reuse(ctx, t, 128, 1)
+
+
+@pytest.mark.parametrize("case", [("srad", dict(rows=128, cols=128, iters=2)), ("bfs", dict(nodes=20000, seed=3)),
+                                  ("rand", dict(seed=12, ctas=30, threads=64, instrs=10, lines=40, pstore=0.3))])
+def test_segment_kernel_equals_tiles(ctx, cadv, case):
+    """CTA segments of <= 256 kept records go to the segment kernel (k_rd_seg);
+    CADV_RD_TILES forces the tile kernels on the same trace: both equal the
+    oracle (histogram, stats incl. streaming and the finite sum), both bin modes."""
+    import os
+    name, kw = case
+    t = tg.generate(name, **kw)
+    load(ctx, cadv, t)
+    for lb, binning, nb in ((128, 0, 66), (32, 1, 20)):
+        ref = orc.reuse(t, lb, 0, binning, nb)
+        seg = ctx.reuse_histogram(lb, 0, binning, nb)
+        os.environ["CADV_RD_TILES"] = "1"
+        try:
+            til = ctx.reuse_histogram(lb, 0, binning, nb)
+        finally:
+            del os.environ["CADV_RD_TILES"]
+        for h, st in (seg, til):
+            assert (h == ref[0]).all() and st == ref[1], (name, lb)
