@@ -437,7 +437,8 @@ def main():
     # ---- e2e: the same step through the C ABI with HOST buffers (H2D inside the timed region)
     e2e = None
     if args.e2e_steps > 0 and not args.profile_run:
-        host = {k: t.cols[k] for k in cadv.COLUMNS}
+        # the step's inputs in pinned host memory (copied to the device inside the timed region)
+        host = {k: torch.from_numpy(t.cols[k]).pin_memory() for k in cadv.COLUMNS}
         step(host, allreduce=False)  # warm the host-copy workspace
         if world > 1:
             dist.barrier()

@@ -377,30 +377,35 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
       // previous use of the line: an earlier lane of this round, else the table
       const uint32_t peers = __match_any_sync(FULL, line);
       const uint32_t lower = peers & lanemask_lt();
-      const uint32_t h0 = (uint32_t)((line * 0x9E3779B97F4A7C15ull) >> 55);
       int32_t pp = -1;
+      uint32_t hs = 0;  // the group's first lane: the line's slot (bit 16: present) or the first empty slot
       if (valid) {
         if (lower) {
           pp = (int32_t)(32 * r + 31 - __clz(lower));
         } else {
-          uint32_t h = h0;
+          uint32_t h = (uint32_t)((line * 0x9E3779B97F4A7C15ull) >> 55);
           while (true) {
             const unsigned long long k = HK[h];
-            if (k == line) { pp = (int32_t)HP[h]; break; }
-            if (k == ~0ull) break;
+            if (k == line) { pp = (int32_t)HP[h]; hs = h | 0x10000u; break; }
+            if (k == ~0ull) { hs = h; break; }
             h = (h + 1) & 511u;
           }
         }
       }
+      hs = __shfl_sync(FULL, hs, __ffs(peers) - 1);
       const bool q = valid && !st && pp >= 0;  // a local query: RD = window - reused in window
       const int32_t P = q ? pp : -1;
       __syncwarp();
       if (valid && (peers >> lane) == 1u) {  // the line's last lane in this round records it
-        uint32_t h = h0;
-        while (true) {  // lanes of other lines insert concurrently: claim slots with CAS
-          const unsigned long long k = atomicCAS(&HK[h], ~0ull, line);
-          if (k == ~0ull || k == line) break;
-          h = (h + 1) & 511u;
+        uint32_t h = hs & 511u;
+        if (!(hs >> 16)) {
+          // new line: claim a slot from the first empty one the probe saw (lanes
+          // of other new lines insert concurrently, so with CAS)
+          while (true) {
+            const unsigned long long k = atomicCAS(&HK[h], ~0ull, line);
+            if (k == ~0ull || k == line) break;
+            h = (h + 1) & 511u;
+          }
         }
         HP[h] = (uint16_t)i;
       }
