@@ -175,12 +175,18 @@ __global__ void __launch_bounds__(RG_NT) k_rg_scatter(const uint32_t* __restrict
   const uint64_t* vr = val + (uint64_t)w * chunk;
   const uint64_t rounds = (m + 31) / 32, per = (rounds + RG_W - 1) / RG_W;
   const uint64_t lo = min(m, q * per * 32), hi = min(m, (q + 1) * per * 32);
-  // (a) count the slice's CTAs
-  for (uint64_t r = lo; r < hi; r += 32) {
-    const bool ok = r + lane < hi;
-    const uint32_t c = ok ? __ldg(kr + r + lane) : RG_EMPTY;
-    const uint32_t peers = __match_any_sync(FULL, c);
-    if (ok && (uint32_t)(__ffs(peers) - 1) == lane) st[q][rg_slot(tk, c)] += __popc(peers);
+  // (a) count the slice's CTAs (loads of 4 rounds issued together)
+  for (uint64_t r0 = lo; r0 < hi; r0 += 128) {
+    uint32_t cb[4];
+#pragma unroll
+    for (int b = 0; b < 4; ++b) cb[b] = r0 + 32 * b + lane < hi ? __ldg(kr + r0 + 32 * b + lane) : RG_EMPTY;
+#pragma unroll
+    for (int b = 0; b < 4; ++b) {
+      const bool ok = r0 + 32 * b + lane < hi;
+      const uint32_t peers = __match_any_sync(FULL, cb[b]);
+      if (ok && (uint32_t)(__ffs(peers) - 1) == lane) st[q][rg_slot(tk, cb[b])] += __popc(peers);
+      __syncwarp();
+    }
   }
   __syncthreads();
   // (b) slice starts = the CTA's region offset + its records in earlier slices
