@@ -357,11 +357,18 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
   uint32_t* const CW8 = RW + 8;
   uint32_t stream = 0;
   unsigned long long rdsum = 0;
-  for (uint32_t sg = __shfl_sync(FULL, lane == 0 ? atomicAdd(next, 1u) : 0u, 0); sg < nseg;
-       sg = __shfl_sync(FULL, lane == 0 ? atomicAdd(next, 1u) : 0u, 0)) {
-    const uint2 sd = seg[sg];
+  // The next segment is claimed (and its descriptor and first round loaded)
+  // while the current one is resolved; round r + 1's records are loaded at
+  // the top of round r.  Segments are independent, so the claim order does
+  // not matter.
+  uint32_t sg = __shfl_sync(FULL, lane == 0 ? atomicAdd(next, 1u) : 0u, 0);
+  uint2 sd = sg < nseg ? seg[sg] : make_uint2(0u, 0u);
+  uint64_t vnext = lane < sd.y ? __ldg(val + sd.x + lane) : 0ull;
+  while (sg < nseg) {
     const uint64_t* const vs = val + sd.x;
     const uint32_t n = sd.y;  // <= 256 (the host checked the longest)
+    const uint32_t sg_n = __shfl_sync(FULL, lane == 0 ? atomicAdd(next, 1u) : 0u, 0);
+    const uint2 sd_n = sg_n < nseg ? seg[sg_n] : make_uint2(0u, 0u);
     for (uint32_t k = lane; k < 512; k += 32) HK[k] = ~0ull;
     if (lane < 8) { RW[lane] = 0; CW8[lane] = 0; }
     __syncwarp();
@@ -370,7 +377,8 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
     for (uint32_t r = 0; 32 * r < n; ++r) {
       const uint32_t i = 32 * r + lane;
       const bool valid = i < n;
-      const uint64_t v = valid ? __ldg(vs + i) : 0ull;
+      const uint64_t v = vnext;
+      vnext = (i + 32 < n) ? __ldg(vs + i + 32) : 0ull;
       const unsigned long long line = valid ? (v & LINE_MASK) : ~0ull;
       const bool st = (v >> VB_STORE) & 1u, hd = (v >> VB_DUP) & 1u;
       const uint32_t w = valid ? (uint32_t)(v >> VB_W) + 1u : 0u;
@@ -474,6 +482,9 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
       if (i < n && !((qbits >> r) & 1u) && !((hbits >> r) & 1u) && !((RW[i >> 5] >> (i & 31u)) & 1u)) stream += 1;
     }
     __syncwarp();
+    sg = sg_n;
+    sd = sd_n;
+    vnext = lane < sd.y ? __ldg(val + sd.x + lane) : 0ull;
   }
   stream = __reduce_add_sync(FULL, stream);
   if (lane == 0 && stream) atomicAdd((unsigned long long*)g_stream, (unsigned long long)stream);
