@@ -329,9 +329,13 @@ struct EntryCols {
 // prefix, reused-position bitmap + bit-sliced compare), but with 64-bit line
 // keys (no tile line range) and no block barrier until the final flush.
 constexpr int SG_NT = 256, SG_W = SG_NT / 32;
+// 384 hash slots per warp (load factor <= 2/3 at 256 distinct lines) keep the
+// CTA under 40 KB of shared memory: 5 CTAs (40 warps) per SM.  The histogram
+// is last so that the launch allocates only the bins it uses.
+constexpr uint32_t SG_HS = 384;
 struct SegSmem {
-  unsigned long long hk[SG_W][512];  // line -> (slot) ; ~0 = empty
-  uint16_t hp[SG_W][512];            // slot -> last position
+  unsigned long long hk[SG_W][SG_HS];  // line -> (slot) ; ~0 = empty
+  uint16_t hp[SG_W][SG_HS];            // slot -> last position
   uint32_t wpi[SG_W][256];           // inclusive weighted prefix by position
   uint32_t rw[SG_W][16];             // reused-position bitmap [8] + word prefix counts [8]
   uint32_t hist[TL_SMEM_BINS];
@@ -369,7 +373,7 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
     const uint32_t n = sd.y;  // <= 256 (the host checked the longest)
     const uint32_t sg_n = __shfl_sync(FULL, lane == 0 ? atomicAdd(next, 1u) : 0u, 0);
     const uint2 sd_n = sg_n < nseg ? seg[sg_n] : make_uint2(0u, 0u);
-    for (uint32_t k = lane; k < 512; k += 32) HK[k] = ~0ull;
+    for (uint32_t k = lane; k < SG_HS; k += 32) HK[k] = ~0ull;
     if (lane < 8) { RW[lane] = 0; CW8[lane] = 0; }
     __syncwarp();
     uint32_t wb = 0, rtot = 0;          // running weight, reused positions (warp-uniform)
@@ -391,12 +395,12 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
         if (lower) {
           pp = (int32_t)(32 * r + 31 - __clz(lower));
         } else {
-          uint32_t h = (uint32_t)((line * 0x9E3779B97F4A7C15ull) >> 55);
+          uint32_t h = __umulhi((uint32_t)((line * 0x9E3779B97F4A7C15ull) >> 32), SG_HS);
           while (true) {
             const unsigned long long k = HK[h];
             if (k == line) { pp = (int32_t)HP[h]; hs = h | 0x10000u; break; }
             if (k == ~0ull) { hs = h; break; }
-            h = (h + 1) & 511u;
+            h = h + 1 == SG_HS ? 0u : h + 1;
           }
         }
       }
@@ -405,14 +409,14 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
       const int32_t P = q ? pp : -1;
       __syncwarp();
       if (valid && (peers >> lane) == 1u) {  // the line's last lane in this round records it
-        uint32_t h = hs & 511u;
+        uint32_t h = hs & 0xffffu;
         if (!(hs >> 16)) {
           // new line: claim a slot from the first empty one the probe saw (lanes
           // of other new lines insert concurrently, so with CAS)
           while (true) {
             const unsigned long long k = atomicCAS(&HK[h], ~0ull, line);
             if (k == ~0ull || k == line) break;
-            h = (h + 1) & 511u;
+            h = h + 1 == SG_HS ? 0u : h + 1;
           }
         }
         HP[h] = (uint16_t)i;
@@ -1555,8 +1559,18 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
             seg_smem_set = true;
           }
           if (hcm[0]) {
-            const unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * 4, (hcm[0] + SG_W - 1) / SG_W);
-            CADV_LAUNCH(c, k_rd_seg<<<grid, SG_NT, sizeof(SegSmem), c->stream>>>(val, seg, seg_cm, seg_cm + 2, log2bins,
+            const uint64_t hbins = (uint64_t)(O.n + 1) * nbins;
+            const size_t smem = offsetof(SegSmem, hist) + (hbins <= TL_SMEM_BINS ? 4 * hbins : 0);
+            static int seg_ctas = 0;
+            static size_t seg_ctas_smem = 0;
+            if (seg_ctas_smem != smem) {
+              if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&seg_ctas, k_rd_seg, SG_NT, smem))) return e;
+              if (seg_ctas < 1) seg_ctas = 1;
+              seg_ctas_smem = smem;
+            }
+            const unsigned grid =
+                (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * seg_ctas, (hcm[0] + SG_W - 1) / SG_W);
+            CADV_LAUNCH(c, k_rd_seg<<<grid, SG_NT, smem, c->stream>>>(val, seg, seg_cm, seg_cm + 2, log2bins,
                                                                                 nbins, d_hist, d_stats, O));
           }
           c->counts[1] = 0;

@@ -526,3 +526,38 @@ def test_segment_kernel_equals_tiles(ctx, cadv, case):
             del os.environ["CADV_RD_TILES"]
         for h, st in (seg, til):
             assert (h == ref[0]).all() and st == ref[1], (name, lb)
+
+
+@pytest.mark.parametrize("reuse_frac", [0.0, 0.25])
+def test_segment_kernel_full_hash_tables(ctx, cadv, reuse_frac):
+    """Every CTA segment holds exactly 256 kept records (the segment kernel's
+    limit) over up to 256 distinct random lines spread across a 2^40-line
+    range: each warp's hash table runs at its highest load, with long probe
+    chains and wrap-around; the result equals the oracle and the tile path."""
+    import os
+    rng = np.random.default_rng(31)
+    nct, per = 300, 256
+    addr, cta = [], []
+    for c in range(nct):
+        nd = per - int(per * reuse_frac)
+        lines = rng.choice(1 << 40, nd, replace=False).astype(np.uint64)
+        seq = np.concatenate([lines, rng.choice(lines, per - nd)])
+        rng.shuffle(seq)
+        for k in range(1, per):  # no two consecutive equal lines (no duplicate-load compression)
+            if seq[k] == seq[k - 1]:
+                seq[k], seq[0] = seq[0], seq[k]
+        addr.append(0x10000000000 + 128 * seq)
+        cta.append(np.full(per, c, dtype=np.uint64))
+    addr, cta = np.concatenate(addr), np.concatenate(cta)
+    meta = np.where(rng.random(len(addr)) < 0.1, (2 << 2) | 1, 2 << 2)
+    t = _mk(addr, cta, tid=rng.integers(0, 256, len(addr)), meta=meta)
+    load(ctx, cadv, t)
+    ref = orc.reuse(t, 128, 0, 0, 66)
+    seg = ctx.reuse_histogram(128, 0, 0, 66)
+    os.environ["CADV_RD_TILES"] = "1"
+    try:
+        til = ctx.reuse_histogram(128, 0, 0, 66)
+    finally:
+        del os.environ["CADV_RD_TILES"]
+    for h, st in (seg, til):
+        assert (h == ref[0]).all() and st == ref[1]
