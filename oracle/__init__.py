@@ -8,6 +8,7 @@ Functions follow PAPER.md (see oracle.cpp header for the passages):
   reuse(trace, ...)        LRU-stack reuse-distance histogram
   reuse_rd(trace, ...)     per-record reuse distances
   reuse_brute(trace, ...)  O(n^2) literal definition
+  reuse_fenwick(trace, ...) Fenwick-tree distinct counts (same outputs; large traces)
   mem_div(trace, ...)      unique lines per warp instruction
   branch_div(trace, ...)   divergent warp-level block executions
   data_centric(trace, objects, ...)  per-data-object RD / MD histograms
@@ -47,11 +48,12 @@ def _load():
     lib.oracle_reuse.argtypes = [P, P, P, P, u64, u32, i32, i32, u32, P, P]
     lib.oracle_reuse_rd.argtypes = [P, P, P, P, u64, u32, i32, P]
     lib.oracle_reuse_brute.argtypes = [P, P, P, P, u64, u32, i32, i32, u32, P, P, P]
+    lib.oracle_reuse_fenwick.argtypes = [P, P, P, P, u64, u32, i32, i32, u32, P, P]
     lib.oracle_mem_div.argtypes = [P, P, P, P, P, P, u64, u32, u32, u32, P, P]
     lib.oracle_branch_div.argtypes = [P, P, P, P, P, u64, u32, u32, P, P]
-    lib.oracle_data_centric.argtypes = [P, P, P, P, P, u64, P, P, u32, u32, i32, i32, u32, u32, P, P]
+    lib.oracle_data_centric.argtypes = [P, P, P, P, P, P, u64, P, P, u32, u32, i32, i32, u32, u32, P, P]
     for f in ("oracle_reuse", "oracle_reuse_rd", "oracle_reuse_brute", "oracle_mem_div",
-              "oracle_branch_div", "oracle_data_centric", "oracle_num_threads"):
+              "oracle_branch_div", "oracle_data_centric", "oracle_num_threads", "oracle_reuse_fenwick"):
         getattr(lib, f).restype = ctypes.c_int
     _lib = lib
     return lib
@@ -77,6 +79,17 @@ def reuse(t, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66):
     st = np.zeros(5, np.uint64)
     _check(lib.oracle_reuse(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.meta), t.n, line_bytes, scope, binning,
                             nbins, _p(hist), _p(st)))
+    return hist, dict(zip(("accesses", "inf", "streaming", "overflow", "finite_sum"), map(int, st)))
+
+
+def reuse_fenwick(t, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66):
+    """Same outputs as reuse(), Fenwick-tree (Bennett-Kruskal) distinct counts:
+    O(n log n) per scope, for kernel scope at full size."""
+    lib = _load()
+    hist = np.zeros(nbins, np.uint64)
+    st = np.zeros(5, np.uint64)
+    _check(lib.oracle_reuse_fenwick(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.meta), t.n, line_bytes, scope, binning,
+                                    nbins, _p(hist), _p(st)))
     return hist, dict(zip(("accesses", "inf", "streaming", "overflow", "finite_sum"), map(int, st)))
 
 
@@ -131,7 +144,7 @@ def data_centric(t, objects, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEA
     k = len(base)
     rh = np.zeros((k + 1, nbins), np.uint64) if rd else None
     mh = np.zeros((k + 1, 2, warp_size + 1), np.uint64) if md else None
-    _check(lib.oracle_data_centric(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.winst), _p(t.meta), t.n, _p(base), _p(nb),
+    _check(lib.oracle_data_centric(_p(t.addr), _p(t.cta), _p(t.tid), _p(t.winst), _p(t.site), _p(t.meta), t.n, _p(base), _p(nb),
                                    k, line_bytes, scope, binning, nbins, warp_size, _p(rh), _p(mh)))
     return rh, mh
 

@@ -16,10 +16,14 @@
 //     accesses "never reused by the same CTA".
 //       - oracle_reuse: explicit LRU stack of renamed (line, write-epoch) keys.
 //       - oracle_reuse_brute: literal O(n^2) definition (tiny traces only).
+//       - oracle_reuse_fenwick: Fenwick-tree (Bennett-Kruskal) distinct
+//         counts, O(n log n) per scope (large traces, kernel scope).
 //   * memory divergence: "the number of unique cache lines touched by each
 //     instruction", per dynamic warp-level instruction, a std::set
 //     of lines per group (group identity = (cta, tid / W, winst), DESIGN.md
 //     reading R9); degree = weighted average left to the caller.
+//     A group's records must share kind and site (one static instruction,
+//     P:L235 / P:L345; reading R19), else BAD_TRACE.
 //   * branch divergence: how many times a block executes, how many threads,
 //     how often it makes the warp diverge; divergent = fewer active
 //     lanes than launched lanes of that warp (reading R12).
@@ -51,8 +55,9 @@ bool pow2(uint32_t x) { return x && !(x & (x - 1)); }
 
 // Per-record validity (include/cadv.h "Per-record validity"), checked over
 // the columns an analysis reads: kind <= 2, reserved meta bits 5..7 zero;
-// memory records: log2 bytes <= 4, naturally aligned, addr < 2^58 (when the
-// address column is read); tid < 1024 (when the tid column is read).
+// memory records: log2 bytes <= 4, naturally aligned (when the address column
+// is read; any 64-bit effective address, "Record(i8* addr, ...)");
+// tid < 1024 (when the tid column is read).
 bool record_ok(const uint64_t* addr, const uint16_t* tid, const uint8_t* meta, uint64_t i) {
   uint32_t kind = meta[i] & 3u;
   if (kind == 3 || (meta[i] >> 5) != 0) return false;
@@ -63,7 +68,6 @@ bool record_ok(const uint64_t* addr, const uint16_t* tid, const uint8_t* meta, u
     if (addr) {
       uint64_t bytes = 1ull << lg;
       if (addr[i] % bytes != 0) return false;
-      if (addr[i] >> 58) return false;
     }
   }
   return true;
@@ -72,6 +76,26 @@ bool record_ok(const uint64_t* addr, const uint16_t* tid, const uint8_t* meta, u
 bool check_all(const uint64_t* addr, const uint16_t* tid, const uint8_t* meta, uint64_t n) {
   for (uint64_t i = 0; i < n; ++i)
     if (!record_ok(addr, tid, meta, i)) return false;
+  return true;
+}
+
+// Group invariant (include/cadv.h "Group validity", reading R19):
+// the records of one dynamic warp-level instruction (cta, tid / 32, winst)
+// of a family (memory or basic block) come from ONE static instruction
+// (P:L235 one Record() call site per instrumented load/store; P:L345 one
+// passBasicBlock() per block), so they share kind and site.  Checked by the
+// divergence analyses over the family they analyse.
+bool groups_uniform(const uint32_t* cta, const uint16_t* tid, const uint32_t* winst, const uint32_t* site,
+                    const uint8_t* meta, uint64_t n, bool bb_family) {
+  std::map<std::tuple<uint32_t, uint32_t, uint32_t>, std::pair<uint32_t, uint32_t>> first;  // -> (kind, site)
+  for (uint64_t i = 0; i < n; ++i) {
+    const uint32_t kind = meta[i] & 3u;
+    if ((kind == KIND_BB) != bb_family) continue;
+    auto key = std::make_tuple(cta[i], (uint32_t)tid[i] / 32u, winst[i]);
+    auto it = first.find(key);
+    if (it == first.end()) first.emplace(key, std::make_pair(kind, site[i]));
+    else if (it->second.first != kind || it->second.second != site[i]) return false;
+  }
   return true;
 }
 
@@ -277,6 +301,82 @@ int oracle_reuse_brute(const uint64_t* addr, const uint32_t* cta, const uint16_t
   return OK;
 }
 
+// Reuse-distance histogram, large-trace variant ("the
+// Fenwick-tree (Bennett-Kruskal) CPU variant ... cross-checked == LRU"):
+// the same definition as oracle_reuse (P:L248 distinct elements between two
+// consecutive uses; the write rule of P:L248/L252 renames the element), with
+// the distinct count taken from a Fenwick tree over the scope's positions
+// that holds a 1 at the LAST access of every renamed element seen so far:
+// RD(k) = number of marks strictly between the previous use p and k (each
+// marked position is a distinct element used in the window, and every
+// element used in the window has its last use there).  O(n log n) per scope
+// instead of the stack walk's O(n * depth), so kernel scope at full size
+// finishes.  Same outputs and error codes as oracle_reuse.
+namespace {
+void fenwick_scope(const std::vector<uint64_t>& idx, const uint64_t* addr, const uint8_t* meta, uint32_t line_bytes,
+                   int binning, uint32_t nbins, std::vector<uint64_t>& h, uint64_t& streaming, uint64_t& fsum) {
+  const size_t m = idx.size();
+  std::vector<uint32_t> bit(m + 1, 0);  // Fenwick tree, 1-based
+  auto add = [&](size_t pos, int32_t v) { for (size_t x = pos + 1; x <= m; x += x & (0 - x)) bit[x] += (uint32_t)v; };
+  auto prefix = [&](size_t pos) {  // marks at positions < pos
+    uint64_t r = 0;
+    for (size_t x = pos; x > 0; x -= x & (0 - x)) r += bit[x];
+    return r;
+  };
+  std::unordered_map<uint64_t, uint64_t> epoch;                 // e(s, line)
+  std::unordered_map<RKey, std::pair<uint64_t, uint64_t>, KeyHash> last;  // key -> (last position, uses)
+  for (size_t k = 0; k < m; ++k) {
+    const uint64_t i = idx[k];
+    const uint64_t line = addr[i] / line_bytes;
+    const bool store = (meta[i] & 3u) == KIND_STORE;
+    RKey key{line, store ? ++epoch[line] : epoch[line]};
+    auto it = last.find(key);
+    if (it == last.end()) {                   // first use of the (renamed) element: ∞
+      h[nbins - 1]++;
+      last.emplace(key, std::make_pair((uint64_t)k, (uint64_t)1));
+    } else {
+      const uint64_t p = it->second.first;
+      const uint64_t d = prefix(k) - prefix(p + 1);
+      h[bin_of(d, binning, nbins)]++;
+      fsum += d;
+      add(p, -1);
+      it->second.first = k;
+      it->second.second++;
+    }
+    add(k, 1);
+  }
+  for (auto& kv : last) if (kv.second.second == 1) streaming++;
+}
+}  // namespace
+
+extern "C" int oracle_reuse_fenwick(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid, const uint8_t* meta,
+                                    uint64_t n, uint32_t line_bytes, int scope, int binning, uint32_t nbins,
+                                    uint64_t* hist, uint64_t* stats) {
+  int rc = check_reuse_args(line_bytes, scope, binning, nbins);
+  if (rc) return rc;
+  if (!check_all(addr, nullptr, meta, n)) return BAD_TRACE;
+  auto sc = scopes_of(cta, meta, n, scope);
+  std::vector<uint64_t> h(nbins, 0);
+  uint64_t streaming = 0, fsum = 0;
+#pragma omp parallel
+  {
+    std::vector<uint64_t> hl(nbins, 0);
+    uint64_t sl = 0, fl = 0;
+#pragma omp for schedule(dynamic, 1)
+    for (int64_t s = 0; s < (int64_t)sc.size(); ++s) fenwick_scope(sc[s], addr, meta, line_bytes, binning, nbins, hl, sl, fl);
+#pragma omp critical
+    {
+      for (uint32_t b = 0; b < nbins; ++b) h[b] += hl[b];
+      streaming += sl;
+      fsum += fl;
+    }
+  }
+  uint64_t acc = 0;
+  for (uint32_t b = 0; b < nbins; ++b) { hist[b] = h[b]; acc += h[b]; }
+  stats[0] = acc; stats[1] = h[nbins - 1]; stats[2] = streaming; stats[3] = h[nbins - 2]; stats[4] = fsum;
+  return OK;
+}
+
 // Memory divergence: per dynamic warp-level load/store, the number
 // of unique cache lines touched.  Group = (cta, tid / W, winst) over memory
 // records.  hist[2][W+1] (row 0 loads, row 1 stores; column = degree);
@@ -287,6 +387,7 @@ int oracle_mem_div(const uint64_t* addr, const uint32_t* cta, const uint16_t* ti
   if (!pow2(line_bytes) || line_bytes > 4096) return INVALID_ARG;
   if (!pow2(warp_size) || warp_size > 32) return INVALID_ARG;
   if (!check_all(addr, tid, meta, n)) return BAD_TRACE;
+  if (!groups_uniform(cta, tid, winst, site, meta, n, false)) return BAD_TRACE;
   for (uint64_t i = 0; i < n; ++i)
     if ((meta[i] & 3u) != KIND_BB && per_site && site[i] >= nsites) return INVALID_ARG;
   const uint32_t W = warp_size;
@@ -349,6 +450,7 @@ int oracle_branch_div(const uint32_t* cta, const uint16_t* tid, const uint32_t* 
                       uint64_t* totals) {
   if (!pow2(warp_size) || warp_size > 32) return INVALID_ARG;
   if (!check_all(nullptr, tid, meta, n)) return BAD_TRACE;
+  if (!groups_uniform(cta, tid, winst, site, meta, n, true)) return BAD_TRACE;
   for (uint64_t i = 0; i < n; ++i)
     if ((meta[i] & 3u) == KIND_BB && per_site && site[i] >= nsites) return INVALID_ARG;
   const uint32_t W = warp_size;
@@ -425,7 +527,7 @@ int oracle_branch_div(const uint32_t* cta, const uint16_t* tid, const uint32_t* 
 //     its first record's line.
 // Rows are found by a linear scan over the table (the definition).
 int oracle_data_centric(const uint64_t* addr, const uint32_t* cta, const uint16_t* tid, const uint32_t* winst,
-                        const uint8_t* meta, uint64_t n, const uint64_t* obj_base, const uint64_t* obj_bytes,
+                        const uint32_t* site, const uint8_t* meta, uint64_t n, const uint64_t* obj_base, const uint64_t* obj_bytes,
                         uint32_t nobj, uint32_t line_bytes, int scope, int binning, uint32_t nbins,
                         uint32_t warp_size, uint64_t* rd_hist, uint64_t* md_hist) {
   if (!rd_hist && !md_hist) return INVALID_ARG;
@@ -439,6 +541,7 @@ int oracle_data_centric(const uint64_t* addr, const uint32_t* cta, const uint16_
     if (k > 0 && (obj_base[k - 1] + obj_bytes[k - 1] - 1) / L >= obj_base[k] / L) return INVALID_ARG;
   }
   if (!check_all(addr, md_hist ? tid : nullptr, meta, n)) return BAD_TRACE;
+  if (md_hist && !groups_uniform(cta, tid, winst, site, meta, n, false)) return BAD_TRACE;
   auto row_of_line = [&](uint64_t line) -> uint32_t {
     const uint64_t lo = line * L, hi = lo + L;  // the line's bytes [lo, hi)
     for (uint32_t k = 0; k < nobj; ++k)

@@ -528,3 +528,126 @@ def test_data_centric_rejects_bad_tables():
             orc.data_centric(t, (np.array(base, np.uint64), np.array(nb, np.uint64)), 128)
     # the same pair is fine at 64 B lines (no line intersects both)
     orc.data_centric(t, (np.array([b, b + 64], np.uint64), np.array([64, 64], np.uint64)), 64)
+
+
+# ----------------------------------------------------------------- round 2 pins
+
+def test_vecadd_md_per_site_closed_form():
+    """Config 1 per site (P:L264 per instruction): each of ld a / ld b / st c
+    is 22 warp-level instructions (683 = 10*64 + 43: warp 0 runs 11 full
+    iterations, warp 1 runs 11, the last with 11 lanes); a full group covers
+    128 contiguous bytes = 1 line at 128 B, 4 at 32 B; the 11-lane group
+    covers bytes 2688..2731 = 1 line at 128 B, 2 at 32 B ->
+    {22, 22} at 128 B and {22, 21*4 + 2 = 86} at 32 B."""
+    t = tg.generate("vecadd")
+    _, ps = orc.mem_div(t, 128)
+    mem_sites = sorted(set(t.site[(t.meta & 3) != BB].tolist()))
+    assert len(mem_sites) == 3
+    for s in mem_sites:
+        assert list(ps[s]) == [22, 22]
+    _, ps = orc.mem_div(t, 32)
+    for s in mem_sites:
+        assert list(ps[s]) == [22, 86]
+    assert ps.sum(axis=0).tolist() == [66, 258]
+
+
+def test_sgemm_md_per_site_closed_form():
+    """Config 2 per site: naive ld A[row*N+k] (2 rows, one k -> 2 lines at any
+    L), ld B[k*N+col] (16 consecutive floats = 64 B, 64-B aligned -> 1 line at
+    128 B, 2 at 32 B), st C (2 rows x 64 B -> 2 / 4); 256 CTAs x 8 warps x 256
+    iterations = 524,288 groups per loop site, 2,048 per store; tiled: 16 tile
+    steps -> 32,768 groups per tile load, each 2 rows x 64 B -> 2 / 4 lines."""
+    t = tg.generate("sgemm", n=256)
+    _, p128 = orc.mem_div(t, 128)
+    _, p32 = orc.mem_div(t, 32)
+    rows128 = [tuple(r) for r in p128.tolist() if r[0]]
+    rows32 = [tuple(r) for r in p32.tolist() if r[0]]
+    assert rows128 == [(524288, 1048576), (524288, 524288), (2048, 4096), (32768, 65536), (32768, 65536), (2048, 4096)]
+    assert rows32 == [(524288, 1048576), (524288, 1048576), (2048, 8192), (32768, 131072), (32768, 131072), (2048, 8192)]
+
+
+def test_address_domain_is_the_full_u64():
+    """P:L242 records an i8* effective address: no upper limit.  Shifting every
+    address by a multiple of the line size (here into [2^62, 2^64)) relabels
+    lines one-to-one, so every analysis must give the same result."""
+    t = tg.generate("rand", seed=5, ctas=3, threads=64, instrs=20, lines=30, pstore=0.3)
+    for shift in (np.uint64(1 << 58), np.uint64(0xC000000000000000)):
+        cols = {k: v.copy() for k, v in t.cols.items()}
+        mem = (cols["meta"] & 3) != BB
+        cols["addr"][mem] = cols["addr"][mem] + shift
+        t2 = tg.from_arrays(*(cols[k] for k, _ in tg.COLUMNS), nsites=t.nsites)
+        for lb in (1, 128):
+            for sc in (0, 1):
+                a, b = orc.reuse(t, lb, sc), orc.reuse(t2, lb, sc)
+                assert (a[0] == b[0]).all() and a[1] == b[1]
+                f = orc.reuse_fenwick(t2, lb, sc)
+                assert (a[0] == f[0]).all() and a[1] == f[1]
+            assert all((x == y).all() for x, y in zip(orc.mem_div(t, lb), orc.mem_div(t2, lb)))
+
+
+def _group_trace(sites, kinds, tids=None):
+    n = len(sites)
+    tids = np.arange(n) if tids is None else np.asarray(tids)
+    addr = 0x7F0000000000 + 4 * np.arange(n)
+    return tg.from_arrays(addr, np.zeros(n), tids, np.asarray(sites), np.zeros(n),
+                          [meta(k) for k in kinds], nsites=max(sites) + 1)
+
+
+def test_group_invariant_enforced():
+    """A dynamic warp-level instruction comes from one static instruction
+    (P:L235 Record() per instrumented load/store, P:L345 passBasicBlock() per
+    block): the records of one (cta, tid/32, winst) group share kind and
+    site; a group that mixes them is a malformed trace (BAD_TRACE), also when
+    the analysis warp size splits the warp (the group is the warp32's)."""
+    ok = _group_trace([3] * 8, [LD] * 8)
+    orc.mem_div(ok, 128)
+    for bad in (_group_trace([3] * 7 + [4], [LD] * 8), _group_trace([3] * 8, [LD] * 7 + [ST])):
+        for W in (32, 4):
+            with pytest.raises(orc.OracleError) as e:
+                orc.mem_div(bad, 128, W)
+            assert e.value.code == 2
+        orc.reuse(bad, 128)           # reuse distance does not read the group columns
+    bb = _group_trace([1] * 5 + [2] * 3, [BB] * 8)
+    with pytest.raises(orc.OracleError) as e:
+        orc.branch_div(bb)
+    assert e.value.code == 2
+    # the two half-warps of one winst are still one warp32 instruction
+    with pytest.raises(orc.OracleError):
+        orc.branch_div(_group_trace([1] * 16 + [2] * 16, [BB] * 32), warp_size=16)
+    # different warps (tid / 32) are different groups: no constraint between them
+    orc.branch_div(_group_trace([1] * 4 + [2] * 4, [BB] * 8, tids=[0, 1, 2, 3, 32, 33, 34, 35]))
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_fenwick_equals_brute_force(seed):
+    """The Fenwick variant against the literal O(n^2) definition on
+    random traces with stores, both scopes, both binnings."""
+    t = tg.generate("rand", seed=100 + seed, ctas=3, threads=40, instrs=12, lines=12, pstore=0.3)
+    for lb in (1, 32, 128):
+        for sc in (0, 1):
+            for b, nb in ((0, 40), (1, 8)):
+                hb, sb, _ = orc.reuse_brute(t, lb, sc, b, nb)
+                hf, sf = orc.reuse_fenwick(t, lb, sc, b, nb)
+                assert (hb == hf).all() and sb == sf, (seed, lb, sc, b)
+
+
+def test_fenwick_pins():
+    """The paper example (RD(B) = 5) and the cyclic closed form."""
+    t = literal(list("ABCCDEFAAAB"))
+    h, st = orc.reuse_fenwick(t, line_bytes=4, nbins=8)
+    assert list(h) == [3, 0, 0, 0, 0, 2, 0, 6] and st["finite_sum"] == 10
+    K, R = 130, 3
+    h, st = orc.reuse_fenwick(literal([f"x{k}" for _ in range(R) for k in range(K)]), line_bytes=4, nbins=K + 3)
+    assert h[-1] == K and h[K - 1] == K * (R - 1) and st["finite_sum"] == K * (R - 1) * (K - 1)
+
+
+@pytest.mark.parametrize("name,kw", [("vecadd", {}), ("sgemm", dict(n=64, bb=1)), ("bfs", dict(nodes=8000, seed=42)),
+                                     ("srad", dict(rows=128, cols=128, iters=2)), ("backprop", {"in": 2048})])
+def test_fenwick_equals_lru_on_configs(name, kw):
+    """the Fenwick variant is cross-checked == LRU on C1-C4
+    (C1 at full size, C2-C4 shapes at reduced size), both scopes."""
+    t = tg.generate(name, **kw)
+    for lb in (32, 128):
+        for sc in (0, 1):
+            a, f = orc.reuse(t, lb, sc), orc.reuse_fenwick(t, lb, sc)
+            assert (a[0] == f[0]).all() and a[1] == f[1], (name, lb, sc)
