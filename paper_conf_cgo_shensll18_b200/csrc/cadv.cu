@@ -100,11 +100,16 @@ static void prof_collect(cadv_ctx* c) {
   }
 }
 
-__global__ void k_agree_flags(const Scalars* s, const uint64_t* f1, const uint64_t* f2, uint32_t* out) {
+// Every rank's per-call status words, max-reduced over the ranks before any
+// exchange: bad record / group (err_code), site id >= nsites, CTA-id range,
+// unsupported reuse line, workspace to grow (`again`, set by the host).
+__global__ void k_agree_flags(const Scalars* s, const uint64_t* f1, const uint64_t* f2, uint32_t again, uint32_t* out) {
   if (threadIdx.x == 0) {
     out[0] = s->err_code;
     out[1] = ((f1 && *f1) || (f2 && *f2)) ? 1u : 0u;
-    out[2] = (uint32_t)s->max_cta;
+    out[2] = (uint32_t)(s->max_cta > 0xffffffffull ? 0xffffffffull : s->max_cta);
+    out[3] = s->unsup_index != ~0ull ? 1u : 0u;
+    out[4] = again;
   }
 }
 
@@ -144,6 +149,7 @@ cadv_status begin_call(cadv_ctx* c) {
   CK(ensure(c, B_SCALARS, sizeof(Scalars), &p), "workspace");
   CK(cudaMemsetAsync(p, 0, sizeof(Scalars), c->stream), "memset");
   CK(cudaMemsetAsync(&((Scalars*)p)->err_index, 0xff, sizeof(unsigned long long), c->stream), "memset");
+  CK(cudaMemsetAsync(&((Scalars*)p)->unsup_index, 0xff, sizeof(unsigned long long), c->stream), "memset");
   c->launches = 0;
   c->nprof = 0;
   for (auto& v : c->counts) v = 0;
@@ -171,9 +177,16 @@ cadv_status end_call(cadv_ctx* c, const void* d_out, size_t nout, void** h_out) 
     snprintf(b, sizeof b, "%s at trace position %llu",
              hs->err_code == 1 ? "invalid record" :
              hs->err_code == 2 ? "warp-level group longer than 32 records or with a repeated lane" :
+             hs->err_code == 4 ? "warp-level group whose records differ in kind or site" :
                                  "trace invariant violated",
              (unsigned long long)(hs->err_index == ~0ull ? 0 : hs->err_index + c->global_offset));
     return fail(c, CADV_ERR_BAD_TRACE, b);
+  }
+  if (hs->unsup_index != ~0ull) {
+    char b[200];
+    snprintf(b, sizeof b, "memory record at trace position %llu: its reuse-distance line (addr / line_bytes) is >= 2^58",
+             (unsigned long long)(hs->unsup_index + c->global_offset));
+    return fail(c, CADV_ERR_UNSUPPORTED, b);
   }
   *h_out = hr;
   return CADV_OK;
@@ -188,6 +201,7 @@ cadv_status load_trace_collective(cadv_ctx* c) {
   CK(ensure(c, B_COMM, 64 + (size_t)G * 64 + 64, &p), "workspace");
   uint32_t* d = (uint32_t*)p;
   uint32_t h[16] = {0};
+  h[0] = c->t.warp_contiguous ? 0u : 1u;
   if (c->t.n) {
     const uint64_t at[2] = {0, c->t.n - 1};
     for (int k = 0; k < 2; ++k) {
@@ -210,9 +224,11 @@ cadv_status load_trace_collective(cadv_ctx* c) {
   CK(cudaMemcpyAsync(all.data(), d + 16, (size_t)G * 64, cudaMemcpyDeviceToHost, c->stream), "D2H");
   CK(cudaStreamSynchronize(c->stream), "collective");
   c->split_group = false;
+  c->noncontig_any = false;
   const uint32_t* prev_last = nullptr;
   for (int r = 0; r < G; ++r) {
     const uint32_t* e = all.data() + (size_t)r * 16;
+    if (e[0]) c->noncontig_any = true;
     if (!e[1]) continue;  // empty shard
     if (prev_last && prev_last[0] && prev_last[1] == e[2] && prev_last[2] == e[3] && prev_last[3] == e[4])
       c->split_group = true;
@@ -459,6 +475,30 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
 cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_stats* rd_stats, uint64_t* md_hist,
                          cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites) {
   if (!c->loaded) return fail(c, CADV_ERR_NO_TRACE, "no trace loaded");
+  const bool noncontig = c->comm ? c->noncontig_any : !c->t.warp_contiguous;
+  if (q.rd && (q.md || q.bd) && noncontig && (c->t.n || c->comm)) {
+    // A non-warp-contiguous trace is reordered by (cta, warp) for the
+    // divergence analyses (regroup_by_warp); reuse distance needs trace order
+    // (reading R2), so it gets its own pass over the original columns.
+    // Outputs are staged and written only when both passes succeed.
+    Req a = q, b = q;
+    a.md = a.bd = a.md_sites = a.bd_sites = false;
+    b.rd = false;
+    const size_t rows = (size_t)q.nobj + 1;
+    std::vector<uint64_t> h(rows * q.nbins);
+    cadv_reuse_stats st{};
+    cadv_status s = run_analyses(c, a, h.data(), rd_stats ? &st : nullptr, nullptr, nullptr, nullptr, nullptr);
+    if (s != CADV_OK) return s;
+    const float ms = c->elapsed_ms;
+    const uint32_t launches = c->launches;
+    s = run_analyses(c, b, nullptr, nullptr, md_hist, md_sites, bd_tot, bd_sites);
+    if (s != CADV_OK) return s;
+    c->elapsed_ms += ms;
+    c->launches += launches;
+    memcpy(rd_hist, h.data(), h.size() * 8);
+    if (rd_stats) *rd_stats = st;
+    return CADV_OK;
+  }
   if (q.bd) {
     // one T_c generation per call (identical on every rank: calls run in lockstep)
     if (++c->tc_gen >= (1u << 21)) {
@@ -477,7 +517,7 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
                      cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites) {
   const bool multi = c->comm != nullptr;  // also a 1-rank NCCL / loopback context (plumbing tests)
   if (multi && (q.md || q.bd)) {
-    if (!c->t.warp_contiguous)
+    if (c->noncontig_any)  // (all-gathered at load: every rank decides alike)
       return fail(c, CADV_ERR_UNSUPPORTED, "multi-rank divergence analyses need warp-contiguous shards");
     if (c->split_group)
       return fail(c, CADV_ERR_BAD_TRACE, "a shard boundary splits a warp-level group (cta, warp, winst)");
@@ -525,6 +565,7 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
     P.cta_scope = q.scope == CADV_SCOPE_CTA;
     P.kout = rs.cta_scope ? rs.k1 : nullptr;
     P.vout = rs.v1;
+    P.kcap = rs.chunk_cap;
     P.blkcnt = rs.blkcnt;
     P.hist0 = d + o_rdh;
   }
@@ -564,6 +605,7 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
   if (flags && t.n) CK(launch_scan(c, flags, P), "scan launch");
   // R0 results of the pass: CTA-id range, T_c / deferred-group capacity; the
   // reuse compaction is queued behind them, so one synchronisation covers both
+  bool again = false;  // workspace grown: run the call again
   {
     Scalars* hsp = (Scalars*)((uint8_t*)c->hstage + 64);
     CK(cudaMemcpyAsync(hsp, scalars(c), sizeof(Scalars), cudaMemcpyDeviceToHost, c->stream), "D2H");
@@ -571,9 +613,15 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
     CK(cudaStreamSynchronize(c->stream), "scan");
     const Scalars hs = *hsp;
     c->max_cta = (uint32_t)hs.max_cta;
+    // one rank: a bad / unsupported record ends the call here (its report
+    // comes from end_call); several ranks first agree (below)
+    if (!multi && (hs.err_code || hs.unsup_index != ~0ull)) {
+      void* h0;
+      s = end_call(c, nullptr, 0, &h0);
+      return s != CADV_OK ? s : fail(c, CADV_ERR_BAD_TRACE, "invalid trace");
+    }
     if (q.bd && t.n) {
-      if (hs.max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
-      bool again = false;
+      if (!multi && hs.max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
       if (hs.tc_overflow) {
         uint64_t cap = (uint64_t)c->tc_cap * 2;
         if (cap < hs.max_cta + 1) cap = hs.max_cta + 1;
@@ -584,8 +632,12 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
         c->defer_cap = hs.ndefer + hs.ndefer / 4 + 4096;
         again = true;
       }
-      if (again && !hs.err_code) return RETRY;
     }
+    if (q.rd && hs.kept_max > rs.chunk_cap) {  // a warp's kept records overflowed its region
+      c->kdiv = 1;
+      again = true;
+    }
+    if (again && !hs.err_code && !multi) return RETRY;
   }
   if (multi) {
     // every rank learns whether any rank found a bad record / site id before
@@ -594,19 +646,22 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
     CK(ensure(c, B_COMM, 64, &fb), "workspace");
     uint32_t* df = (uint32_t*)fb;
     CADV_LAUNCH(c, k_agree_flags<<<1, 32, 0, c->stream>>>(scalars(c), q.md ? d + o_mdf : nullptr,
-                                                          q.bd ? d + o_bdf : nullptr, df));
-    if (c->comm->allreduce_max_u32(df, 3, c->stream)) return fail(c, CADV_ERR_NCCL, c->comm->err);
-    uint32_t hf[3];
-    CK(cudaMemcpyAsync(hf, df, 12, cudaMemcpyDeviceToHost, c->stream), "D2H");
+                                                          q.bd ? d + o_bdf : nullptr, again ? 1u : 0u, df));
+    if (c->comm->allreduce_max_u32(df, 5, c->stream)) return fail(c, CADV_ERR_NCCL, c->comm->err);
+    uint32_t hf[5];
+    CK(cudaMemcpyAsync(hf, df, 20, cudaMemcpyDeviceToHost, c->stream), "D2H");
     CK(cudaStreamSynchronize(c->stream), "scan");
     c->max_cta = hf[2];  // global CTA-id range
-    if (hf[0] || hf[1]) {
+    if (hf[0] || hf[1] || hf[3]) {
       void* h0;
       s = end_call(c, nullptr, 0, &h0);  // reports this rank's own bad record, if it has one
       if (s != CADV_OK) return s;
       if (hf[0]) return fail(c, CADV_ERR_BAD_TRACE, "invalid record or warp-level group on another rank");
+      if (hf[3]) return fail(c, CADV_ERR_UNSUPPORTED, "a reuse-distance line >= 2^58 on another rank");
       return fail(c, CADV_ERR_INVALID_ARG, "a record's site id is >= nsites (on some rank)");
     }
+    if (q.bd && c->max_cta >= (1u << 28)) return fail(c, CADV_ERR_UNSUPPORTED, "CTA ids must be < 2^28");
+    if (hf[4]) return RETRY;  // some rank grew its workspace: every rank runs the call again
   }
   if (q.rd && (t.n || multi)) {
     const ObjTab ot{q.obj_lo, q.obj_hi, q.nobj};

@@ -21,7 +21,10 @@ struct DevBuf {
 // Small per-call device scalars (zeroed at the start of every analysis).
 struct Scalars {
   unsigned long long err_index;  // first offending record (ULLONG_MAX = none)
-  unsigned int err_code;         // 1 = bad record, 2 = run longer than 32 / duplicate lane
+  unsigned int err_code;         // 1 = bad record, 2 = run longer than 32 / duplicate lane,
+                                 // 3 = internal invariant, 4 = group mixes kinds / sites
+  unsigned long long unsup_index;
+  unsigned long long kept_max;   // scan (RD): most kept records of one warp chunk (region capacity check)  // first memory record whose reuse line is >= 2^58 (ULLONG_MAX = none)
   unsigned int tile_counter;     // dynamic tile assignment
   unsigned long long count[8];   // generic counters (kept records, entries, ...)
   unsigned long long max_cta;    // scan: max CTA id of the trace (shard)
@@ -88,6 +91,17 @@ struct cadv_ctx {
   std::vector<float> prof_ms;
   uint32_t nprof = 0;
   uint64_t counts[4] = {0, 0, 0, 0};  // cadv_last_count
+  // max-dynamic-shared-memory opt-ins done on this context's device (the
+  // attribute is per device context, so it is tracked per cadv_ctx):
+  // bits 0-15 k_scan<F>, bit 16 k_rd_seg, 17 k_rd_tile, 18 k_merge_count_block
+  uint32_t attr_set = 0;
+  int seg_ctas = 0;           // k_rd_seg CTAs per SM for seg_ctas_smem bytes of shared memory
+  size_t seg_ctas_smem = 0;
+  bool noncontig_any = false;
+  // kept-record region capacity of a scan warp = chunk / kdiv records (grown
+  // to the whole chunk, for the context's lifetime, the first time a region
+  // overflows: the call then runs again)
+  uint32_t kdiv = 4; // multi-rank: some rank's shard is not warp-contiguous (load_trace)
 };
 
 namespace cadv {
@@ -113,8 +127,9 @@ struct ScanParams {
   // reuse distance: run compression output
   uint32_t lbs_rd = 0;
   int cta_scope = 1;
-  uint32_t* kout = nullptr;    // gapped per-block regions (scan_geometry)
+  uint32_t* kout = nullptr;    // gapped per-warp regions (scan_geometry) of kcap records
   uint64_t* vout = nullptr;
+  uint64_t kcap = 0;
   uint64_t* blkcnt = nullptr;  // kept records per scan warp chunk
   uint64_t* hist0 = nullptr;
   // memory divergence

@@ -27,10 +27,12 @@ __device__ __forceinline__ bool is_bb(uint8_t m) { return (m & 3u) == 2u; }
 __device__ __forceinline__ bool meta_ok(uint8_t m) {
   return (m & 3u) != 3u && (m >> 5) == 0 && (((m & 3u) == 2u) || ((m >> 2) & 7u) <= 4u);
 }
+// (any 64-bit address is valid; the reuse path's own limit on line
+// numbers, < 2^58, is CADV_ERR_UNSUPPORTED, not a bad record)
 __device__ __forceinline__ bool addr_ok(uint64_t a, uint8_t m) {
   if ((m & 3u) == 2u) return true;
   uint64_t bytes = 1ull << ((m >> 2) & 7u);
-  return (a & (bytes - 1)) == 0 && (a >> 58) == 0;
+  return (a & (bytes - 1)) == 0;
 }
 
 // ------------------------------------------------------------------ data objects

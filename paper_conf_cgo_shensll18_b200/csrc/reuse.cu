@@ -1254,8 +1254,6 @@ int bits_for(uint64_t maxv) {
   return b;
 }
 
-int g_tile_smem_set = 0;
-int g_mc_smem_set = 0;
 
 }  // namespace
 
@@ -1267,11 +1265,18 @@ cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st) {
   uint64_t grid, nw, chunk;
   scan_geometry(c, n, &grid, &nw, &chunk);
   st->grid = nw;  // one kept-record region per scan warp
-  st->chunk_cap = chunk;
-  // the scan writes kept records into per-block regions of (k1, v1) (capacity
-  // grid * chunk >= n); the squeeze packs them into (k0, v0); the CTA radix
-  // sort then ping-pongs between the two pairs.
-  const uint64_t gap = nw * chunk + 16, cap = (nmem > gap ? gap : nmem) + 16;
+  // region capacity: chunk / kdiv records (run compression keeps ~7 % of the
+  // paper-shaped traces; a region that overflows makes the call run again
+  // with whole-chunk regions, see run_once), so C5's 4e9 records need 24 B
+  // per kept slot instead of per record
+  uint64_t kcap = chunk / (c->kdiv ? c->kdiv : 1);
+  kcap = ((kcap + 255) / 256) * 256;
+  if (kcap > chunk) kcap = chunk;
+  st->chunk_cap = kcap;
+  // the scan writes kept records into per-warp regions of (k1, v1) (stride
+  // kcap); the regroup / squeeze packs them into (k0, v0); the CTA radix sort
+  // then ping-pongs between the two pairs.
+  const uint64_t gap = nw * kcap + 16, cap = (nmem > gap ? gap : nmem) + 16;
   void *k0 = nullptr, *k1 = nullptr, *v0, *v1, *bc;
   if ((e = ensure(c, B_RD_VAL, (gap > cap ? gap : cap) * 8, &v0)) || (e = ensure(c, B_SORT_V1, gap * 8, &v1))) return e;
   if (st->cta_scope && ((e = ensure(c, B_RD_KEY, (gap > cap ? gap : cap) * 4, &k0)) ||
@@ -1368,7 +1373,13 @@ cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const 
     roff[p] = Kn;
     Kn += rcnt[p];
   }
-  if (Kn >= 0xffffffffull) return cudaErrorNotSupported;  // kept positions are u32
+  // kept positions are u32: decided from the all-gathered matrix, so every
+  // rank takes the same branch (no rank may leave the others in a collective)
+  for (int r = 0; r < G; ++r) {
+    uint64_t kr = 0;
+    for (int p = 0; p < G; ++p) kr += mat[(size_t)p * G + r];
+    if (kr >= 0xffffffffull) return cudaErrorNotSupported;
+  }
   void *rk0, *rk1 = nullptr, *rv0, *rv1;
   if ((e = ensure(c, B_XCH_V0, Kn * 8 + 16, &rv0)) || (e = ensure(c, B_XCH_V1, Kn * 8 + 16, &rv1))) return e;
   if (cta_scope &&
@@ -1552,24 +1563,21 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
         if ((e = cudaMemcpyAsync(hcm, seg_cm, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
         if ((e = cudaStreamSynchronize(c->stream))) return e;
         if (hcm[1] <= 256u && getenv("CADV_RD_TILES") == nullptr) {
-          static bool seg_smem_set = false;
-          if (!seg_smem_set) {
+          if (!(c->attr_set & (1u << 16))) {
             if ((e = cudaFuncSetAttribute(k_rd_seg, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SegSmem))))
               return e;
-            seg_smem_set = true;
+            c->attr_set |= 1u << 16;
           }
           if (hcm[0]) {
             const uint64_t hbins = (uint64_t)(O.n + 1) * nbins;
             const size_t smem = offsetof(SegSmem, hist) + (hbins <= TL_SMEM_BINS ? 4 * hbins : 0);
-            static int seg_ctas = 0;
-            static size_t seg_ctas_smem = 0;
-            if (seg_ctas_smem != smem) {
-              if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&seg_ctas, k_rd_seg, SG_NT, smem))) return e;
-              if (seg_ctas < 1) seg_ctas = 1;
-              seg_ctas_smem = smem;
+            if (c->seg_ctas_smem != smem) {
+              if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c->seg_ctas, k_rd_seg, SG_NT, smem))) return e;
+              if (c->seg_ctas < 1) c->seg_ctas = 1;
+              c->seg_ctas_smem = smem;
             }
             const unsigned grid =
-                (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * seg_ctas, (hcm[0] + SG_W - 1) / SG_W);
+                (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * c->seg_ctas, (hcm[0] + SG_W - 1) / SG_W);
             CADV_LAUNCH(c, k_rd_seg<<<grid, SG_NT, smem, c->stream>>>(val, seg, seg_cm, seg_cm + 2, log2bins,
                                                                                 nbins, d_hist, d_stats, O));
           }
@@ -1667,13 +1675,13 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     En.ff = (uint8_t*)take(K);
     En.lf = (uint8_t*)take(K);
   }
-  if (!g_tile_smem_set) {
+  if (!(c->attr_set & (1u << 17))) {
     if ((e = cudaFuncSetAttribute(k_rd_tile<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))) ||
         (e = cudaFuncSetAttribute(k_rd_tile<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))) ||
         (e = cudaFuncSetAttribute(k_rd_tile<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   (int)sizeof(TileSmemWide))))
       return e;
-    g_tile_smem_set = 1;
+    c->attr_set |= 1u << 17;
   }
   uint32_t* tile_w = (uint32_t*)tw;
   uint32_t* tile_q = (uint32_t*)tq;
@@ -1810,11 +1818,11 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   ka = (uint32_t*)ek0;
   kb = ka + M;
   CADV_LAUNCH(c, k_iota_gather<<<grid_ls, 256, 0, c->stream>>>(ord, X.xq, M, ka, ia, cnt));
-  if (!g_mc_smem_set) {
+  if (!(c->attr_set & (1u << 18))) {
     if ((e = cudaFuncSetAttribute(k_merge_count_block, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                   (int)sizeof(MergeBlockSmem))))
       return e;
-    g_mc_smem_set = 1;
+    c->attr_set |= 1u << 18;
   }
   CADV_LAUNCH(c, k_merge_count_block<<<(unsigned)((M + MC_BLOCK - 1) / MC_BLOCK), 512, sizeof(MergeBlockSmem),
                                        c->stream>>>(ka, ia, kb, ib, M, cnt));

@@ -87,6 +87,7 @@ struct ScanArgs {
   uint32_t* kout;        // gapped output: warp w writes from w * chunk
   uint64_t* vout;
   uint64_t* wcnt;        // kept records per warp
+  uint64_t kcap;         // kept-record region capacity per warp (writes beyond it are dropped; the host reruns)
   uint64_t* hist0;
   // MD
   uint32_t lbs_md, ws_md;
@@ -561,7 +562,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     for (uint32_t p = 0; p < issued; ++p) issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, p);
     // the record before the step (warp-uniform); meta 3 = "no record"
     // p_kb: kind bits of that record (bit 0 memory, 1 store, 2 BB; 0 = invalid / none)
-    uint32_t p_cta = 0xffffffffu, p_t = 0, p_kb = 0, p_winst = 0;
+    uint32_t p_cta = 0xffffffffu, p_t = 0, p_kb = 0, p_winst = 0, p_site = 0;
     uint64_t p_addr = 0;
     if (c_lo > 0) {
       p_cta = __ldg(A.cta + c_lo - 1);
@@ -572,6 +573,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       p_kb = (pm0 & 3u) < 2u ? (1u | ((pm0 & 1u) << 1)) : ((pm0 & 3u) == 2u ? 4u : 0u);
       if (NG) p_t = __ldg(A.tid + c_lo - 1);
       if (NG) p_winst = __ldg(A.winst + c_lo - 1);
+      if (NG) p_site = __ldg(A.site + c_lo - 1);
     }
     // the run open at the step end (warp-uniform); owned iff it starts in the chunk
     bool cr_on = false, cr_own = false;
@@ -579,8 +581,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     uint32_t qn = 0;  // queued complete runs (warp-uniform)
     // RD: the last kept record when its compression run reaches the step end
     bool open_rd = false;
-    uint64_t* wbv = A.vout ? A.vout + gw * A.chunk : nullptr;
-    uint32_t* wbk = A.kout ? A.kout + gw * A.chunk : nullptr;
+    uint64_t* wbv = A.vout ? A.vout + gw * A.kcap : nullptr;
+    uint32_t* wbk = A.kout ? A.kout + gw * A.kcap : nullptr;
 
     for (uint32_t p = 0; p < npieces; ++p) {
       const uint32_t base = p * KR;
@@ -605,6 +607,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       const uint32_t* r_site = (const uint32_t*)(stg + S_SITE);
       const uint8_t* r_meta = stg + S_META;
       uint32_t c[LPR], t[LPR], w[LPR], mmx, mmy, tor = 0;
+      uint32_t sdm = 0;  // NG: site changes (a group's records share their site, reading R19)
       uint64_t a[LPR];
       {
         const uint4 c0 = *(const uint4*)(r_cta + sl), c1 = *(const uint4*)(r_cta + sl + 4);
@@ -619,6 +622,21 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           t[4] = t4.z & 0xffffu; t[5] = t4.z >> 16; t[6] = t4.w & 0xffffu; t[7] = t4.w >> 16;
           const uint4 w0 = *(const uint4*)(r_winst + sl), w1 = *(const uint4*)(r_winst + sl + 4);
           w[0] = w0.x; w[1] = w0.y; w[2] = w0.z; w[3] = w0.w; w[4] = w1.x; w[5] = w1.y; w[6] = w1.z; w[7] = w1.w;
+          {  // site changes, compared at once (the site registers die here)
+            const uint4 s0 = *(const uint4*)(r_site + sl), s1 = *(const uint4*)(r_site + sl + 4);
+            uint32_t psi = __shfl_up_sync(FULL, s1.w, 1);
+            if (lane == 0) psi = p_site;
+            p_site = __shfl_sync(FULL, s1.w, 31);
+            const uint32_t one = A.one;
+            add_if_nz(sdm, s0.x ^ psi, one, 1u);
+            add_if_nz(sdm, s0.y ^ s0.x, one, 2u);
+            add_if_nz(sdm, s0.z ^ s0.y, one, 4u);
+            add_if_nz(sdm, s0.w ^ s0.z, one, 8u);
+            add_if_nz(sdm, s1.x ^ s0.w, one, 16u);
+            add_if_nz(sdm, s1.y ^ s1.x, one, 32u);
+            add_if_nz(sdm, s1.z ^ s1.y, one, 64u);
+            add_if_nz(sdm, s1.w ^ s1.z, one, 128u);
+          }
         } else {
 #pragma unroll
           for (int k = 0; k < LPR; ++k) t[k] = w[k] = 0;
@@ -665,7 +683,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             const uint32_t H = __byte_perm(__byte_perm((uint32_t)(a[i] >> 32), (uint32_t)(a[i + 1] >> 32), 0x0073u),
                                            __byte_perm((uint32_t)(a[i + 2] >> 32), (uint32_t)(a[i + 3] >> 32), 0x0073u),
                                            0x5410u);
-            trig |= ((L | 0x10101010u) & M) | (H & K & 0xfcfcfcfcu);  // misaligned / > 16 B, address >= 2^58
+            // misaligned / > 16 B; RD: address >= 2^58 (a superset of line >= 2^58, the packing limit)
+            trig |= ((L | 0x10101010u) & M) | (RD ? (H & K & 0xfcfcfcfcu) : 0u);
           } else {
             trig |= M & 0x10101010u;
           }
@@ -681,6 +700,9 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             if (!ok) {
               report(A.sc, c_lo + j0 + k, 1);
               okm &= ~(1u << k);
+            } else if (RD && is_mem(m) && ((a[k] >> A.lbs_rd) >> 58)) {
+              // a valid record whose line does not fit the kept-record packing
+              atomicMin(&A.sc->unsup_index, (unsigned long long)(c_lo + j0 + k));
             }
           }
         }
@@ -754,7 +776,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         const uint32_t k0 = ((lt ? sv : 0u) - sb) & 15u;
         uint32_t keepm = (memm & ~dupm & brk) | (k0 < fbk ? (1u << k0) : 0u);
         keepm &= ownm;
-        if (open_rd && lane == 0 && (dupm & 1u)) wbv[kept - 1] |= 1ull << VB_DUP;  // the previous step's open piece
+        if (open_rd && lane == 0 && (dupm & 1u) && kept - 1 < A.kcap) wbv[kept - 1] |= 1ull << VB_DUP;  // the previous step's open piece
         const uint32_t nk = __popc(keepm);
         uint32_t x = nk;
 #pragma unroll
@@ -776,9 +798,11 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           bool hd = nd;
           if (wgt > 16u) { wgt = 16u; hd = false; }      // the chain goes on with another kept store
           else last_open = nb == (uint32_t)KR;           // decided by the next step's first record
-          wbv[pos] = (lds_u64(r_addr + sl + k) >> A.lbs_rd) | ((uint64_t)((stm >> k) & 1u) << VB_STORE) | ((uint64_t)hd << VB_DUP) |
-                     ((uint64_t)(wgt - 1u) << VB_W);
-          if (wbk) wbk[pos] = A.cta_scope ? lds_u32(r_cta + sl + k) : 0u;
+          if (pos < A.kcap) {
+            wbv[pos] = (lds_u64(r_addr + sl + k) >> A.lbs_rd) | ((uint64_t)((stm >> k) & 1u) << VB_STORE) |
+                       ((uint64_t)hd << VB_DUP) | ((uint64_t)(wgt - 1u) << VB_W);
+            if (wbk) wbk[pos] = A.cta_scope ? lds_u32(r_cta + sl + k) : 0u;
+          }
           ++pos;
         }
         open_rd = __ballot_sync(FULL, last_open) != 0;
@@ -811,6 +835,14 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         rsm |= ~inbm & 0xffu;  // every record past the stream is a run of its own (never finalized)
         nlm |= rsm;
         vim &= ~rsm;
+        {
+          // a record continuing a run must have its predecessor's kind and site
+          // (both valid records): else the group mixes static instructions
+          const uint32_t kcm = (stm ^ ((stm << 1) | ((pkb >> 1) & 1u))) & 0xffu;
+          const uint32_t pvm = ((okm << 1) | (pkb ? 1u : 0u)) & 0xffu;
+          const uint32_t gv = (sdm | kcm) & ~rsm & ownm & okm & pvm;
+          if (__any_sync(FULL, gv != 0) && gv) report(A.sc, c_lo + j0 + __ffs(gv) - 1, 4);
+        }
         // lane bits of each in-lane run piece (backward)
         uint32_t rm[LPR];
         uint32_t m = 0;
@@ -937,6 +969,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   }
   if (RD && lane == 0) {
     A.wcnt[gw] = kept;
+    if (kept > A.kcap) atomicMax(&A.sc->kept_max, (unsigned long long)kept);
   }
 
   if (RD && !OBJ) {
@@ -1062,7 +1095,6 @@ size_t scan_smem() {
          (size_t)NWARP * (qcap<F>() * 24 + 16) + (OBJ ? (size_t)OBJ_SMEM * (16 + 4 + (MD ? 66 * 4 : 0)) : 0);
 }
 
-int g_scan_ready[16] = {0};
 const char* const kScanName[16] = {"k_scan<0>", "k_scan<1>", "k_scan<2>", "k_scan<3>", "k_scan<4>", "k_scan<5>",
                                    "k_scan<6>", "k_scan<7>", "k_scan<8>", "k_scan<9>", "k_scan<10>", "k_scan<11>",
                                    "k_scan<12>", "k_scan<13>", "k_scan<14>", "k_scan<15>"};
@@ -1070,10 +1102,10 @@ const char* const kScanName[16] = {"k_scan<0>", "k_scan<1>", "k_scan<2>", "k_sca
 template <int F>
 cudaError_t launch_scan_t(cadv_ctx* c, const ScanArgs& A, uint64_t grid) {
   const size_t smem = scan_smem<F>();
-  if (!g_scan_ready[F]) {
+  if (!(c->attr_set & (1u << F))) {
     cudaError_t e = cudaFuncSetAttribute(k_scan<F>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    g_scan_ready[F] = 1;
+    c->attr_set |= 1u << F;
   }
   CADV_LAUNCH_N(c, kScanName[F], k_scan<F><<<(unsigned)grid, NTHR, smem, c->stream>>>(A));
   return cudaGetLastError();
@@ -1113,6 +1145,7 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
   uint64_t grid, nwarps;
   scan_geometry(c, t.n, &grid, &nwarps, &A.chunk);
   A.lbs_rd = P.lbs_rd; A.cta_scope = P.cta_scope; A.kout = P.kout; A.vout = P.vout; A.wcnt = P.blkcnt;
+  A.kcap = P.kcap;
   A.hist0 = P.hist0;
   A.lbs_md = P.lbs_md; A.ws_md = P.ws_md; A.md_hist = P.md_hist; A.md_sites = P.md_sites;
   A.ws_bd = P.ws_bd; A.tc = P.tc; A.tc_cap = P.tc_cap; A.tc_gen = P.tc_gen; A.defer_cap = P.defer_cap;

@@ -127,6 +127,7 @@ struct Trace {
   std::vector<std::pair<uint64_t, uint64_t>> objs;  // allocated arrays (base, bytes), ascending
   // state shared by the generator closures
   std::vector<std::shared_ptr<void>> keep;
+  uint64_t limit = 0;  // > 0: the trace is truncated to its first `limit` records (C5)
   int scramble = 0;
   uint64_t scramble_seed = 0;
 };
@@ -708,6 +709,7 @@ void wl_nw(Trace& T, const Params& P) {
 // Random well-formed traces for fuzzing / adversarial parity cases.
 //   ctas, threads, instrs (per warp), lines (address pool, in 128 B units),
 //   pstore, pbb, pfull (full-warp mask), launches, seed, stride,
+//   msites / bsites (number of memory / basic-block site ids, default 16 / 8),
 //   lanes=asc|perm (lane order inside a warp-instruction)
 void wl_rand(Trace& T, const Params& P) {
   uint32_t ncta = (uint32_t)P.i("ctas", 4), NT = (uint32_t)P.i("threads", 64);
@@ -715,7 +717,9 @@ void wl_rand(Trace& T, const Params& P) {
   uint32_t nlaunch = (uint32_t)P.i("launches", 1);
   double pstore = P.f("pstore", 0.2), pbb = P.f("pbb", 0.3), pfull = P.f("pfull", 0.5);
   uint64_t seed = (uint64_t)P.i("seed", 1);
-  uint32_t nmsite = 16, nbsite = 8;
+  uint32_t nmsite = (uint32_t)P.i("msites", 16), nbsite = (uint32_t)P.i("bsites", 8);
+  if (!nmsite) nmsite = 1;
+  if (!nbsite) nbsite = 1;
   T.nsites = nmsite + nbsite;
   Alloc A(&T.objs);
   uint64_t pool = A.get(128ull * lines + 4096);
@@ -785,39 +789,64 @@ void wl_literal(Trace& T, const Params& P) {
   T.launches.push_back(L);
 }
 
-// C5-style mixed trace: several workloads back to back (CTA ids continue).
+// C5: the launches of several Rodinia-shaped workloads back
+// to back -- SRAD 4096^2 x 3 iterations, backprop 2^23, SGEMM-naive 512^3,
+// BFS 4M nodes, tiled SGEMM 2048^3, then SRAD 4096^2 iterations -- until
+// exactly `records` (default 4.0e9) records, the last launch truncated.
+// Part k uses seed 42 + k.  CTA ids continue across launches; each part's
+// site ids are offset past the previous parts'.  C5 is the memory trace of
+// the mix (bb=0: the 4.0e9 records are loads/stores, so that the recipe's
+// five parts (3.60e9 records) are followed by SRAD iterations as it states;
+// with BB records the parts alone would exceed 4.0e9; reading R20).
+// div=k divides every linear size by k (edge sizes by sqrt-ish factors) for
+// small parity tests of the mixing and truncation logic.
 void build(Trace& T, const std::string& name, const Params& P);
+uint64_t count_launch(const Launch& L);
 
 void wl_mixed(Trace& T, const Params& P) {
-  // launches in order: SRAD, backprop, SGEMM naive, BFS, SGEMM tiled, SRAD...
-  // scaled by "scale" (1 = the C5 recipe of SURVEY 8(d) sizes divided down).
-  uint32_t scale = (uint32_t)P.i("scale", 1);
+  const uint64_t limit = (uint64_t)P.i("records", 4000000000ll);
+  const uint32_t d = (uint32_t)P.i("div", 1);
+  auto sq = [&](uint32_t x) { uint32_t r = x; for (uint32_t k = 1; k * k < d && r > 16; k *= 2) r /= 2; return r; };
   std::vector<std::pair<std::string, std::string>> parts;
   char b[256];
-  snprintf(b, sizeof b, "rows=%u,cols=%u,iters=1,bb=1", 512 * scale, 512 * scale); parts.push_back({"srad", b});
-  snprintf(b, sizeof b, "in=%u,bb=1", 16384 * scale); parts.push_back({"backprop", b});
-  snprintf(b, sizeof b, "n=%u,tiled=0", 64 * scale); parts.push_back({"sgemm", b});
-  snprintf(b, sizeof b, "nodes=%u,seed=43", 20000 * scale); parts.push_back({"bfs", b});
-  snprintf(b, sizeof b, "n=%u,naive=0", 128 * scale); parts.push_back({"sgemm", b});
+  snprintf(b, sizeof b, "rows=%u,cols=%u,iters=3,bb=0,seed=42", sq(4096), sq(4096)); parts.push_back({"srad", b});
+  snprintf(b, sizeof b, "in=%u,bb=0", (1u << 23) / d); parts.push_back({"backprop", b});
+  snprintf(b, sizeof b, "n=%u,tiled=0,bb=0", sq(512)); parts.push_back({"sgemm", b});
+  snprintf(b, sizeof b, "nodes=%u,seed=45,bb=0", 4000000u / d); parts.push_back({"bfs", b});
+  snprintf(b, sizeof b, "n=%u,naive=0,bb=0", sq(2048)); parts.push_back({"sgemm", b});
   uint32_t site_base = 0;
-  for (auto& pr : parts) {
+  uint64_t total = 0;
+  auto add = [&](const std::string& nm, const std::string& ps) {
     Trace sub;
-    build(sub, pr.first, Params(pr.second.c_str()));
+    build(sub, nm, Params(ps.c_str()));
     for (auto& L : sub.launches) {
       Launch L2 = L;
-      uint32_t sb = site_base;
+      const uint32_t sb = site_base;
       auto g = L.gen;
       L2.gen = [g, sb](uint32_t c, uint32_t w, Prog& p) {
         size_t st = p.p->size();
         g(c, w, p);
         for (size_t k = st; k < p.p->size(); ++k) (*p.p)[k].site += sb;
       };
+      total += count_launch(L);
       T.launches.push_back(L2);
     }
     for (auto& k : sub.keep) T.keep.push_back(k);
     site_base += sub.nsites;
+  };
+  for (auto& pr : parts) add(pr.first, pr.second);
+  if (total < limit) {  // SRAD iterations until the limit (one SRAD launch pair per iteration)
+    Trace one;
+    snprintf(b, sizeof b, "rows=%u,cols=%u,iters=1,bb=0,seed=47", sq(4096), sq(4096));
+    build(one, "srad", Params(b));
+    uint64_t per = 0;
+    for (auto& L : one.launches) per += count_launch(L);
+    const uint64_t it = (limit - total + per - 1) / per;
+    snprintf(b, sizeof b, "rows=%u,cols=%u,iters=%llu,bb=0,seed=47", sq(4096), sq(4096), (unsigned long long)it);
+    add("srad", b);
   }
   T.nsites = site_base;
+  T.limit = limit;
 }
 
 void build(Trace& T, const std::string& name, const Params& P) {
@@ -861,6 +890,10 @@ tg_trace* tg_plan(const char* workload, const char* params, char* err, int errle
     }
     T->nctas = cb;
     T->n = off;
+    if (T->limit && T->n > T->limit) {  // truncation: launches that start past the limit go
+      while (!T->launches.empty() && T->launches.back().offset >= T->limit) T->launches.pop_back();
+      T->n = T->limit;
+    }
     return reinterpret_cast<tg_trace*>(T);
   } catch (std::exception& e) {
     if (err && errlen > 0) snprintf(err, errlen, "%s", e.what());
