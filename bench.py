@@ -42,9 +42,11 @@ WORKLOADS = {
     "c2_sgemm": ("sgemm", dict(n=256, bb=1)),
     "c3_bfs": ("bfs", dict(nodes=1000000, seed=42)),
     "c4_backprop": ("backprop", {"in": 4194304}),
+    # C5 per GPU: 5e8 records of the mixed trace; at N = 8 the global trace is C5 (4.0e9)
+    "c5_mixed": ("mixed", {"records": 500000000}),
 }
 # how a workload grows with N for position-range weak scaling (param, factor per GPU)
-SCALE = {"c4_srad": "iters", "c4_backprop": "in"}
+SCALE = {"c4_srad": "iters", "c4_backprop": "in", "c5_mixed": "records"}
 METRIC = "trace records analysed/sec (reuse+divergence)"
 UNIT = "records/s"
 
@@ -68,6 +70,9 @@ def parse():
     ap.add_argument("--no-data-centric", action="store_true", help="skip the data-centric attribution leg")
     ap.add_argument("--separate", action="store_true",
                     help="one library call per analysis (three passes) instead of the fused cadv_analyze")
+    ap.add_argument("--scaling", default="weak", choices=["weak", "strong"],
+                    help="N>1 position sharding: weak = N times the N=1 workload, strong = the N=1 workload split N ways")
+    ap.add_argument("--no-per-analysis", action="store_true", help="skip the per-analysis (separate) rates")
     return ap.parse_args()
 
 
@@ -153,22 +158,22 @@ def peaks():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
-def workload_params(workload, world, sharding):
+def workload_params(workload, world, sharding, scaling="weak"):
     """(generator, params) of the global trace analysed by `world` GPUs."""
     name, params = WORKLOADS[workload]
     params = dict(params)
-    if world > 1 and sharding == "position" and workload in SCALE:
+    if world > 1 and sharding == "position" and workload in SCALE and scaling == "weak":
         params[SCALE[workload]] = params[SCALE[workload]] * world
     return name, params
 
 
-def make_trace(workload, rank, world, sharding, pinned):
+def make_trace(workload, rank, world, sharding, pinned, scaling="weak"):
     """This rank's trace: its position-range shard of the global trace, or
     (independent / unscalable workloads) a whole trace of its own.  Returns
     (trace, global_offset, global_records, mode)."""
     import tracegen as tg
-    name, params = workload_params(workload, world, sharding)
-    mode = "position" if (world > 1 and sharding == "position" and workload in SCALE) else (
+    name, params = workload_params(workload, world, sharding, scaling)
+    mode = "position" if (world > 1 and sharding == "position" and (workload in SCALE or scaling == "strong")) else (
         "independent" if world > 1 else "single")
     if mode == "independent" and rank:
         params["seed"] = params.get("seed", 42) + rank
@@ -192,40 +197,74 @@ def make_trace(workload, rank, world, sharding, pinned):
     return t, off, total, mode
 
 
-# Algorithmic bytes per launch of each kernel.
+# Algorithmic bytes per launch of each kernel, SURVEY.md 8(d) "Algorithmic
+# bytes per record" (what the method must move): MD 23 B per memory record
+# (addr 8, cta 4, tid 2, winst 4, site 4, meta 1), BD 15 B per BB record
+# (cta, tid, winst, site, meta), reuse 13 B per memory record read (addr,
+# cta, meta) + the previous-occurrence array P (4 B written + 4 B read).
+# The fused pass k_scan<7> streams the trace once: 23 B x mem + 15 B x BB.
+# Its other bytes (the BB records' addr column, the kept records it writes
+# for the reuse tail) are implementation passes, reported separately.
 def algorithmic_bytes(kname, st):
-    n, kept, mgroups, bgroups = st["n"], st["kept"], st["md_groups"], st["bd_groups"]
+    mem, bb, kept = st["n_mem"], st["n_bb"], st["kept"]
     table = {
-        "k_scan<7>": 23 * n + 12 * kept,            # every column once + kept records written (fused pass)
-        "k_scan<1>": 13 * n + 12 * kept,            # addr, cta, meta + kept records
-        "k_scan<2>": 23 * n,                        # addr, cta, tid, winst, site, meta
-        "k_scan<4>": 15 * n,                        # cta, tid, winst, site, meta
-        "k_scan<11>": 19 * n + 12 * kept,           # data-centric: addr, cta, tid, winst, meta + kept records
-        "k_rd_tile<0>": 12 * kept,                  # key 4 + value 8 per kept record
-        "k_squeeze": 24 * kept,                     # kept records read and written once
+        "k_scan<7>": 23 * mem + 15 * bb,
+        "k_scan<1>": 13 * mem,
+        "k_scan<2>": 23 * mem,
+        "k_scan<4>": 15 * bb,
+        "k_scan<11>": 23 * mem,                     # data-centric (reuse + MD per object)
+        "k_rd_seg": 8 * kept,                       # P of the kept records (4 B in + 4 B out, in registers)
+        "k_rd_tile<0>": 8 * kept,
     }
     return table.get(kname)
 
 
-def ncu_traffic(kname):
-    """DRAM bytes (read + write) per launch of `kname` from the committed
-    `ncu --set full` summary of this bench's workload, or None."""
-    import csv
-    p = os.path.join(os.path.dirname(os.path.abspath(__file__)), "profiles", "ncu_full_latest.csv")
+def implementation_bytes(kname, st):
+    """Bytes the kernel moves beyond algorithmic_bytes (not counted in frac)."""
+    if kname in ("k_scan<7>", "k_scan<1>", "k_scan<11>"):
+        return {"bb_addr_column": 8 * st["n_bb"] if kname == "k_scan<7>" else 0, "kept_record_writes": 12 * st["kept"]}
+    return {}
+
+
+def src_sha():
+    """Identity of the library build: hash of its sources and Makefile."""
+    import glob
+    import hashlib
+    h = hashlib.sha256()
+    files = sorted(glob.glob(os.path.join(ROOT, "paper_conf_cgo_shensll18_b200", "csrc", "*"))) + \
+        [os.path.join(ROOT, "include", "cadv.h"), os.path.join(ROOT, "Makefile")]
+    for f in files:
+        with open(f, "rb") as fh:
+            h.update(os.path.basename(f).encode())
+            h.update(fh.read())
+    return h.hexdigest()[:16]
+
+
+def ncu_traffic(kname, workload):
+    """DRAM bytes (read + write) per launch of `kname` from profiles/ncu_traffic.json,
+    written by tools/ncu_capture.sh from one `ncu --set full` capture of this
+    bench's workload -- used only when it was taken on the SAME library
+    sources (src_sha) and workload; else (None, reason)."""
+    p = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
-        with open(p) as f:
-            rows = list(csv.reader(f))
+        d = json.load(open(p))
+    except (OSError, ValueError):
+        return None, "no profiles/ncu_traffic.json"
+    if d.get("src_sha") != src_sha():
+        return None, f"profiles/ncu_traffic.json is from sources {d.get('src_sha')}, not {src_sha()}"
+    k = d.get("workloads", {}).get(workload, {}).get(kname)
+    if k is None:
+        return None, f"no {kname} capture for {workload}"
+    return int(k), f"profiles/ncu_traffic.json ({d.get('capture', 'ncu --set full')}, sources {d['src_sha']})"
+
+
+def cpu_model():
+    try:
+        for ln in open("/proc/cpuinfo"):
+            if ln.startswith("model name"):
+                return ln.split(":", 1)[1].strip()
     except OSError:
-        return None
-    hdr, units = rows[0], rows[1]
-    scale = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12, "": 1}
-    for r in rows[2:]:
-        if r[0] == kname:
-            tot = 0.0
-            for m in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
-                i = hdr.index(m)
-                tot += float(r[i]) * scale.get(units[i], 1)
-            return int(tot)
+        pass
     return None
 
 
@@ -250,6 +289,22 @@ def oracle_sample(t, target_s, line_bytes):
         n = min(t.n, int(n * max(2.0, min(8.0, (target_s / 3) / max(dt, 1e-3)))))
 
 
+def oracle_one_thread(t, nrec, line_bytes):
+    """The same oracle calls on the first nrec records with ONE thread."""
+    import oracle as orc
+    import tracegen as tg
+    sub = tg.from_arrays(*(t.cols[k][:nrec] for k, _ in tg.COLUMNS), nsites=t.nsites)
+    orc.set_num_threads(1)
+    try:
+        t0 = time.time()
+        orc.reuse(sub, line_bytes, 0, 0, 66)
+        orc.mem_div(sub, line_bytes, 32)
+        orc.branch_div(sub, 32)
+        return time.time() - t0
+    finally:
+        orc.set_num_threads(0)
+
+
 # ----------------------------------------------------------------- main
 
 def main():
@@ -266,8 +321,10 @@ def main():
     torch.cuda.set_device(local)
     if world > 1:
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-    t, goff, gtotal, mode = make_trace(args.workload, rank, world, args.sharding, pinned=True)
+    t, goff, gtotal, mode = make_trace(args.workload, rank, world, args.sharding, pinned=True, scaling=args.scaling)
     n = t.n
+    n_mem = int(((t.meta & 3) < 2).sum())
+    n_bb = n - n_mem
     nsites = t.nsites
     dev = {k: torch.from_numpy(t.cols[k]).to(f"cuda:{local}", non_blocking=True) for k in cadv.COLUMNS}
     torch.cuda.synchronize()
@@ -307,7 +364,8 @@ def main():
             r = torch.from_numpy(np.concatenate([h, hm.ravel(), tot]).astype(np.int64)).cuda()
             dist.all_reduce(r)
             launches += 1
-        return launches, ktimes, dict(n=n, kept=kept, md_groups=int(hm.sum()), bd_groups=int(tot[0]))
+        return launches, ktimes, dict(n=n, n_mem=n_mem, n_bb=n_bb, kept=kept, md_groups=int(hm.sum()),
+                                      bd_groups=int(tot[0]))
 
     # ---- warm-up (allocates the library workspace)
     for _ in range(max(args.warmup, 0)):
@@ -353,6 +411,11 @@ def main():
         total_records = int(sm[1])
     ms_step = ms_max / max(args.steps, 1)
     value = total_records * args.steps / (ms_max / 1e3)
+    total_mem = n_mem
+    if world > 1:
+        v = torch.tensor([float(n_mem)], dtype=torch.float64, device="cuda")
+        dist.all_reduce(v)
+        total_mem = int(v[0])
 
     # ---- dominant kernel roofline (live CUDA-event durations of the timed region)
     agg = {}
@@ -369,11 +432,19 @@ def main():
         avg_ms = tot_ms / cnt
         if per is not None:
             gbs = per / (avg_ms / 1e3) / 1e9
+            traffic, tsrc = ncu_traffic(dom, args.workload)
+            # the whole step by SURVEY 8(d) bytes: 31 B per memory record (23 B read
+            # once + the P array 4 B written and read) + 15 B per BB record
+            step_bytes = 31 * n_mem + 15 * n_bb
             roof = {"bound": "hbm", "kernel": dom, "achieved": round(gbs, 1), "peak": peak, "unit": "GB/s",
-                    "frac": round(gbs / peak, 4), "traffic": ncu_traffic(dom), "peak_source": peak_src,
-                    "traffic_source": "profiles/ncu_full_latest.csv (dram read+write bytes per launch, ncu --set full)",
-                    "avg_launch_ms": round(avg_ms, 4), "algorithmic_bytes_per_launch": per,
-                    "share_of_step": round(tot_ms / (ms * 1.0), 4)}
+                    "frac": round(gbs / peak, 4), "traffic": traffic, "peak_source": peak_src,
+                    "traffic_source": tsrc, "avg_launch_ms": round(avg_ms, 4),
+                    "algorithmic_bytes_per_launch": per,
+                    "algorithmic_bytes_rule": "SURVEY 8(d): 23 B x memory records + 15 B x BB records (k_scan<7>)",
+                    "implementation_bytes_per_launch": implementation_bytes(dom, stats),
+                    "share_of_step": round(tot_ms / (ms * 1.0), 4),
+                    "step_algorithmic_frac": round(step_bytes / (ms_step / 1e3) / 1e9 / peak, 4),
+                    "step_algorithmic_bytes": step_bytes}
     # ---- per-kernel breakdown of the step: a separate, untimed pass with
     # events around every launch
     kernels = {}
@@ -391,6 +462,36 @@ def main():
         ctx.set_profiling(False)
         kernels = {k: {"launches_per_step": v[1] / nb, "ms_per_step": round(v[0] / nb, 4)}
                    for k, v in sorted(kall.items(), key=lambda kv: -kv[1][0])}
+
+    # ---- per-analysis rates (reuse, MD and BD records/s
+    # separately, and "reuse+divergence" = memory records / (t_reuse + t_md)),
+    # each analysis alone through its own C-ABI call, CUDA events, untimed
+    # for the headline value
+    per_an = None
+    if world == 1 and not args.profile_run and not args.no_per_analysis:
+        calls = {"reuse": lambda: ctx.reuse_histogram(lb, SC, cadv.BINS_LINEAR, NB),
+                 "mem_div": lambda: ctx.mem_divergence(lb, 32, nsites),
+                 "branch_div": lambda: ctx.branch_divergence(32, nsites)}
+        per_an = {}
+        ksteps = max(3, min(args.steps, 10))
+        for nm, fn in calls.items():
+            fn()
+            torch.cuda.synchronize()
+            a0, a1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a0.record(stream)
+            for _ in range(ksteps):
+                fn()
+            a1.record(stream)
+            torch.cuda.synchronize()
+            ams = a0.elapsed_time(a1) / ksteps
+            recs = n_bb if nm == "branch_div" else n_mem
+            per_an[nm] = {"ms_per_call": round(ams, 4), "records": recs,
+                          "records_per_s": round(recs / (ams / 1e3), 1),
+                          "record_kind": "BB records" if nm == "branch_div" else "memory records"}
+        per_an["reuse_plus_divergence"] = {
+            "records_per_s": round(n_mem / ((per_an["reuse"]["ms_per_call"] + per_an["mem_div"]["ms_per_call"]) / 1e3), 1),
+            "definition": "memory records / (t_reuse + t_mem_div), SURVEY 8(d)"}
+        per_an["fused_mem_records_per_s"] = round(n_mem * args.steps / (ms / 1e3), 1)
 
     # ---- data-centric attribution: the same trace, per-object
     # RD + MD rows over the workload's allocation table (one fused pass)
@@ -424,7 +525,7 @@ def main():
                 a[0] += t_ms
                 a[1] += 1
             ddom = max(dagg.items(), key=lambda kv: kv[1][0])[0]
-            per = algorithmic_bytes(ddom, dict(n=n, kept=dkept, md_groups=0, bd_groups=0))
+            per = algorithmic_bytes(ddom, dict(n=n, n_mem=n_mem, n_bb=n_bb, kept=dkept, md_groups=0, bd_groups=0))
             davg = dagg[ddom][0] / dagg[ddom][1]
             dcen = {"value": round(n / (dms / 1e3), 1), "unit": UNIT, "ms_per_step": round(dms, 3),
                     "objects": int(len(objs[0])), "call": "cadv_data_centric(rd + md rows per object)",
@@ -463,29 +564,34 @@ def main():
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu_baseline and not args.profile_run:
         rec, dt, cores, desc = oracle_sample(t, args.cpu_seconds, lb)
+        n1 = max(1, rec // max(1, cores))
+        dt1 = oracle_one_thread(t, n1, lb)
         cpu = {"value": round(rec / dt, 1), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc,
-               "seconds": round(dt, 2)}
+               "seconds": round(dt, 2), "cpu_model": cpu_model(),
+               "one_thread": {"value": round(n1 / dt1, 1), "unit": UNIT, "records": n1, "seconds": round(dt1, 2)}}
 
     if rank == 0:
         name, params = WORKLOADS[args.workload]
         line = {
             "metric": METRIC, "value": round(value, 1), "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": round(ms_step, 3), "higher_is_better": True,
-            "scaling": "weak", "vs_baseline": None, "dtype": "u64", "data": "synthetic",
+            "scaling": args.scaling if world > 1 else "weak", "vs_baseline": None, "dtype": "u64",
+            "data": "synthetic",
+            "mem_records_per_s": round(total_mem * args.steps / (ms_max / 1e3), 1),
             "config": {"workload": args.workload, "generator": name, "params": params,
                        "records_per_gpu": n, "mem_records_per_gpu": int(((t.meta & 3) < 2).sum()),
                        "line_bytes": lb, "warp_size": 32, "rd_scope": args.rd_scope, "rd_bins": "linear 66",
                        "analyses": ("load_trace + reuse + mem_div + branch_div (three calls)" if args.separate else
                                     "load_trace + cadv_analyze(reuse, mem_div, branch_div: one fused pass)"),
                        "l2": "inputs larger than L2 (trace >> 126 MB), no flush needed",
-                       "global_records": gtotal, "sharding": mode,
+                       "global_records": gtotal, "sharding": mode, "src_sha": src_sha(),
                        "parallelism": (f"position-range shards of one trace over {world} GPUs (library NCCL: "
                                        "kept records exchanged by CTA range, T_c max, histograms all-reduced)"
                                        if mode == "position" else
                                        f"dp{world} (independent trace per GPU, histograms all-reduced)"
                                        if world > 1 else "single GPU")},
             "roofline": roof, "cpu_baseline": cpu, "e2e": e2e, "gpu_launches": launches,
-            "clocks": ck, "kernels": kernels, "data_centric": dcen,
+            "clocks": ck, "kernels": kernels, "per_analysis": per_an, "data_centric": dcen,
         }
         print(json.dumps(line), flush=True)
     ctx.destroy()
@@ -525,7 +631,7 @@ def run_reference(args, rank, world):
         "config": {"workload": args.workload, "generator": name, "params": params, "line_bytes": lb,
                    "sample_records": nsamp},
         "cpu_baseline": {"value": round(value, 1), "unit": UNIT, "cores": cores, "kind": "oracle",
-                         "sample": desc},
+                         "sample": desc, "cpu_model": cpu_model()},
         "e2e": {"value": round(value, 1), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)

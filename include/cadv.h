@@ -127,6 +127,23 @@ CADV_API cadv_status cadv_create(cadv_ctx **out, int device, void *cuda_stream,
  * it to the other ranks, e.g. with torch.distributed, before cadv_create). */
 CADV_API cadv_status cadv_nccl_unique_id(void *out128);
 
+/* Multi-rank context over the library's OWN collectives (no NCCL): every
+ * collective is one kernel that reads the peers' staged device buffers
+ * through CUDA IPC mappings (NVLink / NVSwitch between GPUs; local HBM when
+ * ranks share a GPU), with a host TCP bootstrap for the IPC handles,
+ * offsets and barriers: bootstrap_addr = "a.b.c.d:port" of rank 0 (every
+ * rank passes the same string; rank 0 listens there).  One process per rank;
+ * collective like cadv_create.  CADV_ERR_NCCL if the bootstrap fails within
+ * 120 s. */
+CADV_API cadv_status cadv_create_peer(cadv_ctx **out, int device, void *cuda_stream, const char *bootstrap_addr,
+                                      int rank, int nranks);
+
+/* Host-only check of the peer backend's TCP bootstrap (no GPU needed):
+ * allgathers `bytes` bytes from every rank into out[nranks * bytes] and
+ * returns 0 on success. */
+CADV_API int cadv_bootstrap_selftest(const char *bootstrap_addr, int rank, int nranks, const void *in, void *out,
+                                     uint64_t bytes);
+
 /* In-process multi-rank contexts for testing on one GPU: a group of nranks
  * ranks that exchange data through host staging instead of NCCL.  Each rank
  * is a thread of the calling process holding its own context (created with

@@ -12,7 +12,7 @@
  * analyses group by (reading R9).
  *
  * Usage inside a kernel (the buffer lives in device memory; see
- * paper_conf_cgo_shensll18_b200/producer.py for a host-side allocator):
+ * paper_conf_cgo_shensll18_b200/producer/__init__.py for a host-side allocator):
  *     cadv_record_bb(T, SITE_LOOP);                 // a basic block entered
  *     cadv_record_load(T, &a[i], sizeof a[i], SITE_LD_A);  float x = a[i];
  *     cadv_record_store(T, &c[i], sizeof c[i], SITE_ST_C); c[i] = x;

@@ -55,6 +55,8 @@ def _load():
     for f in ("oracle_reuse", "oracle_reuse_rd", "oracle_reuse_brute", "oracle_mem_div",
               "oracle_branch_div", "oracle_data_centric", "oracle_num_threads", "oracle_reuse_fenwick"):
         getattr(lib, f).restype = ctypes.c_int
+    lib.oracle_set_num_threads.restype = None
+    lib.oracle_set_num_threads.argtypes = [ctypes.c_int]
     _lib = lib
     return lib
 
@@ -70,6 +72,11 @@ def _check(rc):
 
 def num_threads() -> int:
     return int(_load().oracle_num_threads())
+
+
+def set_num_threads(k: int) -> None:
+    """OpenMP threads of the following oracle calls (0 = all cores)."""
+    _load().oracle_set_num_threads(int(k))
 
 
 def reuse(t, line_bytes=128, scope=SCOPE_CTA, binning=BINS_LINEAR, nbins=66):

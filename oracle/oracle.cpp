@@ -323,29 +323,37 @@ void fenwick_scope(const std::vector<uint64_t>& idx, const uint64_t* addr, const
     for (size_t x = pos; x > 0; x -= x & (0 - x)) r += bit[x];
     return r;
   };
-  std::unordered_map<uint64_t, uint64_t> epoch;                 // e(s, line)
-  std::unordered_map<RKey, std::pair<uint64_t, uint64_t>, KeyHash> last;  // key -> (last position, uses)
+  // per line: its CURRENT renamed element (the one a load would use: the
+  // latest store's, or the never-written one) -> (last position, uses);
+  // an element replaced by a store is never used again, so only its use
+  // count (streaming) is settled then -- its mark stays in the tree
+  struct Cur { uint64_t last, uses; };
+  std::unordered_map<uint64_t, Cur> cur;
   for (size_t k = 0; k < m; ++k) {
     const uint64_t i = idx[k];
     const uint64_t line = addr[i] / line_bytes;
     const bool store = (meta[i] & 3u) == KIND_STORE;
-    RKey key{line, store ? ++epoch[line] : epoch[line]};
-    auto it = last.find(key);
-    if (it == last.end()) {                   // first use of the (renamed) element: ∞
+    auto it = cur.find(line);
+    if (store || it == cur.end()) {           // first use of a (renamed) element: ∞
       h[nbins - 1]++;
-      last.emplace(key, std::make_pair((uint64_t)k, (uint64_t)1));
+      if (it == cur.end()) {
+        cur.emplace(line, Cur{(uint64_t)k, 1});
+      } else {
+        if (it->second.uses == 1) streaming++;  // the replaced element was used once
+        it->second = Cur{(uint64_t)k, 1};
+      }
     } else {
-      const uint64_t p = it->second.first;
+      const uint64_t p = it->second.last;
       const uint64_t d = prefix(k) - prefix(p + 1);
       h[bin_of(d, binning, nbins)]++;
       fsum += d;
       add(p, -1);
-      it->second.first = k;
-      it->second.second++;
+      it->second.last = k;
+      it->second.uses++;
     }
     add(k, 1);
   }
-  for (auto& kv : last) if (kv.second.second == 1) streaming++;
+  for (auto& kv : cur) if (kv.second.uses == 1) streaming++;
 }
 }  // namespace
 
@@ -610,6 +618,16 @@ int oracle_num_threads(void) {
   return omp_get_max_threads();
 #else
   return 1;
+#endif
+}
+
+// Thread count of the following calls (bench.py's 1-thread baseline); 0 = all cores.
+void oracle_set_num_threads(int k) {
+#ifdef _OPENMP
+  static const int all = omp_get_max_threads();
+  omp_set_num_threads(k > 0 ? k : all);
+#else
+  (void)k;
 #endif
 }
 

@@ -103,6 +103,10 @@ def lib():
     L.cadv_loopback_group_destroy.restype = i32
     L.cadv_create_loopback.argtypes = [ctypes.POINTER(P), i32, P, P, i32]
     L.cadv_create_loopback.restype = i32
+    L.cadv_create_peer.argtypes = [ctypes.POINTER(P), i32, P, ctypes.c_char_p, i32, i32]
+    L.cadv_create_peer.restype = i32
+    L.cadv_bootstrap_selftest.argtypes = [ctypes.c_char_p, i32, i32, P, P, u64]
+    L.cadv_bootstrap_selftest.restype = i32
     _lib = L
     return L
 
@@ -129,10 +133,13 @@ class Context:
     """One analysis context (one per GPU / rank): cadv_create ... cadv_destroy."""
 
     def __init__(self, device: int = 0, stream=None, nccl_id: bytes | None = None, rank: int = 0, nranks: int = 1,
-                 loopback=None):
+                 loopback=None, peer_addr: str | None = None):
         L = lib()
         h = ctypes.c_void_p()
-        if loopback is not None:
+        if peer_addr is not None:
+            s = L.cadv_create_peer(ctypes.byref(h), int(device), ctypes.c_void_p(stream or 0), peer_addr.encode(),
+                                   int(rank), int(nranks))
+        elif loopback is not None:
             s = L.cadv_create_loopback(ctypes.byref(h), int(device), ctypes.c_void_p(stream or 0), loopback.handle,
                                        int(rank))
             nranks = loopback.nranks
@@ -284,10 +291,24 @@ class Context:
         self.destroy()
 
 
-def create(device: int = 0, stream=None, nccl_id: bytes | None = None, rank: int = 0, nranks: int = 1) -> Context:
+def create(device: int = 0, stream=None, nccl_id: bytes | None = None, rank: int = 0, nranks: int = 1,
+           peer_addr: str | None = None) -> Context:
     """cadv_create.  nranks > 1: one process per GPU, all ranks pass the same
-    nccl_id (from nccl_unique_id() on rank 0)."""
-    return Context(device, stream, nccl_id, rank, nranks)
+    nccl_id (from nccl_unique_id() on rank 0) -- or the same peer_addr
+    ("127.0.0.1:port" of rank 0) for cadv_create_peer, the library's own
+    collectives over CUDA IPC peer memory."""
+    return Context(device, stream, nccl_id, rank, nranks, peer_addr=peer_addr)
+
+
+def bootstrap_selftest(addr: str, rank: int, nranks: int, payload: bytes) -> bytes:
+    """cadv_bootstrap_selftest: host-only allgather over the peer backend's TCP
+    bootstrap (no GPU); returns the nranks payloads concatenated in rank order."""
+    out = ctypes.create_string_buffer(len(payload) * nranks)
+    rc = lib().cadv_bootstrap_selftest(addr.encode(), int(rank), int(nranks), ctypes.c_char_p(payload), out,
+                                       len(payload))
+    if rc != 0:
+        raise CadvError(CADV_ERR_NCCL, f"bootstrap self-test failed ({rc})")
+    return out.raw
 
 
 def nccl_unique_id() -> bytes:

@@ -248,11 +248,11 @@ CADV_API const char* cadv_version(void) { return "cadv 0.1 (sm_100a)"; }
 namespace {
 
 cadv_status create_ctx(cadv_ctx** out, int device, void* cuda_stream, const void* nccl_unique_id,
-                       LoopbackGroup* group, int rank, int nranks) {
+                       LoopbackGroup* group, int rank, int nranks, const char* peer_addr = nullptr) {
   if (!out) return CADV_ERR_INVALID_ARG;
   *out = nullptr;
   if (nranks < 1 || rank < 0 || rank >= nranks) return CADV_ERR_INVALID_ARG;
-  if (nranks > 1 && !nccl_unique_id && !group) return CADV_ERR_INVALID_ARG;
+  if (nranks > 1 && !nccl_unique_id && !group && !peer_addr) return CADV_ERR_INVALID_ARG;
   int ndev = 0;
   if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
     cudaGetLastError();
@@ -277,6 +277,17 @@ cadv_status create_ctx(cadv_ctx** out, int device, void* cuda_stream, const void
   }
   if (group) {
     c->comm = make_loopback_comm(group, rank);
+  } else if (peer_addr) {
+    std::string err;
+    c->comm = make_peer_comm(peer_addr, rank, nranks, &err);
+    if (!c->comm) {
+      fprintf(stderr, "cadv_create_peer: %s\n", err.c_str());
+      cudaEventDestroy(c->ev0);
+      cudaEventDestroy(c->ev1);
+      cudaFreeHost(c->hstage);
+      delete c;
+      return CADV_ERR_NCCL;
+    }
   } else if (nccl_unique_id) {
     std::string err;
     c->comm = make_nccl_comm(nccl_unique_id, rank, nranks, &err);
@@ -310,6 +321,27 @@ CADV_API cadv_status cadv_nccl_unique_id(void* out128) {
     return CADV_ERR_NCCL;
   }
   return CADV_OK;
+}
+
+CADV_API cadv_status cadv_create_peer(cadv_ctx** out, int device, void* cuda_stream, const char* bootstrap_addr,
+                                     int rank, int nranks) {
+  if (!bootstrap_addr) return CADV_ERR_INVALID_ARG;
+  return create_ctx(out, device, cuda_stream, nullptr, nullptr, rank, nranks, bootstrap_addr);
+}
+
+CADV_API int cadv_bootstrap_selftest(const char* bootstrap_addr, int rank, int nranks, const void* in, void* out,
+                                     uint64_t bytes) {
+  if (!bootstrap_addr || nranks < 1 || rank < 0 || rank >= nranks || (bytes && (!in || !out))) return 1;
+  std::string err;
+  Bootstrap* b = make_tcp_bootstrap(bootstrap_addr, rank, nranks, 60, &err);
+  if (!b) {
+    fprintf(stderr, "cadv_bootstrap_selftest: %s\n", err.c_str());
+    return 2;
+  }
+  int e = b->allgather(in, out, bytes);
+  e |= b->barrier();
+  delete b;
+  return e ? 3 : 0;
 }
 
 CADV_API void* cadv_loopback_group_create(int nranks) { return nranks >= 1 ? loopback_group_new(nranks) : nullptr; }
@@ -634,7 +666,7 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
       }
     }
     if (q.rd && hs.kept_max > rs.chunk_cap) {  // a warp's kept records overflowed its region
-      c->kdiv = 1;
+      c->kcap_min = hs.kept_max + hs.kept_max / 8;
       again = true;
     }
     if (again && !hs.err_code && !multi) return RETRY;

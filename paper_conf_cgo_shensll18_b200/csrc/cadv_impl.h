@@ -98,10 +98,10 @@ struct cadv_ctx {
   int seg_ctas = 0;           // k_rd_seg CTAs per SM for seg_ctas_smem bytes of shared memory
   size_t seg_ctas_smem = 0;
   bool noncontig_any = false;
-  // kept-record region capacity of a scan warp = chunk / kdiv records (grown
-  // to the whole chunk, for the context's lifetime, the first time a region
-  // overflows: the call then runs again)
-  uint32_t kdiv = 4; // multi-rank: some rank's shard is not warp-contiguous (load_trace)
+  // kept-record region capacity of a scan warp = max(chunk / 4, kcap_min)
+  // records; a region that overflows raises kcap_min to its kept count + 1/8
+  // (for the context's lifetime) and the call runs again
+  uint64_t kcap_min = 0; // multi-rank: some rank's shard is not warp-contiguous (load_trace)
 };
 
 namespace cadv {

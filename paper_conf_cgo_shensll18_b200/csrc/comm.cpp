@@ -6,9 +6,11 @@
 //             already loaded (torch's), so libcadv has no link-time NCCL
 //             dependency and there is one NCCL per process.
 //   loopback  N ranks = N threads of one process (tests on a single GPU):
-//             buffers are exchanged through host staging under a
-//             barrier.  Same call sequence as NCCL, so the analysis code that
-//             drives the collectives is the one the NCCL path runs.
+//             the peer backend's device kernels (comm_peer.cu) over the
+//             ranks' buffers, with the group's host barrier as bootstrap.
+//             Same call sequence as NCCL, so the analysis code that drives
+//             the collectives is the one the NCCL path runs.
+// (A third backend, peer over TCP bootstrap + CUDA IPC, is in comm_peer.cu.)
 #include <cuda_runtime.h>
 #include <dlfcn.h>
 #include <nccl.h>
@@ -82,9 +84,6 @@ class NcclComm : public Comm {
  public:
   NcclComm(int rank, int nranks, ncclComm_t c) : Comm(rank, nranks), comm_(c) {}
   ~NcclComm() override {
-    for (auto& v : cache_)
-      for (auto& m : v)
-        if (m.ptr) cudaIpcCloseMemHandle(m.ptr);
     if (dev_) cudaFree(dev_);
     if (comm_) g_nccl.CommDestroy(comm_);
   }
@@ -109,43 +108,32 @@ class NcclComm : public Comm {
     return e;
   }
   int map_peers(int slot, void* local, void** peers, cudaStream_t s) override {
-    cudaIpcMemHandle_t h;
-    if (cu(cudaIpcGetMemHandle(&h, local))) return 1;
+    (void)slot;
+    IpcRef h;
+    if (ipc_export(local, &h, &err)) return 1;
     if (!dev_) {
       if (cu(cudaMalloc(&dev_, (size_t)(nranks + 1) * sizeof h))) return 1;
     }
     uint8_t* d = (uint8_t*)dev_;
     if (cu(cudaMemcpyAsync(d, &h, sizeof h, cudaMemcpyHostToDevice, s))) return 1;
     if (ck(g_nccl.AllGather(d, d + sizeof h, sizeof h, ncclUint8, comm_, s))) return 1;
-    std::vector<cudaIpcMemHandle_t> all(nranks);
+    std::vector<IpcRef> all(nranks);
     if (cu(cudaMemcpyAsync(all.data(), d + sizeof h, nranks * sizeof h, cudaMemcpyDeviceToHost, s))) return 1;
     if (cu(cudaStreamSynchronize(s))) return 1;
-    if ((int)cache_.size() <= slot) cache_.resize(slot + 1, std::vector<Mapped>(nranks));
     for (int p = 0; p < nranks; ++p) {
       if (p == rank) { peers[p] = local; continue; }
-      Mapped& m = cache_[slot][p];
-      if (!m.ptr || memcmp(&m.h, &all[p], sizeof h)) {
-        if (m.ptr) cudaIpcCloseMemHandle(m.ptr);
-        m.ptr = nullptr;
-        if (cu(cudaIpcOpenMemHandle(&m.ptr, all[p], cudaIpcMemLazyEnablePeerAccess))) return 1;
-        m.h = all[p];
-      }
-      peers[p] = m.ptr;
+      if (!(peers[p] = ipc_.open(all[p], &err))) return 1;
     }
     return 0;
   }
   int barrier(cudaStream_t s) override {
-    if (!dev_ && cu(cudaMalloc(&dev_, (size_t)(nranks + 1) * sizeof(cudaIpcMemHandle_t)))) return 1;
+    if (!dev_ && cu(cudaMalloc(&dev_, (size_t)(nranks + 1) * sizeof(IpcRef)))) return 1;
     if (ck(g_nccl.AllReduce(dev_, dev_, 1, ncclUint32, ncclMax, comm_, s))) return 1;
     return cu(cudaStreamSynchronize(s));
   }
 
  private:
-  struct Mapped {
-    cudaIpcMemHandle_t h;
-    void* ptr = nullptr;
-  };
-  std::vector<std::vector<Mapped>> cache_;
+  IpcCache ipc_;
   void* dev_ = nullptr;
   int cu(cudaError_t e) {
     if (e == cudaSuccess) return 0;
@@ -189,15 +177,13 @@ Comm* make_nccl_comm(const void* id128, int rank, int nranks, std::string* err) 
 
 // ------------------------------------------------------------------ loopback
 struct LoopbackGroup {
-  explicit LoopbackGroup(int n) : n(n), slot(n), soff(n), scnt(n), ptr(n, nullptr) {}
+  explicit LoopbackGroup(int n) : n(n), slot(n) {}
   int n;
   std::mutex mu;
   std::condition_variable cv;
   int arrived = 0;
   uint64_t generation = 0;
-  std::vector<std::vector<uint8_t>> slot;  // per-rank host staging of the contribution
-  std::vector<std::vector<uint64_t>> soff, scnt;
-  std::vector<void*> ptr;  // map_peers: the ranks' device buffers (one process, one address space)
+  std::vector<std::vector<uint8_t>> slot;  // per-rank host blob (bootstrap allgather)
   void barrier() {
     std::unique_lock<std::mutex> lk(mu);
     const uint64_t g = generation;
@@ -217,97 +203,30 @@ int loopback_group_size(const LoopbackGroup* g) { return g->n; }
 
 namespace {
 
-class LoopbackComm : public Comm {
+// The loopback group as a bootstrap: thread ranks exchange host blobs
+// through the group's slots under its barrier.  The data path is PeerComm's
+// (device kernels reading the other ranks' staging buffers directly: one
+// process, one address space), the same kernels the multi-process peer
+// backend runs over CUDA IPC mappings.
+class LoopbackBootstrap : public Bootstrap {
  public:
-  LoopbackComm(LoopbackGroup* g, int rank) : Comm(rank, g->n), g_(g) {}
-  int allreduce_sum_u64(uint64_t* d, size_t n, cudaStream_t s) override { return reduce(d, n * 8, s, true); }
-  int allreduce_max_u32(uint32_t* d, size_t n, cudaStream_t s) override { return reduce(d, n * 4, s, false); }
-  int allgather(const void* send, void* recv, size_t bytes, cudaStream_t s) override {
-    const int e0 = publish(send, bytes, s);
+  LoopbackBootstrap(LoopbackGroup* g, int rank) : Bootstrap(rank, g->n), g_(g) {}
+  int allgather(const void* in, void* out, size_t bytes) override {
+    g_->slot[rank].assign((const uint8_t*)in, (const uint8_t*)in + bytes);
     g_->barrier();
-    if (e0) return finish(1);
-    for (int p = 0; p < nranks; ++p)
-      if (bytes && cuda(cudaMemcpyAsync((uint8_t*)recv + (size_t)p * bytes, g_->slot[p].data(), bytes,
-                                        cudaMemcpyHostToDevice, s)))
-        return finish(1);
-    return finish(cuda(cudaStreamSynchronize(s)));
-  }
-  int alltoallv(const void* send, const uint64_t* soff, const uint64_t* scnt, void* recv, const uint64_t* roff,
-                const uint64_t* rcnt, cudaStream_t s) override {
-    uint64_t end = 0;
-    for (int p = 0; p < nranks; ++p) end = soff[p] + scnt[p] > end ? soff[p] + scnt[p] : end;
-    const int e0 = publish(send, end, s);
-    g_->soff[rank].assign(soff, soff + nranks);
-    g_->scnt[rank].assign(scnt, scnt + nranks);
-    g_->barrier();
-    if (e0) return finish(1);
-    for (int p = 0; p < nranks; ++p) {
-      if (g_->scnt[p][rank] != rcnt[p]) {
-        err = "loopback alltoallv: send / receive counts disagree";
-        return finish(1);
-      }
-      if (rcnt[p] && cuda(cudaMemcpyAsync((uint8_t*)recv + roff[p], g_->slot[p].data() + g_->soff[p][rank], rcnt[p],
-                                          cudaMemcpyHostToDevice, s)))
-        return finish(1);
-    }
-    return finish(cuda(cudaStreamSynchronize(s)));
-  }
-  int map_peers(int slot, void* local, void** peers, cudaStream_t s) override {
-    (void)slot;
-    const int e0 = cuda(cudaStreamSynchronize(s));
-    g_->ptr[rank] = local;
-    g_->barrier();
-    for (int p = 0; p < nranks; ++p) peers[p] = g_->ptr[p];
-    return finish(e0);
-  }
-  int barrier(cudaStream_t s) override {
-    const int e0 = cuda(cudaStreamSynchronize(s));
-    return finish(e0);
+    for (int p = 0; p < nranks; ++p) memcpy((uint8_t*)out + (size_t)p * bytes, g_->slot[p].data(), bytes);
+    g_->barrier();  // nobody rewrites a slot before every rank has read it
+    return 0;
   }
 
  private:
-  int cuda(cudaError_t e) {
-    if (e == cudaSuccess) return 0;
-    err = std::string("loopback: ") + cudaGetErrorString(e);
-    return 1;
-  }
-  // the rank's contribution -> its host slot
-  int publish(const void* d, size_t bytes, cudaStream_t s) {
-    g_->slot[rank].resize(bytes);
-    if (bytes && cuda(cudaMemcpyAsync(g_->slot[rank].data(), d, bytes, cudaMemcpyDeviceToHost, s))) return 1;
-    return cuda(cudaStreamSynchronize(s));
-  }
-  // second barrier: nobody rewrites a slot before every rank has read it.
-  // A rank that failed still takes part in both barriers (no deadlock).
-  int finish(int e) {
-    g_->barrier();
-    return e;
-  }
-  int reduce(void* d, size_t bytes, cudaStream_t s, bool sum64) {
-    const int e0 = publish(d, bytes, s);
-    g_->barrier();
-    if (e0) return finish(1);
-    std::vector<uint8_t> acc(g_->slot[0]);
-    for (int p = 1; p < nranks; ++p) {
-      if (sum64) {
-        uint64_t* a = (uint64_t*)acc.data();
-        const uint64_t* b = (const uint64_t*)g_->slot[p].data();
-        for (size_t i = 0; i < bytes / 8; ++i) a[i] += b[i];
-      } else {
-        uint32_t* a = (uint32_t*)acc.data();
-        const uint32_t* b = (const uint32_t*)g_->slot[p].data();
-        for (size_t i = 0; i < bytes / 4; ++i) a[i] = a[i] > b[i] ? a[i] : b[i];
-      }
-    }
-    int e = bytes ? cuda(cudaMemcpyAsync(d, acc.data(), bytes, cudaMemcpyHostToDevice, s)) : 0;
-    if (!e) e = cuda(cudaStreamSynchronize(s));
-    return finish(e);
-  }
   LoopbackGroup* g_;
 };
 
 }  // namespace
 
-Comm* make_loopback_comm(LoopbackGroup* g, int rank) { return new LoopbackComm(g, rank); }
+Comm* make_loopback_comm(LoopbackGroup* g, int rank) {
+  return new PeerComm(new LoopbackBootstrap(g, rank), true, true);
+}
 
 }  // namespace cadv

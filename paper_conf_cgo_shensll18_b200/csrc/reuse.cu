@@ -1265,11 +1265,11 @@ cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st) {
   uint64_t grid, nw, chunk;
   scan_geometry(c, n, &grid, &nw, &chunk);
   st->grid = nw;  // one kept-record region per scan warp
-  // region capacity: chunk / kdiv records (run compression keeps ~7 % of the
-  // paper-shaped traces; a region that overflows makes the call run again
-  // with whole-chunk regions, see run_once), so C5's 4e9 records need 24 B
-  // per kept slot instead of per record
-  uint64_t kcap = chunk / (c->kdiv ? c->kdiv : 1);
+  // region capacity: max(chunk / 4, kcap_min) records (run compression keeps
+  // ~7 % of the paper-shaped traces; a region that overflows raises kcap_min
+  // and the call runs again, see run_once), so C5's 4e9 records need 24 B per
+  // kept slot, not per record
+  uint64_t kcap = chunk / 4 > c->kcap_min ? chunk / 4 : c->kcap_min;
   kcap = ((kcap + 255) / 256) * 256;
   if (kcap > chunk) kcap = chunk;
   st->chunk_cap = kcap;

@@ -283,10 +283,6 @@ __device__ __forceinline__ uint32_t run_hi(uint32_t tid, uint32_t meta) {
 }
 
 // ------------------------------------------------------------------ group finishing
-struct Acc {              // per-lane BD accumulators, reduced at the end
-  uint32_t bd_exec, bd_threads;
-};
-
 // row (F_OBJ): the object row of the group's first record
 template <int F>
 __device__ __forceinline__ void finish_md(const ScanArgs& A, const Counters& C, uint32_t* whist, bool sites_smem,
@@ -305,66 +301,80 @@ __device__ __forceinline__ void finish_md(const ScanArgs& A, const Counters& C, 
   }
 }
 
-// One BB group: exec / threads, T_c candidate, per-site counters; groups with
-// fewer than W active lanes are deferred until T_c is known (k_bd_resolve).
-__device__ __forceinline__ void finish_bd(const ScanArgs& A, const Counters& C, Acc& acc, bool sites_smem,
-                                          uint32_t cnt, uint32_t s, uint32_t cta, uint32_t wsub, uint32_t maxtid) {
-  acc.bd_exec += 1;
-  acc.bd_threads += cnt;
-  tc_update(A, cta, maxtid);
-  atomicMax(&A.sc->max_cta, (unsigned long long)cta);  // rare (exact walk) path
+// BD per-site counters of one complete group (exec, threads)
+__device__ __forceinline__ void bd_sites_add(const ScanArgs& A, const Counters& C, bool sites_smem, uint32_t s,
+                                             uint32_t cnt) {
   if (sites_smem) {
     if (s < A.nsites) { atomicAdd(&C.bd_sites[3 * s], 1u); atomicAdd(&C.bd_sites[3 * s + 2], cnt); }
     else *A.site_flag = 1;
   } else if (A.nsites) {
     site_add(A, nullptr, A.bd_sites, 3, s, 1, cnt);
   }
-  if (cnt < (1u << A.ws_bd)) {
-    const unsigned long long k = atomicAdd(A.ndefer, 1ull);
-    if (k < A.defer_cap) A.defer[k] = make_uint4(cta, wsub, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
-  }
 }
 
-
-// Exact resolution of one run [j0, j0 + nrec) read back from the ring: every
-// sub-warp group's distinct lines (MD) / lanes (BD) by pairwise comparison.
-// Used for runs whose lines are not non-decreasing (MD), for analysis warp
-// sizes below 32 and to report runs with more than 32 records (a lane must
-// repeat).  Reads the run from global memory (rare path).
-template <int F>
-__device__ __noinline__ void walk_run(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
-                                      uint64_t g0, uint32_t nrec) {
-  if (nrec > 32) { report(A.sc, g0, 2); return; }
-  Acc acc{0, 0};
-  const bool bb = (__ldg(A.meta + g0) & 3u) == 2u;
+// Warp-cooperative exact resolution of ONE run [g0, g0 + nrec), nrec <= 32,
+// re-read from global memory (recently streamed: L2) one record per lane:
+// the run's sub-warp groups (tid % 32 >> ws, analysis warp size 2^ws) with
+// their distinct lines (MD: __match_any_sync on the line within the group,
+// first lane of each line counted) or their lane sets (BD).  Used for runs
+// whose lines are not non-decreasing (MD: the fast path counts line changes)
+// and for analysis warp sizes below 32; the whole warp calls it with
+// warp-uniform arguments.  The run's records share kind, CTA and site (the
+// scan checks R19).  exec / thr / mxc: the caller's BD accumulators.
+// The run's records come from global memory (SMEM = false: g0 = trace
+// position; queued runs whose stage was recycled) or from the warp's ring
+// stage (SMEM = true: ta / aa point at the run's first record there).
+template <int F, bool SMEM>
+__device__ __forceinline__ void walk_warp(const ScanArgs& A, const Counters& C, uint32_t* whist, bool sites_smem,
+                                          uint64_t g0, const uint16_t* ta, const uint64_t* aa, uint32_t nrec,
+                                          uint32_t kind, uint32_t cta, uint32_t s, uint32_t& exec, uint32_t& thr,
+                                          uint32_t& mxc) {
+  const uint32_t lane = lane_id();
+  const bool bb = kind == 2u;
   const uint32_t ws = bb ? A.ws_bd : A.ws_md;
-  for (uint32_t r = 0; r < nrec; ++r) {
-    const uint32_t tr = __ldg(A.tid + g0 + r), sub = (tr & 31u) >> ws;
-    bool leader = true;
-    for (uint32_t q = 0; q < r && leader; ++q) leader = ((__ldg(A.tid + g0 + q) & 31u) >> ws) != sub;
-    if (!leader) continue;
-    uint32_t deg = 0, cnt = 0, mask = 0, maxt = 0;
-    for (uint32_t q = r; q < nrec; ++q) {
-      const uint32_t tq = __ldg(A.tid + g0 + q);
-      if (((tq & 31u) >> ws) != sub) continue;
-      cnt++;
-      mask |= 1u << (tq & 31u);
-      maxt = max(maxt, tq);
-      if (!bb) {
-        const uint64_t lq = __ldg(A.addr + g0 + q) >> A.lbs_md;
-        bool first = true;
-        for (uint32_t u = r; u < q && first; ++u)
-          if (((__ldg(A.tid + g0 + u) & 31u) >> ws) == sub && (__ldg(A.addr + g0 + u) >> A.lbs_md) == lq) first = false;
-        deg += first;
-      }
-    }
-    if ((uint32_t)__popc(mask) != cnt) { report(A.sc, g0 + r, 2); continue; }
-    const uint32_t s = A.nsites ? __ldg(A.site + g0 + r) : 0u;
-    if (bb) finish_bd(A, C, acc, sites_smem, cnt, s, __ldg(A.cta + g0 + r), tr >> ws, maxt);
-    else finish_md<F>(A, C, whist, sites_smem, __ldg(A.meta + g0 + r) & 3u, deg, s,
-                      (F & F_OBJ) ? row_of(A, C, __ldg(A.addr + g0 + r) >> A.lbs_md) : 0u);
+  const bool v = lane < nrec;
+  const uint32_t vm = nrec >= 32u ? FULL : ((1u << nrec) - 1u);
+  const uint32_t t = v ? (SMEM ? (uint32_t)ta[lane] : (uint32_t)__ldg(A.tid + g0 + lane)) : 0u;
+  const uint32_t lb = t & 31u;
+  // lane set of the run; a repeated lane makes the popcount fall short
+  const uint32_t M = __reduce_or_sync(FULL, v ? 1u << lb : 0u);
+  if ((uint32_t)__popc(M) != nrec) {
+    if (lane == 0) report(A.sc, g0, 2);
+    return;
   }
-  if (acc.bd_exec) { atomicAdd(&C.bd_tot[0], acc.bd_exec); atomicAdd(&C.bd_tot[2], acc.bd_threads); }
+  const uint32_t sub = v ? (lb >> ws) : 32u;                 // the record's sub-warp group
+  const uint32_t ps = __match_any_sync(FULL, sub) & vm;     // lanes of the same group
+  const bool lead = v && (ps & lanemask_lt()) == 0u;        // the group's first record
+  const uint32_t c = __popc(ps);
+  if (bb) {
+    const uint32_t W = 1u << ws;
+    const uint32_t gm = M & ((W == 32u ? FULL : ((1u << W) - 1u)) << ((lb >> ws) << ws));  // the group's lanes
+    if (lead) {
+      exec += 1;
+      thr += c;
+      mxc = max(mxc, cta);
+      tc_update(A, cta, (t & ~31u) | (31u - __clz(gm)));
+      bd_sites_add(A, C, sites_smem, s, c);
+    }
+    // groups with fewer than W lanes wait for T_c (warp-aggregated append)
+    const bool need = lead && c < W;
+    const uint32_t dm = __ballot_sync(FULL, need);
+    if (dm) {
+      const uint32_t leader = __ffs(dm) - 1;
+      unsigned long long b = 0;
+      if (lane == leader) b = atomicAdd(A.ndefer, (unsigned long long)__popc(dm));
+      b = __shfl_sync(FULL, b, leader);
+      const unsigned long long slot = b + __popc(dm & lanemask_lt());
+      if (need && slot < A.defer_cap)
+        A.defer[slot] = make_uint4(cta, t >> ws, c, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
+    }
+  } else {
+    const uint64_t line = v ? ((SMEM ? aa[lane] : __ldg(A.addr + g0 + lane)) >> A.lbs_md) : 0ull;
+    const uint32_t pl = __match_any_sync(FULL, line) & ps;  // same group, same line
+    const bool first = v && (pl & lanemask_lt()) == 0u;
+    const uint32_t deg = __popc(__ballot_sync(FULL, first) & ps);
+    if (lead) finish_md<F>(A, C, whist, sites_smem, kind, deg, s, (F & F_OBJ) ? row_of(A, C, line) : 0u);
+  }
 }
 
 // run aggregates packed for the segmented scans: deg | cnt << 10 | viol << 20
@@ -391,14 +401,15 @@ struct RunQueue {  // six columns of QCAP words from one base (one live register
 
 template <int F>
 __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
-                                        const RunQueue<F> Q, uint32_t qn, uint64_t c_lo) {
+                                        const RunQueue<F> Q, uint32_t qn, uint64_t c_lo, const uint8_t* stg,
+                                        uint32_t sbase) {
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
   const uint32_t lane = lane_id();
   uint32_t exec = 0, thr = 0, mxc = 0;
   for (uint32_t q0 = 0; q0 < qn; q0 += 32) {
     const uint32_t q = q0 + lane;
-    bool md = false, bd = false;
-    uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0;
+    bool md = false, bd = false, slow = false;
+    uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0, cnt = 0;
     if (q < qn) {
       j = Q.j(q);
       u = Q.u(q);
@@ -408,10 +419,11 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
       t = kt & 0xffffu;
       cta = Q.cta(q);
       s = Q.site(q);
-    const bool bb = kind == 2u;
+      const bool bb = kind == 2u;
+      cnt = (u >> PK_CNT) & PK_M;
       if (bb ? BD : MD) {
-        const uint32_t cnt = (u >> PK_CNT) & PK_M;
-        if ((u >> PK_VIOL) || (bb ? A.ws_bd : A.ws_md) != 5u || cnt > 32) walk_run<F>(A, C, whist, sites_smem, c_lo + j, cnt);
+        if (cnt > 32) report(A.sc, c_lo + j, 2);  // a lane must repeat
+        else if (bb ? A.ws_bd != 5u : ((u >> PK_VIOL) || A.ws_md != 5u)) slow = true;  // (BB: no address test)
         else if ((uint32_t)__popc(m) != cnt) report(A.sc, c_lo + j, 2);
         else if (bb) bd = true;
         else md = true;
@@ -422,18 +434,12 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
       finish_md<F>(A, C, whist, sites_smem, kind, u & PK_M, s,
                    (F & F_OBJ) ? row_of(A, C, __ldg(A.addr + c_lo + j) >> A.lbs_md) : 0u);
     if (BD) {
-      const uint32_t cnt = (u >> PK_CNT) & PK_M;
       if (bd) {
         exec += 1;
         thr += cnt;
         mxc = max(mxc, cta);
         tc_update(A, cta, (t & ~31u) | (31u - __clz(m)));
-        if (sites_smem) {
-          if (s < A.nsites) { atomicAdd(&C.bd_sites[3 * s], 1u); atomicAdd(&C.bd_sites[3 * s + 2], cnt); }
-          else *A.site_flag = 1;
-        } else if (A.nsites) {
-          site_add(A, nullptr, A.bd_sites, 3, s, 1, cnt);
-        }
+        bd_sites_add(A, C, sites_smem, s, cnt);
       }
       // groups with fewer than 32 active lanes wait for T_c (warp-aggregated append)
       const bool need = bd && cnt < 32u;
@@ -447,6 +453,21 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uin
         if (need && slot < A.defer_cap)
           A.defer[slot] = make_uint4(cta, t >> 5, cnt, (A.nsites && s < A.nsites) ? s : 0xffffffffu);
       }
+    }
+    // runs that need the exact walk: the whole warp takes them one by one,
+    // from the ring when the run lies in the current step's stage (records
+    // [sbase, sbase + KR) of the chunk: usually every queued run of an
+    // irregular trace, whose queue fills each step), else from global memory
+    for (uint32_t sm = __ballot_sync(FULL, slow); sm; sm &= sm - 1) {
+      const uint32_t src = __ffs(sm) - 1;
+      const uint32_t rj = __shfl_sync(FULL, j, src), rn = __shfl_sync(FULL, cnt, src);
+      const uint32_t rk = __shfl_sync(FULL, kind, src), rc = __shfl_sync(FULL, cta, src);
+      const uint32_t rs = __shfl_sync(FULL, s, src);
+      if (rj >= sbase && rj + rn <= sbase + KR)
+        walk_warp<F, true>(A, C, whist, sites_smem, 0, (const uint16_t*)(stg + S_TID) + (rj - sbase),
+                           (const uint64_t*)(stg + S_ADDR) + (rj - sbase), rn, rk, rc, rs, exec, thr, mxc);
+      else
+        walk_warp<F, false>(A, C, whist, sites_smem, c_lo + rj, nullptr, nullptr, rn, rk, rc, rs, exec, thr, mxc);
     }
   }
   if (BD) {
@@ -895,7 +916,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           if (!bm) break;
           if (qn > QCAP - 32) {  // room for one more round
             __syncwarp();
-            flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
+            flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo, stg, base);
             qn = 0;
             __syncwarp();
           }
@@ -919,7 +940,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         }
         if (qn >= 32) {
           __syncwarp();
-          flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
+          flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo, stg, base);
           qn = 0;
         }
         // ---- the last head lane's open run becomes the carry
@@ -962,7 +983,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     }
     if (NG && qn) {
       __syncwarp();
-      flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo);
+      flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo, nullptr, 0xffffffffu);
     }
     // no bulk copy may still target the ring when the CTA exits
     for (uint32_t q = waited; q < issued; ++q) mbar_wait(&bar[q % KS], (q / KS) & 1u);

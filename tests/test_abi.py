@@ -65,3 +65,33 @@ def test_product_path_is_independent_of_the_oracle():
 def test_sm100a_only_build():
     mk = open(os.path.join(ROOT, "Makefile")).read()
     assert "arch=compute_100a,code=sm_100a" in mk
+
+
+def _boot_worker(addr, rank, nranks, q):
+    import paper_conf_cgo_shensll18_b200 as cadv
+    try:
+        q.put((rank, cadv.bootstrap_selftest(addr, rank, nranks, bytes([rank + 1]) * 5)))
+    except Exception as e:  # noqa: BLE001
+        q.put((rank, repr(e)))
+
+
+@pytest.mark.parametrize("nranks", [2, 3])
+def test_peer_bootstrap_multiprocess(nranks):
+    """The peer backend's host bootstrap (TCP star through rank 0, the part of
+    cadv_create_peer that needs no GPU): nranks processes allgather a blob."""
+    import multiprocessing as mp
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    ps = [ctx.Process(target=_boot_worker, args=(f"127.0.0.1:{port}", r, nranks, q)) for r in range(nranks)]
+    for p in ps:
+        p.start()
+    got = dict(q.get(timeout=60) for _ in range(nranks))
+    for p in ps:
+        p.join(timeout=30)
+    want = b"".join(bytes([r + 1]) * 5 for r in range(nranks))
+    assert all(got[r] == want for r in range(nranks)), got

@@ -4,11 +4,13 @@ times (one fused cadv_analyze on the whole trace resident in HBM).
 * C3 (BFS, 1 M nodes) and C4 (SRAD 2048^2 x 6): every histogram and per-site
   counter element by element against the oracle (CTA scope; the oracle's
   LRU stack is per CTA, so it finishes in seconds to a minute).
-* Kernel scope at full size, where the LRU oracle cannot finish: properties
-  that hold at any size -- histogram mass = memory records; ∞ = stores +
-  lines whose first access is a load (each renamed element's first use);
-  streaming = renamed elements used exactly once -- computed from the
-  definition with numpy; plus exact oracle parity on a 4 M-record prefix.
+* C4-backprop (input 2^22, 1.02 G records with its BB trace): the same.
+* Sub-warp analysis warp sizes (W = 8, 16) on C3 at full size (the
+  warp-cooperative exact walk of every run).
+* Kernel scope at full size, exact: the Fenwick-tree oracle variant
+  (oracle.reuse_fenwick, pinned == LRU in test_oracle_pins.py) finishes
+  where the LRU stack cannot; plus the size-free properties (mass, ∞,
+  streaming) computed from the definition with numpy.
 """
 import numpy as np
 import pytest
@@ -57,17 +59,37 @@ def test_c4_srad_full(ctx, cadv):
     fused_vs_oracle(ctx, cadv, t, 128)
 
 
-def test_kernel_scope_full_properties(ctx, cadv):
-    t = tg.generate("srad", rows=2048, cols=2048, iters=6, bb=1)
+@pytest.mark.parametrize("name,kw", [("bfs", dict(nodes=1000000, seed=42)),
+                                     ("srad", dict(rows=2048, cols=2048, iters=6, bb=1))])
+def test_kernel_scope_full_exact(ctx, cadv, name, kw):
+    """Kernel scope (the paper's "traditional definition") on C3 and
+    C4 at full size, bit-exact against the Fenwick oracle; log2 and linear bins."""
+    t = tg.generate(name, **kw)
     ctx.load_trace(cadv.to_device(t))
-    h, st = ctx.reuse_histogram(128, 1, 1, 40)
+    for binning, nb in ((1, 40), (0, 66)):
+        h, st = ctx.reuse_histogram(128, 1, binning, nb)
+        h_ref, s_ref = orc.reuse_fenwick(t, 128, 1, binning, nb)
+        assert (h == h_ref).all(), (name, binning, np.nonzero(h != h_ref))
+        assert st == s_ref
     mass, inf, streaming = kernel_scope_properties(t, 128)
-    assert int(h.sum()) == mass == st["accesses"]
-    assert int(h[-1]) == inf == st["inf"]
-    assert st["streaming"] == streaming
-    # exact parity on a prefix the LRU oracle finishes
-    p = tg.from_arrays(*(t.cols[k][:4_000_000] for k, _ in tg.COLUMNS), nsites=t.nsites)
-    ctx.load_trace(cadv.to_device(p))
-    h2, s2 = ctx.reuse_histogram(128, 1, 1, 40)
-    h_ref, s_ref = orc.reuse(p, 128, 1, 1, 40)
-    assert (h2 == h_ref).all() and s2 == s_ref
+    assert int(h.sum()) == mass == st["accesses"] and int(h[-1]) == inf == st["inf"] and st["streaming"] == streaming
+
+
+def test_c4_backprop_full(ctx, cadv):
+    """C4's second shape: backprop, input 2^22, hidden 16, with BB records."""
+    t = tg.generate("backprop", **{"in": 4194304})
+    assert t.n > 1_000_000_000
+    fused_vs_oracle(ctx, cadv, t, 128)
+
+
+def test_c3_bfs_full_subwarp(ctx, cadv):
+    """W = 16 and 8 (sub-warp groups: every run goes through the exact
+    warp-cooperative walk) for memory and branch divergence at full size."""
+    t = tg.generate("bfs", nodes=1000000, seed=42)
+    ctx.load_trace(cadv.to_device(t))
+    for W in (16, 8):
+        o = ctx.analyze(rd=None, md=(128, W), bd=W, nsites=t.nsites)
+        mh, ms = orc.mem_div(t, 128, W)
+        assert (o["mem_div"][0] == mh).all() and (o["mem_div"][1] == ms).all(), W
+        bs, bt = orc.branch_div(t, W)
+        assert (o["branch_div"][0] == bs).all() and (o["branch_div"][1] == bt).all(), W

@@ -561,3 +561,19 @@ def test_segment_kernel_full_hash_tables(ctx, cadv, reuse_frac):
         del os.environ["CADV_RD_TILES"]
     for h, st in (seg, til):
         assert (h == ref[0]).all() and st == ref[1]
+
+
+@pytest.mark.parametrize("seed", [1, 2])
+def test_many_sites_global_counters(ctx, cadv, seed):
+    """More than 512 sites (NSITE_SMEM): the per-site counters of memory and
+    branch divergence take the global-atomic path; fused and separate calls,
+    W = 32 and 8, against the oracle."""
+    t = tg.generate("rand", seed=seed, ctas=20, threads=256, instrs=40, lines=100, msites=3000, bsites=1000,
+                    pbb=0.4, pstore=0.2)
+    assert t.nsites == 4000
+    full_check(ctx, cadv, t, lbs=(32, 128), scopes=(0,), W=(32, 8))
+    out = ctx.analyze(rd=(128, 0, 0, 66), md=(128, 16), bd=16, nsites=t.nsites)
+    mh, ms = orc.mem_div(t, 128, 16)
+    assert (out["mem_div"][0] == mh).all() and (out["mem_div"][1] == ms).all()
+    bs, bt = orc.branch_div(t, 16)
+    assert (out["branch_div"][0] == bs).all() and (out["branch_div"][1] == bt).all()

@@ -207,6 +207,26 @@ def generate(workload: str, lo: int | None = None, hi: int | None = None, alloc=
         lib.tg_free(h)
 
 
+def generate_ranges(workload: str, ranges, alloc=None, **params):
+    """Yields the Trace of every [lo, hi) in `ranges`, planning the workload
+    once (C5's plan counts 4e9 records; full-size tests generate it in
+    launch-aligned chunks)."""
+    lib = _load()
+    h, n_total, nsites, nctas, nl, info = plan(workload, **params)
+    try:
+        alloc = alloc or (lambda m, dt: np.empty(m, dtype=dt))
+        for lo, hi in ranges:
+            lo, hi = int(lo), int(hi)
+            cols = {name: alloc(hi - lo, dt) for name, dt in COLUMNS}
+            if hi > lo:
+                rc = lib.tg_fill_range(h, lo, hi, *[cols[name].ctypes.data for name, _ in COLUMNS])
+                if rc != 0:
+                    raise ValueError(f"tg_fill_range failed ({rc})")
+            yield Trace(workload, dict(params), hi - lo, n_total, nsites, nctas, nl, info, lo, cols)
+    finally:
+        lib.tg_free(h)
+
+
 def from_arrays(addr, cta, tid, site, winst, meta, nsites=None, workload="custom") -> Trace:
     """Wraps hand-built columns (tests, golden fixtures) as a Trace."""
     cols = {}
@@ -232,4 +252,5 @@ CONFIGS = {
     "c3_bfs": ("bfs", {"nodes": 1000000, "seed": 42}),
     "c4_srad": ("srad", {"rows": 2048, "cols": 2048, "iters": 6}),
     "c4_backprop": ("backprop", {"in": 4194304}),
+    "c5_mixed": ("mixed", {}),
 }

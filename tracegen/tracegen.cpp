@@ -835,13 +835,14 @@ void wl_mixed(Trace& T, const Params& P) {
     site_base += sub.nsites;
   };
   for (auto& pr : parts) add(pr.first, pr.second);
-  if (total < limit) {  // SRAD iterations until the limit (one SRAD launch pair per iteration)
+  if (limit && total < limit) {  // SRAD iterations until the limit (records=0: the five parts only)
     Trace one;
     snprintf(b, sizeof b, "rows=%u,cols=%u,iters=1,bb=0,seed=47", sq(4096), sq(4096));
     build(one, "srad", Params(b));
     uint64_t per = 0;
     for (auto& L : one.launches) per += count_launch(L);
     const uint64_t it = (limit - total + per - 1) / per;
+    if (it > 4096) throw std::runtime_error("mixed: records too large for the SRAD fill");
     snprintf(b, sizeof b, "rows=%u,cols=%u,iters=%llu,bb=0,seed=47", sq(4096), sq(4096), (unsigned long long)it);
     add("srad", b);
   }
