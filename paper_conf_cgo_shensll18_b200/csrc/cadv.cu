@@ -19,11 +19,12 @@ cudaError_t ensure(cadv_ctx* c, BufId id, size_t bytes, void** out) {
     if (b.p) {
       cudaError_t e = cudaStreamSynchronize(c->stream);
       if (e != cudaSuccess) return e;
-      cudaFree(b.p);
+      if (b.exported) c->graveyard.push_back(b.p);
+      else cudaFree(b.p);
       b.p = nullptr;
       b.bytes = 0;
     }
-    size_t want = bytes + bytes / 8;  // headroom so slightly larger calls do not reallocate
+    size_t want = b.exported ? 2 * bytes : bytes + bytes / 8;  // headroom so slightly larger calls do not reallocate
     cudaError_t e = cudaMalloc(&b.p, want);
     if (e != cudaSuccess) {
       cudaGetLastError();
@@ -269,6 +270,7 @@ cadv_status create_ctx(cadv_ctx** out, int device, void* cuda_stream, const void
   c->nranks = nranks;
   c->num_sms = prop.multiProcessorCount;
   if (const char* e = getenv("CADV_SCAN_CTAS")) c->scan_ctas = atoi(e);
+  if (const char* e = getenv("CADV_SCAN_SPLIT")) c->scan_split = atoi(e);
   if (cudaEventCreate(&c->ev0) != cudaSuccess || cudaEventCreate(&c->ev1) != cudaSuccess ||
       cudaMallocHost(&c->hstage, 512) != cudaSuccess) {
     if (c->hstage) cudaFreeHost(c->hstage);
@@ -362,15 +364,17 @@ CADV_API cadv_status cadv_destroy(cadv_ctx* c) {
   if (!c) return CADV_ERR_INVALID_ARG;
   cudaSetDevice(c->device);
   cudaStreamSynchronize(c->stream);
+  delete c->comm;  // (closes its peer mappings before the buffers go)
+  c->comm = nullptr;
   for (auto& b : c->buf)
     if (b.p) cudaFree(b.p);
+  for (void* p : c->graveyard) cudaFree(p);
   if (c->host_pinned) cudaFreeHost(c->host_pinned);
   if (c->hstage) cudaFreeHost(c->hstage);
   if (c->ev0) cudaEventDestroy(c->ev0);
   if (c->ev1) cudaEventDestroy(c->ev1);
   for (auto e : c->prof_ev) cudaEventDestroy(e);
   if (c->tc_buf) cudaFree(c->tc_buf);
-  delete c->comm;
   delete c;
   return CADV_OK;
 }
@@ -548,12 +552,9 @@ cadv_status run_analyses(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reus
 cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_stats* rd_stats, uint64_t* md_hist,
                      cadv_site_mem* md_sites, uint64_t* bd_tot, cadv_site_branch* bd_sites) {
   const bool multi = c->comm != nullptr;  // also a 1-rank NCCL / loopback context (plumbing tests)
-  if (multi && (q.md || q.bd)) {
-    if (c->noncontig_any)  // (all-gathered at load: every rank decides alike)
-      return fail(c, CADV_ERR_UNSUPPORTED, "multi-rank divergence analyses need warp-contiguous shards");
-    if (c->split_group)
-      return fail(c, CADV_ERR_BAD_TRACE, "a shard boundary splits a warp-level group (cta, warp, winst)");
-  }
+  // (noncontig_any and split_group are all-gathered at load: every rank decides alike)
+  if (multi && (q.md || q.bd) && !c->noncontig_any && c->split_group)
+    return fail(c, CADV_ERR_BAD_TRACE, "a shard boundary splits a warp-level group (cta, warp, winst)");
   CK(cudaSetDevice(c->device), "cudaSetDevice");
   cadv_status s = begin_call(c);
   if (s != CADV_OK) return s;
@@ -571,7 +572,17 @@ cadv_status run_once(cadv_ctx* c, const Req& q, uint64_t* rd_hist, cadv_reuse_st
   CK(cudaMemsetAsync(dv, 0, total * 8 + 64, c->stream), "memset");
   uint64_t* d = (uint64_t*)dv;
   cadv_trace_desc t = c->t;
-  if ((q.md || q.bd) && !t.warp_contiguous && t.n) CK(regroup_by_warp(c, &t), "regroup by warp");
+  if ((q.md || q.bd) && multi && c->noncontig_any) {
+    // every (cta, warp32) stream to one rank, in trace order (collective)
+    cudaError_t e = exchange_by_warp(c, &t);
+    if (e != cudaSuccess) {
+      if (!c->comm->err.empty()) return fail(c, CADV_ERR_NCCL, c->comm->err);
+      if (e == cudaErrorNotSupported) return fail(c, CADV_ERR_UNSUPPORTED, "a rank would receive >= 2^32 records");
+      return cuda_fail(c, e, "exchange by warp");
+    }
+  } else if ((q.md || q.bd) && !t.warp_contiguous && t.n) {
+    CK(regroup_by_warp(c, &t), "regroup by warp");
+  }
   // the scan's 1-D TMA copies need 16-byte aligned column bases
   if (t.n && (((uintptr_t)t.addr | (uintptr_t)t.cta | (uintptr_t)t.tid | (uintptr_t)t.site | (uintptr_t)t.winst |
                (uintptr_t)t.meta) & 15)) {

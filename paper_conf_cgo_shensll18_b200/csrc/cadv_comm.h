@@ -106,6 +106,7 @@ class PeerComm : public Comm {
   void* stage_ = nullptr;
   size_t stage_cap_ = 0;
   void* tmp_ = nullptr;
+  std::vector<void*> graveyard_;
   IpcCache ipc_;
 };
 Comm* make_peer_comm(const char* addr, int rank, int nranks, std::string* err);

@@ -16,6 +16,10 @@ namespace cadv {
 struct DevBuf {
   void* p = nullptr;
   size_t bytes = 0;
+  // exported to peer processes (CUDA IPC, map_peers): never freed while the
+  // context lives (an importer may still map it, and a freed range that the
+  // driver hands out again would collide with that mapping); grown 2x
+  bool exported = false;
 };
 
 // Small per-call device scalars (zeroed at the start of every analysis).
@@ -24,7 +28,8 @@ struct Scalars {
   unsigned int err_code;         // 1 = bad record, 2 = run longer than 32 / duplicate lane,
                                  // 3 = internal invariant, 4 = group mixes kinds / sites
   unsigned long long unsup_index;
-  unsigned long long kept_max;   // scan (RD): most kept records of one warp chunk (region capacity check)  // first memory record whose reuse line is >= 2^58 (ULLONG_MAX = none)
+  unsigned long long kept_max;   // scan (RD): most kept records of one chunk (region capacity check)
+  unsigned long long chunk_next; // scan: next chunk to claim  // first memory record whose reuse line is >= 2^58 (ULLONG_MAX = none)
   unsigned int tile_counter;     // dynamic tile assignment
   unsigned long long count[8];   // generic counters (kept records, entries, ...)
   unsigned long long max_cta;    // scan: max CTA id of the trace (shard)
@@ -45,6 +50,8 @@ enum BufId {
   B_ALIGN0, B_ALIGN1, B_ALIGN2, B_ALIGN3, B_ALIGN4, B_ALIGN5,
   B_XCH_K0, B_XCH_K1, B_XCH_V0, B_XCH_V1, B_XCH_CNT, B_COMM, B_OBJ, B_RD_ENT_ALL,
   B_RG_PK, B_RG_PN, B_RG_NP, B_RG_SORT, B_RG_SEG,
+  B_WX_RECV, B_WX_K0, B_WX_K1, B_WX_V0, B_WX_V1, B_WX_COLS,
+  B_XE_OWN, B_XE_SEND, B_XE_CNT, B_XE_ALLP, B_RD_XQR,
   B_COUNT
 };
 
@@ -59,6 +66,7 @@ struct cadv_ctx {
   bool split_group = false;              // a shard boundary splits a warp-level group (load_trace)
   int num_sms = 148;
   int scan_ctas = 0;     // CADV_SCAN_CTAS (testing): cap on the scan grid, 0 = one CTA per SM
+  int scan_split = 0;    // CADV_SCAN_SPLIT: chunks per scan warp (0 = default 4)
   // registered trace (device pointers)
   bool loaded = false;
   cadv_trace_desc t{};
@@ -95,6 +103,7 @@ struct cadv_ctx {
   // attribute is per device context, so it is tracked per cadv_ctx):
   // bits 0-15 k_scan<F>, bit 16 k_rd_seg, 17 k_rd_tile, 18 k_merge_count_block
   uint32_t attr_set = 0;
+  std::vector<void*> graveyard;  // replaced exported buffers (freed at cadv_destroy)
   int seg_ctas = 0;           // k_rd_seg CTAs per SM for seg_ctas_smem bytes of shared memory
   size_t seg_ctas_smem = 0;
   bool noncontig_any = false;
@@ -117,6 +126,9 @@ Scalars* scalars(cadv_ctx* c);
 // Stable (cta, tid/32) ordering of a non-warp-contiguous trace: fills `out`
 // with device copies of every column in that order.
 cudaError_t regroup_by_warp(cadv_ctx* c, cadv_trace_desc* out);
+// Multi-rank, non-warp-contiguous shards: every (cta, warp32) stream moved
+// to one rank and sorted there (collective); *out = this rank's records.
+cudaError_t exchange_by_warp(cadv_ctx* c, cadv_trace_desc* out);
 
 // ---- the fused streaming pass (scan.cu)
 // F_OBJ: data-centric attribution (cadv_data_centric): the RD bin-0 counts
@@ -154,7 +166,7 @@ struct ScanParams {
   uint32_t rd_nbins = 0;
 };
 uint64_t scan_tiles(uint64_t n);
-void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nwarps, uint64_t* chunk);
+void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, uint64_t* chunk);
 cudaError_t launch_squeeze(cadv_ctx* c, const uint32_t* kin, const uint64_t* vin, uint32_t* kout, uint64_t* vout,
                            const uint64_t* cnt, const uint64_t* off, uint64_t nblocks, uint64_t chunk_cap);
 cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P);

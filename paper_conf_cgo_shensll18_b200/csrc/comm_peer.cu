@@ -255,6 +255,7 @@ PeerComm::PeerComm(Bootstrap* b, bool owns, bool same_process)
 
 PeerComm::~PeerComm() {
   if (stage_) cudaFree(stage_);
+  for (void* p : graveyard_) cudaFree(p);
   if (tmp_) cudaFree(tmp_);
   if (owns_) delete boot_;
 }
@@ -273,10 +274,11 @@ int PeerComm::boot(int e) {
 
 int PeerComm::grow(void** buf, size_t* cap, size_t bytes) {
   if (*cap >= bytes) return 0;
-  if (*buf) cudaFree(*buf);
+  // an exported buffer is never freed while the communicator lives (see DevBuf::exported)
+  if (*buf) graveyard_.push_back(*buf);
   *buf = nullptr;
   *cap = 0;
-  const size_t want = bytes + bytes / 4 + 256;
+  const size_t want = 2 * bytes + 256;
   if (cu(cudaMalloc(buf, want))) return 1;
   *cap = want;
   return 0;

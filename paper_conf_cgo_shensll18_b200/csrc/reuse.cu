@@ -1264,7 +1264,7 @@ cudaError_t rd_begin(cadv_ctx* c, int scope, RdState* st) {
   st->cta_scope = scope == CADV_SCOPE_CTA;
   uint64_t grid, nw, chunk;
   scan_geometry(c, n, &grid, &nw, &chunk);
-  st->grid = nw;  // one kept-record region per scan warp
+  st->grid = nw;  // one kept-record region per scan chunk (scan_geometry: nchunks)
   // region capacity: max(chunk / 4, kcap_min) records (run compression keeps
   // ~7 % of the paper-shaped traces; a region that overflows raises kcap_min
   // and the call runs again, see run_once), so C5's 4e9 records need 24 B per
@@ -1381,6 +1381,7 @@ cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const 
     if (kr >= 0xffffffffull) return cudaErrorNotSupported;
   }
   void *rk0, *rk1 = nullptr, *rv0, *rv1;
+  c->buf[B_XCH_V0].exported = c->buf[B_XCH_K0].exported = true;  // mapped by the peers (k_push)
   if ((e = ensure(c, B_XCH_V0, Kn * 8 + 16, &rv0)) || (e = ensure(c, B_XCH_V1, Kn * 8 + 16, &rv1))) return e;
   if (cta_scope &&
       ((e = ensure(c, B_XCH_K0, Kn * 4 + 16, &rk0)) || (e = ensure(c, B_XCH_K1, Kn * 4 + 16, &rk1))))
@@ -1442,61 +1443,254 @@ cudaError_t rd_exchange(cadv_ctx* c, int cta_scope, const uint32_t** key, const 
   return cudaSuccess;
 }
 
-// Spread kernel scope: every rank's cross-tile entries gathered on rank 0
-// (column by column, in rank order); *En / *nent become the gathered set
-// there and nent = 0 elsewhere.  Collective.
-cudaError_t gather_entries(cadv_ctx* c, EntryCols* En, unsigned long long* nent) {
-  cudaError_t e;
+// ---- kernel scope over ranks, distributed cross-tile phase
+namespace {
+
+__device__ __forceinline__ uint32_t line_owner(uint64_t line, int G) {
+  uint64_t z = line + 0x9E3779B97F4A7C15ull;  // splitmix64 finaliser: lines spread evenly over the ranks
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  z ^= z >> 31;
+  return (uint32_t)(((z >> 32) * (uint64_t)G) >> 32);
+}
+
+__global__ void k_ent_owner(const uint64_t* __restrict__ line, uint64_t n, int G, uint32_t* own, uint32_t* idx,
+                            unsigned long long* cnt) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t o = line_owner(__ldg(line + i), G);
+    own[i] = o;
+    idx[i] = (uint32_t)i;
+    atomicAdd(&cnt[o], 1ull);
+  }
+}
+
+// entry columns permuted: dst[k] = src[perm[k]]
+__global__ void k_ent_permute(const uint32_t* __restrict__ perm, uint64_t n, EntryCols S, EntryCols D) {
+  for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < n; k += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t i = perm[k];
+    D.line[k] = S.line[i]; D.seg[k] = S.seg[i]; D.tile[k] = S.tile[i];
+    D.f[k] = S.f[i]; D.fa[k] = S.fa[i]; D.fw[k] = S.fw[i]; D.ff[k] = S.ff[i];
+    D.l[k] = S.l[i]; D.lw[k] = S.lw[i]; D.ld[k] = S.ld[i]; D.lf[k] = S.lf[i];
+  }
+}
+
+// cross queries permuted into position order (send layout): dst[k] = src[perm[k]]
+__global__ void k_xq_permute(const uint32_t* __restrict__ perm, uint64_t n, CrossOut S, CrossOut D) {
+  for (uint64_t k = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; k < n; k += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t i = perm[k];
+    D.xpos[k] = S.xpos[i]; D.xq[k] = S.xq[i]; D.part[k] = S.part[i]; D.xline[k] = S.xline[i];
+  }
+}
+
+// cnt[j] += number of the queries of ranks before this one whose previous
+// use lies after query j's (their positions all precede j's): per earlier
+// rank r, M_r minus the upper bound of xq[j] in r's sorted previous uses
+__global__ void k_count_greater(const uint32_t* __restrict__ xq, uint64_t M, const uint32_t* __restrict__ allp,
+                                const uint64_t* __restrict__ off, int me, uint32_t* cnt) {
+  for (uint64_t j = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; j < M; j += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t x = xq[j];
+    uint32_t add = 0;
+    for (int r = 0; r < me; ++r) {
+      uint64_t lo = off[r], hi = off[r + 1];
+      const uint64_t b = hi;
+      while (lo < hi) {
+        const uint64_t md = (lo + hi) >> 1;
+        if (allp[md] <= x) lo = md + 1;
+        else hi = md;
+      }
+      add += (uint32_t)(b - lo);
+    }
+    cnt[j] += add;
+  }
+}
+
+EntryCols carve_entries(void* base, uint64_t n) {
+  EntryCols E;
+  uint8_t* p = (uint8_t*)base;
+  auto take = [&](size_t bytes) { uint8_t* q = p; p += (bytes + 15) & ~size_t(15); return q; };
+  E.line = (uint64_t*)take(n * 8);
+  E.seg = (uint32_t*)take(n * 4);
+  E.tile = (uint32_t*)take(n * 4);
+  E.f = (uint32_t*)take(n * 4);
+  E.fa = (uint32_t*)take(n * 4);
+  E.fw = (uint32_t*)take(n * 4);
+  E.l = (uint32_t*)take(n * 4);
+  E.lw = (uint32_t*)take(n * 4);
+  E.ld = (uint32_t*)take(n * 4);
+  E.ff = (uint8_t*)take(n);
+  E.lf = (uint8_t*)take(n);
+  return E;
+}
+constexpr size_t ENT_BYTES = 4 + 8 + 4 + 4 + 4 + 4 + 1 + 4 + 4 + 4 + 1;
+
+CrossOut carve_queries(void* base, uint64_t n) {
+  CrossOut X;
+  X.xpos = (uint32_t*)base;
+  X.xq = X.xpos + n;
+  X.part = (int64_t*)(((uintptr_t)(X.xq + n) + 15) & ~(uintptr_t)15);
+  X.xline = (uint64_t*)(X.part + n);
+  return X;
+}
+
+// send counts (per destination rank, in the sender's order) -> the G x G
+// matrix all-gathered; fills soff / scnt / roff / rcnt (in elements) and
+// returns the number of elements this rank receives
+int counts_matrix(cadv_ctx* c, const std::vector<uint64_t>& scnt, std::vector<uint64_t>* soff,
+                  std::vector<uint64_t>* roff, std::vector<uint64_t>* rcnt, uint64_t* total, cudaError_t* e) {
   const int G = c->nranks, me = c->rank;
   void* cb;
-  if ((e = ensure(c, B_COMM, (size_t)(2 + 2 * G) * 8 + 64, &cb))) return e;
-  uint64_t* d = (uint64_t*)cb;
-  const uint64_t mine = *nent;
-  if ((e = cudaMemcpyAsync(d, &mine, 8, cudaMemcpyHostToDevice, c->stream))) return e;
-  if (c->comm->allgather(d, d + 1, 8, c->stream)) return cudaErrorUnknown;
-  std::vector<uint64_t> cnt(G);
-  if ((e = cudaMemcpyAsync(cnt.data(), d + 1, 8 * G, cudaMemcpyDeviceToHost, c->stream))) return e;
-  if ((e = cudaStreamSynchronize(c->stream))) return e;
-  std::vector<uint64_t> off(G + 1, 0);
-  for (int r = 0; r < G; ++r) off[r + 1] = off[r] + cnt[r];
-  const uint64_t N = off[G];
-  if (N == 0) { *nent = 0; return cudaSuccess; }
-  EntryCols A{};
-  if (me == 0) {
-    void* ent;
-    if ((e = ensure(c, B_RD_ENT_ALL, N * (4 + 8 + 4 + 4 + 4 + 4 + 1 + 4 + 4 + 4 + 1) + 16 * 16, &ent))) return e;
-    uint8_t* p = (uint8_t*)ent;
-    auto take = [&](size_t bytes) { uint8_t* q = p; p += (bytes + 15) & ~size_t(15); return q; };
-    A.line = (uint64_t*)take(N * 8);
-    A.seg = (uint32_t*)take(N * 4);
-    A.tile = (uint32_t*)take(N * 4);
-    A.f = (uint32_t*)take(N * 4);
-    A.fa = (uint32_t*)take(N * 4);
-    A.fw = (uint32_t*)take(N * 4);
-    A.l = (uint32_t*)take(N * 4);
-    A.lw = (uint32_t*)take(N * 4);
-    A.ld = (uint32_t*)take(N * 4);
-    A.ff = (uint8_t*)take(N);
-    A.lf = (uint8_t*)take(N);
+  if ((*e = ensure(c, B_COMM, (size_t)(G + 2) * 8 + (size_t)G * G * 8 + 64, &cb))) return 1;
+  uint64_t* d_send = (uint64_t*)cb;
+  uint64_t* d_mat = d_send + G + 2;
+  std::vector<uint64_t> mat((size_t)G * G);
+  if ((*e = cudaMemcpyAsync(d_send, scnt.data(), G * 8, cudaMemcpyHostToDevice, c->stream))) return 1;
+  if (c->comm->allgather(d_send, d_mat, G * 8, c->stream)) { *e = cudaErrorUnknown; return 1; }
+  if ((*e = cudaMemcpyAsync(mat.data(), d_mat, (size_t)G * G * 8, cudaMemcpyDeviceToHost, c->stream)) ||
+      (*e = cudaStreamSynchronize(c->stream)))
+    return 1;
+  soff->assign(G, 0);
+  roff->assign(G, 0);
+  rcnt->assign(G, 0);
+  uint64_t a = 0, b = 0;
+  for (int p = 0; p < G; ++p) {
+    (*soff)[p] = a;
+    a += scnt[p];
+    (*rcnt)[p] = mat[(size_t)p * G + me];
+    (*roff)[p] = b;
+    b += (*rcnt)[p];
   }
-  auto col = [&](const void* src, void* dst, size_t es) -> int {
-    std::vector<uint64_t> soff(G, 0), scnt(G, 0), roff(G, 0), rcnt(G, 0);
-    scnt[0] = mine * es;
-    if (me == 0)
-      for (int r = 0; r < G; ++r) { roff[r] = off[r] * es; rcnt[r] = cnt[r] * es; }
-    return c->comm->alltoallv(src, soff.data(), scnt.data(), dst, roff.data(), rcnt.data(), c->stream);
-  };
-  if (col(En->line, A.line, 8) || col(En->seg, A.seg, 4) || col(En->tile, A.tile, 4) || col(En->f, A.f, 4) ||
-      col(En->fa, A.fa, 4) || col(En->fw, A.fw, 4) || col(En->l, A.l, 4) || col(En->lw, A.lw, 4) ||
-      col(En->ld, A.ld, 4) || col(En->ff, A.ff, 1) || col(En->lf, A.lf, 1))
+  *total = b;
+  return 0;
+}
+
+int a2av_col(cadv_ctx* c, const void* src, void* dst, size_t es, const std::vector<uint64_t>& soff,
+             const std::vector<uint64_t>& scnt, const std::vector<uint64_t>& roff, const std::vector<uint64_t>& rcnt) {
+  const int G = c->nranks;
+  std::vector<uint64_t> so(G), sc(G), ro(G), rc(G);
+  for (int p = 0; p < G; ++p) { so[p] = soff[p] * es; sc[p] = scnt[p] * es; ro[p] = roff[p] * es; rc[p] = rcnt[p] * es; }
+  return c->comm->alltoallv(src, so.data(), sc.data(), dst, ro.data(), rc.data(), c->stream);
+}
+
+}  // namespace
+
+// Every rank's cross-tile entries to the owner of their line (line hash):
+// all entries of one line meet on one rank, which links them (k_link) and
+// emits the cross-tile queries locally.  Collective; *En / *nent become the
+// entries this rank owns.
+cudaError_t exchange_entries_by_line(cadv_ctx* c, EntryCols* En, unsigned long long* nent) {
+  cudaError_t e;
+  const int G = c->nranks;
+  const uint64_t n = *nent;
+  void *ob, *sb, *cb2;
+  if ((e = ensure(c, B_XE_OWN, n * 16 + 64, &ob)) || (e = ensure(c, B_XE_SEND, n * ENT_BYTES + 16 * 16, &sb)) ||
+      (e = ensure(c, B_XE_CNT, (size_t)G * 8 + 64, &cb2)))
+    return e;
+  uint32_t* own0 = (uint32_t*)ob;
+  uint32_t* idx0 = own0 + n;
+  uint32_t* own1 = idx0 + n;
+  uint32_t* idx1 = own1 + n;
+  unsigned long long* dcnt = (unsigned long long*)cb2;
+  if ((e = cudaMemsetAsync(dcnt, 0, (size_t)G * 8, c->stream))) return e;
+  EntryCols S = carve_entries(sb, n);
+  if (n) {
+    CADV_LAUNCH(c, k_ent_owner<<<c->num_sms * 4, 256, 0, c->stream>>>(En->line, n, G, own0, idx0, dcnt));
+    int res, bits = bits_for((uint64_t)(G - 1));
+    if (bits == 0) bits = 1;
+    if ((e = radix_sort_pairs<uint32_t, uint32_t>(c, own0, idx0, own1, idx1, n, 0, bits, &res))) return e;
+    CADV_LAUNCH(c, k_ent_permute<<<c->num_sms * 4, 256, 0, c->stream>>>(res ? idx1 : idx0, n, *En, S));
+  }
+  std::vector<uint64_t> scnt(G), soff, roff, rcnt;
+  if ((e = cudaMemcpyAsync(scnt.data(), dcnt, (size_t)G * 8, cudaMemcpyDeviceToHost, c->stream)) ||
+      (e = cudaStreamSynchronize(c->stream)))
+    return e;
+  uint64_t N = 0;
+  if (counts_matrix(c, scnt, &soff, &roff, &rcnt, &N, &e)) return e ? e : cudaErrorUnknown;
+  void* rb;
+  if ((e = ensure(c, B_RD_ENT_ALL, N * ENT_BYTES + 16 * 16, &rb))) return e;
+  EntryCols R = carve_entries(rb, N);
+  if (a2av_col(c, S.line, R.line, 8, soff, scnt, roff, rcnt) || a2av_col(c, S.seg, R.seg, 4, soff, scnt, roff, rcnt) ||
+      a2av_col(c, S.tile, R.tile, 4, soff, scnt, roff, rcnt) || a2av_col(c, S.f, R.f, 4, soff, scnt, roff, rcnt) ||
+      a2av_col(c, S.fa, R.fa, 4, soff, scnt, roff, rcnt) || a2av_col(c, S.fw, R.fw, 4, soff, scnt, roff, rcnt) ||
+      a2av_col(c, S.l, R.l, 4, soff, scnt, roff, rcnt) || a2av_col(c, S.lw, R.lw, 4, soff, scnt, roff, rcnt) ||
+      a2av_col(c, S.ld, R.ld, 4, soff, scnt, roff, rcnt) || a2av_col(c, S.ff, R.ff, 1, soff, scnt, roff, rcnt) ||
+      a2av_col(c, S.lf, R.lf, 1, soff, scnt, roff, rcnt))
     return cudaErrorUnknown;
-  if (me == 0) {
-    *En = A;
-    *nent = N;
-  } else {
-    *nent = 0;
-  }
+  *En = R;
+  *nent = N;
   return cudaSuccess;
+}
+
+// The cross-tile queries to the rank holding their position ([base[r],
+// base[r+1]) of the global kept sequence).  Collective; *X / *M become this
+// rank's queries (capacity in B_RD_XQR).
+cudaError_t exchange_queries_by_pos(cadv_ctx* c, CrossOut* X, unsigned long long* M, const std::vector<uint64_t>& base) {
+  cudaError_t e;
+  const int G = c->nranks;
+  const uint64_t m = *M;
+  void *kb, *sb, *db;
+  if ((e = ensure(c, B_XE_OWN, m * 16 + 64, &kb)) || (e = ensure(c, B_XE_SEND, m * 24 + 256, &sb)) ||
+      (e = ensure(c, B_XE_CNT, (size_t)(2 * G + 4) * 8 + 64, &db)))
+    return e;
+  uint32_t* k0 = (uint32_t*)kb;
+  uint32_t* i0 = k0 + m;
+  uint32_t* k1 = i0 + m;
+  uint32_t* i1 = k1 + m;
+  CrossOut S = carve_queries(sb, m);
+  std::vector<uint64_t> pos(G + 1, 0);
+  pos[G] = m;
+  if (m) {
+    if ((e = cudaMemcpyAsync(k0, X->xpos, m * 4, cudaMemcpyDeviceToDevice, c->stream))) return e;
+    CADV_LAUNCH(c, k_iota<<<c->num_sms * 4, 256, 0, c->stream>>>(i0, m));
+    int res;
+    if ((e = radix_sort_pairs<uint32_t, uint32_t>(c, k0, i0, k1, i1, m, 0, 32, &res))) return e;
+    const uint32_t* sk = res ? k1 : k0;
+    CADV_LAUNCH(c, k_xq_permute<<<c->num_sms * 4, 256, 0, c->stream>>>(res ? i1 : i0, m, *X, S));
+    if (G > 1) {
+      uint64_t* d_bnd = (uint64_t*)db;
+      if ((e = cudaMemcpyAsync(d_bnd, base.data() + 1, (G - 1) * 8, cudaMemcpyHostToDevice, c->stream))) return e;
+      CADV_LAUNCH(c, k_lower_bounds<<<1, 64, 0, c->stream>>>(sk, m, 0, d_bnd, G - 1, d_bnd + G));
+      if ((e = cudaMemcpyAsync(pos.data() + 1, d_bnd + G, (G - 1) * 8, cudaMemcpyDeviceToHost, c->stream)) ||
+          (e = cudaStreamSynchronize(c->stream)))
+        return e;
+    }
+  }
+  std::vector<uint64_t> scnt(G), soff, roff, rcnt;
+  for (int r = 0; r < G; ++r) scnt[r] = pos[r + 1] - pos[r];
+  uint64_t N = 0;
+  if (counts_matrix(c, scnt, &soff, &roff, &rcnt, &N, &e)) return e ? e : cudaErrorUnknown;
+  void* rb;
+  if ((e = ensure(c, B_RD_XQR, N * 24 + 256, &rb))) return e;
+  CrossOut R = carve_queries(rb, N);
+  R.part = (int64_t*)(((uintptr_t)(R.xq + N) + 15) & ~(uintptr_t)15);
+  if (a2av_col(c, S.xpos, R.xpos, 4, soff, scnt, roff, rcnt) || a2av_col(c, S.xq, R.xq, 4, soff, scnt, roff, rcnt) ||
+      a2av_col(c, S.part, R.part, 8, soff, scnt, roff, rcnt) ||
+      a2av_col(c, S.xline, R.xline, 8, soff, scnt, roff, rcnt))
+    return cudaErrorUnknown;
+  *X = R;
+  *M = N;
+  return cudaSuccess;
+}
+
+// cnt[j] += the queries of earlier ranks (smaller positions) with a larger
+// previous use than query j's: every rank's previous uses, sorted, are
+// all-gathered and each query counts the larger ones by binary search.
+// Collective (sorted = this rank's M previous uses in ascending order).
+cudaError_t add_earlier_ranks(cadv_ctx* c, const uint32_t* sorted, uint64_t M, const uint32_t* xq, uint32_t* cnt) {
+  cudaError_t e;
+  const int G = c->nranks, me = c->rank;
+  std::vector<uint64_t> scnt(G, M), soff(G, 0), roff, rcnt, dummy;
+  uint64_t N = 0;
+  if (counts_matrix(c, scnt, &dummy, &roff, &rcnt, &N, &e)) return e ? e : cudaErrorUnknown;
+  void *ab, *ob;
+  if ((e = ensure(c, B_XE_ALLP, N * 4 + 64, &ab)) || (e = ensure(c, B_XE_CNT, (size_t)(G + 2) * 8 + 64, &ob))) return e;
+  if (a2av_col(c, sorted, ab, 4, soff, scnt, roff, rcnt)) return cudaErrorUnknown;
+  std::vector<uint64_t> off(G + 1, 0);
+  for (int p = 0; p < G; ++p) off[p + 1] = off[p] + rcnt[p];
+  if ((e = cudaMemcpyAsync(ob, off.data(), (G + 1) * 8, cudaMemcpyHostToDevice, c->stream))) return e;
+  if (M && me > 0)
+    CADV_LAUNCH(c, k_count_greater<<<c->num_sms * 4, 256, 0, c->stream>>>(xq, M, (const uint32_t*)ab,
+                                                                             (const uint64_t*)ob, me, cnt));
+  return cudaGetLastError();
 }
 
 cudaError_t rd_compact(cadv_ctx* c, const RdState& S) {
@@ -1722,12 +1916,13 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_w, w64, ntiles, ntiles + 1));
     CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_q, q64, ntiles, ntiles + 1));
     if (c->comm->allreduce_sum_u64((uint64_t*)w64, 2 * (ntiles + 2), c->stream)) return cudaErrorUnknown;
-    if ((e = gather_entries(c, &En, &nent))) return e;  // rank 0: everyone's entries; others: nent = 0
+    // each rank links the entries of the lines it owns (line hash)
+    if ((e = exchange_entries_by_line(c, &En, &nent))) return e;
   } else if (nent) {
     CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_w, w64, ntiles, ntiles + 1));
     CADV_LAUNCH(c, k_widen<<<64, 256, 0, c->stream>>>(tile_q, q64, ntiles, ntiles + 1));
   }
-  if (nent == 0) return cudaSuccess;
+  if (nent == 0 && !spread) return cudaSuccess;
   // ---- cross-tile phase
   // tile prefix sums of weights and local query counts
   unsigned long long* twb = (unsigned long long*)((uint8_t*)tw + (ntiles + 2) * 8);
@@ -1749,8 +1944,10 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   int lb = bits_for(hmm[1] - hmm[0]);
   int tb = bits_for(ntiles);
   int sb = cta_scope ? bits_for(c->max_cta) : 0;
-  const uint32_t* order;
-  if (sb + lb + tb <= 64) {
+  const uint32_t* order = nullptr;
+  if (nent == 0) {
+    // (spread: this rank owns no line; it still takes part in the exchanges below)
+  } else if (sb + lb + tb <= 64) {
     CADV_LAUNCH(c, k_ent_key<<<grid_ls, 256, 0, c->stream>>>(En.seg, En.line, En.tile, nent, minl, lb, tb, -1, nullptr,
                                                              (uint64_t*)ek0, (uint32_t*)ei0));
     int res;
@@ -1788,23 +1985,34 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   X.xq = X.xpos + nent;
   X.part = (int64_t*)(((uintptr_t)(X.xq + nent) + 15) & ~(uintptr_t)15);
   X.xline = (uint64_t*)(X.part + nent);
-  CADV_LAUNCH(c, k_link<<<grid_ls, 256, 0, c->stream>>>(order, nent, En, twb, tqb, nbins, d_hist, d_stats, X, sc, O));
-  unsigned long long M;
+  if (nent)
+    CADV_LAUNCH(c, k_link<<<grid_ls, 256, 0, c->stream>>>(order, nent, En, twb, tqb, nbins, d_hist, d_stats, X, sc, O));
+  unsigned long long M = 0;
   if ((e = cudaMemcpyAsync(&M, &sc->count[2], 8, cudaMemcpyDeviceToHost, c->stream))) return e;
   if ((e = cudaStreamSynchronize(c->stream))) return e;
+  if (!nent) M = 0;
+  if (spread) {
+    // the queries to the ranks holding their positions (collective)
+    std::vector<uint64_t> base(c->nranks + 1, 0);
+    for (int r = 0; r < c->nranks; ++r) base[r + 1] = base[r] + kk[2 * r];
+    if ((e = exchange_queries_by_pos(c, &X, &M, base))) return e;
+  }
   c->counts[2] = M;
-  if (M == 0) return cudaSuccess;
+  if (M == 0 && !spread) return cudaSuccess;
+  if ((e = ensure(c, B_RD_ENT_IDX0, M * 4 + 64, &ei0)) || (e = ensure(c, B_RD_ENT_IDX1, M * 4 + 64, &ei1))) return e;
   // sort cross queries by position, then count inversions of their previous uses
   if ((e = ensure(c, B_RD_ENT_KEY1, M * 8 + nent * 8, &ek1))) return e;
   if ((e = ensure(c, B_SORT_K0, M * 4 * 2 + 64, &xq2))) return e;
   uint32_t* pk0 = (uint32_t*)xq2;
   uint32_t* pk1 = pk0 + M;
-  uint32_t* pi0 = (uint32_t*)ei0;  // nent >= M
+  uint32_t* pi0 = (uint32_t*)ei0;
   uint32_t* pi1 = (uint32_t*)ei1;
-  if ((e = cudaMemcpyAsync(pk0, X.xpos, M * 4, cudaMemcpyDeviceToDevice, c->stream))) return e;
-  CADV_LAUNCH(c, k_iota<<<grid_ls, 256, 0, c->stream>>>(pi0, M));
-  int res;
-  if ((e = radix_sort_pairs<uint32_t, uint32_t>(c, pk0, pi0, pk1, pi1, M, 0, 32, &res))) return e;
+  int res = 0;
+  if (M) {
+    if ((e = cudaMemcpyAsync(pk0, X.xpos, M * 4, cudaMemcpyDeviceToDevice, c->stream))) return e;
+    CADV_LAUNCH(c, k_iota<<<grid_ls, 256, 0, c->stream>>>(pi0, M));
+    if ((e = radix_sort_pairs<uint32_t, uint32_t>(c, pk0, pi0, pk1, pi1, M, 0, 32, &res))) return e;
+  }
   const uint32_t* ord = res ? pi1 : pi0;
   // keys = previous use in position order; ids = cross-query index
   uint32_t* ka = (uint32_t*)ek0;
@@ -1817,24 +2025,30 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   if ((e = ensure(c, B_RD_ENT_KEY0, M * 8 + 64, &ek0))) return e;
   ka = (uint32_t*)ek0;
   kb = ka + M;
-  CADV_LAUNCH(c, k_iota_gather<<<grid_ls, 256, 0, c->stream>>>(ord, X.xq, M, ka, ia, cnt));
-  if (!(c->attr_set & (1u << 18))) {
-    if ((e = cudaFuncSetAttribute(k_merge_count_block, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                  (int)sizeof(MergeBlockSmem))))
-      return e;
-    c->attr_set |= 1u << 18;
-  }
-  CADV_LAUNCH(c, k_merge_count_block<<<(unsigned)((M + MC_BLOCK - 1) / MC_BLOCK), 512, sizeof(MergeBlockSmem),
-                                       c->stream>>>(ka, ia, kb, ib, M, cnt));
-  std::swap(ka, kb);
-  std::swap(ia, ib);
-  for (uint64_t w = MC_BLOCK; w < M; w <<= 1) {
-    CADV_LAUNCH(c, k_merge_count<<<grid_ls, 256, 0, c->stream>>>(ka, ia, kb, ib, M, w, cnt));
+  if (M) {
+    CADV_LAUNCH(c, k_iota_gather<<<grid_ls, 256, 0, c->stream>>>(ord, X.xq, M, ka, ia, cnt));
+    if (!(c->attr_set & (1u << 18))) {
+      if ((e = cudaFuncSetAttribute(k_merge_count_block, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)sizeof(MergeBlockSmem))))
+        return e;
+      c->attr_set |= 1u << 18;
+    }
+    CADV_LAUNCH(c, k_merge_count_block<<<(unsigned)((M + MC_BLOCK - 1) / MC_BLOCK), 512, sizeof(MergeBlockSmem),
+                                         c->stream>>>(ka, ia, kb, ib, M, cnt));
     std::swap(ka, kb);
     std::swap(ia, ib);
+    for (uint64_t w = MC_BLOCK; w < M; w <<= 1) {
+      CADV_LAUNCH(c, k_merge_count<<<grid_ls, 256, 0, c->stream>>>(ka, ia, kb, ib, M, w, cnt));
+      std::swap(ka, kb);
+      std::swap(ia, ib);
+    }
   }
-  CADV_LAUNCH(c, k_cross_final<<<grid_ls, 256, 0, c->stream>>>(X.part, cnt, M, log2bins, nbins, d_hist, d_stats, sc, O,
-                                                                      X.xline));
+  // ka: this rank's previous uses in ascending order; with ranks, the queries
+  // of the earlier ranks (all at smaller positions) add their larger ones
+  if (spread && (e = add_earlier_ranks(c, ka, M, X.xq, cnt))) return e;
+  if (M)
+    CADV_LAUNCH(c, k_cross_final<<<grid_ls, 256, 0, c->stream>>>(X.part, cnt, M, log2bins, nbins, d_hist, d_stats, sc,
+                                                                        O, X.xline));
   return cudaGetLastError();
 }
 

@@ -63,11 +63,8 @@ constexpr uint32_t S_META = S_SITE + KR * 4;
 constexpr uint32_t STG_BYTES = S_META + KR;
 constexpr uint32_t R_BYTES = KS * STG_BYTES;
 
-// chunk-relative record j -> byte offset of its stage in the ring
-__device__ __forceinline__ uint32_t stage_off(uint32_t j) {
-  const uint32_t p = j / KR;
-  return (p - (p / KS) * KS) * STG_BYTES;
-}
+// piece number g of the warp (counted over all its chunks) -> its ring stage
+__device__ __forceinline__ uint32_t stage_of(uint32_t g) { return (g % KS) * STG_BYTES; }
 
 constexpr uint64_t LINE_MASK = (1ull << 58) - 1;
 constexpr int VB_STORE = 58, VB_DUP = 59, VB_W = 60;
@@ -80,7 +77,8 @@ struct ScanArgs {
   const uint32_t* winst;
   const uint8_t* meta;
   uint64_t n;
-  uint64_t chunk;        // records per warp chunk (multiple of KR)
+  uint64_t chunk;        // records per chunk (multiple of KR); warps claim chunks dynamically
+  uint64_t nchunks;
   // RD
   uint32_t lbs_rd;
   int cta_scope;
@@ -153,6 +151,8 @@ struct Counters {        // block-level shared-memory accumulators
   const uint64_t* ohi;
   uint32_t* mdo;         // [rows][2][33] MD histogram per object row
   uint32_t* dup;         // [rows] dropped duplicate loads (RD 0) per object row
+  uint32_t* wh_all;      // per-warp MD histograms [NWARP][68], then the run queues
+  bool sites_smem;       // per-site counters in shared memory (nsites <= NSITE_SMEM)
 };
 
 // row of a line among the data objects (F_OBJ)
@@ -247,8 +247,9 @@ __device__ __noinline__ void issue_partial(const ScanArgs& A, uint32_t dst, uint
 }
 template <int F>
 __device__ __forceinline__ void issue_piece(const ScanArgs& A, uint32_t ring, uint32_t bar0, uint64_t c_lo,
-                                            uint64_t s_end, uint32_t p) {
-  const uint32_t stg = p % KS, bar = bar0 + stg * 8, dst = ring + stg * STG_BYTES;
+                                            uint64_t s_end, uint32_t p, uint32_t g) {
+  // piece p of the chunk = the warp's piece g (ring stage and mbarrier by g)
+  const uint32_t stg = g % KS, bar = bar0 + stg * 8, dst = ring + stg * STG_BYTES;
   const uint32_t q0 = (uint32_t)c_lo + p * KR;  // < n < 2^32 (cadv_load_trace)
   if ((uint64_t)q0 + KR <= s_end) issue_full<F>(A, dst, bar, q0);
   else issue_partial<F>(A, dst, bar, q0, (uint32_t)(s_end - q0));
@@ -400,11 +401,16 @@ struct RunQueue {  // six columns of QCAP words from one base (one live register
 };
 
 template <int F>
-__device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters C, uint32_t* whist, bool sites_smem,
-                                        const RunQueue<F> Q, uint32_t qn, uint64_t c_lo, const uint8_t* stg,
-                                        uint32_t sbase) {
+__device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters* Cp, uint32_t qn, uint64_t c_lo,
+                                        const uint8_t* stg, uint32_t sbase) {
+  // (the block's counter table lives in shared memory: the streaming loop
+  // keeps no register for it across the call)
   constexpr bool MD = (F & F_MD) != 0, BD = (F & F_BD) != 0;
-  const uint32_t lane = lane_id();
+  const Counters C = *Cp;
+  const bool sites_smem = C.sites_smem;
+  const uint32_t lane = lane_id(), warp = threadIdx.x >> 5;
+  uint32_t* const whist = C.wh_all + warp * 68;
+  const RunQueue<F> Q{C.wh_all + NWARP * 68 + warp * (RunQueue<F>::C * 6 + 4)};
   uint32_t exec = 0, thr = 0, mxc = 0;
   for (uint32_t q0 = 0; q0 < qn; q0 += 32) {
     const uint32_t q = q0 + lane;
@@ -530,10 +536,13 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   uint64_t* s_ohi = s_olo + OBJ_SMEM;
   uint32_t* s_dup = (uint32_t*)(s_ohi + OBJ_SMEM);
   uint32_t* s_mdo = s_dup + OBJ_SMEM;
-  const Counters C{s_md_hist, (MD && sites_smem) ? sites : nullptr, s_bd_tot,
+  __shared__ Counters s_C;
+  if (tx == 0)
+    s_C = Counters{s_md_hist, (MD && sites_smem) ? sites : nullptr, s_bd_tot,
                    (BD && sites_smem) ? sites + (MD ? 2 * NSITE_SMEM : 0) : nullptr,
                    obj_sm ? s_olo : nullptr, obj_sm ? s_ohi : nullptr, (obj_sm && MD) ? s_mdo : nullptr,
-                   obj_sm ? s_dup : nullptr};
+                   obj_sm ? s_dup : nullptr, wh_all, sites_smem};
+  const Counters& C = s_C;
   if (obj_sm) {
     for (uint32_t k = tx; k < A.nobj; k += NTHR) { s_olo[k] = A.obj_lo[k]; s_ohi[k] = A.obj_hi[k]; }
     for (uint32_t k = tx; k < OBJ_SMEM; k += NTHR) s_dup[k] = 0;
@@ -552,10 +561,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
 
   uint8_t* ring = smem + warp * R_BYTES;
   uint64_t* bar = bars[warp];
-  const uint64_t gw = (uint64_t)blockIdx.x * NWARP + warp;
-  const uint64_t c_lo = gw * A.chunk;
-  const uint64_t c_hi = c_lo + A.chunk < A.n ? c_lo + A.chunk : A.n;
-  uint32_t kept = 0, ndup = 0;
+  uint32_t ndup = 0;
   // F_OBJ: duplicate loads counted per object row (run of one line per lane)
   uint64_t dc_line = ~0ull;
   uint32_t dc_row = 0, dc_cnt = 0;
@@ -566,21 +572,31 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       dc_cnt = 0;
     }
   };
-  if (c_lo < A.n) {
+  if (lane == 0) {
+    for (int s = 0; s < KS; ++s) mbar_init(&bar[s], 1);
+    fence_barrier_init();
+  }
+  __syncwarp();
+  const uint32_t ring_s = smem_u32(ring), bar_s = smem_u32(bar);
+  // Chunks are claimed dynamically (irregular traces have very uneven work
+  // per record); each chunk is one reuse-distance region in trace order.
+  // pg: pieces this warp issued before the current chunk (ring stage and
+  // mbarrier phase run on across chunks).
+  uint32_t pg = 0;
+  for (uint64_t cid = __shfl_sync(FULL, lane == 0 ? atomicAdd(&A.sc->chunk_next, 1ull) : 0ull, 0); cid < A.nchunks;
+       cid = __shfl_sync(FULL, lane == 0 ? atomicAdd(&A.sc->chunk_next, 1ull) : 0ull, 0)) {
+    const uint64_t c_lo = cid * A.chunk;
+    const uint64_t c_hi = c_lo + A.chunk < A.n ? c_lo + A.chunk : A.n;
+    uint32_t kept = 0;
     const uint32_t clen = (uint32_t)(c_hi - c_lo);
     // the chunk's last run may reach 32 records past its end; one more record
     // decides whether the last kept reuse record is followed by a duplicate
     const uint64_t s_end = c_hi + 32 < A.n ? c_hi + 32 : A.n;
     const uint32_t slen = (uint32_t)(s_end - c_lo);
     const uint32_t npieces = (slen + KR - 1) / KR;
-    if (lane == 0) {
-      for (int s = 0; s < KS; ++s) mbar_init(&bar[s], 1);
-      fence_barrier_init();
-    }
-    __syncwarp();
-    const uint32_t ring_s = smem_u32(ring), bar_s = smem_u32(bar);
     uint32_t issued = npieces < (uint32_t)KS ? npieces : (uint32_t)KS, waited = 0;
-    for (uint32_t p = 0; p < issued; ++p) issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, p);
+    fence_proxy_async();  // (the previous chunk's last reads of these stages precede the copies)
+    for (uint32_t p = 0; p < issued; ++p) issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, p, pg + p);
     // the record before the step (warp-uniform); meta 3 = "no record"
     // p_kb: kind bits of that record (bit 0 memory, 1 store, 2 BB; 0 = invalid / none)
     uint32_t p_cta = 0xffffffffu, p_t = 0, p_kb = 0, p_winst = 0, p_site = 0;
@@ -602,8 +618,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     uint32_t qn = 0;  // queued complete runs (warp-uniform)
     // RD: the last kept record when its compression run reaches the step end
     bool open_rd = false;
-    uint64_t* wbv = A.vout ? A.vout + gw * A.kcap : nullptr;
-    uint32_t* wbk = A.kout ? A.kout + gw * A.kcap : nullptr;
+    uint64_t* wbv = A.vout ? A.vout + cid * A.kcap : nullptr;
+    uint32_t* wbk = A.kout ? A.kout + cid * A.kcap : nullptr;
 
     for (uint32_t p = 0; p < npieces; ++p) {
       const uint32_t base = p * KR;
@@ -611,15 +627,15 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
       // piece p + 1 goes into the stage of piece p - 1 (consumed)
       if (p >= 1 && issued < npieces) {
         fence_proxy_async();
-        issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, issued);
+        issue_piece<F>(A, ring_s, bar_s, c_lo, s_end, issued, pg + issued);
         ++issued;
       }
-      mbar_wait(&bar[p % KS], (p / KS) & 1u);
+      mbar_wait(&bar[(pg + p) % KS], ((pg + p) / KS) & 1u);
       waited = p + 1;
       // ---- this lane's LPR consecutive records (vector shared-memory loads)
       const uint32_t j0 = base + lane * LPR;
       // this step's stage in the ring; the lane's records start at slot lane * LPR
-      const uint8_t* stg = ring + stage_off(base);
+      const uint8_t* stg = ring + stage_of(pg + p);
       const uint32_t sl = lane * LPR;
       const uint64_t* r_addr = (const uint64_t*)(stg + S_ADDR);
       const uint32_t* r_cta = (const uint32_t*)(stg + S_CTA);
@@ -808,9 +824,8 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         const uint32_t tot = __shfl_sync(FULL, x, 31);
         uint32_t pos = kept + x - nk;
         bool last_open = false;
-#pragma unroll
-        for (int k = 0; k < LPR; ++k) {
-          if (!((keepm >> k) & 1u)) continue;
+        for (uint32_t km = keepm; km; km &= km - 1) {  // (~7 % of the records are kept)
+          const uint32_t k = __ffs(km) - 1;
           const uint32_t after = brk & (0xffu << (k + 1)) & 0xffu;
           const uint32_t ab = after ? (uint32_t)(__ffs(after) - 1) : 0u;
           const uint32_t nb = after ? sb + ab : nb_l;   // the first break after record k
@@ -916,7 +931,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
           if (!bm) break;
           if (qn > QCAP - 32) {  // room for one more round
             __syncwarp();
-            flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo, stg, base);
+            flush_runs<F>(A, &s_C, qn, c_lo, stg, base);
             qn = 0;
             __syncwarp();
           }
@@ -940,7 +955,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         }
         if (qn >= 32) {
           __syncwarp();
-          flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo, stg, base);
+          flush_runs<F>(A, &s_C, qn, c_lo, stg, base);
           qn = 0;
         }
         // ---- the last head lane's open run becomes the carry
@@ -983,14 +998,16 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
     }
     if (NG && qn) {
       __syncwarp();
-      flush_runs<F>(A, C, whist, sites_smem, Q, qn, c_lo, nullptr, 0xffffffffu);
+      flush_runs<F>(A, &s_C, qn, c_lo, nullptr, 0xffffffffu);
     }
-    // no bulk copy may still target the ring when the CTA exits
-    for (uint32_t q = waited; q < issued; ++q) mbar_wait(&bar[q % KS], (q / KS) & 1u);
-  }
-  if (RD && lane == 0) {
-    A.wcnt[gw] = kept;
-    if (kept > A.kcap) atomicMax(&A.sc->kept_max, (unsigned long long)kept);
+    // no bulk copy may still target the ring when the chunk (CTA) is done
+    for (uint32_t q = waited; q < issued; ++q) mbar_wait(&bar[(pg + q) % KS], ((pg + q) / KS) & 1u);
+    pg += issued;
+    if (RD && lane == 0) {
+      A.wcnt[cid] = kept;
+      if (kept > A.kcap) atomicMax(&A.sc->kept_max, (unsigned long long)kept);
+    }
+    __syncwarp();
   }
 
   if (RD && !OBJ) {
@@ -1134,20 +1151,27 @@ cudaError_t launch_scan_t(cadv_ctx* c, const ScanArgs& A, uint64_t grid) {
 
 }  // namespace
 
-// One CTA per SM; every warp a contiguous chunk whose length is a multiple of KR.
-void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nwarps, uint64_t* chunk) {
+// One CTA per SM; the trace is cut into chunks of a multiple of KR records,
+// 1-4 per warp (CADV_SCAN_SPLIT overrides), which the warps claim
+// dynamically; *nchunks = number of chunks (= reuse-distance regions).
+void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, uint64_t* chunk) {
   uint64_t g = (uint64_t)c->num_sms;
   if (c->scan_ctas > 0 && (uint64_t)c->scan_ctas < g) g = (uint64_t)c->scan_ctas;
-  const uint64_t tw = g * NWARP;
+  // up to 4 chunks per warp, none shorter than 64 steps (16 K records):
+  // each chunk start waits for its first bulk copy with nothing to overlap
+  uint64_t split = n / (g * NWARP * 16384);
+  split = split < 1 ? 1 : (split > 4 ? 4 : split);
+  if (c->scan_split > 0) split = (uint64_t)c->scan_split;
+  const uint64_t tw = g * NWARP * split;
   uint64_t ch = (n + tw - 1) / tw;
   ch = ((ch + KR - 1) / KR) * KR;
   if (ch == 0) ch = KR;
   *chunk = ch;
-  const uint64_t need = (n + ch - 1) / ch;  // warps with records
-  g = (need + NWARP - 1) / NWARP;
-  if (g == 0) g = 1;
-  *grid = g;
-  *nwarps = g * NWARP;
+  const uint64_t need = (n + ch - 1) / ch;
+  *nchunks = need ? need : 1;
+  uint64_t gg = (need + NWARP - 1) / NWARP;
+  if (gg > g) gg = g;
+  *grid = gg ? gg : 1;
 }
 
 cudaError_t launch_squeeze(cadv_ctx* c, const uint32_t* kin, const uint64_t* vin, uint32_t* kout, uint64_t* vout,
@@ -1163,8 +1187,8 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
   ScanArgs A{};
   A.addr = t.addr; A.cta = t.cta; A.tid = t.tid; A.site = t.site; A.winst = t.winst; A.meta = t.meta;
   A.n = t.n;
-  uint64_t grid, nwarps;
-  scan_geometry(c, t.n, &grid, &nwarps, &A.chunk);
+  uint64_t grid;
+  scan_geometry(c, t.n, &grid, &A.nchunks, &A.chunk);
   A.lbs_rd = P.lbs_rd; A.cta_scope = P.cta_scope; A.kout = P.kout; A.vout = P.vout; A.wcnt = P.blkcnt;
   A.kcap = P.kcap;
   A.hist0 = P.hist0;

@@ -268,6 +268,190 @@ template cudaError_t radix_sort_pairs<uint64_t, uint32_t>(cadv_ctx*, uint64_t*, 
 template cudaError_t radix_sort_pairs<uint32_t, uint32_t>(cadv_ctx*, uint32_t*, uint32_t*, uint32_t*, uint32_t*,
                                                           uint64_t, int, int, int*);
 
+namespace {
+
+__global__ void k_bucket_count64(const uint64_t* __restrict__ key, uint64_t n, int shift, unsigned long long* cnt) {
+  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < n; i += (uint64_t)gridDim.x * blockDim.x) {
+    const uint32_t b = (uint32_t)(__ldg(key + i) >> shift);  // sorted keys: one atomic per run of a bucket in the warp
+    const uint32_t peers = __match_any_sync(__activemask(), b);
+    if (lane_id() == (uint32_t)(__ffs(peers) - 1)) atomicAdd(&cnt[b], (unsigned long long)__popc(peers));
+  }
+}
+
+// out[r] = first position whose bucket >= bnd[r] (keys sorted)
+__global__ void k_lower_bounds64(const uint64_t* __restrict__ key, uint64_t n, int shift, const uint64_t* bnd, int m,
+                                 uint64_t* out) {
+  const int r = blockIdx.x * blockDim.x + threadIdx.x;
+  if (r >= m) return;
+  uint64_t lo = 0, hi = n;
+  while (lo < hi) {
+    const uint64_t md = (lo + hi) >> 1;
+    if ((key[md] >> shift) < bnd[r]) lo = md + 1;
+    else hi = md;
+  }
+  out[r] = lo;
+}
+
+__global__ void k_max_key(const uint64_t* __restrict__ key, uint64_t n, uint32_t* out) {
+  if (threadIdx.x == 0) *out = n ? (uint32_t)(key[n - 1] >> 5) : 0u;  // sorted: the last key is the largest
+}
+
+int bits_of(uint64_t v) {
+  int b = 0;
+  while (b < 64 && (v >> b)) ++b;
+  return b;
+}
+
+// Stable sort of t's records by (cta << 5 | tid / 32): sorted keys in *keys,
+// the permuted columns in `cols` (B_GATHER layout of regroup_by_warp).
+cudaError_t sort_by_warp(cadv_ctx* c, const cadv_trace_desc& t, BufId kb0, BufId kb1, BufId vb0, BufId vb1, BufId gb,
+                         const uint64_t** keys, cadv_trace_desc* out) {
+  const uint64_t n = t.n;
+  void *k0, *k1, *v0, *v1, *g;
+  cudaError_t e;
+  if ((e = ensure(c, kb0, n * 8, &k0)) || (e = ensure(c, kb1, n * 8, &k1)) || (e = ensure(c, vb0, n * 4, &v0)) ||
+      (e = ensure(c, vb1, n * 4, &v1)) || (e = ensure(c, gb, n * 24 + 128, &g)))
+    return e;
+  const int grid = c->num_sms * 8;
+  *out = t;
+  if (n) {
+    CADV_LAUNCH(c, k_warp_keys<<<grid, 256, 0, c->stream>>>(t.cta, t.tid, n, (uint64_t*)k0, (uint32_t*)v0));
+    int res;
+    if ((e = radix_sort_pairs<uint64_t, uint32_t>(c, (uint64_t*)k0, (uint32_t*)v0, (uint64_t*)k1, (uint32_t*)v1, n, 0,
+                                                  37, &res)))
+      return e;
+    *keys = res ? (const uint64_t*)k1 : (const uint64_t*)k0;
+    const uint32_t* idx = res ? (const uint32_t*)v1 : (const uint32_t*)v0;
+    uint8_t* p = (uint8_t*)g;
+    auto al = [&](uint64_t off) { return (off + 15) & ~uint64_t(15); };
+    const uint64_t oa = 0, oc = al(n * 8), os = al(oc + n * 4), ow = al(os + n * 4), ot = al(ow + n * 4),
+                   om = al(ot + n * 2);
+    out->addr = (uint64_t*)(p + oa);
+    out->cta = (uint32_t*)(p + oc);
+    out->site = (uint32_t*)(p + os);
+    out->winst = (uint32_t*)(p + ow);
+    out->tid = (uint16_t*)(p + ot);
+    out->meta = (uint8_t*)(p + om);
+    CADV_LAUNCH(c, k_gather_all<<<grid, 256, 0, c->stream>>>(t, idx, (uint64_t*)out->addr, (uint32_t*)out->cta,
+                                                             (uint16_t*)out->tid, (uint32_t*)out->site,
+                                                             (uint32_t*)out->winst, (uint8_t*)out->meta));
+  } else {
+    *keys = (const uint64_t*)k0;
+  }
+  out->warp_contiguous = 1;
+  return cudaGetLastError();
+}
+
+}  // namespace
+
+// Multi-rank divergence on non-warp-contiguous shards: every
+// (cta, warp32) record stream moves to ONE rank, so that each warp-level
+// group is whole there.  Each rank sorts its shard stably by the stream key,
+// the key space is cut into equal shares of the global record count (bucket
+// histogram all-reduced), every rank sends its slice for rank r to r
+// (alltoallv of the seven columns incl. the key), and r stably re-sorts what
+// it received: slices arrive in rank order = trace order, so every stream
+// keeps its trace order.  Collective; *out = this rank's streams.
+cudaError_t exchange_by_warp(cadv_ctx* c, cadv_trace_desc* out) {
+  cudaError_t e;
+  Comm* cm = c->comm;
+  const int G = c->nranks, me = c->rank;
+  const uint64_t* keys = nullptr;
+  cadv_trace_desc loc;
+  if ((e = sort_by_warp(c, c->t, B_SORT_K0, B_SORT_K1, B_SORT_V0, B_SORT_V1, B_GATHER, &keys, &loc))) return e;
+  const uint64_t n = c->t.n;
+  void* cb;
+  if ((e = ensure(c, B_COMM, (size_t)(2 * G + 4) * 8 + (size_t)G * G * 8 + 64, &cb))) return e;
+  uint64_t* d_send = (uint64_t*)cb;
+  uint64_t* d_mat = d_send + G + 2;
+  // global key range -> bucket width (<= 2^20 buckets)
+  uint32_t* dm = (uint32_t*)d_mat;
+  CADV_LAUNCH(c, k_max_key<<<1, 32, 0, c->stream>>>(keys, n, dm));
+  if (cm->allreduce_max_u32(dm, 1, c->stream)) return cudaErrorUnknown;
+  uint32_t gmax = 0;
+  if ((e = cudaMemcpyAsync(&gmax, dm, 4, cudaMemcpyDeviceToHost, c->stream)) || (e = cudaStreamSynchronize(c->stream)))
+    return e;
+  const int kbits = bits_of(((uint64_t)gmax << 5) | 31u);
+  const int shift = kbits > 20 ? kbits - 20 : 0;
+  const uint64_t nb = ((((uint64_t)gmax << 5) | 31u) >> shift) + 1;
+  void* cntb;
+  if ((e = ensure(c, B_XCH_CNT, (nb + 2 * G + 4) * 8 + 64, &cntb))) return e;
+  unsigned long long* cnt = (unsigned long long*)cntb;
+  uint64_t* d_bnd = (uint64_t*)(cnt + nb);
+  if ((e = cudaMemsetAsync(cnt, 0, nb * 8, c->stream))) return e;
+  if (n) CADV_LAUNCH(c, k_bucket_count64<<<c->num_sms * 4, 256, 0, c->stream>>>(keys, n, shift, cnt));
+  if (cm->allreduce_sum_u64((uint64_t*)cnt, nb, c->stream)) return cudaErrorUnknown;
+  std::vector<uint64_t> h(nb);
+  if ((e = cudaMemcpyAsync(h.data(), cnt, nb * 8, cudaMemcpyDeviceToHost, c->stream)) ||
+      (e = cudaStreamSynchronize(c->stream)))
+    return e;
+  uint64_t total = 0;
+  for (uint64_t b = 0; b < nb; ++b) total += h[b];
+  std::vector<uint64_t> bnd(G + 1, nb), pos(G + 1, 0);
+  bnd[0] = 0;
+  {
+    uint64_t acc = 0, b = 0;
+    for (int r = 1; r < G; ++r) {
+      const uint64_t target = (uint64_t)((unsigned __int128)total * r / G);
+      while (b < nb && acc + h[b] <= target) acc += h[b++];
+      bnd[r] = b;
+    }
+  }
+  pos[G] = n;
+  if (n && G > 1) {
+    if ((e = cudaMemcpyAsync(d_bnd, bnd.data() + 1, (G - 1) * 8, cudaMemcpyHostToDevice, c->stream))) return e;
+    CADV_LAUNCH(c, k_lower_bounds64<<<1, 64, 0, c->stream>>>(keys, n, shift, d_bnd, G - 1, d_bnd + G));
+    if ((e = cudaMemcpyAsync(pos.data() + 1, d_bnd + G, (G - 1) * 8, cudaMemcpyDeviceToHost, c->stream)) ||
+        (e = cudaStreamSynchronize(c->stream)))
+      return e;
+  }
+  std::vector<uint64_t> scnt(G), soff(G), rcnt(G), roff(G), mat((size_t)G * G);
+  for (int r = 0; r < G; ++r) { soff[r] = pos[r]; scnt[r] = pos[r + 1] - pos[r]; }
+  if ((e = cudaMemcpyAsync(d_send, scnt.data(), G * 8, cudaMemcpyHostToDevice, c->stream))) return e;
+  if (cm->allgather(d_send, d_mat, G * 8, c->stream)) return cudaErrorUnknown;
+  if ((e = cudaMemcpyAsync(mat.data(), d_mat, (size_t)G * G * 8, cudaMemcpyDeviceToHost, c->stream)) ||
+      (e = cudaStreamSynchronize(c->stream)))
+    return e;
+  uint64_t Kn = 0;
+  for (int p = 0; p < G; ++p) { rcnt[p] = mat[(size_t)p * G + me]; roff[p] = Kn; Kn += rcnt[p]; }
+  for (int r = 0; r < G; ++r) {  // u32 positions per shard (decided alike on every rank)
+    uint64_t kr = 0;
+    for (int p = 0; p < G; ++p) kr += mat[(size_t)p * G + r];
+    if (kr >= 0xffffffffull) return cudaErrorNotSupported;
+  }
+  // receive buffers: the key and the six columns, 16-byte aligned slices
+  auto al = [](uint64_t x) { return (x + 15) & ~uint64_t(15); };
+  const size_t es[7] = {8, 8, 4, 2, 4, 4, 1};
+  size_t off[8];
+  off[0] = 0;
+  for (int k = 0; k < 7; ++k) off[k + 1] = al(off[k] + es[k] * Kn);
+  void* rb;
+  if ((e = ensure(c, B_WX_RECV, off[7] + 64, &rb))) return e;
+  uint8_t* R = (uint8_t*)rb;
+  const void* src[7] = {keys, loc.addr, loc.cta, loc.tid, loc.site, loc.winst, loc.meta};
+  for (int k = 0; k < 7; ++k) {
+    std::vector<uint64_t> so(G), sc(G), ro(G), rc(G);
+    for (int p = 0; p < G; ++p) {
+      so[p] = soff[p] * es[k]; sc[p] = scnt[p] * es[k]; ro[p] = roff[p] * es[k]; rc[p] = rcnt[p] * es[k];
+    }
+    if (cm->alltoallv(src[k], so.data(), sc.data(), R + off[k], ro.data(), rc.data(), c->stream))
+      return cudaErrorUnknown;
+  }
+  cadv_trace_desc recv = c->t;
+  recv.n = Kn;
+  recv.addr = (const uint64_t*)(R + off[1]);
+  recv.cta = (const uint32_t*)(R + off[2]);
+  recv.tid = (const uint16_t*)(R + off[3]);
+  recv.site = (const uint32_t*)(R + off[4]);
+  recv.winst = (const uint32_t*)(R + off[5]);
+  recv.meta = (const uint8_t*)(R + off[6]);
+  // stable re-sort of the received slices (rank order = trace order)
+  const uint64_t* k2;
+  if ((e = sort_by_warp(c, recv, B_WX_K0, B_WX_K1, B_WX_V0, B_WX_V1, B_WX_COLS, &k2, out))) return e;
+  out->n = Kn;
+  return cudaSuccess;
+}
+
 cudaError_t regroup_by_warp(cadv_ctx* c, cadv_trace_desc* out) {
   const cadv_trace_desc& t = c->t;
   uint64_t n = t.n;

@@ -37,21 +37,27 @@ def _free_port():
     return p
 
 
-def _worker(addr, rank, nranks, name, kw, snap, env, q):
+def _worker(addr, rank, nranks, name, kw, snap, env, q, contiguous=True):
     try:
         os.environ.update(env)
         import torch
         import paper_conf_cgo_shensll18_b200 as cadv
         torch.cuda.set_device(0)
-        cuts = tg.position_bounds(name, nranks, snap=snap, **kw)
-        t = tg.generate(name, cuts[rank], cuts[rank + 1], **kw)
+        if contiguous:
+            cuts = tg.position_bounds(name, nranks, snap=snap, **kw)
+        else:  # (scrambled traces are generated whole: unsnapped equal cuts)
+            n = tg.generate(name, **kw).n
+            cuts = [r * n // nranks for r in range(nranks)] + [n]
+        t = tg.generate(name, **kw) if not contiguous else None
+        t = tg.from_arrays(*(t.cols[k][cuts[rank]:cuts[rank + 1]] for k, _ in tg.COLUMNS), nsites=t.nsites) \
+            if t is not None else tg.generate(name, cuts[rank], cuts[rank + 1], **kw)
         ctx = cadv.create(0, peer_addr=addr, rank=rank, nranks=nranks)
-        ctx.load_trace(cadv.to_device(t), global_offset=cuts[rank])
+        ctx.load_trace(cadv.to_device(t), global_offset=cuts[rank], warp_contiguous=contiguous)
         out = {}
         for lb, sc in ((128, 0), (32, 0), (128, 1)):
             h, st = ctx.reuse_histogram(lb, sc, 0, 66)
             out[("rd", lb, sc)] = (h, st)
-        if snap:
+        if snap or not contiguous:
             o = ctx.analyze(rd=(128, 0, 1, 20), md=(128, 32), bd=32, nsites=t.nsites)
             out["fused"] = (o["reuse"][0], o["mem_div"][0], o["mem_div"][1], o["branch_div"][0], o["branch_div"][1])
             out["md16"] = ctx.mem_divergence(32, 16, t.nsites)
@@ -63,11 +69,12 @@ def _worker(addr, rank, nranks, name, kw, snap, env, q):
         q.put((rank, "ERR " + repr(e) + traceback.format_exc()))
 
 
-def _run(name, kw, nranks, snap, env=None):
+def _run(name, kw, nranks, snap, env=None, contiguous=True):
     addr = f"127.0.0.1:{_free_port()}"
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
-    ps = [ctx.Process(target=_worker, args=(addr, r, nranks, name, kw, snap, env or {}, q)) for r in range(nranks)]
+    ps = [ctx.Process(target=_worker, args=(addr, r, nranks, name, kw, snap, env or {}, q, contiguous))
+          for r in range(nranks)]
     for p in ps:
         p.start()
     res = {}
@@ -115,3 +122,20 @@ def test_peer_processes_unsnapped_reuse_and_alltoallv():
             h, st = orc.reuse(t, k[1], k[2], 0, 66)
             for r in range(2):
                 assert (res[r][k][0] == h).all() and res[r][k][1] == st, (env, r, k)
+
+
+def test_peer_processes_non_contiguous():
+    """warp_contiguous = 0 shards in two processes: the per-warp stream
+    exchange (exchange_by_warp) runs over the peer collectives."""
+    kw = dict(seed=2, ctas=8, threads=128, instrs=15, lines=30, pstore=0.3, pbb=0.3, scramble=1, scramble_seed=2)
+    t = tg.generate("rand", **kw)
+    res = _run("rand", kw, 2, snap=False, contiguous=False)
+    rh20 = orc.reuse(t, 128, 0, 1, 20)[0]
+    mh, ms = orc.mem_div(t, 128, 32)
+    bs, bt = orc.branch_div(t, 32)
+    for r in range(2):
+        f = res[r]["fused"]
+        assert (f[0] == rh20).all() and (f[1] == mh).all() and (f[2] == ms).all()
+        assert (f[3] == bs).all() and (f[4] == bt).all()
+        assert (res[r]["md16"][0] == orc.mem_div(t, 32, 16)[0]).all()
+        assert (res[r]["bd8"][1] == orc.branch_div(t, 8)[1]).all()

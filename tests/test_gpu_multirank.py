@@ -21,7 +21,7 @@ def cadv():
     return m
 
 
-def run_ranks(cadv, t, cuts, fn):
+def run_ranks(cadv, t, cuts, fn, contiguous=True):
     """fn(ctx) on every rank r with shard [cuts[r], cuts[r+1]); returns per-rank results."""
     import torch
     G = len(cuts) - 1
@@ -36,7 +36,7 @@ def run_ranks(cadv, t, cuts, fn):
             torch.cuda.synchronize()
             ctx = grp.context(r, stream=stream.cuda_stream)
             try:
-                ctx.load_trace(cols, global_offset=lo)
+                ctx.load_trace(cols, global_offset=lo, warp_contiguous=contiguous)
                 out[r] = fn(ctx)
             finally:
                 ctx.destroy()
@@ -233,3 +233,27 @@ def test_kernel_scope_spread_cyclic(cadv, G):
     for h, s in out:
         assert h[-1] == K and h[K - 1] == K * (R - 1) and h.sum() == n
         assert s["streaming"] == 0 and s["finite_sum"] == K * (R - 1) * (K - 1)
+
+
+@pytest.mark.parametrize("G", [2, 3])
+@pytest.mark.parametrize("seed", [0, 1])
+def test_non_contiguous_shards(cadv, G, seed):
+    """warp_contiguous = 0 on several ranks, unsnapped cuts (a warp-level
+    group may lie on two ranks): every (cta, warp32) stream moves to one rank
+    (exchange_by_warp), reuse distance keeps the trace order -- one fused call
+    per rank equals the whole-trace oracle."""
+    t = tg.generate("rand", seed=seed, ctas=8, threads=128, instrs=15, lines=30, pstore=0.3, pbb=0.3, scramble=1,
+                    scramble_seed=seed)
+    cuts = random_cuts(t.n, G, seed=seed + 11, empty=(G == 3))
+    ref = (orc.reuse(t, 128, 0, 0, 66)[0], orc.mem_div(t, 128, 32)[0], orc.mem_div(t, 128, 32)[1],
+           orc.branch_div(t, 32)[0], orc.branch_div(t, 32)[1], orc.mem_div(t, 32, 16)[0], orc.branch_div(t, 8)[1])
+
+    def fn(c):
+        o = c.analyze(rd=(128, 0, 0, 66), md=(128, 32), bd=32, nsites=t.nsites)
+        m16, _ = c.mem_divergence(32, 16, t.nsites)
+        _, b8 = c.branch_divergence(8, t.nsites)
+        return o["reuse"][0], o["mem_div"][0], o["mem_div"][1], o["branch_div"][0], o["branch_div"][1], m16, b8
+
+    out, err = run_ranks(cadv, t, cuts, fn, contiguous=False)
+    assert not any(err), err
+    check_all_equal(out, ref)
