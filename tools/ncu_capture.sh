@@ -11,7 +11,7 @@
 TAG=${1:-latest}; WL=${2:-c4_srad}; shift 2 2>/dev/null
 cd "$(dirname "$0")/.."
 O=gpurun_out
-R=/tmp/ncu_$TAG_$WL
+R=/tmp/ncu_${TAG}_$WL
 mkdir -p $O $R
 timeout 900 ncu --profile-from-start off --metrics gpu__time_duration.sum --clock-control none --csv \
     --log-file $O/${TAG}_launches_${WL}.csv \

@@ -15,6 +15,8 @@ for l in dis:
     if m and line is not None: offs[int(m.group(1),16)]=line
 rows=list(csv.reader(open(csvf)))
 h=rows[1]; data=rows[2:]
+for i,r in enumerate(data):  # first kernel section only
+    if r and r[0]=='Kernel Name': data=data[:i]; break
 ia=h.index('Address'); ie=h.index('Instructions Executed'); iss=h.index('Warp Stall Sampling (All Samples)')
 stalls=[i for i,n in enumerate(h) if n.startswith('stall_') and 'Not Issued' not in n]
 base=int(data[0][ia],16)
