@@ -27,9 +27,9 @@ struct Scalars {
   unsigned long long err_index;  // first offending record (ULLONG_MAX = none)
   unsigned int err_code;         // 1 = bad record, 2 = run longer than 32 / duplicate lane,
                                  // 3 = internal invariant, 4 = group mixes kinds / sites
-  unsigned long long unsup_index;
+  unsigned long long unsup_index;  // first memory record whose reuse line is >= 2^58 (ULLONG_MAX = none)
   unsigned long long kept_max;   // scan (RD): most kept records of one chunk (region capacity check)
-  unsigned long long chunk_next; // scan: next chunk to claim  // first memory record whose reuse line is >= 2^58 (ULLONG_MAX = none)
+  unsigned long long chunk_next; // scan: next chunk to claim
   unsigned int tile_counter;     // dynamic tile assignment
   unsigned long long count[8];   // generic counters (kept records, entries, ...)
   unsigned long long max_cta;    // scan: max CTA id of the trace (shard)
@@ -166,7 +166,8 @@ struct ScanParams {
   uint32_t rd_nbins = 0;
 };
 uint64_t scan_tiles(uint64_t n);
-void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, uint64_t* chunk);
+void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, uint64_t* chunk, uint64_t* nbig = nullptr,
+                   uint64_t* chunk_s = nullptr);
 cudaError_t launch_squeeze(cadv_ctx* c, const uint32_t* kin, const uint64_t* vin, uint32_t* kout, uint64_t* vout,
                            const uint64_t* cnt, const uint64_t* off, uint64_t nblocks, uint64_t chunk_cap);
 cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P);
@@ -178,6 +179,11 @@ cudaError_t launch_bd_resolve(cadv_ctx* c, const void* defer, const unsigned lon
 // R1 regroup by CTA through per-region CTA tables (regroup.cu; CTA scope on
 // one rank): a region = one scan warp's kept records
 constexpr uint32_t RG_MAX = 768;  // distinct CTAs per region (more: squeeze + radix sort)
+// CTA segments (CTA scope, one rank): <= SEG_WARP_MAX kept records go to the
+// segment kernel (one warp each), <= SEG_TILE_MAX to one tile each (k_rd_tile
+// over a segment list, no cross-tile queries); any longer segment sends the
+// whole call to the tiled CTA-major sequence (bounds, keys, cross-tile phase)
+constexpr uint32_t SEG_WARP_MAX = 256, SEG_TILE_MAX = 4096;
 struct RgState {
   uint32_t* pk = nullptr;    // [region][RG_MAX] CTA ids
   uint32_t* pn = nullptr;    // [region][RG_MAX] record counts, later output offsets
@@ -191,7 +197,7 @@ cudaError_t rg_count(cadv_ctx* c, const uint32_t* key, const uint64_t* cnt, uint
 // seg_cm[0] = their number, seg_cm[1] = the longest (device)
 cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, const uint32_t* key,
                       const uint64_t* val, const uint64_t* cnt, uint64_t chunk, uint32_t* kout, uint64_t* vout,
-                      uint2* seg, unsigned int* seg_cm);
+                      uint2* seg, uint2* seg_long, unsigned int* seg_cm);
 
 struct RdState {
   int cta_scope = 1;

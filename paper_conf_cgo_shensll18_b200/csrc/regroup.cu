@@ -153,17 +153,23 @@ __global__ void k_rg_offsets(const uint32_t* __restrict__ sv, const uint32_t* __
 //    their slices' CTAs, a prefix over the warps turns the region offsets of
 //    the CTAs into per-slice starts, then every warp writes its slice in
 //    order (rank among a round's peers by __match_any_sync; the peer group's
-//    leader probes the table once).
+//    leader probes the table once).  Keys are written only when a later
+//    kernel reads them (no segment list, or a segment longer than
+//    SEG_TILE_MAX kept records).  (A variant that staged each region in
+//    shared memory and wrote every (CTA, region) run contiguously was
+//    measured slower, 0.23 -> 0.40 ms on C4: half the resident CTAs and four
+//    block barriers per window.)
 constexpr int RG_W = RG_NT / 32;
 __global__ void __launch_bounds__(RG_NT) k_rg_scatter(const uint32_t* __restrict__ key,
                                                       const uint64_t* __restrict__ val,
                                                       const uint64_t* __restrict__ cnt, uint64_t chunk,
                                                       const uint32_t* __restrict__ pk, const uint32_t* __restrict__ po,
-                                                      const uint32_t* __restrict__ np, uint32_t* __restrict__ kout,
-                                                      uint64_t* __restrict__ vout) {
+                                                      const uint32_t* __restrict__ np, const unsigned int* seg_cm,
+                                                      uint32_t* __restrict__ kout, uint64_t* __restrict__ vout) {
   __shared__ uint32_t tk[RG_SLOTS];
   __shared__ uint32_t st[RG_W][RG_SLOTS];  // per slice: CTA counts, then starts
   const uint32_t lane = lane_id(), tx = threadIdx.x, q = tx >> 5, w = blockIdx.x;
+  const bool keys = seg_cm == nullptr || seg_cm[1] > SEG_TILE_MAX;  // (only the bounds-tiled path reads keys)
   for (uint32_t k = tx; k < RG_SLOTS; k += RG_NT) tk[k] = RG_EMPTY;
   for (uint32_t k = tx; k < RG_W * RG_SLOTS; k += RG_NT) (&st[0][0])[k] = 0;
   __syncthreads();
@@ -225,7 +231,7 @@ __global__ void __launch_bounds__(RG_NT) k_rg_scatter(const uint32_t* __restrict
       uint32_t dst = 0;
       if (ok) {
         dst = to[s] + __popc(peers & lanemask_lt());
-        kout[dst] = c;
+        if (keys) kout[dst] = c;
         vout[dst] = vb[b];
       }
       __syncwarp();
@@ -236,21 +242,38 @@ __global__ void __launch_bounds__(RG_NT) k_rg_scatter(const uint32_t* __restrict
 }
 
 // 4. the CTA segments of the output: for every CTA's first sorted pair,
-//    (start, length) appended to seg (unordered: segments are independent);
-//    cnt_max[0] = number of segments, cnt_max[1] = longest segment
+//    (start, length) appended to seg (<= SEG_WARP_MAX kept records, or every
+//    segment when seg_long is null) or to seg_long (unordered: segments are
+//    independent); cm[0] = |seg|, cm[1] = longest, cm[3] = |seg_long|
+//    (warp-aggregated counters)
 __global__ void k_rg_segments(const uint32_t* __restrict__ sk, const uint32_t* __restrict__ sn,
                               const uint32_t* __restrict__ so, uint64_t P, uint2* __restrict__ seg,
-                              unsigned int* __restrict__ cnt_max) {
-  for (uint64_t s = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; s < P; s += (uint64_t)gridDim.x * blockDim.x) {
-    const uint32_t c = sk[s];
-    if (s > 0 && sk[s - 1] == c) continue;
+                              uint2* __restrict__ seg_long, unsigned int* __restrict__ cm) {
+  const uint32_t lane = lane_id();
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  uint32_t mx = 0;
+  for (uint64_t base = ((blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5) * 32; base < P; base += nw * 32) {
+    const uint64_t s = base + lane;
     uint32_t len = 0;
-    for (uint64_t x = s; x < P && sk[x] == c; ++x) len += sn[x];
-    if (len == 0) continue;
-    const uint32_t k = atomicAdd(&cnt_max[0], 1u);
-    seg[k] = make_uint2(so[s], len);
-    atomicMax(&cnt_max[1], len);
+    if (s < P && (s == 0 || sk[s - 1] != sk[s])) {
+      const uint32_t c = sk[s];
+      for (uint64_t x = s; x < P && sk[x] == c; ++x) len += sn[x];
+    }
+    mx = max(mx, len);
+    const bool lg = len > SEG_WARP_MAX && seg_long != nullptr;
+    const uint32_t bs = __ballot_sync(FULL, len && !lg), bl = __ballot_sync(FULL, lg);
+    uint32_t os = 0, ol = 0;
+    if (lane == 0) {
+      if (bs) os = atomicAdd(&cm[0], (unsigned)__popc(bs));
+      if (bl) ol = atomicAdd(&cm[3], (unsigned)__popc(bl));
+    }
+    os = __shfl_sync(FULL, os, 0);
+    ol = __shfl_sync(FULL, ol, 0);
+    if (len && !lg) seg[os + __popc(bs & lanemask_lt())] = make_uint2(so[s], len);
+    if (lg) seg_long[ol + __popc(bl & lanemask_lt())] = make_uint2(so[s], len);
   }
+  mx = __reduce_max_sync(FULL, mx);
+  if (lane == 0 && mx) atomicMax(&cm[1], mx);
 }
 
 }  // namespace
@@ -279,7 +302,7 @@ cudaError_t rg_count(cadv_ctx* c, const uint32_t* key, const uint64_t* cnt, uint
 // Phases 2-3 (after the synchronisation; P = total pairs, no overflow).
 cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, const uint32_t* key,
                       const uint64_t* val, const uint64_t* cnt, uint64_t chunk, uint32_t* kout, uint64_t* vout,
-                      uint2* seg, unsigned int* seg_cm) {
+                      uint2* seg, uint2* seg_long, unsigned int* seg_cm) {
   void *b;
   cudaError_t e;
   // packed pairs (ping-pong for the sort) + counts + offsets
@@ -299,12 +322,15 @@ cudaError_t rg_finish(cadv_ctx* c, const RgState& st, uint64_t P, int bits, cons
   if ((e = exclusive_scan_u32(c, n1, n0, P, nullptr))) return e;
   // the offsets overwrite the pair counts (pn is no longer needed)
   CADV_LAUNCH(c, k_rg_offsets<<<grid, 256, 0, c->stream>>>(sv, n0, P, st.pn));
-  CADV_LAUNCH(c, k_rg_scatter<<<(unsigned)st.nregions, RG_NT, 0, c->stream>>>(key, val, cnt, chunk, st.pk, st.pn, st.np,
-                                                                           kout, vout));
   if (seg) {  // the CTA segments of the output (count and longest in seg_cm)
     if ((e = cudaMemsetAsync(seg_cm, 0, 16, c->stream))) return e;
-    CADV_LAUNCH(c, k_rg_segments<<<grid, 256, 0, c->stream>>>(res ? k1 : k0, n1, n0, P, seg, seg_cm));
+    CADV_LAUNCH(c, k_rg_segments<<<grid, 256, 0, c->stream>>>(res ? k1 : k0, n1, n0, P, seg, seg_long, seg_cm));
   }
+  // keys are written for the bounds-tiled path only (no segment list, a segment longer than
+  // SEG_TILE_MAX, or CADV_RD_TILES)
+  const unsigned int* keys_flag = (seg && getenv("CADV_RD_TILES") == nullptr) ? seg_cm : nullptr;
+  CADV_LAUNCH(c, k_rg_scatter<<<(unsigned)st.nregions, RG_NT, 0, c->stream>>>(
+                     key, val, cnt, chunk, st.pk, st.pn, st.np, keys_flag, kout, vout));
   return cudaGetLastError();
 }
 

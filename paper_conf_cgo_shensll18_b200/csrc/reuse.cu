@@ -341,25 +341,87 @@ struct SegSmem {
   uint32_t hist[TL_SMEM_BINS];
 };
 
-__global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ val, const uint2* __restrict__ seg,
-                                                  const unsigned int* __restrict__ seg_cm, unsigned int* next,
-                                                  int log2bins, uint32_t nbins, uint64_t* __restrict__ g_hist,
-                                                  uint64_t* __restrict__ g_stream, ObjTab O) {
+// dynamic shared memory of k_rd_seg: the histogram only when it fits, then
+// the object extents of a data-centric call with <= SG_OBJ_SMEM objects
+constexpr uint32_t SG_OBJ_SMEM = 64;
+// histogram words: one private copy per warp when they fit (no shared-memory
+// atomics between warps on the hot bins), else one per CTA, else none (global)
+__host__ __device__ constexpr uint64_t seg_hist_words(uint64_t hbins) {
+  return hbins * SG_W <= TL_SMEM_BINS ? hbins * SG_W : (hbins <= TL_SMEM_BINS ? hbins : 0);
+}
+__host__ __device__ constexpr size_t seg_obj_offset(uint64_t hbins) {
+  return (offsetof(SegSmem, hist) + 4 * seg_hist_words(hbins) + 15) & ~(size_t)15;
+}
+__host__ __device__ constexpr size_t seg_smem_bytes(uint64_t hbins, uint32_t nobj) {
+  return nobj && nobj <= SG_OBJ_SMEM ? seg_obj_offset(hbins) + 16 * SG_OBJ_SMEM
+                                     : offsetof(SegSmem, hist) + 4 * seg_hist_words(hbins);
+}
+
+// Shared-memory accesses by 32-bit shared-window address (computed once per
+// warp): no generic-to-shared conversion (S2UR SR_CgaCtaId + ULEA) inside the
+// round loop.
+__device__ __forceinline__ uint64_t sh_ld64(uint32_t a) {
+  uint64_t v;
+  asm volatile("ld.shared.u64 %0, [%1];" : "=l"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t sh_ld32(uint32_t a) {
+  uint32_t v;
+  asm volatile("ld.shared.u32 %0, [%1];" : "=r"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint32_t sh_ld16(uint32_t a) {
+  uint16_t v;
+  asm volatile("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a) : "memory");
+  return v;
+}
+__device__ __forceinline__ void sh_st32(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sh_st16(uint32_t a, uint32_t v) {
+  asm volatile("st.shared.u16 [%0], %1;" ::"r"(a), "h"((uint16_t)v) : "memory");
+}
+__device__ __forceinline__ void sh_add32(uint32_t a, uint32_t v) {
+  asm volatile("red.shared.add.u32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ void sh_or32(uint32_t a, uint32_t v) {
+  asm volatile("red.shared.or.b32 [%0], %1;" ::"r"(a), "r"(v) : "memory");
+}
+__device__ __forceinline__ uint64_t sh_cas64(uint32_t a, uint64_t cmp, uint64_t v) {
+  uint64_t o;
+  asm volatile("atom.shared.cas.b64 %0, [%1], %2, %3;" : "=l"(o) : "r"(a), "l"(cmp), "l"(v) : "memory");
+  return o;
+}
+
+// OBJ: data-centric rows (O.n > 0); the reuse-only instance carries none of it.
+template <bool OBJ>
+__global__ void __launch_bounds__(SG_NT, 5) k_rd_seg(const uint64_t* __restrict__ val, const uint2* __restrict__ seg,
+                                                     const unsigned int* __restrict__ seg_cm, unsigned int* next,
+                                                     int log2bins, uint32_t nbins, uint64_t* __restrict__ g_hist,
+                                                     uint64_t* __restrict__ g_stream, ObjTab O) {
   extern __shared__ __align__(16) uint8_t sg_smem[];
   SegSmem& S = *reinterpret_cast<SegSmem*>(sg_smem);
   const uint32_t tx = threadIdx.x, warp = tx >> 5, lane = lane_id();
-  const uint32_t hbins = (O.n + 1) * nbins;
-  const bool smem_hist = hbins <= TL_SMEM_BINS;
-  if (smem_hist)
-    for (uint32_t k = tx; k < hbins; k += SG_NT) S.hist[k] = 0;
+  const uint32_t nobj = OBJ ? O.n : 0u;
+  const uint32_t hbins = (nobj + 1) * nbins;
+  const uint32_t hwords = (uint32_t)seg_hist_words(hbins);
+  const bool smem_hist = hwords != 0, whist = hwords > hbins;
+  for (uint32_t k = tx; k < hwords; k += SG_NT) S.hist[k] = 0;
+  if (OBJ && nobj <= SG_OBJ_SMEM) {  // data-centric rows: the object extents in shared memory (seg_smem_bytes)
+    uint64_t* so = reinterpret_cast<uint64_t*>(sg_smem + seg_obj_offset(hbins));
+    for (uint32_t k = tx; k < nobj; k += SG_NT) { so[k] = O.lo[k]; so[SG_OBJ_SMEM + k] = O.hi[k]; }
+    O.lo = so;
+    O.hi = so + SG_OBJ_SMEM;
+  }
   __syncthreads();
   const uint32_t nseg = seg_cm[0];
-  unsigned long long* const HK = S.hk[warp];
-  uint16_t* const HP = S.hp[warp];
-  uint32_t* const WPI = S.wpi[warp];
-  uint32_t* const RW = S.rw[warp];
-  uint32_t* const CW8 = RW + 8;
-  uint32_t stream = 0;
+  const uint32_t HK = smem_u32(S.hk[warp]);   // u64 [SG_HS]
+  const uint32_t HP = smem_u32(S.hp[warp]);   // u16 [SG_HS]
+  const uint32_t WPI = smem_u32(S.wpi[warp]); // u32 [256]
+  const uint32_t RW = smem_u32(S.rw[warp]);   // u32 [8] bitmap words, then [8] word prefix counts
+  const uint32_t CW8 = RW + 32;
+  const uint32_t H = smem_u32(S.hist) + (whist ? 4 * warp * hbins : 0u);
+  uint32_t stream = 0, ninf = 0;  // ninf: the infinity bin (reuse-only instance) counted in a register
   unsigned long long rdsum = 0;
   // The next segment is claimed (and its descriptor and first round loaded)
   // while the current one is resolved; round r + 1's records are loaded at
@@ -369,12 +431,13 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
   uint2 sd = sg < nseg ? seg[sg] : make_uint2(0u, 0u);
   uint64_t vnext = lane < sd.y ? __ldg(val + sd.x + lane) : 0ull;
   while (sg < nseg) {
-    const uint64_t* const vs = val + sd.x;
-    const uint32_t n = sd.y;  // <= 256 (the host checked the longest)
+    const uint64_t* const vs = val + sd.x + lane;
+    const uint32_t n = sd.y;  // <= SEG_WARP_MAX (k_rg_segments lists longer ones apart)
     const uint32_t sg_n = __shfl_sync(FULL, lane == 0 ? atomicAdd(next, 1u) : 0u, 0);
     const uint2 sd_n = sg_n < nseg ? seg[sg_n] : make_uint2(0u, 0u);
-    for (uint32_t k = lane; k < SG_HS; k += 32) HK[k] = ~0ull;
-    if (lane < 8) { RW[lane] = 0; CW8[lane] = 0; }
+    for (uint32_t k = lane; k < SG_HS; k += 32)
+      asm volatile("st.shared.u64 [%0], %1;" ::"r"(HK + 8 * k), "l"(~0ull) : "memory");
+    if (lane < 16) sh_st32(RW + 4 * lane, 0u);
     __syncwarp();
     uint32_t wb = 0, rtot = 0;          // running weight, reused positions (warp-uniform)
     uint32_t qbits = 0, hbits = 0;      // this lane's positions 32 r + lane: query / has-dup flags
@@ -382,12 +445,23 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
       const uint32_t i = 32 * r + lane;
       const bool valid = i < n;
       const uint64_t v = vnext;
-      vnext = (i + 32 < n) ? __ldg(vs + i + 32) : 0ull;
+      vnext = (i + 32 < n) ? __ldg(vs + 32 * (r + 1)) : 0ull;
       const unsigned long long line = valid ? (v & LINE_MASK) : ~0ull;
       const bool st = (v >> VB_STORE) & 1u, hd = (v >> VB_DUP) & 1u;
       const uint32_t w = valid ? (uint32_t)(v >> VB_W) + 1u : 0u;
       // previous use of the line: an earlier lane of this round, else the table
-      const uint32_t peers = __match_any_sync(FULL, line);
+      // lines that share their high half (every lane, the usual case): a 32-bit
+      // match, much cheaper than the 64-bit one (k_rd_seg 0.49 -> 0.37 ms on C4)
+      const uint32_t lhi = (uint32_t)(line >> 32);
+      const uint32_t peers = __all_sync(FULL, lhi == __shfl_sync(FULL, lhi, 0))
+                                 ? __match_any_sync(FULL, (uint32_t)line) : __match_any_sync(FULL, line);
+      // weighted prefix (inclusive) by position (independent of the match: overlaps its latency)
+      uint32_t xw = w;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, xw, o);
+        if (lane >= (uint32_t)o) xw += y;
+      }
       const uint32_t lower = peers & lanemask_lt();
       int32_t pp = -1;
       uint32_t hs = 0;  // the group's first lane: the line's slot (bit 16: present) or the first empty slot
@@ -397,8 +471,8 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
         } else {
           uint32_t h = __umulhi((uint32_t)((line * 0x9E3779B97F4A7C15ull) >> 32), SG_HS);
           while (true) {
-            const unsigned long long k = HK[h];
-            if (k == line) { pp = (int32_t)HP[h]; hs = h | 0x10000u; break; }
+            const unsigned long long k = sh_ld64(HK + 8 * h);
+            if (k == line) { pp = (int32_t)sh_ld16(HP + 2 * h); hs = h | 0x10000u; break; }
             if (k == ~0ull) { hs = h; break; }
             h = h + 1 == SG_HS ? 0u : h + 1;
           }
@@ -414,76 +488,91 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
           // new line: claim a slot from the first empty one the probe saw (lanes
           // of other new lines insert concurrently, so with CAS)
           while (true) {
-            const unsigned long long k = atomicCAS(&HK[h], ~0ull, line);
+            const unsigned long long k = sh_cas64(HK + 8 * h, ~0ull, line);
             if (k == ~0ull || k == line) break;
             h = h + 1 == SG_HS ? 0u : h + 1;
           }
         }
-        HP[h] = (uint16_t)i;
+        sh_st16(HP + 2 * h, i);
       }
-      // weighted prefix (inclusive) by position
-      uint32_t xw = w;
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, xw, o);
-        if (lane >= (uint32_t)o) xw += y;
-      }
-      if (valid) WPI[i] = wb + xw;
+      if (valid) sh_st32(WPI + 4 * i, wb + xw);
       // reused positions inside the window (P, i): earlier rounds (bitmap R) ...
       uint32_t cnt = 0;
       if (q && (uint32_t)P < 32 * r) {
         const uint32_t pw = (uint32_t)P >> 5, pb = (uint32_t)P & 31u;
-        cnt = rtot - (CW8[pw] + __popc(RW[pw] & (0xffffffffu >> (31u - pb))));
+        cnt = rtot - (sh_ld32(CW8 + 4 * pw) + __popc(sh_ld32(RW + 4 * pw) & (0xffffffffu >> (31u - pb))));
       }
       // ... and this round: lanes s < lane with P(s) > P (bit-sliced compare)
+      // (MSB first over the bits positions of this round can have: P < 32 (r + 1))
       const uint32_t qm = __ballot_sync(FULL, q);
       const uint32_t pv = q ? (uint32_t)P : 0u;
       uint32_t gt = 0, eq = FULL;
-#pragma unroll
-      for (int kb = 7; kb >= 0; --kb) {
-        const uint32_t bk = __ballot_sync(FULL, (pv >> kb) & 1u);
-        if ((pv >> kb) & 1u) eq &= bk;
-        else { gt |= eq & bk; eq &= ~bk; }
+  // one ballot and three predicated logic ops per bit: with my bit 0 the lanes
+  // still equal above that have it set are greater; eq keeps the lanes whose
+  // bit equals mine
+#define SG_CMP_BIT(kb)                                                       \
+  asm("{\n\t.reg .pred p;\n\t.reg .b32 b, t;\n\t"                          \
+      "and.b32 t, %2, %3;\n\tsetp.ne.u32 p, t, 0;\n\t"                        \
+      "vote.sync.ballot.b32 b, p, 0xffffffff;\n\t"                            \
+      "@!p lop3.b32 %1, %1, %0, b, 0xF8;\n\t"                                 \
+      "@p and.b32 %0, %0, b;\n\t@!p lop3.b32 %0, %0, b, 0, 0x30;\n\t}"          \
+      : "+r"(eq), "+r"(gt)                                                   \
+      : "r"(pv), "n"(1u << (kb)));
+      switch (r) {
+        default: SG_CMP_BIT(7);  // fall through
+        case 2: case 3: SG_CMP_BIT(6);  // fall through
+        case 1: SG_CMP_BIT(5);  // fall through
+        case 0: SG_CMP_BIT(4); SG_CMP_BIT(3); SG_CMP_BIT(2); SG_CMP_BIT(1); SG_CMP_BIT(0);
       }
+#undef SG_CMP_BIT
       cnt += __popc(gt & qm & lanemask_lt());
       __syncwarp();
       // R4
       if (valid) {
-        uint32_t bin, cntb = 1;
         if (q) {
-          const uint32_t rd = (wb + xw - w) - WPI[P] - cnt;
-          bin = rd_bin(rd, log2bins, nbins);
+          const uint32_t rd = (wb + xw - w) - sh_ld32(WPI + 4 * (uint32_t)P) - cnt;
+          uint32_t bin = rd_bin(rd, log2bins, nbins);
           rdsum += rd;
+          if (OBJ) bin += obj_row(O, line) * nbins;
+          if (smem_hist) sh_add32(H + 4 * bin, 1u);
+          else atomicAdd((unsigned long long*)&g_hist[bin], 1ull);
         } else {
-          bin = nbins - 1;
-          if (st) cntb = w;
+          const uint32_t cntb = st ? w : 1u;
+          if (!OBJ) {
+            ninf += cntb;
+          } else {
+            const uint32_t bin = nbins - 1 + obj_row(O, line) * nbins;
+            if (smem_hist) sh_add32(H + 4 * bin, cntb);
+            else atomicAdd((unsigned long long*)&g_hist[bin], (unsigned long long)cntb);
+          }
         }
-        if (O.n) bin += obj_row(O, line) * nbins;
-        if (smem_hist) atomicAdd(&S.hist[bin], cntb);
-        else atomicAdd((unsigned long long*)&g_hist[bin], (unsigned long long)cntb);
         if (st) stream += w - 1;  // all but the last of merged stores are one-shot elements
       }
       qbits |= (uint32_t)q << r;
       hbits |= (uint32_t)hd << r;
       // R += { P(s) } of this round's queries; word prefix counts
-      if (q) atomicOr(&RW[(uint32_t)P >> 5], 1u << (P & 31));
+      if (q) sh_or32(RW + 4 * ((uint32_t)P >> 5), 1u << (P & 31));
       __syncwarp();
-      const uint32_t nr = lane < 8 ? RW[lane] : 0u;
+      const uint32_t nr = lane < 8 ? sh_ld32(RW + 4 * lane) : 0u;
       uint32_t pc = __popc(nr), xc = pc;
 #pragma unroll
       for (int o = 1; o < 8; o <<= 1) {
         const uint32_t y = __shfl_up_sync(FULL, xc, o);
         if (lane >= (uint32_t)o) xc += y;
       }
-      if (lane < 8) CW8[lane] = xc - pc;
-      rtot = __shfl_sync(FULL, xc, 7);
+      if (lane < 8) sh_st32(CW8 + 4 * lane, xc - pc);
+      rtot += __popc(qm);  // every position is reused at most once: the round's P are new bits
       wb += __shfl_sync(FULL, xw, 31);
       __syncwarp();
     }
-    // streaming: positions whose element is never used again (not reused, no dup)
-    for (uint32_t r = 0; 32 * r < n; ++r) {
-      const uint32_t i = 32 * r + lane;
-      if (i < n && !((qbits >> r) & 1u) && !((hbits >> r) & 1u) && !((RW[i >> 5] >> (i & 31u)) & 1u)) stream += 1;
+    // streaming: positions whose element is never used again (not reused, no dup);
+    // bit r of this lane's masks = position 32 r + lane
+    {
+      uint32_t reused = 0;
+#pragma unroll
+      for (int k = 0; k < 8; ++k) reused |= ((sh_ld32(RW + 4 * k) >> lane) & 1u) << k;
+      const uint32_t nr = n > lane ? (n - lane + 31) / 32 : 0u;  // this lane's positions
+      stream += __popc(((1u << nr) - 1u) & ~(qbits | hbits | reused));
     }
     __syncwarp();
     sg = sg_n;
@@ -495,10 +584,21 @@ __global__ void __launch_bounds__(SG_NT) k_rd_seg(const uint64_t* __restrict__ v
 #pragma unroll
   for (int o = 16; o; o >>= 1) rdsum += __shfl_xor_sync(FULL, rdsum, o);
   if (lane == 0 && rdsum) atomicAdd((unsigned long long*)g_stream + 1, rdsum);
+  if (!OBJ) {
+    ninf = __reduce_add_sync(FULL, ninf);
+    if (lane == 0 && ninf) {
+      if (smem_hist) sh_add32(H + 4 * (nbins - 1), ninf);
+      else atomicAdd((unsigned long long*)&g_hist[nbins - 1], (unsigned long long)ninf);
+    }
+  }
   __syncthreads();
   if (smem_hist)
-    for (uint32_t k = tx; k < hbins; k += SG_NT)
-      if (S.hist[k]) atomicAdd((unsigned long long*)&g_hist[k], (unsigned long long)S.hist[k]);
+    for (uint32_t k = tx; k < hbins; k += SG_NT) {
+      uint32_t v = S.hist[k];
+      if (whist)
+        for (int x = 1; x < SG_W; ++x) v += S.hist[x * hbins + k];
+      if (v) atomicAdd((unsigned long long*)&g_hist[k], (unsigned long long)v);
+    }
 }
 
 template <int MODE>
@@ -507,13 +607,14 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
               const uint32_t* __restrict__ bounds, uint32_t ntiles, int log2bins, uint32_t nbins,
               uint64_t* __restrict__ g_hist, uint64_t* __restrict__ g_stream, uint32_t* __restrict__ tile_w,
               uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc, uint32_t* wide_list, ObjTab O,
-              TilePos TP) {
+              TilePos TP, const uint2* __restrict__ tl) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
   const uint32_t tx = threadIdx.x;
   constexpr bool WIDE = MODE == 2;
   const uint32_t tile = MODE == 0 ? blockIdx.x : MODE == 1 ? wide_list[ntiles + 2 + blockIdx.x] : wide_list[blockIdx.x];
-  const uint64_t b = bounds[tile], e = bounds[tile + 1];
+  // tl (segment list, CTA scope on one rank): the tile is one whole segment
+  const uint64_t b = tl ? tl[tile].x : bounds[tile], e = tl ? b + tl[tile].y : bounds[tile + 1];
   const uint32_t m = (uint32_t)(e - b);
   // data-centric attribution: one row of nbins per object + 1 (O.n = 0: one row)
   const uint32_t hbins = (O.n + 1) * nbins;
@@ -569,7 +670,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   for (int j = 0; j < IPT; ++j) {
     uint32_t x = tx * IPT + j;
     uint64_t gx = b + x;
-    bool sflag = x < m && (TP.pos_base + gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1)));
+    bool sflag = x < m && (tl ? x == 0 : (TP.pos_base + gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1))));
     if (sflag) { ssm |= 1u << j; ss_local = x; }
   }
   uint32_t* tmax = reinterpret_cast<uint32_t*>(S.es);
@@ -588,8 +689,8 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     }
   }
   // (kernel scope over ranks: the one segment continues across the shards' kept records)
-  const bool head_cont = m > 0 && TP.pos_base + b > 0 && (!key || __ldg(key + b) == __ldg(key + b - 1));
-  const bool tail_cont = m > 0 && TP.pos_base + e < TP.k_glob && (!key || __ldg(key + e) == __ldg(key + e - 1));
+  const bool head_cont = !tl && m > 0 && TP.pos_base + b > 0 && (!key || __ldg(key + b) == __ldg(key + b - 1));
+  const bool tail_cont = !tl && m > 0 && TP.pos_base + e < TP.k_glob && (!key || __ldg(key + e) == __ldg(key + e - 1));
   __syncthreads();
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) S.es[x] = 0;
   // ---- warp path (MODE 0): the tile holds whole segments of <= 256 kept
@@ -794,10 +895,13 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
     TileSmemWide& SW = *reinterpret_cast<TileSmemWide*>(smem_raw);
     r = block_merge_sort<TL_NT, IPT, uint64_t, uint16_t, false>(S.key[0], SW.ps[0], S.key[1], SW.ps[1], nullptr,
                                                                 ~0ull);
-  } else if (MODE == 1) {
-    r = block_sort_keys<TL_NT, uint64_t, false>(S.key[0], S.key[1], nullptr, ~0ull);
   } else {
-    r = block_sort_keys<TL_NT, uint32_t, false>(K32a, K32b, nullptr, 0xffffffffu);
+    // only the first N1 keys (m records + pads, a power of two) take part: a
+    // short tile (one segment of the segment list) sorts fewer levels
+    uint32_t N1 = 256;
+    while (N1 < m) N1 <<= 1;
+    if (MODE == 1) r = block_sort_keys<TL_NT, uint64_t, false>(S.key[0], S.key[1], nullptr, ~0ull, N1);
+    else r = block_sort_keys<TL_NT, uint32_t, false>(K32a, K32b, nullptr, 0xffffffffu, N1);
   }
   const uint64_t* KS = S.key[r];
   const uint32_t* KS32 = r ? K32b : K32a;
@@ -1083,29 +1187,50 @@ __global__ void k_link(const uint32_t* __restrict__ order, uint64_t E, EntryCols
 
 // one level of a device-wide merge sort with inversion counting: runs of
 // width w are merged pairwise; items of the right run add the number of
-// larger items in the left run to cnt[id].
-__global__ void k_merge_count(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ iin,
-                              uint32_t* __restrict__ kout, uint32_t* __restrict__ iout, uint64_t M, uint64_t w,
-                              uint32_t* __restrict__ cnt) {
-  for (uint64_t i = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; i < M; i += (uint64_t)gridDim.x * blockDim.x) {
-    uint64_t s = (i / (2 * w)) * (2 * w);
-    uint32_t k = kin[i];
-    uint64_t dst;
-    if (i < s + w) {
-      uint64_t b0 = s + w, b1 = s + 2 * w < M ? s + 2 * w : M;
-      uint64_t lo = b0, hi = b1 > b0 ? b1 : b0;
-      while (lo < hi) { uint64_t md = (lo + hi) >> 1; if (kin[md] < k) lo = md + 1; else hi = md; }
-      dst = s + (i - s) + (lo - b0);
-    } else {
-      uint64_t a0 = s, a1 = s + w;
-      uint64_t lo = a0, hi = a1;
-      while (lo < hi) { uint64_t md = (lo + hi) >> 1; if (kin[md] < k) lo = md + 1; else hi = md; }
-      uint64_t less = lo - a0;
-      cnt[iin[i]] += (uint32_t)(w - less);
-      dst = s + (i - s - w) + less;
+// larger items in the left run to cnt[id] (keys are distinct).  Merge path:
+// each thread finds where its MP_IT consecutive output positions start in the
+// two runs with one binary search along its diagonal, then merges them
+// sequentially - a right-run item leaves lenA - a larger left items behind.
+constexpr int MP_IT = 8;
+__global__ void __launch_bounds__(256) k_merge_count(const uint32_t* __restrict__ kin, const uint32_t* __restrict__ iin,
+                                                     uint32_t* __restrict__ kout, uint32_t* __restrict__ iout,
+                                                     uint64_t M, uint64_t w, uint32_t* __restrict__ cnt) {
+  const uint64_t nthr = (M + MP_IT - 1) / MP_IT;
+  for (uint64_t t = blockIdx.x * (uint64_t)blockDim.x + threadIdx.x; t < nthr; t += (uint64_t)gridDim.x * blockDim.x) {
+    const uint64_t d0 = t * MP_IT;
+    const uint64_t s = (d0 / (2 * w)) * (2 * w);
+    const uint64_t d = d0 - s;
+    const uint64_t lenA = M - s < w ? M - s : w;
+    const uint64_t lenB = M - s > w ? (M - s - w < w ? M - s - w : w) : 0;
+    const uint32_t* A = kin + s;
+    const uint32_t* B = kin + s + lenA;
+    // a = number of left-run items among the pair's first d outputs
+    uint64_t lo = d > lenB ? d - lenB : 0, hi = d < lenA ? d : lenA;
+    while (lo < hi) {
+      const uint64_t mid = (lo + hi) >> 1;
+      if (__ldg(A + mid) <= __ldg(B + (d - 1 - mid))) lo = mid + 1;
+      else hi = mid;
     }
-    kout[dst] = k;
-    iout[dst] = iin[i];
+    uint64_t ia = lo, ib = d - lo;
+    uint32_t ka = ia < lenA ? __ldg(A + ia) : 0u, kb = ib < lenB ? __ldg(B + ib) : 0u;
+#pragma unroll
+    for (int k = 0; k < MP_IT; ++k) {
+      const uint64_t o = d + k;
+      if (o >= lenA + lenB) break;
+      if (ia < lenA && (ib >= lenB || ka <= kb)) {
+        kout[s + o] = ka;
+        iout[s + o] = __ldg(iin + s + ia);
+        ++ia;
+        if (ia < lenA) ka = __ldg(A + ia);
+      } else {
+        const uint32_t id = __ldg(iin + s + lenA + ib);
+        kout[s + o] = kb;
+        iout[s + o] = id;
+        if (lenA - ia) cnt[id] += (uint32_t)(lenA - ia);
+        ++ib;
+        if (ib < lenB) kb = __ldg(B + ib);
+      }
+    }
   }
 }
 
@@ -1718,6 +1843,49 @@ cudaError_t rd_compact(cadv_ctx* c, const RdState& S) {
   return cudaMemcpyAsync(&h[1], &scalars(c)->max_cta, 8, cudaMemcpyDeviceToHost, c->stream);
 }
 
+// One tile per listed segment (<= SEG_TILE_MAX kept records each, CTA scope,
+// one rank): k_rd_tile's block path over the whole segment, no entries (no
+// piece is cut); tiles whose line range is too wide for packed keys go to the
+// MODE 1 / 2 instances as in the bounds-tiled path.
+cudaError_t rd_segment_tiles(cadv_ctx* c, const uint64_t* val, const uint2* tl, uint32_t ntl, int log2bins,
+                             uint32_t nbins, uint64_t* d_hist, uint64_t* d_stats, const ObjTab& O) {
+  cudaError_t e;
+  Scalars* sc = scalars(c);
+  void *lst, *tw, *tq;
+  if ((e = ensure(c, B_RD_XTMP, (3 * (uint64_t)ntl + 8) * 4 + 64, &lst)) ||
+      (e = ensure(c, B_RD_TILEW, ((uint64_t)ntl + 2) * 8 * 2, &tw)) ||
+      (e = ensure(c, B_RD_TILEQ, ((uint64_t)ntl + 2) * 8 * 2, &tq)))
+    return e;
+  if (!(c->attr_set & (1u << 17))) {
+    if ((e = cudaFuncSetAttribute(k_rd_tile<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))) ||
+        (e = cudaFuncSetAttribute(k_rd_tile<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))) ||
+        (e = cudaFuncSetAttribute(k_rd_tile<2>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                  (int)sizeof(TileSmemWide))))
+      return e;
+    c->attr_set |= 1u << 17;
+  }
+  const EntryCols En{};
+  const TilePos TP{0, 0, 0};
+  uint32_t* wide_list = (uint32_t*)lst + 2;
+  CADV_LAUNCH(c, k_rd_tile<0><<<ntl, TL_NT, sizeof(TileSmem), c->stream>>>(
+                     nullptr, val, 0, nullptr, ntl, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq, En,
+                     sc, wide_list, O, TP, tl));
+  static_assert(64 + sizeof(Scalars) + 64 + 16 <= 512, "pinned staging (cadv_create: 512 bytes)");
+  unsigned long long* cnt = (unsigned long long*)((uint8_t*)c->hstage + 64 + sizeof(Scalars) + 64);
+  if ((e = cudaMemcpyAsync(cnt, &sc->count[3], 16, cudaMemcpyDeviceToHost, c->stream)) ||
+      (e = cudaStreamSynchronize(c->stream)))
+    return e;
+  if (cnt[1])
+    CADV_LAUNCH(c, k_rd_tile<1><<<(unsigned)cnt[1], TL_NT, sizeof(TileSmem), c->stream>>>(
+                       nullptr, val, 0, nullptr, ntl, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq,
+                       En, sc, wide_list, O, TP, tl));
+  if (cnt[0])
+    CADV_LAUNCH(c, k_rd_tile<2><<<(unsigned)cnt[0], TL_NT, sizeof(TileSmemWide), c->stream>>>(
+                       nullptr, val, 0, nullptr, ntl, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq,
+                       En, sc, wide_list, O, TP, tl));
+  return cudaGetLastError();
+}
+
 cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbins, uint64_t* d_hist,
                       uint64_t* d_stats, const ObjTab* obj) {
   cudaError_t e;
@@ -1744,39 +1912,47 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
       if (hs[3] == 0) {  // every region's CTAs fit its table
         const uint64_t P = hs[2];
         void* sb;
-        if ((e = ensure(c, B_RG_SEG, (P + 16) * 8 + 64, &sb))) return e;
-        uint2* seg = (uint2*)sb;
-        unsigned int* seg_cm = (unsigned int*)((uint8_t*)sb + (P + 16) * 8);  // count, longest, next
+        if ((e = ensure(c, B_RG_SEG, (P + 16) * 16 + 64, &sb))) return e;
+        uint2* seg = (uint2*)sb;                  // segments of <= SEG_WARP_MAX kept records
+        uint2* seg_long = seg + (P + 16);         // longer ones
+        unsigned int* seg_cm = (unsigned int*)(seg_long + (P + 16));  // |seg|, longest, next, |seg_long|
         if ((e = rg_finish(c, S.rgs, P, bits, (const uint32_t*)k1, (const uint64_t*)v1, S.blkcnt, S.chunk_cap,
-                           (uint32_t*)k0, (uint64_t*)v0, seg, seg_cm)))
+                           (uint32_t*)k0, (uint64_t*)v0, seg, seg_long, seg_cm)))
           return e;
         key = (const uint32_t*)k0;
         val = (const uint64_t*)v0;
-        // every CTA segment <= 256 kept records: the segment kernel, no tiles
+        // every CTA segment <= SEG_TILE_MAX kept records: no cross-segment term
+        // exists, so every segment is resolved alone - short ones by a warp of
+        // the segment kernel, long ones by a CTA of the tile kernel
         unsigned int* hcm = (unsigned int*)((uint8_t*)c->hstage + 40);
-        if ((e = cudaMemcpyAsync(hcm, seg_cm, 8, cudaMemcpyDeviceToHost, c->stream))) return e;
+        if ((e = cudaMemcpyAsync(hcm, seg_cm, 16, cudaMemcpyDeviceToHost, c->stream))) return e;
         if ((e = cudaStreamSynchronize(c->stream))) return e;
-        if (hcm[1] <= 256u && getenv("CADV_RD_TILES") == nullptr) {
+        if (hcm[1] <= SEG_TILE_MAX && getenv("CADV_RD_TILES") == nullptr) {
+          const uint32_t nshort = hcm[0], nlong = hcm[3];
+          const auto kseg = O.n ? k_rd_seg<true> : k_rd_seg<false>;
           if (!(c->attr_set & (1u << 16))) {
-            if ((e = cudaFuncSetAttribute(k_rd_seg, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(SegSmem))))
-              return e;
+            for (const auto kf : {k_rd_seg<true>, k_rd_seg<false>})
+              if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                            (int)(sizeof(SegSmem) + 16 * SG_OBJ_SMEM + 16))))
+                return e;
             c->attr_set |= 1u << 16;
           }
-          if (hcm[0]) {
+          if (nshort) {
             const uint64_t hbins = (uint64_t)(O.n + 1) * nbins;
-            const size_t smem = offsetof(SegSmem, hist) + (hbins <= TL_SMEM_BINS ? 4 * hbins : 0);
+            const size_t smem = seg_smem_bytes(hbins, O.n);
             if (c->seg_ctas_smem != smem) {
-              if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c->seg_ctas, k_rd_seg, SG_NT, smem))) return e;
+              if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c->seg_ctas, kseg, SG_NT, smem))) return e;
               if (c->seg_ctas < 1) c->seg_ctas = 1;
               c->seg_ctas_smem = smem;
             }
             const unsigned grid =
-                (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * c->seg_ctas, (hcm[0] + SG_W - 1) / SG_W);
-            CADV_LAUNCH(c, k_rd_seg<<<grid, SG_NT, smem, c->stream>>>(val, seg, seg_cm, seg_cm + 2, log2bins,
+                (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * c->seg_ctas, (nshort + SG_W - 1) / SG_W);
+            CADV_LAUNCH_N(c, "k_rd_seg", kseg<<<grid, SG_NT, smem, c->stream>>>(val, seg, seg_cm, seg_cm + 2, log2bins,
                                                                                 nbins, d_hist, d_stats, O));
           }
+          if (nlong && (e = rd_segment_tiles(c, val, seg_long, nlong, log2bins, nbins, d_hist, d_stats, O))) return e;
           c->counts[1] = 0;
-          c->counts[3] = 0;
+          c->counts[3] = nlong;
           return cudaGetLastError();
         }
       } else {  // overflow: pack, then the radix sort
@@ -1883,7 +2059,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   if (ntiles_loc) {
     CADV_LAUNCH(c, k_rd_tile<0><<<(unsigned)ntiles_loc, TL_NT, sizeof(TileSmem), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
-                       tile_w, tile_q, En, sc, wide_list, O, TP));
+                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr));
     if ((e = cudaGetLastError())) return e;
   }
   unsigned long long cnt14[4];  // count[1..4]: entries, cross queries, MODE 2 tiles, MODE 1 tiles
@@ -1892,13 +2068,13 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   if (cnt14[3]) {
     CADV_LAUNCH(c, k_rd_tile<1><<<(unsigned)cnt14[3], TL_NT, sizeof(TileSmem), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
-                       tile_w, tile_q, En, sc, wide_list, O, TP));
+                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr));
     if ((e = cudaGetLastError())) return e;
   }
   if (cnt14[2]) {
     CADV_LAUNCH(c, k_rd_tile<2><<<(unsigned)cnt14[2], TL_NT, sizeof(TileSmemWide), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
-                       tile_w, tile_q, En, sc, wide_list, O, TP));
+                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr));
     if ((e = cudaGetLastError())) return e;
   }
   unsigned long long nent = cnt14[0];

@@ -79,6 +79,8 @@ struct ScanArgs {
   uint64_t n;
   uint64_t chunk;        // records per chunk (multiple of KR); warps claim chunks dynamically
   uint64_t nchunks;
+  uint64_t nbig;         // chunks [0, nbig) have `chunk` records, the rest chunk_s (the tail: less imbalance)
+  uint64_t chunk_s;
   // RD
   uint32_t lbs_rd;
   int cta_scope;
@@ -155,10 +157,6 @@ struct Counters {        // block-level shared-memory accumulators
   bool sites_smem;       // per-site counters in shared memory (nsites <= NSITE_SMEM)
 };
 
-// row of a line among the data objects (F_OBJ)
-__device__ __forceinline__ uint32_t row_of(const ScanArgs& A, const Counters& C, uint64_t line) {
-  return C.olo ? obj_row(C.olo, C.ohi, A.nobj, line) : obj_row(A.obj_lo, A.obj_hi, A.nobj, line);
-}
 
 // Per-site counter update: shared-memory counters when the site table fits,
 // global counters otherwise; an out-of-range site raises the site flag.
@@ -268,6 +266,20 @@ __device__ __forceinline__ uint32_t lds_u32(const uint32_t* p) {
   return v;
 }
 
+// row of a line among the data objects (F_OBJ): binary search of the extents,
+// with explicit shared-memory loads when the table is in shared memory (a
+// generic load would wait on the long scoreboard)
+__device__ __forceinline__ uint32_t row_of(const ScanArgs& A, const Counters& C, uint64_t line) {
+  if (!C.olo) return obj_row(A.obj_lo, A.obj_hi, A.nobj, line);
+  uint32_t a = 0, b = A.nobj;  // a = number of extents starting at or before the line
+  while (a < b) {
+    const uint32_t m = (a + b) >> 1;
+    if (lds_u64(C.olo + m) <= line) a = m + 1;
+    else b = m;
+  }
+  return (a && line < lds_u64(C.ohi + a - 1)) ? a - 1 : A.nobj;
+}
+
 // Mask building off the integer ALU pipe (the scan's bottleneck): m += bit
 // when the condition holds, as a predicated IMAD by an opaque 1 (FMA pipe)
 // instead of SEL + IADD3 on the ALU pipe.
@@ -371,7 +383,10 @@ __device__ __forceinline__ void walk_warp(const ScanArgs& A, const Counters& C, 
     }
   } else {
     const uint64_t line = v ? ((SMEM ? aa[lane] : __ldg(A.addr + g0 + lane)) >> A.lbs_md) : 0ull;
-    const uint32_t pl = __match_any_sync(FULL, line) & ps;  // same group, same line
+    // same group, same line (a 32-bit match when every lane's line has the same high half)
+    const uint32_t lhi = (uint32_t)(line >> 32);
+    const uint32_t pl = (__all_sync(FULL, lhi == __shfl_sync(FULL, lhi, 0)) ? __match_any_sync(FULL, (uint32_t)line)
+                                                                             : __match_any_sync(FULL, line)) & ps;
     const bool first = v && (pl & lanemask_lt()) == 0u;
     const uint32_t deg = __popc(__ballot_sync(FULL, first) & ps);
     if (lead) finish_md<F>(A, C, whist, sites_smem, kind, deg, s, (F & F_OBJ) ? row_of(A, C, line) : 0u);
@@ -415,14 +430,15 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters* Cp, u
   for (uint32_t q0 = 0; q0 < qn; q0 += 32) {
     const uint32_t q = q0 + lane;
     bool md = false, bd = false, slow = false;
-    uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0, cnt = 0;
+    uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0, cnt = 0, row = 0;
     if (q < qn) {
       j = Q.j(q);
       u = Q.u(q);
       m = Q.m(q);
       const uint32_t kt = Q.kt(q);
-      kind = kt >> 16;
+      kind = (kt >> 16) & 3u;
       t = kt & 0xffffu;
+      row = kt >> 18;
       cta = Q.cta(q);
       s = Q.site(q);
       const bool bb = kind == 2u;
@@ -435,10 +451,11 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters* Cp, u
         else md = true;
       }
     }
-    // F_OBJ: the group's object from its first record's address (global; recently streamed, L2)
+    // F_OBJ: the group's object row (queued with it when the table is in shared
+    // memory, else from its first record's address: global, recently streamed, L2)
     if (MD && md)
       finish_md<F>(A, C, whist, sites_smem, kind, u & PK_M, s,
-                   (F & F_OBJ) ? row_of(A, C, __ldg(A.addr + c_lo + j) >> A.lbs_md) : 0u);
+                   (F & F_OBJ) ? (C.olo ? row : row_of(A, C, __ldg(A.addr + c_lo + j) >> A.lbs_md)) : 0u);
     if (BD) {
       if (bd) {
         exec += 1;
@@ -585,8 +602,9 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
   uint32_t pg = 0;
   for (uint64_t cid = __shfl_sync(FULL, lane == 0 ? atomicAdd(&A.sc->chunk_next, 1ull) : 0ull, 0); cid < A.nchunks;
        cid = __shfl_sync(FULL, lane == 0 ? atomicAdd(&A.sc->chunk_next, 1ull) : 0ull, 0)) {
-    const uint64_t c_lo = cid * A.chunk;
-    const uint64_t c_hi = c_lo + A.chunk < A.n ? c_lo + A.chunk : A.n;
+    const uint64_t c_lo = cid < A.nbig ? cid * A.chunk : A.nbig * A.chunk + (cid - A.nbig) * A.chunk_s;
+    const uint64_t c_len = cid < A.nbig ? A.chunk : A.chunk_s;
+    const uint64_t c_hi = c_lo + c_len < A.n ? c_lo + c_len : A.n;
     uint32_t kept = 0;
     const uint32_t clen = (uint32_t)(c_hi - c_lo);
     // the chunk's last run may reach 32 records past its end; one more record
@@ -844,19 +862,19 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
         open_rd = __ballot_sync(FULL, last_open) != 0;
         kept += tot;
         if (OBJ) {
-          const uint32_t dm = dupm & ownm;
-          if (dm) {
-#pragma unroll
-            for (int k = 0; k < LPR; ++k) {
-              if (!((dm >> k) & 1u)) continue;
-              const uint64_t ln = lds_u64(r_addr + sl + k) >> A.lbs_rd;
-              if (ln != dc_line) {
-                dc_flush();
-                dc_line = ln;
-                dc_row = row_of(A, C, ln);
-              }
-              ++dc_cnt;
+          // runs of consecutive duplicate loads: a duplicate repeats its
+          // predecessor's line, so a run is one line (one lookup, one count)
+          uint32_t dm = dupm & ownm;
+          while (dm) {
+            const uint32_t k = __ffs(dm) - 1, len = __ffs(~(dm >> k)) - 1;
+            const uint64_t ln = lds_u64(r_addr + sl + k) >> A.lbs_rd;
+            if (ln != dc_line) {
+              dc_flush();
+              dc_line = ln;
+              dc_row = row_of(A, C, ln);
             }
+            dc_cnt += len;
+            dm &= ~(((1u << len) - 1u) << k);
           }
         } else {
           ndup += __popc(dupm & ownm);
@@ -947,7 +965,10 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             Q.j(pos) = j0 + k;
             Q.u(pos) = u2;
             Q.m(pos) = m2;
-            Q.kt(pos) = ((r_meta[sl + k] & 3u) << 16) | r_tid[sl + k];
+            uint32_t kt = ((r_meta[sl + k] & 3u) << 16) | r_tid[sl + k];
+            // F_OBJ, table in shared memory: the memory group's object row rides in kt
+            if (OBJ && MD && C.olo && (kt >> 16) < 2u) kt |= row_of(A, C, lds_u64(r_addr + sl + k) >> A.lbs_md) << 18;
+            Q.kt(pos) = kt;
             Q.cta(pos) = r_cta[sl + k];
             Q.site(pos) = A.nsites ? r_site[sl + k] : 0u;
           }
@@ -969,7 +990,9 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             if (lane < 31) { tu += S_next; tmk |= M_next; }
             // the carried run's first record (its stage is recycled before the run closes)
             const uint32_t sl0 = sl + lastk;
-            Q.carry()[0] = ((r_meta[sl0] & 3u) << 16) | r_tid[sl0];
+            uint32_t kt0 = ((r_meta[sl0] & 3u) << 16) | r_tid[sl0];
+            if (OBJ && MD && C.olo && (kt0 >> 16) < 2u) kt0 |= row_of(A, C, lds_u64(r_addr + sl0) >> A.lbs_md) << 18;
+            Q.carry()[0] = kt0;
             Q.carry()[1] = r_cta[sl0];
             Q.carry()[2] = A.nsites ? r_site[sl0] : 0u;
           }
@@ -1153,8 +1176,13 @@ cudaError_t launch_scan_t(cadv_ctx* c, const ScanArgs& A, uint64_t grid) {
 
 // One CTA per SM; the trace is cut into chunks of a multiple of KR records,
 // 1-4 per warp (CADV_SCAN_SPLIT overrides), which the warps claim
-// dynamically; *nchunks = number of chunks (= reuse-distance regions).
-void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, uint64_t* chunk) {
+// dynamically; *nchunks = number of chunks (= reuse-distance regions).  With
+// more than one chunk per warp, the last half chunk per warp of the trace is
+// cut into quarter chunks: warps that claim late finish at nearly the same
+// time even when the work per record is very uneven (irregular traces).
+// Chunks [0, *nbig) have *chunk records, the others *chunk_s.
+void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, uint64_t* chunk, uint64_t* nbig,
+                   uint64_t* chunk_s) {
   uint64_t g = (uint64_t)c->num_sms;
   if (c->scan_ctas > 0 && (uint64_t)c->scan_ctas < g) g = (uint64_t)c->scan_ctas;
   // up to 4 chunks per warp, none shorter than 64 steps (16 K records):
@@ -1166,10 +1194,19 @@ void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, u
   uint64_t ch = (n + tw - 1) / tw;
   ch = ((ch + KR - 1) / KR) * KR;
   if (ch == 0) ch = KR;
+  uint64_t nb = (n + ch - 1) / ch, cs = ch, nc = nb;
+  if (split > 1 && getenv("CADV_SCAN_NOTAIL") == nullptr) {
+    cs = ((ch / 4 + KR - 1) / KR) * KR;
+    const uint64_t tail = g * NWARP * (ch / 2);
+    nb = n > tail ? (n - tail) / ch : 0;
+    const uint64_t rest = n - nb * ch;
+    nc = nb + (rest + cs - 1) / cs;
+  }
   *chunk = ch;
-  const uint64_t need = (n + ch - 1) / ch;
-  *nchunks = need ? need : 1;
-  uint64_t gg = (need + NWARP - 1) / NWARP;
+  *nchunks = nc ? nc : 1;
+  if (nbig) *nbig = nb;
+  if (chunk_s) *chunk_s = cs;
+  uint64_t gg = (*nchunks + NWARP - 1) / NWARP;
   if (gg > g) gg = g;
   *grid = gg ? gg : 1;
 }
@@ -1188,7 +1225,7 @@ cudaError_t launch_scan(cadv_ctx* c, int flags, const ScanParams& P) {
   A.addr = t.addr; A.cta = t.cta; A.tid = t.tid; A.site = t.site; A.winst = t.winst; A.meta = t.meta;
   A.n = t.n;
   uint64_t grid;
-  scan_geometry(c, t.n, &grid, &A.nchunks, &A.chunk);
+  scan_geometry(c, t.n, &grid, &A.nchunks, &A.chunk, &A.nbig, &A.chunk_s);
   A.lbs_rd = P.lbs_rd; A.cta_scope = P.cta_scope; A.kout = P.kout; A.vout = P.vout; A.wcnt = P.blkcnt;
   A.kcap = P.kcap;
   A.hist0 = P.hist0;

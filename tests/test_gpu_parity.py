@@ -563,6 +563,46 @@ def test_segment_kernel_full_hash_tables(ctx, cadv, reuse_frac):
         assert (h == ref[0]).all() and st == ref[1]
 
 
+@pytest.mark.parametrize("longest", [4096, 4097])
+def test_segment_lists_mixed_lengths(ctx, cadv, longest):
+    """CTA segments of every length class in one trace: <= 256 kept records
+    (segment kernel), 257 .. 4096 (one tile each from the segment list, no
+    cross-tile queries; line ranges for all three tile key widths) and, with
+    longest = 4097, one segment that sends the call to the bounds-tiled path
+    with its cross-tile phase.  Both scopes, both bin modes, against the
+    oracle and the forced tile path."""
+    import os
+    rng = np.random.default_rng(longest)
+    lens = [1, 2, 255, 256, 257, 300, 1000, 2048, 4095, longest] + list(rng.integers(1, 700, 60))
+    addr, cta = [], []
+    for c, n in enumerate(lens):
+        span = [1 << 12, 1 << 30, 1 << 55][c % 3]  # MODE 0 / 1 / 2 tiles (line range < 2^20, < 2^52, wider)
+        nd = max(1, int(n * rng.uniform(0.2, 0.9)))
+        lines = np.sort(rng.choice(span, nd, replace=False).astype(np.uint64))
+        seq = rng.choice(lines, int(n))
+        for k in range(1, int(n)):  # no two consecutive equal lines: every record is kept
+            if seq[k] == seq[k - 1]:
+                seq[k] = lines[(np.searchsorted(lines, seq[k]) + 1) % nd] if nd > 1 else seq[k]
+        addr.append(128 * seq)
+        cta.append(np.full(int(n), c, dtype=np.uint64))
+    order = rng.permutation(len(lens))  # CTAs interleaved in blocks, as resident CTAs would be
+    addr = np.concatenate([addr[i] for i in order])
+    cta = np.concatenate([cta[i] for i in order])
+    meta = np.where(rng.random(len(addr)) < 0.15, (2 << 2) | 1, 2 << 2)
+    t = _mk(addr, cta, tid=rng.integers(0, 256, len(addr)), meta=meta)
+    load(ctx, cadv, t)
+    for lb, scope, binning, nb in ((128, 0, 0, 66), (128, 0, 1, 20), (128, 1, 0, 66)):
+        ref = orc.reuse(t, lb, scope, binning, nb)
+        got = ctx.reuse_histogram(lb, scope, binning, nb)
+        os.environ["CADV_RD_TILES"] = "1"
+        try:
+            til = ctx.reuse_histogram(lb, scope, binning, nb)
+        finally:
+            del os.environ["CADV_RD_TILES"]
+        for h, st in (got, til):
+            assert (h == ref[0]).all() and st == ref[1], (lb, scope, binning)
+
+
 @pytest.mark.parametrize("seed", [1, 2])
 def test_many_sites_global_counters(ctx, cadv, seed):
     """More than 512 sites (NSITE_SMEM): the per-site counters of memory and
