@@ -256,8 +256,18 @@ __global__ void k_rg_segments(const uint32_t* __restrict__ sk, const uint32_t* _
     const uint64_t s = base + lane;
     uint32_t len = 0;
     if (s < P && (s == 0 || sk[s - 1] != sk[s])) {
+      // the CTA's pairs are [s, x): galloping then binary search for x (a CTA
+      // spread over many regions has a long run), length from the offsets
       const uint32_t c = sk[s];
-      for (uint64_t x = s; x < P && sk[x] == c; ++x) len += sn[x];
+      uint64_t lo = s, step = 1;  // sk[lo] == c
+      while (lo + step < P && sk[lo + step] == c) { lo += step; step <<= 1; }
+      uint64_t hi = lo + step < P ? lo + step : P;  // sk[hi] != c or hi == P
+      while (hi - lo > 1) {
+        const uint64_t md = (lo + hi) >> 1;
+        if (sk[md] == c) lo = md;
+        else hi = md;
+      }
+      len = so[lo] + sn[lo] - so[s];
     }
     mx = max(mx, len);
     const bool lg = len > SEG_WARP_MAX && seg_long != nullptr;

@@ -255,6 +255,7 @@ __device__ int block_sort_keys(K* ka, K* kb, uint16_t* cnt, K pad_key, uint32_t 
 
 // ------------------------------------------------------------------ R2-R4 tile kernel
 constexpr int TL_NT = 512;            // 8 keys per thread -> TL_CAP
+constexpr int TL_LSEG = 16;           // segments per segment-list tile
 constexpr int TL_SMEM_BINS = 1024;
 
 // Shared memory of one tile (<= 113 KB so that two CTAs fit on an SM).
@@ -274,6 +275,10 @@ struct TileSmem {
   uint32_t ws[TL_NT / 32 + 1];
   uint32_t misc[8];
   unsigned long long lmin, lmax;
+  // segment-list tiles: the tile's segments (global start, local start), <= TL_LSEG
+  uint32_t lsb[TL_LSEG];
+  uint32_t lsp[TL_LSEG + 1];
+  uint32_t nls;
 };
 // the warp path of k_rd_tile keeps 256 u32 per warp in pl + qx
 static_assert(offsetof(TileSmem, qx) == offsetof(TileSmem, pl) + sizeof(uint16_t) * TL_CAP, "pl, qx adjacent");
@@ -607,15 +612,50 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
               const uint32_t* __restrict__ bounds, uint32_t ntiles, int log2bins, uint32_t nbins,
               uint64_t* __restrict__ g_hist, uint64_t* __restrict__ g_stream, uint32_t* __restrict__ tile_w,
               uint32_t* __restrict__ tile_q, EntryCols E, Scalars* sc, uint32_t* wide_list, ObjTab O,
-              TilePos TP, const uint2* __restrict__ tl) {
+              TilePos TP, const uint2* __restrict__ tl, const uint32_t* __restrict__ tofs) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   TileSmem& S = *reinterpret_cast<TileSmem*>(smem_raw);
   const uint32_t tx = threadIdx.x;
   constexpr bool WIDE = MODE == 2;
   const uint32_t tile = MODE == 0 ? blockIdx.x : MODE == 1 ? wide_list[ntiles + 2 + blockIdx.x] : wide_list[blockIdx.x];
-  // tl (segment list, CTA scope on one rank): the tile is one whole segment
-  const uint64_t b = tl ? tl[tile].x : bounds[tile], e = tl ? b + tl[tile].y : bounds[tile + 1];
+  // tl (segment list, CTA scope on one rank): the tile is whole segments
+  // tl[tofs[tile] .. tofs[tile + 1]) (one segment when tofs is null), placed
+  // one after the other; gpos maps a tile position to its kept record
+  uint64_t b = 0, e = 0;
+  if (!tl) {
+    b = bounds[tile];
+    e = bounds[tile + 1];
+  } else {
+    if (tx == 0) {
+      const uint32_t j0 = tofs ? tofs[tile] : tile, j1 = tofs ? tofs[tile + 1] : tile + 1;
+      uint32_t acc = 0;
+      for (uint32_t j = j0; j < j1; ++j) {
+        const uint2 d = tl[j];
+        S.lsb[j - j0] = d.x;
+        S.lsp[j - j0] = acc;
+        acc += d.y;
+      }
+      S.lsp[j1 - j0] = acc;
+      S.nls = j1 - j0;
+    }
+    __syncthreads();
+    e = S.lsp[S.nls];
+  }
   const uint32_t m = (uint32_t)(e - b);
+  auto lseg = [&](uint32_t x) {  // the list segment holding tile position x
+    uint32_t lo = 0, hi = S.nls - 1;
+    while (lo < hi) {
+      const uint32_t md = (lo + hi + 1) >> 1;
+      if (S.lsp[md] <= x) lo = md;
+      else hi = md - 1;
+    }
+    return lo;
+  };
+  auto gpos = [&](uint32_t x) -> uint64_t {
+    if (!tl) return b + x;
+    const uint32_t j = lseg(x);
+    return (uint64_t)S.lsb[j] + (x - S.lsp[j]);
+  };
   // data-centric attribution: one row of nbins per object + 1 (O.n = 0: one row)
   const uint32_t hbins = (O.n + 1) * nbins;
   const bool smem_hist = hbins <= TL_SMEM_BINS;
@@ -630,7 +670,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   {
     uint64_t mn = ~0ull, mx = 0;
     for (uint32_t x = tx; x < m; x += TL_NT) {
-      uint64_t l = __ldg(val + b + x) & LINE_MASK;
+      uint64_t l = __ldg(val + gpos(x)) & LINE_MASK;
       mn = l < mn ? l : mn;
       mx = l > mx ? l : mx;
     }
@@ -670,7 +710,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   for (int j = 0; j < IPT; ++j) {
     uint32_t x = tx * IPT + j;
     uint64_t gx = b + x;
-    bool sflag = x < m && (tl ? x == 0 : (TP.pos_base + gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1))));
+    bool sflag = x < m && (tl ? S.lsp[lseg(x)] == x : (TP.pos_base + gx == 0 || (key && __ldg(key + gx) != __ldg(key + gx - 1))));
     if (sflag) { ssm |= 1u << j; ss_local = x; }
   }
   uint32_t* tmax = reinterpret_cast<uint32_t*>(S.es);
@@ -699,7 +739,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   //      two sorts as below over <= 256 keys (<= 5 merge levels instead of 9,
   //      warp syncs only).  Segments cut by a tile boundary, longer segments
   //      and the wider key modes take the block path.
-  if (MODE == 0 && !head_cont && !tail_cont && m) {
+  if (MODE == 0 && !tl && !head_cont && !tail_cont && m) {
     uint32_t ml = 0;
 #pragma unroll
     for (int j = 0; j < IPT; ++j) {
@@ -868,7 +908,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
   uint16_t* PSW = WIDE ? reinterpret_cast<TileSmemWide*>(smem_raw)->ps[0] : nullptr;
   for (uint32_t x = tx; x < TL_CAP; x += TL_NT) {
     if (x < m) {
-      uint64_t v = __ldg(val + b + x);
+      uint64_t v = __ldg(val + gpos(x));
       uint64_t l = v & LINE_MASK;
       if (MODE == 0) K32a[swz<uint32_t>(x)] = (uint32_t)(((l - lmin) << 12) | x);
       else S.key[0][WIDE ? x : swz<uint64_t>(x)] = WIDE ? l : (((l - lmin) << 12) | x);
@@ -1038,7 +1078,7 @@ __global__ void __launch_bounds__(TL_NT, MODE == 2 ? 1 : 2)
       bin = nbins - 1;
     }
     if (bin != 0xffffffffu) {
-      if (O.n) bin += obj_row(O, __ldg(val + b + x) & LINE_MASK) * nbins;
+      if (O.n) bin += obj_row(O, __ldg(val + gpos(x)) & LINE_MASK) * nbins;
       if (smem_hist) atomicAdd(&S.hist[bin], cntb);
       else atomicAdd((unsigned long long*)&g_hist[bin], (unsigned long long)cntb);
     }
@@ -1843,19 +1883,42 @@ cudaError_t rd_compact(cadv_ctx* c, const RdState& S) {
   return cudaMemcpyAsync(&h[1], &scalars(c)->max_cta, 8, cudaMemcpyDeviceToHost, c->stream);
 }
 
-// One tile per listed segment (<= SEG_TILE_MAX kept records each, CTA scope,
-// one rank): k_rd_tile's block path over the whole segment, no entries (no
-// piece is cut); tiles whose line range is too wide for packed keys go to the
-// MODE 1 / 2 instances as in the bounds-tiled path.
+// The listed segments (257 .. SEG_TILE_MAX kept records each, CTA scope, one
+// rank) packed next-fit, in list order, into tiles of <= TL_CAP kept records
+// and <= TL_LSEG segments (the host reads the lengths back: a few hundred KB
+// at most); k_rd_tile's block path resolves each tile without entries (no
+// segment is cut); tiles whose line range is too wide for packed keys go to
+// the MODE 1 / 2 instances as in the bounds-tiled path.
 cudaError_t rd_segment_tiles(cadv_ctx* c, const uint64_t* val, const uint2* tl, uint32_t ntl, int log2bins,
                              uint32_t nbins, uint64_t* d_hist, uint64_t* d_stats, const ObjTab& O) {
   cudaError_t e;
   Scalars* sc = scalars(c);
-  void *lst, *tw, *tq;
-  if ((e = ensure(c, B_RD_XTMP, (3 * (uint64_t)ntl + 8) * 4 + 64, &lst)) ||
-      (e = ensure(c, B_RD_TILEW, ((uint64_t)ntl + 2) * 8 * 2, &tw)) ||
-      (e = ensure(c, B_RD_TILEQ, ((uint64_t)ntl + 2) * 8 * 2, &tq)))
+  std::vector<uint2> hs(ntl);
+  if ((e = cudaMemcpyAsync(hs.data(), tl, (size_t)ntl * sizeof(uint2), cudaMemcpyDeviceToHost, c->stream)) ||
+      (e = cudaStreamSynchronize(c->stream)))
     return e;
+  std::vector<uint32_t> tofs;
+  tofs.reserve(ntl / 2 + 2);
+  uint32_t acc = TL_CAP + 1, nin = 0;
+  for (uint32_t j = 0; j < ntl; ++j) {
+    if (acc + hs[j].y > (uint32_t)TL_CAP || nin == (uint32_t)TL_LSEG) {
+      tofs.push_back(j);
+      acc = 0;
+      nin = 0;
+    }
+    acc += hs[j].y;
+    ++nin;
+  }
+  tofs.push_back(ntl);
+  const uint32_t nt = (uint32_t)tofs.size() - 1;
+  void *lst, *tw, *tq;
+  if ((e = ensure(c, B_RD_XTMP, (3 * (uint64_t)nt + 8 + (uint64_t)nt + 2) * 4 + 64, &lst)) ||
+      (e = ensure(c, B_RD_TILEW, ((uint64_t)nt + 2) * 8 * 2, &tw)) ||
+      (e = ensure(c, B_RD_TILEQ, ((uint64_t)nt + 2) * 8 * 2, &tq)))
+    return e;
+  uint32_t* wide_list = (uint32_t*)lst + 2;
+  uint32_t* d_tofs = (uint32_t*)lst + 3 * (uint64_t)nt + 8;
+  if ((e = cudaMemcpyAsync(d_tofs, tofs.data(), tofs.size() * 4, cudaMemcpyHostToDevice, c->stream))) return e;
   if (!(c->attr_set & (1u << 17))) {
     if ((e = cudaFuncSetAttribute(k_rd_tile<0>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))) ||
         (e = cudaFuncSetAttribute(k_rd_tile<1>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)sizeof(TileSmem))) ||
@@ -1866,10 +1929,9 @@ cudaError_t rd_segment_tiles(cadv_ctx* c, const uint64_t* val, const uint2* tl, 
   }
   const EntryCols En{};
   const TilePos TP{0, 0, 0};
-  uint32_t* wide_list = (uint32_t*)lst + 2;
-  CADV_LAUNCH(c, k_rd_tile<0><<<ntl, TL_NT, sizeof(TileSmem), c->stream>>>(
-                     nullptr, val, 0, nullptr, ntl, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq, En,
-                     sc, wide_list, O, TP, tl));
+  CADV_LAUNCH(c, k_rd_tile<0><<<nt, TL_NT, sizeof(TileSmem), c->stream>>>(
+                     nullptr, val, 0, nullptr, nt, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq, En,
+                     sc, wide_list, O, TP, tl, d_tofs));
   static_assert(64 + sizeof(Scalars) + 64 + 16 <= 512, "pinned staging (cadv_create: 512 bytes)");
   unsigned long long* cnt = (unsigned long long*)((uint8_t*)c->hstage + 64 + sizeof(Scalars) + 64);
   if ((e = cudaMemcpyAsync(cnt, &sc->count[3], 16, cudaMemcpyDeviceToHost, c->stream)) ||
@@ -1877,12 +1939,12 @@ cudaError_t rd_segment_tiles(cadv_ctx* c, const uint64_t* val, const uint2* tl, 
     return e;
   if (cnt[1])
     CADV_LAUNCH(c, k_rd_tile<1><<<(unsigned)cnt[1], TL_NT, sizeof(TileSmem), c->stream>>>(
-                       nullptr, val, 0, nullptr, ntl, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq,
-                       En, sc, wide_list, O, TP, tl));
+                       nullptr, val, 0, nullptr, nt, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq,
+                       En, sc, wide_list, O, TP, tl, d_tofs));
   if (cnt[0])
     CADV_LAUNCH(c, k_rd_tile<2><<<(unsigned)cnt[0], TL_NT, sizeof(TileSmemWide), c->stream>>>(
-                       nullptr, val, 0, nullptr, ntl, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq,
-                       En, sc, wide_list, O, TP, tl));
+                       nullptr, val, 0, nullptr, nt, log2bins, nbins, d_hist, d_stats, (uint32_t*)tw, (uint32_t*)tq,
+                       En, sc, wide_list, O, TP, tl, d_tofs));
   return cudaGetLastError();
 }
 
@@ -2059,7 +2121,7 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   if (ntiles_loc) {
     CADV_LAUNCH(c, k_rd_tile<0><<<(unsigned)ntiles_loc, TL_NT, sizeof(TileSmem), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
-                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr));
+                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr, nullptr));
     if ((e = cudaGetLastError())) return e;
   }
   unsigned long long cnt14[4];  // count[1..4]: entries, cross queries, MODE 2 tiles, MODE 1 tiles
@@ -2068,13 +2130,13 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   if (cnt14[3]) {
     CADV_LAUNCH(c, k_rd_tile<1><<<(unsigned)cnt14[3], TL_NT, sizeof(TileSmem), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
-                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr));
+                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr, nullptr));
     if ((e = cudaGetLastError())) return e;
   }
   if (cnt14[2]) {
     CADV_LAUNCH(c, k_rd_tile<2><<<(unsigned)cnt14[2], TL_NT, sizeof(TileSmemWide), c->stream>>>(
                        key, val, K, (const uint32_t*)bnd, (uint32_t)ntiles_loc, log2bins, nbins, d_hist, d_stats,
-                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr));
+                       tile_w, tile_q, En, sc, wide_list, O, TP, nullptr, nullptr));
     if ((e = cudaGetLastError())) return e;
   }
   unsigned long long nent = cnt14[0];
@@ -2187,7 +2249,8 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   if (M) {
     if ((e = cudaMemcpyAsync(pk0, X.xpos, M * 4, cudaMemcpyDeviceToDevice, c->stream))) return e;
     CADV_LAUNCH(c, k_iota<<<grid_ls, 256, 0, c->stream>>>(pi0, M));
-    if ((e = radix_sort_pairs<uint32_t, uint32_t>(c, pk0, pi0, pk1, pi1, M, 0, 32, &res))) return e;
+    // (positions < the global kept count: only its bits, 3 passes instead of 4 below 2^27)
+    if ((e = radix_sort_pairs<uint32_t, uint32_t>(c, pk0, pi0, pk1, pi1, M, 0, bits_for(TP.k_glob), &res))) return e;
   }
   const uint32_t* ord = res ? pi1 : pi0;
   // keys = previous use in position order; ids = cross-query index

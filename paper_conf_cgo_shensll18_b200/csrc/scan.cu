@@ -383,10 +383,7 @@ __device__ __forceinline__ void walk_warp(const ScanArgs& A, const Counters& C, 
     }
   } else {
     const uint64_t line = v ? ((SMEM ? aa[lane] : __ldg(A.addr + g0 + lane)) >> A.lbs_md) : 0ull;
-    // same group, same line (a 32-bit match when every lane's line has the same high half)
-    const uint32_t lhi = (uint32_t)(line >> 32);
-    const uint32_t pl = (__all_sync(FULL, lhi == __shfl_sync(FULL, lhi, 0)) ? __match_any_sync(FULL, (uint32_t)line)
-                                                                             : __match_any_sync(FULL, line)) & ps;
+    const uint32_t pl = __match_any_sync(FULL, line) & ps;  // same group, same line
     const bool first = v && (pl & lanemask_lt()) == 0u;
     const uint32_t deg = __popc(__ballot_sync(FULL, first) & ps);
     if (lead) finish_md<F>(A, C, whist, sites_smem, kind, deg, s, (F & F_OBJ) ? row_of(A, C, line) : 0u);
@@ -430,15 +427,14 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters* Cp, u
   for (uint32_t q0 = 0; q0 < qn; q0 += 32) {
     const uint32_t q = q0 + lane;
     bool md = false, bd = false, slow = false;
-    uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0, cnt = 0, row = 0;
+    uint32_t j = 0, u = 0, m = 0, t = 0, kind = 0, cta = 0, s = 0, cnt = 0;
     if (q < qn) {
       j = Q.j(q);
       u = Q.u(q);
       m = Q.m(q);
       const uint32_t kt = Q.kt(q);
-      kind = (kt >> 16) & 3u;
+      kind = kt >> 16;
       t = kt & 0xffffu;
-      row = kt >> 18;
       cta = Q.cta(q);
       s = Q.site(q);
       const bool bb = kind == 2u;
@@ -451,11 +447,12 @@ __device__ __noinline__ void flush_runs(const ScanArgs& A, const Counters* Cp, u
         else md = true;
       }
     }
-    // F_OBJ: the group's object row (queued with it when the table is in shared
-    // memory, else from its first record's address: global, recently streamed, L2)
+    // F_OBJ: the group's object from its first record's address (global; recently streamed, L2).
+    // (Computing the row when the run is queued, from the ring, was measured slower:
+    // k_scan<11> 3.95 -> 4.27 ms - the streaming loop carries the search.)
     if (MD && md)
       finish_md<F>(A, C, whist, sites_smem, kind, u & PK_M, s,
-                   (F & F_OBJ) ? (C.olo ? row : row_of(A, C, __ldg(A.addr + c_lo + j) >> A.lbs_md)) : 0u);
+                   (F & F_OBJ) ? row_of(A, C, __ldg(A.addr + c_lo + j) >> A.lbs_md) : 0u);
     if (BD) {
       if (bd) {
         exec += 1;
@@ -965,10 +962,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             Q.j(pos) = j0 + k;
             Q.u(pos) = u2;
             Q.m(pos) = m2;
-            uint32_t kt = ((r_meta[sl + k] & 3u) << 16) | r_tid[sl + k];
-            // F_OBJ, table in shared memory: the memory group's object row rides in kt
-            if (OBJ && MD && C.olo && (kt >> 16) < 2u) kt |= row_of(A, C, lds_u64(r_addr + sl + k) >> A.lbs_md) << 18;
-            Q.kt(pos) = kt;
+            Q.kt(pos) = ((r_meta[sl + k] & 3u) << 16) | r_tid[sl + k];
             Q.cta(pos) = r_cta[sl + k];
             Q.site(pos) = A.nsites ? r_site[sl + k] : 0u;
           }
@@ -990,9 +984,7 @@ __global__ void __launch_bounds__(NTHR, 1) k_scan(const __grid_constant__ ScanAr
             if (lane < 31) { tu += S_next; tmk |= M_next; }
             // the carried run's first record (its stage is recycled before the run closes)
             const uint32_t sl0 = sl + lastk;
-            uint32_t kt0 = ((r_meta[sl0] & 3u) << 16) | r_tid[sl0];
-            if (OBJ && MD && C.olo && (kt0 >> 16) < 2u) kt0 |= row_of(A, C, lds_u64(r_addr + sl0) >> A.lbs_md) << 18;
-            Q.carry()[0] = kt0;
+            Q.carry()[0] = ((r_meta[sl0] & 3u) << 16) | r_tid[sl0];
             Q.carry()[1] = r_cta[sl0];
             Q.carry()[2] = A.nsites ? r_site[sl0] : 0u;
           }
@@ -1178,8 +1170,8 @@ cudaError_t launch_scan_t(cadv_ctx* c, const ScanArgs& A, uint64_t grid) {
 // 1-4 per warp (CADV_SCAN_SPLIT overrides), which the warps claim
 // dynamically; *nchunks = number of chunks (= reuse-distance regions).  With
 // more than one chunk per warp, the last half chunk per warp of the trace is
-// cut into quarter chunks: warps that claim late finish at nearly the same
-// time even when the work per record is very uneven (irregular traces).
+// cut into quarter chunks (n < 2^31): warps that claim late finish at nearly
+// the same time even when the work per record is very uneven.
 // Chunks [0, *nbig) have *chunk records, the others *chunk_s.
 void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, uint64_t* chunk, uint64_t* nbig,
                    uint64_t* chunk_s) {
@@ -1195,9 +1187,13 @@ void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, u
   ch = ((ch + KR - 1) / KR) * KR;
   if (ch == 0) ch = KR;
   uint64_t nb = (n + ch - 1) / ch, cs = ch, nc = nb;
-  if (split > 1 && getenv("CADV_SCAN_NOTAIL") == nullptr) {
+  // (n < 2^31: the tail's extra regions cost kept-record workspace, which a
+  // 4e9-record context cannot spare)
+  if (split > 1 && n < (1ull << 31) && getenv("CADV_SCAN_NOTAIL") == nullptr) {
     cs = ((ch / 4 + KR - 1) / KR) * KR;
-    const uint64_t tail = g * NWARP * (ch / 2);
+    uint64_t tq = 2;  // tail quarter chunks per warp
+    if (const char* ev = getenv("CADV_SCAN_TAIL")) tq = (uint64_t)atoi(ev);
+    const uint64_t tail = g * NWARP * (ch / 4) * tq;
     nb = n > tail ? (n - tail) / ch : 0;
     const uint64_t rest = n - nb * ch;
     nc = nb + (rest + cs - 1) / cs;
