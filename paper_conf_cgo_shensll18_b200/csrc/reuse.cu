@@ -80,6 +80,47 @@ __global__ void k_tile_bounds(const uint32_t* __restrict__ key, uint64_t K, uint
   }
 }
 
+// The CTA segments of a CTA-major kept sequence (multi-rank CTA scope, after
+// the exchange): every position where the key changes starts one; its end by
+// galloping + binary search; appended as k_rg_segments does (short list
+// <= SEG_WARP_MAX, long list, cm[0] / cm[3] counts, cm[1] longest).
+__global__ void k_key_segments(const uint32_t* __restrict__ key, uint64_t K, uint2* __restrict__ seg,
+                               uint2* __restrict__ seg_long, unsigned int* __restrict__ cm) {
+  const uint32_t lane = lane_id();
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  uint32_t mx = 0;
+  for (uint64_t base = ((blockIdx.x * (uint64_t)blockDim.x + threadIdx.x) >> 5) * 32; base < K; base += nw * 32) {
+    const uint64_t s = base + lane;
+    uint32_t len = 0;
+    if (s < K && (s == 0 || key[s - 1] != key[s])) {
+      const uint32_t c = key[s];
+      uint64_t lo = s, step = 1;
+      while (lo + step < K && key[lo + step] == c) { lo += step; step <<= 1; }
+      uint64_t hi = lo + step < K ? lo + step : K;
+      while (hi - lo > 1) {
+        const uint64_t md = (lo + hi) >> 1;
+        if (key[md] == c) lo = md;
+        else hi = md;
+      }
+      len = (uint32_t)(lo + 1 - s);
+    }
+    mx = max(mx, len);
+    const bool lg = len > SEG_WARP_MAX;
+    const uint32_t bs = __ballot_sync(FULL, len && !lg), bl = __ballot_sync(FULL, lg);
+    uint32_t os = 0, ol = 0;
+    if (lane == 0) {
+      if (bs) os = atomicAdd(&cm[0], (unsigned)__popc(bs));
+      if (bl) ol = atomicAdd(&cm[3], (unsigned)__popc(bl));
+    }
+    os = __shfl_sync(FULL, os, 0);
+    ol = __shfl_sync(FULL, ol, 0);
+    if (len && !lg) seg[os + __popc(bs & lanemask_lt())] = make_uint2((uint32_t)s, len);
+    if (lg) seg_long[ol + __popc(bl & lanemask_lt())] = make_uint2((uint32_t)s, len);
+  }
+  mx = __reduce_max_sync(FULL, mx);
+  if (lane == 0 && mx) atomicMax(&cm[1], mx);
+}
+
 // ------------------------------------------------------------------ block merge sort (shared memory)
 // Stable merge sort of N = NT*IPT items held in (ka, pa); result ends in the
 // buffer returned (0 = a, 1 = b).  COUNT: for every item from the right run
@@ -406,6 +447,7 @@ __global__ void __launch_bounds__(SG_NT, 5) k_rd_seg(const uint64_t* __restrict_
                                                      uint64_t* __restrict__ g_stream, ObjTab O) {
   extern __shared__ __align__(16) uint8_t sg_smem[];
   SegSmem& S = *reinterpret_cast<SegSmem*>(sg_smem);
+  if (seg_cm[1] > SEG_TILE_MAX) return;  // the call takes the bounds-tiled path (queued before the host knew)
   const uint32_t tx = threadIdx.x, warp = tx >> 5, lane = lane_id();
   const uint32_t nobj = OBJ ? O.n : 0u;
   const uint32_t hbins = (nobj + 1) * nbins;
@@ -1948,6 +1990,52 @@ cudaError_t rd_segment_tiles(cadv_ctx* c, const uint64_t* val, const uint2* tl, 
   return cudaGetLastError();
 }
 
+// Every CTA segment <= SEG_TILE_MAX kept records (CTA scope): no
+// cross-segment term exists, so every segment is resolved alone - short ones
+// by a warp of the segment kernel, long ones by the tile kernel over the
+// packed segment list.  The segment kernel is queued before the host reads
+// the segment counts (persistent grid: it reads them on the device and does
+// nothing when a segment is longer than SEG_TILE_MAX), so the read-back
+// overlaps it.  *done = false: a longer segment (or CADV_RD_TILES) - the
+// caller takes the bounds-tiled path.  nseg_max: an upper bound of the
+// number of segments (grid size).
+cudaError_t rd_segments(cadv_ctx* c, const uint64_t* val, const uint2* seg, const uint2* seg_long,
+                        unsigned int* seg_cm, uint64_t nseg_max, int log2bins, uint32_t nbins, uint64_t* d_hist,
+                        uint64_t* d_stats, const ObjTab& O, bool* done) {
+  cudaError_t e;
+  *done = false;
+  if (getenv("CADV_RD_TILES") != nullptr) return cudaSuccess;
+  const auto kseg = O.n ? k_rd_seg<true> : k_rd_seg<false>;
+  if (!(c->attr_set & (1u << 16))) {
+    for (const auto kf : {k_rd_seg<true>, k_rd_seg<false>})
+      if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                    (int)(sizeof(SegSmem) + 16 * SG_OBJ_SMEM + 16))))
+        return e;
+    c->attr_set |= 1u << 16;
+  }
+  const uint64_t hbins = (uint64_t)(O.n + 1) * nbins;
+  const size_t smem = seg_smem_bytes(hbins, O.n);
+  if (c->seg_ctas_smem != smem) {
+    if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c->seg_ctas, kseg, SG_NT, smem))) return e;
+    if (c->seg_ctas < 1) c->seg_ctas = 1;
+    c->seg_ctas_smem = smem;
+  }
+  const unsigned grid = (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * c->seg_ctas, (nseg_max + SG_W - 1) / SG_W);
+  if (grid)
+    CADV_LAUNCH_N(c, "k_rd_seg", kseg<<<grid, SG_NT, smem, c->stream>>>(val, seg, seg_cm, seg_cm + 2, log2bins, nbins,
+                                                                        d_hist, d_stats, O));
+  unsigned int* hcm = (unsigned int*)((uint8_t*)c->hstage + 40);
+  if ((e = cudaMemcpyAsync(hcm, seg_cm, 16, cudaMemcpyDeviceToHost, c->stream))) return e;
+  if ((e = cudaStreamSynchronize(c->stream))) return e;
+  if (hcm[1] > SEG_TILE_MAX) return cudaSuccess;
+  const uint32_t nlong = hcm[3];
+  if (nlong && (e = rd_segment_tiles(c, val, seg_long, nlong, log2bins, nbins, d_hist, d_stats, O))) return e;
+  c->counts[1] = 0;
+  c->counts[3] = nlong;
+  *done = true;
+  return cudaGetLastError();
+}
+
 cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbins, uint64_t* d_hist,
                       uint64_t* d_stats, const ObjTab* obj) {
   cudaError_t e;
@@ -1983,40 +2071,9 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
           return e;
         key = (const uint32_t*)k0;
         val = (const uint64_t*)v0;
-        // every CTA segment <= SEG_TILE_MAX kept records: no cross-segment term
-        // exists, so every segment is resolved alone - short ones by a warp of
-        // the segment kernel, long ones by a CTA of the tile kernel
-        unsigned int* hcm = (unsigned int*)((uint8_t*)c->hstage + 40);
-        if ((e = cudaMemcpyAsync(hcm, seg_cm, 16, cudaMemcpyDeviceToHost, c->stream))) return e;
-        if ((e = cudaStreamSynchronize(c->stream))) return e;
-        if (hcm[1] <= SEG_TILE_MAX && getenv("CADV_RD_TILES") == nullptr) {
-          const uint32_t nshort = hcm[0], nlong = hcm[3];
-          const auto kseg = O.n ? k_rd_seg<true> : k_rd_seg<false>;
-          if (!(c->attr_set & (1u << 16))) {
-            for (const auto kf : {k_rd_seg<true>, k_rd_seg<false>})
-              if ((e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                            (int)(sizeof(SegSmem) + 16 * SG_OBJ_SMEM + 16))))
-                return e;
-            c->attr_set |= 1u << 16;
-          }
-          if (nshort) {
-            const uint64_t hbins = (uint64_t)(O.n + 1) * nbins;
-            const size_t smem = seg_smem_bytes(hbins, O.n);
-            if (c->seg_ctas_smem != smem) {
-              if ((e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&c->seg_ctas, kseg, SG_NT, smem))) return e;
-              if (c->seg_ctas < 1) c->seg_ctas = 1;
-              c->seg_ctas_smem = smem;
-            }
-            const unsigned grid =
-                (unsigned)std::min<uint64_t>((uint64_t)c->num_sms * c->seg_ctas, (nshort + SG_W - 1) / SG_W);
-            CADV_LAUNCH_N(c, "k_rd_seg", kseg<<<grid, SG_NT, smem, c->stream>>>(val, seg, seg_cm, seg_cm + 2, log2bins,
-                                                                                nbins, d_hist, d_stats, O));
-          }
-          if (nlong && (e = rd_segment_tiles(c, val, seg_long, nlong, log2bins, nbins, d_hist, d_stats, O))) return e;
-          c->counts[1] = 0;
-          c->counts[3] = nlong;
-          return cudaGetLastError();
-        }
+        bool done = false;
+        if ((e = rd_segments(c, val, seg, seg_long, seg_cm, P, log2bins, nbins, d_hist, d_stats, O, &done))) return e;
+        if (done) return cudaSuccess;
       } else {  // overflow: pack, then the radix sort
         if ((e = launch_squeeze(c, (const uint32_t*)k1, (const uint64_t*)v1, (uint32_t*)k0, (uint64_t*)v0, S.blkcnt,
                                 S.blkcnt + S.grid + 4, S.grid, S.chunk_cap)))
@@ -2047,6 +2104,19 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
   // redistributes the kept records by CTA range instead (rd_exchange).
   const bool spread = c->comm != nullptr && !cta_scope;
   if (c->comm && !spread && (e = rd_exchange(c, cta_scope, &key, &val, &K))) return e;
+  if (c->comm && cta_scope && K) {
+    // the rank's CTA range, CTA-major: the same segment path as one rank
+    void* sb;
+    if ((e = ensure(c, B_RG_SEG, (K + 16) * 16 + 64, &sb))) return e;
+    uint2* seg = (uint2*)sb;
+    uint2* seg_long = seg + (K + 16);
+    unsigned int* seg_cm = (unsigned int*)(seg_long + (K + 16));
+    if ((e = cudaMemsetAsync(seg_cm, 0, 16, c->stream))) return e;
+    CADV_LAUNCH(c, k_key_segments<<<grid_ls, 256, 0, c->stream>>>(key, K, seg, seg_long, seg_cm));
+    bool done = false;
+    if ((e = rd_segments(c, val, seg, seg_long, seg_cm, K, log2bins, nbins, d_hist, d_stats, O, &done))) return e;
+    if (done) return cudaSuccess;
+  }
   const uint64_t ntiles_loc = (K + TL_NOM - 1) / TL_NOM;
   uint64_t ntiles = ntiles_loc;  // tiles of all ranks (global tile ids)
   TilePos TP{0, 0, K};

@@ -91,10 +91,38 @@ __global__ void __launch_bounds__(SCAN_NT) k_scan_chunk(const T* in, T* out, uin
   if (d_total && blockIdx.x == gridDim.x - 1 && threadIdx.x == SCAN_NT - 1) *d_total = run;
 }
 
+// Exclusive scan of up to SCAN_SMALL elements in ONE launch (one block of
+// 1024 threads, each a contiguous run): the scans of the reuse path's
+// region counts, pair counts and radix digit matrices are this size, and a
+// single launch beats reduce + scan-of-partials + chunk (three dependent
+// launches, each a few microseconds of latency).  In place is allowed.
+constexpr int SCAN_SMALL_NT = 1024;
+constexpr uint64_t SCAN_SMALL = 128 * 1024;
+template <typename T>
+__global__ void __launch_bounds__(SCAN_SMALL_NT) k_scan_small(const T* in, T* out, uint64_t n, T* d_total) {
+  __shared__ T ws[SCAN_SMALL_NT / 32];
+  const uint64_t per = (n + SCAN_SMALL_NT - 1) / SCAN_SMALL_NT;
+  const uint64_t lo = threadIdx.x * per, hi = lo + per < n ? lo + per : n;
+  T s = 0;
+  for (uint64_t i = lo; i < hi; ++i) s += in[i];
+  T tot;
+  T run = block_scan_t<T, SCAN_SMALL_NT>(s, ws, &tot);
+  for (uint64_t i = lo; i < hi; ++i) {
+    const T v = in[i];
+    out[i] = run;
+    run += v;
+  }
+  if (d_total && threadIdx.x == 0) *d_total = tot;
+}
+
 template <typename T>
 cudaError_t scan_impl(cadv_ctx* c, const T* in, T* out, uint64_t n, T* d_total, int depth) {
   if (n == 0) return cudaSuccess;
   uint64_t nb = (n + SCAN_CH - 1) / SCAN_CH;
+  if (nb > 1 && n <= SCAN_SMALL && depth == 0) {
+    CADV_LAUNCH(c, k_scan_small<T><<<1, SCAN_SMALL_NT, 0, c->stream>>>(in, out, n, d_total));
+    return cudaGetLastError();
+  }
   if (nb == 1) {
     CADV_LAUNCH(c, k_scan_chunk<T><<<1, SCAN_NT, 0, c->stream>>>(in, out, n, nullptr, d_total));
     return cudaGetLastError();
