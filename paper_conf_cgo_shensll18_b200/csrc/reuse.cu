@@ -439,6 +439,17 @@ __device__ __forceinline__ uint64_t sh_cas64(uint32_t a, uint64_t cmp, uint64_t 
   return o;
 }
 
+// Inclusive warp scan step: x += the value o lanes below (when that lane
+// exists), with the shuffle's in-range predicate guarding the add (no SEL).
+__device__ __forceinline__ uint32_t scan_up_add(uint32_t x, uint32_t o) {
+  asm("{\n\t.reg .pred p;\n\t.reg .b32 y;\n\t"
+      "shfl.sync.up.b32 y|p, %0, %1, 0, 0xffffffff;\n\t"
+      "@p add.u32 %0, %0, y;\n\t}"
+      : "+r"(x)
+      : "r"(o));
+  return x;
+}
+
 // OBJ: data-centric rows (O.n > 0); the reuse-only instance carries none of it.
 template <bool OBJ>
 __global__ void __launch_bounds__(SG_NT, 5) k_rd_seg(const uint64_t* __restrict__ val, const uint2* __restrict__ seg,
@@ -505,10 +516,7 @@ __global__ void __launch_bounds__(SG_NT, 5) k_rd_seg(const uint64_t* __restrict_
       // weighted prefix (inclusive) by position (independent of the match: overlaps its latency)
       uint32_t xw = w;
 #pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, xw, o);
-        if (lane >= (uint32_t)o) xw += y;
-      }
+      for (int o = 1; o < 32; o <<= 1) xw = scan_up_add(xw, o);
       const uint32_t lower = peers & lanemask_lt();
       int32_t pp = -1;
       uint32_t hs = 0;  // the group's first lane: the line's slot (bit 16: present) or the first empty slot
@@ -603,10 +611,7 @@ __global__ void __launch_bounds__(SG_NT, 5) k_rd_seg(const uint64_t* __restrict_
       const uint32_t nr = lane < 8 ? sh_ld32(RW + 4 * lane) : 0u;
       uint32_t pc = __popc(nr), xc = pc;
 #pragma unroll
-      for (int o = 1; o < 8; o <<= 1) {
-        const uint32_t y = __shfl_up_sync(FULL, xc, o);
-        if (lane >= (uint32_t)o) xc += y;
-      }
+      for (int o = 1; o < 8; o <<= 1) xc = scan_up_add(xc, o);
       if (lane < 8) sh_st32(CW8 + 4 * lane, xc - pc);
       rtot += __popc(qm);  // every position is reused at most once: the round's P are new bits
       wb += __shfl_sync(FULL, xw, 31);
@@ -1312,6 +1317,73 @@ __global__ void __launch_bounds__(256) k_merge_count(const uint32_t* __restrict_
         ++ib;
         if (ib < lenB) kb = __ldg(B + ib);
       }
+    }
+  }
+}
+
+// The same level with shared-memory staging: block b produces the pair's
+// outputs [MPB_T b', MPB_T (b' + 1)) - the two input stretches that feed them
+// (found by one merge-path search per block boundary) are loaded coalesced
+// into shared memory, each thread merges MP_IT outputs from there.
+constexpr int MPB_NT = 256, MPB_T = MPB_NT * MP_IT;  // 2048 outputs per block
+__device__ __forceinline__ uint64_t merge_split(const uint32_t* A, uint64_t lenA, const uint32_t* B, uint64_t lenB,
+                                                uint64_t d) {
+  uint64_t lo = d > lenB ? d - lenB : 0, hi = d < lenA ? d : lenA;
+  while (lo < hi) {
+    const uint64_t mid = (lo + hi) >> 1;
+    if (A[mid] <= B[d - 1 - mid]) lo = mid + 1;
+    else hi = mid;
+  }
+  return lo;
+}
+__global__ void __launch_bounds__(MPB_NT) k_merge_count_tiled(const uint32_t* __restrict__ kin,
+                                                              const uint32_t* __restrict__ iin,
+                                                              uint32_t* __restrict__ kout, uint32_t* __restrict__ iout,
+                                                              uint64_t M, uint64_t w, uint32_t* __restrict__ cnt) {
+  __shared__ uint32_t sk[MPB_T], si[MPB_T];
+  __shared__ uint64_t s_a[2];
+  const uint64_t o0 = (uint64_t)blockIdx.x * MPB_T;  // blocks never straddle a pair: 2 w is a multiple of MPB_T
+  const uint64_t s = (o0 / (2 * w)) * (2 * w);
+  const uint64_t lenA = M - s < w ? M - s : w;
+  const uint64_t lenB = M - s > w ? (M - s - w < w ? M - s - w : w) : 0;
+  const uint64_t d0 = o0 - s;
+  const uint64_t dn = d0 + MPB_T < lenA + lenB ? d0 + MPB_T : lenA + lenB;
+  const uint32_t* A = kin + s;
+  const uint32_t* B = kin + s + lenA;
+  if (threadIdx.x < 2) s_a[threadIdx.x] = merge_split(A, lenA, B, lenB, threadIdx.x ? dn : d0);
+  __syncthreads();
+  const uint64_t a0 = s_a[0], a1 = s_a[1], b0 = d0 - a0, b1 = dn - a1;
+  const uint32_t na = (uint32_t)(a1 - a0), nt = (uint32_t)(dn - d0);
+  for (uint32_t x = threadIdx.x; x < nt; x += MPB_NT) {
+    if (x < na) { sk[x] = A[a0 + x]; si[x] = iin[s + a0 + x]; }
+    else { sk[x] = B[b0 + x - na]; si[x] = iin[s + lenA + b0 + x - na]; }
+  }
+  __syncthreads();
+  // local merge of sk[0, na) and sk[na, nt): this thread's outputs [d, d + MP_IT)
+  const uint32_t nb = nt - na, d = threadIdx.x * MP_IT;
+  if (d >= nt) return;
+  uint32_t lo = d > nb ? d - nb : 0, hi = d < na ? d : na;
+  while (lo < hi) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (sk[mid] <= sk[na + d - 1 - mid]) lo = mid + 1;
+    else hi = mid;
+  }
+  uint32_t ia = lo, ib = d - lo;
+#pragma unroll
+  for (int k = 0; k < MP_IT; ++k) {
+    const uint32_t o = d + k;
+    if (o >= nt) break;
+    if (ia < na && (ib >= nb || sk[ia] <= sk[na + ib])) {
+      kout[o0 + o] = sk[ia];
+      iout[o0 + o] = si[ia];
+      ++ia;
+    } else {
+      const uint32_t id = si[na + ib];
+      kout[o0 + o] = sk[na + ib];
+      iout[o0 + o] = id;
+      const uint64_t left = lenA - (a0 + ia);  // left-run items still unmerged: all larger
+      if (left) cnt[id] += (uint32_t)left;
+      ++ib;
     }
   }
 }
@@ -2347,7 +2419,11 @@ cudaError_t rd_finish(cadv_ctx* c, const RdState& S, int log2bins, uint32_t nbin
     std::swap(ka, kb);
     std::swap(ia, ib);
     for (uint64_t w = MC_BLOCK; w < M; w <<= 1) {
-      CADV_LAUNCH(c, k_merge_count<<<grid_ls, 256, 0, c->stream>>>(ka, ia, kb, ib, M, w, cnt));
+      if (getenv("CADV_MERGE_UNTILED"))
+        CADV_LAUNCH(c, k_merge_count<<<grid_ls, 256, 0, c->stream>>>(ka, ia, kb, ib, M, w, cnt));
+      else
+        CADV_LAUNCH(c, k_merge_count_tiled<<<(unsigned)((M + MPB_T - 1) / MPB_T), MPB_NT, 0, c->stream>>>(
+                           ka, ia, kb, ib, M, w, cnt));
       std::swap(ka, kb);
       std::swap(ia, ib);
     }

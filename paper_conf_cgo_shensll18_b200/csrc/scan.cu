@@ -1179,8 +1179,14 @@ void scan_geometry(cadv_ctx* c, uint64_t n, uint64_t* grid, uint64_t* nchunks, u
   if (c->scan_ctas > 0 && (uint64_t)c->scan_ctas < g) g = (uint64_t)c->scan_ctas;
   // up to 4 chunks per warp, none shorter than 64 steps (16 K records):
   // each chunk start waits for its first bulk copy with nothing to overlap
+  // (8 K-record chunks cost C2 0.38 -> 0.49 ms).  A trace below 2^28 records
+  // that already has 4 full chunks per warp gets 6: with fewer records per
+  // warp the cost variance between chunks is a larger share of the kernel
+  // (C3 BFS 2.19 -> 2.03 ms), while on C4 the extra regions cost the regroup
+  // more than they save.
   uint64_t split = n / (g * NWARP * 16384);
   split = split < 1 ? 1 : (split > 4 ? 4 : split);
+  if (split == 4 && n < (1ull << 28)) split = 6;
   if (c->scan_split > 0) split = (uint64_t)c->scan_split;
   const uint64_t tw = g * NWARP * split;
   uint64_t ch = (n + tw - 1) / tw;

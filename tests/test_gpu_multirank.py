@@ -257,3 +257,34 @@ def test_non_contiguous_shards(cadv, G, seed):
     out, err = run_ranks(cadv, t, cuts, fn, contiguous=False)
     assert not any(err), err
     check_all_equal(out, ref)
+
+
+@pytest.mark.parametrize("G", [2, 3])
+def test_cta_scope_segment_paths_per_rank(cadv, G):
+    """CTA scope over ranks: after the CTA-range exchange each rank resolves its
+    own CTA segments - segment kernel (<= 256 kept records), packed
+    segment-list tiles (<= 4096) - unless one of its segments is longer, which
+    sends that rank alone to the bounds-tiled path.  Short and medium CTAs
+    first, long (5000-record) CTAs last, so the ranks take different paths."""
+    rng = np.random.default_rng(G)
+    lens = list(rng.integers(1, 257, 40)) + list(rng.integers(257, 4097, 8)) + [5000, 4096, 5000]
+    addr, cta = [], []
+    for c, n in enumerate(lens):
+        lines = np.sort(rng.choice(1 << 20, max(2, int(n) // 3), replace=False)).astype(np.uint64)
+        seq = rng.choice(lines, int(n))
+        for k in range(1, int(n)):  # no two consecutive equal lines: every record is kept
+            if seq[k] == seq[k - 1]:
+                seq[k] = lines[(np.searchsorted(lines, seq[k]) + 1) % len(lines)]
+        addr.append(0x7F0000000000 + 128 * seq)
+        cta.append(np.full(int(n), c, dtype=np.uint64))
+    addr, cta = np.concatenate(addr), np.concatenate(cta)
+    n = len(addr)
+    meta = np.where(rng.random(n) < 0.1, (2 << 2) | 1, 2 << 2)
+    t = tg.from_arrays(addr, cta, rng.integers(0, 256, n), np.zeros(n), np.arange(n), meta, nsites=1)
+    cuts = random_cuts(t.n, G, seed=11 * G)
+    for binning, nb in ((0, 66), (1, 20)):
+        h_ref, s_ref = orc.reuse(t, 128, 0, binning, nb)
+        out, err = run_ranks(cadv, t, cuts, lambda c: c.reuse_histogram(128, 0, binning, nb))
+        assert not any(err), err
+        for h, s in out:
+            assert (h == h_ref).all() and s == s_ref
