@@ -132,3 +132,33 @@ def test_fused_non_contiguous(ctx, cadv, seed):
         rh, mh = ctx.data_centric(objs, 128, scope, 0, 66, 32)
         rr, mr = orc.data_centric(t, objs, 128, scope, 0, 66, 32)
         assert (rh == rr).all() and (mh == mr).all()
+
+
+@pytest.mark.parametrize("top", [(1 << 28) - 1, 1 << 28])
+def test_bd_cta_id_boundary(ctx, cadv, top):
+    """Branch divergence keeps T_c per CTA id: ids up to 2^28 - 1 are exact,
+    an id of 2^28 is CADV_ERR_UNSUPPORTED (include/cadv.h) - for the separate
+    and the fused call - while reuse and memory divergence take any id."""
+    t0 = tg.generate("rand", seed=9, ctas=4, threads=96, instrs=20, lines=40, pstore=0.2, pbb=0.4)
+    cols = {k: v.copy() for k, v in t0.cols.items()}
+    cols["cta"] = (cols["cta"].astype(np.int64) + (top - int(cols["cta"].max()))).astype(np.uint32)
+    t = tg.from_arrays(*(cols[k] for k, _ in tg.COLUMNS), nsites=t0.nsites)
+    assert int(t.cta.max()) == top
+    ctx.load_trace(cadv.to_device(t))
+    h, st = ctx.reuse_histogram(128, 0, 0, 66)
+    hr, sr = orc.reuse(t, 128, 0, 0, 66)
+    assert (h == hr).all() and st == sr
+    m, ps = ctx.mem_divergence(128, 32, t.nsites)
+    assert (m == orc.mem_div(t, 128, 32)[0]).all()
+    if top < (1 << 28):
+        ps, tot = ctx.branch_divergence(32, t.nsites)
+        psr, totr = orc.branch_div(t, 32)
+        assert (tot == totr).all() and (ps == psr).all()
+        out = ctx.analyze(rd=(128, 0, 0, 66), md=(128, 32), bd=32, nsites=t.nsites)
+        assert (out["branch_div"][1] == totr).all()
+    else:
+        for call in (lambda: ctx.branch_divergence(32, t.nsites),
+                     lambda: ctx.analyze(rd=(128, 0, 0, 66), md=(128, 32), bd=32, nsites=t.nsites)):
+            with pytest.raises(cadv.CadvError) as e:
+                call()
+            assert e.value.status == cadv.CADV_ERR_UNSUPPORTED
